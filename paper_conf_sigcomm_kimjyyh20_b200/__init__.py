@@ -1,0 +1,181 @@
+"""B200-native LiveNAS super-resolution hot path (SIGCOMM '20, Kim et al.).
+
+`SRContext` is a thin Python face of the C ABI in include/sr.h (libsr.so): torch is used for device memory
+and streams only; all compute runs in the library's sm_100a kernels.  See DESIGN.md.
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+from . import _lib
+from ._lib import MODELS, SRError, check, load, sr_options, sr_quality  # noqa: F401
+
+__all__ = ["SRContext", "load", "SRError", "MODELS"]
+
+
+def _ptr(t):
+    return C.c_void_p(t.data_ptr()) if t is not None else None
+
+
+def _stream(stream):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return C.c_void_p(s.cuda_stream)
+
+
+def _model(m):
+    return MODELS[m] if isinstance(m, str) else int(m)
+
+
+class SRContext:
+    """One per-stream SR network (sr_create).  Tensors passed in must be CUDA uint8 NHWC, contiguous."""
+
+    def __init__(self, scale: int, blocks: int, channels: int, seed: int = 0, lr: float = 0.0,
+                 world: int = 1, rank: int = 0, dp_weight: float = 0.0, recent_k: int = 0, recent_w: int = 0,
+                 pool_capacity: int = 0):
+        import torch
+        if not torch.cuda.is_available():
+            raise SRError("SRContext needs a CUDA device (no CPU fallback)")
+        self.lib = load()
+        self.scale, self.blocks, self.channels = scale, blocks, channels
+        opt = sr_options(seed=seed, lr=lr, world=world, rank=rank, dp_weight=dp_weight, recent_k=recent_k,
+                         recent_w=recent_w, pool_capacity=pool_capacity)
+        h = C.c_void_p()
+        st = self.lib.sr_create(scale, blocks, channels, C.byref(opt), C.byref(h))
+        if st != 0:
+            raise SRError(f"sr_create({scale},{blocks},{channels}) failed with status {st}")
+        self.h = h
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.sr_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---------------------------------------------------------------- parameters
+    @property
+    def num_params(self) -> int:
+        return int(self.lib.sr_num_params(self.h))
+
+    def get_params(self, which="train"):
+        import numpy as np
+        out = np.empty(self.num_params, dtype=np.float32)
+        check(self.lib.sr_get_params(self.h, _model(which), out.ctypes.data_as(C.c_void_p), out.size), self.h,
+              "sr_get_params")
+        return out
+
+    def set_params(self, flat):
+        import numpy as np
+        a = np.ascontiguousarray(flat, dtype=np.float32)
+        check(self.lib.sr_set_params(self.h, a.ctypes.data_as(C.c_void_p), a.size), self.h, "sr_set_params")
+
+    # ---------------------------------------------------------------- inference
+    def infer(self, lr, which="serve", out=None, stream=None):
+        import torch
+        n, h, w, _ = lr.shape
+        s = self.scale
+        if out is None:
+            out = torch.empty((n, s * h, s * w, 3), dtype=torch.uint8, device=lr.device)
+        check(self.lib.sr_infer(self.h, _model(which), _ptr(lr), n, h, w, _ptr(out), _stream(stream)), self.h,
+              "sr_infer")
+        return out
+
+    def infer_host(self, lr_host, out_host, which="serve", stream=None):
+        """lr_host / out_host: CPU uint8 tensors (pinned for speed)."""
+        n, h, w, _ = lr_host.shape
+        check(self.lib.sr_infer_host(self.h, _model(which), _ptr(lr_host), n, h, w, _ptr(out_host),
+                                     _stream(stream)), self.h, "sr_infer_host")
+        return out_host
+
+    def infer_rows(self, lr_frame, row0, row1, hr_frame, which="serve", stream=None):
+        h, w, _ = lr_frame.shape
+        check(self.lib.sr_infer_rows(self.h, _model(which), _ptr(lr_frame), h, w, row0, row1, _ptr(hr_frame),
+                                     _stream(stream)), self.h, "sr_infer_rows")
+        return hr_frame
+
+    # ---------------------------------------------------------------- training
+    def train_step(self, lr, hr, loss=None, stream=None):
+        n, p = lr.shape[0], lr.shape[1]
+        check(self.lib.sr_train_step(self.h, _ptr(lr), _ptr(hr), n, p, _ptr(loss), _stream(stream)), self.h,
+              "sr_train_step")
+
+    def train_grad(self, lr, hr, loss=None, stream=None):
+        n, p = lr.shape[0], lr.shape[1]
+        check(self.lib.sr_train_grad(self.h, _ptr(lr), _ptr(hr), n, p, _ptr(loss), _stream(stream)), self.h,
+              "sr_train_grad")
+
+    def grad_buffer(self):
+        """torch view of the flat fp32 gradient (for an NCCL allreduce via torch.distributed)."""
+        import torch
+        ptr = self.lib.sr_grad_buffer(self.h)
+        n = self.num_params
+        return _wrap_device_f32(ptr, n, torch.cuda.current_device())
+
+    def train_apply(self, grad_scale=1.0, stream=None):
+        check(self.lib.sr_train_apply(self.h, C.c_float(grad_scale), _stream(stream)), self.h, "sr_train_apply")
+
+    def pool_push(self, lr, hr, stream=None):
+        n, pp = lr.shape[0], lr.shape[1]
+        check(self.lib.sr_pool_push(self.h, _ptr(lr), _ptr(hr), n, pp, None, _stream(stream)), self.h,
+              "sr_pool_push")
+
+    @property
+    def pool_size(self) -> int:
+        return int(self.lib.sr_pool_size(self.h))
+
+    def sample_batch(self, step, batch, p, out=None, stream=None):
+        import torch
+        s = self.scale
+        if out is None:
+            lr = torch.empty((batch, p, p, 3), dtype=torch.uint8, device="cuda")
+            hr = torch.empty((batch, s * p, s * p, 3), dtype=torch.uint8, device="cuda")
+            idx = torch.empty(batch, dtype=torch.int32, device="cuda")
+        else:
+            lr, hr, idx = out
+        check(self.lib.sr_sample_batch(self.h, step, batch, p, _ptr(lr), _ptr(hr), _ptr(idx), _stream(stream)),
+              self.h, "sr_sample_batch")
+        return lr, hr, idx
+
+    def train_sampled(self, iters, batch, p, loss=None, stream=None):
+        check(self.lib.sr_train_sampled(self.h, iters, batch, p, _ptr(loss), _stream(stream)), self.h,
+              "sr_train_sampled")
+
+    def publish(self, stream=None):
+        check(self.lib.sr_publish(self.h, _stream(stream)), self.h, "sr_publish")
+
+    def psnr_gain(self, lr, hr, a="serve", b="bilinear", stream=None):
+        q = sr_quality()
+        n, p = lr.shape[0], lr.shape[1]
+        check(self.lib.sr_psnr_gain(self.h, _model(a), _model(b), _ptr(lr), _ptr(hr), n, p, C.byref(q),
+                                    _stream(stream)), self.h, "sr_psnr_gain")
+        return q.psnr_a, q.psnr_b, q.gain
+
+    def kernel_timing(self, enable=True):
+        check(self.lib.sr_kernel_timing(self.h, int(enable)), self.h, "sr_kernel_timing")
+
+    def kernel_stats(self):
+        import json
+        buf = C.create_string_buffer(1 << 16)
+        n = self.lib.sr_kernel_stats(self.h, buf, len(buf))
+        if n < 0:
+            raise SRError(f"sr_kernel_stats failed: {n}")
+        return json.loads(buf.value.decode())
+
+    @property
+    def launches(self) -> int:
+        return int(self.lib.sr_launch_count(self.h))
+
+
+def _wrap_device_f32(ptr, n, device):
+    """Zero-copy torch tensor over a device pointer owned by the ctx (via __cuda_array_interface__)."""
+    import torch
+
+    class _Arr:
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "<f4", "data": (ptr, False), "version": 3,
+                                    "strides": None}
+    return torch.as_tensor(_Arr(), device=f"cuda:{device}")

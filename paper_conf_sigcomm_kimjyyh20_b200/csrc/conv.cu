@@ -1,0 +1,633 @@
+// 3x3 convolutions on the 5th-gen tensor cores (tcgen05) for sm_100a: implicit GEMM, TMA-staged NHWC bf16
+// tiles, fp32 accumulators in TMEM, fused epilogues.
+//
+//   forward / data-grad:  D[pixel, co] = sum_{tap, ci} X[pixel + tap, ci] * W[tap, ci, co]
+//       M = 128 output positions per MMA tile, N = Cout (padded to 16), K = 9 taps x Cin.
+//       The tap shift is free: the A operand of tap (dy,dx) is the same smem tile with the descriptor start
+//       address moved by (dy*P + dx) * 16 bytes (SWIZZLE_NONE K-major layout = one 16-byte row per pixel).
+//   weight-grad:  D[(dy, ci), co] (for each dx) = sum_pixel X[pixel + (dy,dx), ci] * dY[pixel, co]
+//       K = pixels, both operands MN-major from row-planar smem tiles; split-K over CTAs, deterministic
+//       reduction in a second kernel.
+//
+// Warp roles (192 threads): warp 0 = TMA producer, warp 1 = TMEM allocator + single-thread MMA issuer,
+// warps 2..5 = epilogue (TMEM -> registers -> bias/ReLU/residual/mask or pixel-shuffle tail -> HBM).
+#include <cuda.h>
+#include "ptx.cuh"
+#include "tmap.h"
+#include "sr_internal.h"
+#include "kernels.h"
+
+namespace sr {
+
+static constexpr int kConvThreads = 192;
+static constexpr int kStages = 2;
+static constexpr int kSmemLimit = 227 * 1024;
+
+int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+// ------------------------------------------------------------------------------------------ geometry
+static size_t conv_smem(int cinp, int coutp, int R, int P, int n_mt, int MS) {
+  size_t wbytes = (size_t)9 * cinp * coutp * 2;
+  size_t stage = ((size_t)(cinp / 8) * (R + 2) * P * 16 + 1023) / 1024 * 1024;  // TMA dst: 128-B aligned
+  long over = (long)(n_mt - 1) * MS + 128 + 2 * P + 2 - (long)(R + 2) * P;  // positions read past a plane
+  size_t slack = over > 0 ? (size_t)over * 16 : 0;
+  return 1024 + wbytes + kStages * stage + slack + 16 + coutp * 4;
+}
+
+ConvGeom make_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes) {
+  ConvGeom g{};
+  g.N = N; g.H = H; g.W = W;
+  if (W >= 96) {  // wide: one 128-pixel output row segment per M-tile
+    g.TW = 128; g.P = 130; g.wide = 1; g.MS = g.P;
+    int R = 4;
+    while (R > 1 && conv_smem(cinp, coutp, R, g.P, R, g.MS) > (size_t)kSmemLimit) --R;
+    g.R = R < H ? R : H;
+    g.n_mt = g.R;
+  } else {        // narrow (training patches): M-tiles run across rows of a pitch-(W+2) tile
+    g.TW = W; g.P = W + 2; g.wide = 0; g.MS = 128;
+    int R = (640 + g.P - 1) / g.P;
+    if (R > H) R = H;
+    for (;;) {
+      int n_mt = (R * g.P + 127) / 128;
+      if (R == 1 || conv_smem(cinp, coutp, R, g.P, n_mt, 128) <= (size_t)kSmemLimit) break;
+      --R;
+    }
+    g.R = R;
+    g.n_mt = (R * g.P + 127) / 128;
+  }
+  g.tiles_x = (W + g.TW - 1) / g.TW;
+  g.tiles_y = (H + g.R - 1) / g.R;
+  g.units = N * g.tiles_x * g.tiles_y;
+  if (smem_bytes) *smem_bytes = conv_smem(cinp, coutp, g.R, g.P, g.n_mt, g.MS);
+  return g;
+}
+
+// ------------------------------------------------------------------------------------------ epilogues
+template <int COUTP>
+__device__ __forceinline__ void load_bf16_row(const bf16* p, float* v) {
+  const uint4* q = reinterpret_cast<const uint4*>(p);
+#pragma unroll
+  for (int i = 0; i < COUTP / 8; ++i) {
+    uint4 u = __ldg(q + i);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      float2 f = __bfloat1622float2(h[j]);
+      v[i * 8 + 2 * j] = f.x;
+      v[i * 8 + 2 * j + 1] = f.y;
+    }
+  }
+}
+
+template <int COUTP>
+__device__ __forceinline__ void store_bf16_row(bf16* p, const float* v) {
+  uint4* q = reinterpret_cast<uint4*>(p);
+#pragma unroll
+  for (int i = 0; i < COUTP / 8; ++i) {
+    uint4 u;
+    u.x = pack_bf16x2(v[i * 8 + 0], v[i * 8 + 1]);
+    u.y = pack_bf16x2(v[i * 8 + 2], v[i * 8 + 3]);
+    u.z = pack_bf16x2(v[i * 8 + 4], v[i * 8 + 5]);
+    u.w = pack_bf16x2(v[i * 8 + 6], v[i * 8 + 7]);
+    q[i] = u;
+  }
+}
+
+template <int COUTP>
+__device__ __forceinline__ void epi_act(const EpiParams& ep, const float* sbias, size_t pix, float* v) {
+  if (ep.bias) {
+#pragma unroll
+    for (int c = 0; c < COUTP; ++c) v[c] += sbias[c];
+  }
+  if (ep.res1) {
+    float r[COUTP];
+    load_bf16_row<COUTP>(ep.res1 + pix * COUTP, r);
+#pragma unroll
+    for (int c = 0; c < COUTP; ++c) v[c] += r[c];
+  }
+  if (ep.res2) {
+    float r[COUTP];
+    load_bf16_row<COUTP>(ep.res2 + pix * COUTP, r);
+#pragma unroll
+    for (int c = 0; c < COUTP; ++c) v[c] += r[c];
+  }
+  if (ep.relu) {
+#pragma unroll
+    for (int c = 0; c < COUTP; ++c) v[c] = fmaxf(v[c], 0.f);
+  }
+  if (ep.mask) {
+    float r[COUTP];
+    load_bf16_row<COUTP>(ep.mask + pix * COUTP, r);
+#pragma unroll
+    for (int c = 0; c < COUTP; ++c) v[c] = r[c] > 0.f ? v[c] : 0.f;
+  }
+  store_bf16_row<COUTP>(ep.out + pix * COUTP, v);
+}
+
+// Bilinear skip by output phase (half-pixel centres, edge replicate == PyTorch align_corners=False):
+//   x2: phase 0 -> 0.25 v[i-1] + 0.75 v[i];  phase 1 -> 0.75 v[i] + 0.25 v[i+1]
+//   x3: phase 0 -> v[i-1]/3 + 2 v[i]/3;  phase 1 -> v[i];  phase 2 -> 2 v[i]/3 + v[i+1]/3
+template <int S>
+__device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp) {
+  if (S == 2) {
+    wm = ph == 0 ? 0.25f : 0.f;
+    w0 = 0.75f;
+    wp = ph == 1 ? 0.25f : 0.f;
+  } else {
+    const float t = 1.f / 3.f, tt = 2.f / 3.f;
+    wm = ph == 0 ? t : 0.f;
+    w0 = ph == 1 ? 1.f : tt;
+    wp = ph == 2 ? t : 0.f;
+  }
+}
+
+// Tail: y = acc + b (3 s^2 channels, index c*s^2 + i*s + j = pixel-shuffle phase (i,j) of colour c);
+// skip = bilinear_s(v) at HR (sY+i, sX+j).  Inference: u8 = RNE(clamp(255 y + skip, 0, 255)).
+// Training: o = y + skip/255, d = o - hr/255 -> loss += d^2, dy[c s^2 + i s + j] = 2 d.
+template <int S, int COUTP, bool TRAIN>
+__device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias, int n, int Y, int X, int H,
+                                         int W, float* v, float& lsum) {
+  const uint8_t* lr = ep.lr + (size_t)n * H * W * 3;
+  float nb[3][3][3];  // [dy][dx][c] neighbourhood of LR pixel (Y,X), clamped (edge replicate)
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    int yy = min(max(Y + a - 1, 0), H - 1);
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      int xx = min(max(X + b - 1, 0), W - 1);
+      const uint8_t* p = lr + ((size_t)yy * W + xx) * 3;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) nb[a][b][c] = (float)__ldg(p + c);
+    }
+  }
+  const int sH = S * H, sW = S * W;
+  float dyv[COUTP];
+#pragma unroll
+  for (int k = 0; k < COUTP; ++k) dyv[k] = 0.f;
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    float ym, y0, yp;
+    phase_w<S>(i, ym, y0, yp);
+    uint8_t* hrow = TRAIN ? nullptr : ep.hr + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3;
+    const uint8_t* trow =
+        TRAIN ? ep.hr_ref + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3 : nullptr;
+#pragma unroll
+    for (int j = 0; j < S; ++j) {
+      float xm, x0, xp;
+      phase_w<S>(j, xm, x0, xp);
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        // horizontal pass on the three LR rows, then vertical
+        float h0 = xm * nb[0][0][c] + x0 * nb[0][1][c] + xp * nb[0][2][c];
+        float h1 = xm * nb[1][0][c] + x0 * nb[1][1][c] + xp * nb[1][2][c];
+        float h2 = xm * nb[2][0][c] + x0 * nb[2][1][c] + xp * nb[2][2][c];
+        float skip = ym * h0 + y0 * h1 + yp * h2;
+        const int k = c * S * S + i * S + j;
+        float y = v[k] + sbias[k];
+        if (TRAIN) {
+          float o = y + skip * (1.f / 255.f);
+          float d = o - (float)__ldg(trow + j * 3 + c) * (1.f / 255.f);
+          lsum += d * d;
+          dyv[k] = 2.f * d;
+        } else {
+          float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
+          hrow[j * 3 + c] = (uint8_t)__float2int_rn(o);
+        }
+      }
+    }
+  }
+  if (TRAIN) store_bf16_row<COUTP>(ep.dy + (((size_t)n * H + Y) * W + X) * COUTP, dyv);
+}
+
+// ------------------------------------------------------------------------------------------ conv kernel
+template <int CINP, int COUTP, int EPI, int S>
+__global__ void __launch_bounds__(kConvThreads, 1)
+k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wpk, const ConvGeom g,
+          const EpiParams ep) {
+  constexpr int CCH = CINP / 8;
+  constexpr int KSTEPS = CINP / 16;
+  constexpr uint32_t WBYTES = 9u * CINP * COUTP * 2u;
+  constexpr int SLOT = COUTP <= 32 ? 32 : (COUTP <= 64 ? 64 : 128);
+  constexpr int NSLOT = 4;
+  constexpr uint32_t TMEM_COLS = SLOT * NSLOT;
+  constexpr uint32_t IDESC = make_idesc(128, COUTP, 0, 0);
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], tfull_bar[NSLOT], tempty_bar[NSLOT];
+  __shared__ __align__(8) uint64_t w_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ float sbias[COUTP];
+
+  const int P = g.P;
+  const uint32_t plane = (uint32_t)(g.R + 2) * P * 16;
+  const uint32_t stage_bytes = plane * CCH;                            // TMA box bytes
+  const uint32_t stage_stride = (stage_bytes + 1023u) & ~1023u;        // smem stage stride (TMA dst alignment)
+  uint8_t* sW = smem;
+  uint8_t* sStage = smem + WBYTES;
+
+  const int warp = warp_id();
+  if (threadIdx.x < COUTP) sbias[threadIdx.x] = ep.bias ? ep.bias[threadIdx.x] : 0.f;
+  if (warp == 0 && lane_id() == 0) {
+    for (int s = 0; s < kStages; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
+    for (int s = 0; s < NSLOT; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4); }
+    mbar_init(&w_bar, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<TMEM_COLS>(&tmem_base_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const int tiles_xy = g.tiles_x * g.tiles_y;
+
+  if (warp == 0) {
+    // ===================== TMA producer =====================
+    if (elect_one()) {
+      tma_prefetch_desc(&tm_in);
+      mbar_arrive_expect_tx(&w_bar, WBYTES);
+      bulk_load(sW, wpk, WBYTES, &w_bar);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+        const int n = u / tiles_xy, rem = u - n * tiles_xy;
+        const int ty = rem / g.tiles_x, tx = rem - ty * g.tiles_x;
+        mbar_wait(&empty_bar[s], ph ^ 1);
+        mbar_arrive_expect_tx(&full_bar[s], stage_bytes);
+        tma_load_5d(sStage + s * stage_stride, &tm_in, &full_bar[s], 0, tx * g.TW - 1, ty * g.R - 1, 0, n);
+        if (++s == kStages) { s = 0; ph ^= 1; }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    // ===================== MMA issuer (one thread) =====================
+    if (elect_one()) {
+      mbar_wait(&w_bar, 0);
+      const uint64_t bdesc0 = make_desc(smem_u32(sW), COUTP * 16, 128);
+      int s = 0, slot = 0;
+      uint32_t ph = 0, tph = 0;
+      for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+        mbar_wait(&full_bar[s], ph);
+        tc_fence_after();
+        const uint64_t adesc0 = make_desc(smem_u32(sStage + s * stage_stride), plane, 128);
+        for (int mt = 0; mt < g.n_mt; ++mt) {
+          mbar_wait(&tempty_bar[slot], tph ^ 1);
+          tc_fence_after();
+          const uint32_t d = tmem + slot * SLOT;
+#pragma unroll
+          for (int tap = 0; tap < 9; ++tap) {
+            const uint32_t aoff = (uint32_t)(mt * g.MS + (tap / 3) * P + (tap % 3)) * 16u;
+#pragma unroll
+            for (int ks = 0; ks < KSTEPS; ++ks) {
+              mma_bf16_ss(d, desc_add(adesc0, aoff + ks * 2 * plane),
+                          desc_add(bdesc0, (uint32_t)(tap * CCH + 2 * ks) * COUTP * 16u), IDESC,
+                          (tap | ks) != 0);
+            }
+          }
+          mma_commit(&tfull_bar[slot]);
+          if (++slot == NSLOT) { slot = 0; tph ^= 1; }
+        }
+        mma_commit(&empty_bar[s]);
+        if (++s == kStages) { s = 0; ph ^= 1; }
+      }
+    }
+    __syncwarp();
+  } else {
+    // ===================== epilogue (warps 2..5) =====================
+    const int quarter = warp & 3;  // TMEM lane quarter this warp may access
+    const int row = quarter * 32 + lane_id();
+    int slot = 0;
+    uint32_t tph = 0;
+    float lsum = 0.f;
+    for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+      const int n = u / tiles_xy, rem = u - n * tiles_xy;
+      const int ty = rem / g.tiles_x, tx = rem - ty * g.tiles_x;
+      const int y0 = ty * g.R, x0 = tx * g.TW;
+      for (int mt = 0; mt < g.n_mt; ++mt) {
+        mbar_wait(&tfull_bar[slot], tph);
+        tc_fence_after();
+        float v[COUTP];
+#pragma unroll
+        for (int c0 = 0; c0 < COUTP; c0 += 16)
+          tmem_ld16(tmem + ((uint32_t)(quarter * 32) << 16) + slot * SLOT + c0, v + c0);
+        tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&tempty_bar[slot]);
+        if (++slot == NSLOT) { slot = 0; tph ^= 1; }
+        int r, x;
+        if (g.wide) { r = mt; x = row; }
+        else { const int q = mt * 128 + row; r = q / P; x = q - r * P; }
+        const int Y = y0 + r, X = x0 + x;
+        const bool valid = x < g.TW && r < g.R && Y < g.H && X < g.W;
+        if (!valid) continue;
+        if (EPI == EPI_ACT) {
+          epi_act<COUTP>(ep, sbias, ((size_t)n * g.H + Y) * g.W + X, v);
+        } else if (EPI == EPI_TAIL_U8) {
+          if (Y >= ep.hr_row0 && Y < ep.hr_row1) epi_tail<S, COUTP, false>(ep, sbias, n, Y, X, g.H, g.W, v, lsum);
+        } else {
+          epi_tail<S, COUTP, true>(ep, sbias, n, Y, X, g.H, g.W, v, lsum);
+        }
+      }
+    }
+    if (EPI == EPI_TAIL_TRAIN) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, o);
+      if (lane_id() == 0) atomicAdd(ep.loss_sum, (double)lsum);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<TMEM_COLS>(tmem);
+}
+
+template <int CINP, int COUTP, int EPI, int S>
+static cudaError_t launch_conv_t(const CUtensorMap& tm, const bf16* wpk, const ConvGeom& g, const EpiParams& ep,
+                                 size_t smem, int grid, cudaStream_t st) {
+  auto kern = k_conv3x3<CINP, COUTP, EPI, S>;
+  static size_t configured = 0;
+  if (smem > configured) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    configured = smem;
+  }
+  kern<<<grid, kConvThreads, smem, st>>>(tm, wpk, g, ep);
+  return cudaGetLastError();
+}
+
+#define SR_CONV_CASE(CI, CO)                                                                 \
+  if (cinp == CI && coutp == CO) {                                                           \
+    if (epi == EPI_ACT) return launch_conv_t<CI, CO, EPI_ACT, 1>(tm, wpk, g, ep, smem, grid, st); \
+  }
+#define SR_TAIL_CASE(CI, CO, S)                                                                          \
+  if (cinp == CI && coutp == CO && ep.scale == S) {                                                      \
+    if (epi == EPI_TAIL_U8) return launch_conv_t<CI, CO, EPI_TAIL_U8, S>(tm, wpk, g, ep, smem, grid, st);  \
+    if (epi == EPI_TAIL_TRAIN)                                                                           \
+      return launch_conv_t<CI, CO, EPI_TAIL_TRAIN, S>(tm, wpk, g, ep, smem, grid, st);                   \
+  }
+
+cudaError_t launch_conv(int cinp, int coutp, int epi, const void* in, const bf16* wpk, const ConvGeom& g,
+                        const EpiParams& ep, size_t smem, int grid, cudaStream_t st) {
+  CUtensorMap tm;
+  if (make_act_tmap(&tm, in, g.N, g.H, g.W, cinp, g.P, g.R + 2, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
+    return cudaErrorInvalidValue;
+  // head (16 -> C), body/blocks (C -> C), data-grad of the up conv (16/32 -> C)
+  SR_CONV_CASE(16, 16) SR_CONV_CASE(16, 32) SR_CONV_CASE(16, 48) SR_CONV_CASE(16, 64)
+  SR_CONV_CASE(32, 16) SR_CONV_CASE(32, 32) SR_CONV_CASE(32, 48) SR_CONV_CASE(32, 64)
+  SR_CONV_CASE(48, 16) SR_CONV_CASE(48, 32) SR_CONV_CASE(48, 48)
+  SR_CONV_CASE(64, 16) SR_CONV_CASE(64, 32) SR_CONV_CASE(64, 64)
+  // up conv + tail (C -> 3 s^2 padded: 12 -> 16, 27 -> 32)
+  SR_TAIL_CASE(16, 16, 2) SR_TAIL_CASE(32, 16, 2) SR_TAIL_CASE(48, 16, 2) SR_TAIL_CASE(64, 16, 2)
+  SR_TAIL_CASE(16, 32, 3) SR_TAIL_CASE(32, 32, 3) SR_TAIL_CASE(48, 32, 3) SR_TAIL_CASE(64, 32, 3)
+  return cudaErrorNotSupported;
+}
+
+// ------------------------------------------------------------------------------------------ weight grad
+// Stage: X tile (R+2) rows x P=TW+2 px, row-planar [row][chunk][px]; dY tile R rows x TW px row-planar.
+// A (MN-major) = X^T: 8-row groups g = dy*CCH + j at stride SBO = P*16 (rows are consecutive planes), K =
+// pixel at 16 B, K-groups LBO = 128.  B (MN-major) = dY: N-groups (co chunks) SBO = TW*16, LBO = 128.
+// D[dx][mt] (128 lanes = 16 groups of 8 (dy,ci) rows, COUTP columns), accumulated over all of this CTA's
+// K (split-K); written as a per-CTA partial, summed by k_wgrad_reduce in CTA order (deterministic).
+static size_t wgrad_smem(int cinp, int coutp, int R, int TW) {
+  const int P = TW + 2;
+  const int cch = cinp / 8, och = coutp / 8;
+  const int n_mt = (3 * cch + 15) / 16;
+  size_t xs = ((size_t)(R + 2) * cch * P * 16 + 1023) / 1024 * 1024;
+  size_t ys = ((size_t)R * och * TW * 16 + 1023) / 1024 * 1024;
+  long over = (long)(16 * n_mt - 3 * cch) * P * 16 + 64;  // rows read past the X tile by padded M-tiles
+  return 1024 + kStages * (xs + ys) + (over > 0 ? (size_t)over : 0) + 256;
+}
+
+WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes) {
+  WgradGeom g{};
+  g.N = N; g.H = H; g.W = W;
+  g.TW = W >= 64 ? 64 : ((W + 15) / 16) * 16;
+  g.P = g.TW + 2;
+  int R = 4;
+  while (R > 1 && wgrad_smem(cinp, coutp, R, g.TW) > (size_t)kSmemLimit) --R;
+  g.R = R < H ? R : H;
+  g.tiles_x = (W + g.TW - 1) / g.TW;
+  g.tiles_y = (H + g.R - 1) / g.R;
+  g.units = N * g.tiles_x * g.tiles_y;
+  if (smem_bytes) *smem_bytes = wgrad_smem(cinp, coutp, g.R, g.TW);
+  return g;
+}
+
+template <int CINP, int COUTP>
+__global__ void __launch_bounds__(kConvThreads, 1)
+k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_dy, const WgradGeom g,
+        float* __restrict__ ws_w, float* __restrict__ ws_b) {
+  constexpr int CCH = CINP / 8, OCH = COUTP / 8;
+  constexpr int NMT = (3 * CCH + 15) / 16;
+  constexpr uint32_t TMEM_NEED = 3 * NMT * COUTP;
+  constexpr uint32_t TMEM_COLS = TMEM_NEED <= 32 ? 32 : TMEM_NEED <= 64 ? 64 : TMEM_NEED <= 128 ? 128
+                                 : TMEM_NEED <= 256 ? 256 : 512;
+  static_assert(TMEM_NEED <= 512, "wgrad accumulators exceed TMEM");
+  constexpr uint32_t IDESC = make_idesc(128, COUTP, 1, 1);
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], done_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ float sdb[8][COUTP];
+
+  const int TW = g.TW, P = g.P, R = g.R;
+  const uint32_t xbox = (uint32_t)(R + 2) * CCH * P * 16, ybox = (uint32_t)R * OCH * TW * 16;  // TMA box bytes
+  const uint32_t xbytes = (xbox + 1023u) & ~1023u;      // dY tile offset inside a stage (128-B TMA alignment)
+  const uint32_t ybytes = (ybox + 1023u) & ~1023u;
+  const uint32_t stage_bytes = xbytes + ybytes;
+  const int warp = warp_id();
+  if (warp == 0 && lane_id() == 0) {
+    for (int s = 0; s < kStages; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 2); }
+    mbar_init(&done_bar, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<TMEM_COLS>(&tmem_base_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const int tiles_xy = g.tiles_x * g.tiles_y;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      tma_prefetch_desc(&tm_x);
+      tma_prefetch_desc(&tm_dy);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+        const int n = u / tiles_xy, rem = u - n * tiles_xy;
+        const int ty = rem / g.tiles_x, tx = rem - ty * g.tiles_x;
+        mbar_wait(&empty_bar[s], ph ^ 1);
+        mbar_arrive_expect_tx(&full_bar[s], xbox + ybox);
+        uint8_t* base = smem + s * stage_bytes;
+        tma_load_5d(base, &tm_x, &full_bar[s], 0, tx * TW - 1, 0, ty * R - 1, n);
+        tma_load_5d(base + xbytes, &tm_dy, &full_bar[s], 0, tx * TW, 0, ty * R, n);
+        if (++s == kStages) { s = 0; ph ^= 1; }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (elect_one()) {
+      int s = 0;
+      uint32_t ph = 0;
+      uint32_t acc = 0;
+      for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+        mbar_wait(&full_bar[s], ph);
+        tc_fence_after();
+        const uint32_t xb = smem_u32(smem + s * stage_bytes);
+        const uint32_t yb = xb + xbytes;
+        const uint64_t a0 = make_desc(xb, 128, P * 16);
+        const uint64_t b0 = make_desc(yb, 128, TW * 16);
+        for (int r = 0; r < R; ++r) {
+          for (int k16 = 0; k16 < TW / 16; ++k16) {
+            const uint32_t boff = (uint32_t)(r * OCH * TW + k16 * 16) * 16u;
+#pragma unroll
+            for (int dx = 0; dx < 3; ++dx) {
+#pragma unroll
+              for (int mt = 0; mt < NMT; ++mt) {
+                const uint32_t aoff = (uint32_t)((r * CCH + 16 * mt) * P + k16 * 16 + dx) * 16u;
+                mma_bf16_ss(tmem + (dx * NMT + mt) * COUTP, desc_add(a0, aoff), desc_add(b0, boff), IDESC, acc);
+              }
+            }
+            acc = 1;
+          }
+        }
+        mma_commit(&empty_bar[s]);
+        if (++s == kStages) { s = 0; ph ^= 1; }
+      }
+      mma_commit(&done_bar);
+    }
+    __syncwarp();
+  } else {
+    // epilogue warps: bias gradient from the dY tiles while the MMAs run, then drain the accumulators
+    const int et = threadIdx.x - 64;  // 0..127
+    const int c = et % COUTP;
+    const int part = et / COUTP;      // thread groups summing disjoint pixel subsets
+    const int nparts = 128 / COUTP;
+    float dbsum = 0.f;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+      mbar_wait(&full_bar[s], ph);
+      if (part < nparts) {
+        const bf16* yt = reinterpret_cast<const bf16*>(smem + s * stage_bytes + xbytes);
+        for (int q = part; q < R * TW; q += nparts) {
+          const int r = q / TW, p = q - r * TW;
+          dbsum += __bfloat162float(yt[((size_t)(r * OCH + c / 8) * TW + p) * 8 + (c % 8)]);
+        }
+      }
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (et == 0) mbar_arrive(&empty_bar[s]);
+      if (++s == kStages) { s = 0; ph ^= 1; }
+    }
+    if (part < nparts) sdb[part][c] = dbsum;
+    asm volatile("bar.sync 1, 128;" ::: "memory");
+    if (et < COUTP) {
+      float t = 0.f;
+      for (int p2 = 0; p2 < nparts; ++p2) t += sdb[p2][et];
+      ws_b[(size_t)blockIdx.x * COUTP + et] = t;
+    }
+    // drain: lane m of M-tile mt = row (16*mt + m/8 -> (dy, j)), ci = 8 j + m % 8
+    mbar_wait(&done_bar, 0);
+    tc_fence_after();
+    const int quarter = warp & 3;
+    const int m = quarter * 32 + lane_id();
+    float* outp = ws_w + (size_t)blockIdx.x * 9 * CINP * COUTP;
+#pragma unroll
+    for (int dx = 0; dx < 3; ++dx) {
+#pragma unroll
+      for (int mt = 0; mt < NMT; ++mt) {
+        const int grp = 16 * mt + m / 8;
+        const bool ok = grp < 3 * CCH;
+        const int dy = grp / CCH, j = grp % CCH;
+        const int ci = 8 * j + (m % 8);
+#pragma unroll
+        for (int c0 = 0; c0 < COUTP; c0 += 16) {
+          float v[16];
+          tmem_ld16(tmem + ((uint32_t)(quarter * 32) << 16) + (dx * NMT + mt) * COUTP + c0, v);
+          tmem_ld_wait();
+          if (ok) {
+            float* o = outp + ((size_t)(dy * 3 + dx) * CINP + ci) * COUTP + c0;
+#pragma unroll
+            for (int q = 0; q < 16; ++q) o[q] = v[q];
+          }
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<TMEM_COLS>(tmem);
+}
+
+template <int CINP, int COUTP>
+static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, const WgradGeom& g, float* ws_w,
+                                  float* ws_b, size_t smem, int grid, cudaStream_t st) {
+  auto kern = k_wgrad<CINP, COUTP>;
+  static size_t configured = 0;
+  if (smem > configured) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    configured = smem;
+  }
+  kern<<<grid, kConvThreads, smem, st>>>(tx, ty, g, ws_w, ws_b);
+  return cudaGetLastError();
+}
+
+#define SR_WG_CASE(CI, CO) \
+  if (cinp == CI && coutp == CO) return launch_wgrad_t<CI, CO>(tx, ty, g, ws_w, ws_b, smem, grid, st);
+
+cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, float* ws_w,
+                         float* ws_b, size_t smem, int grid, cudaStream_t st) {
+  CUtensorMap tx, ty;
+  if (make_act_tmap(&tx, x, g.N, g.H, g.W, cinp, g.P, g.R + 2, cinp / 8, ROW_CHUNK_PIX) != CUDA_SUCCESS)
+    return cudaErrorInvalidValue;
+  if (make_act_tmap(&ty, dy, g.N, g.H, g.W, coutp, g.TW, g.R, coutp / 8, ROW_CHUNK_PIX) != CUDA_SUCCESS)
+    return cudaErrorInvalidValue;
+  SR_WG_CASE(16, 16) SR_WG_CASE(16, 32) SR_WG_CASE(16, 48) SR_WG_CASE(16, 64)
+  SR_WG_CASE(32, 16) SR_WG_CASE(32, 32) SR_WG_CASE(32, 48) SR_WG_CASE(32, 64)
+  SR_WG_CASE(48, 16) SR_WG_CASE(48, 32) SR_WG_CASE(48, 48)
+  SR_WG_CASE(64, 16) SR_WG_CASE(64, 32) SR_WG_CASE(64, 64)
+  return cudaErrorNotSupported;
+}
+
+// ------------------------------------------------------------------------------------------ bilinear only
+// SR_BILINEAR "model" (the WebRTC baseline): the tail with y = 0.
+template <int S>
+__global__ void k_bilinear_u8(const uint8_t* __restrict__ lr, int n, int h, int w, uint8_t* __restrict__ hr) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (long long)n * h * w) return;
+  const int X = (int)(i % w);
+  const long long r = i / w;
+  const int Y = (int)(r % h), img = (int)(r / h);
+  EpiParams ep{};
+  ep.lr = lr;
+  ep.hr = hr;
+  float v[32];
+#pragma unroll
+  for (int k = 0; k < 32; ++k) v[k] = 0.f;
+  const float zb[32] = {0.f};
+  float ls = 0.f;
+  epi_tail<S, 32, false>(ep, zb, img, Y, X, h, w, v, ls);
+}
+
+cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st) {
+  long long tot = (long long)n * h * w;
+  unsigned blocks = (unsigned)((tot + 255) / 256);
+  if (s == 2) k_bilinear_u8<2><<<blocks, 256, 0, st>>>(lr, n, h, w, hr);
+  else if (s == 3) k_bilinear_u8<3><<<blocks, 256, 0, st>>>(lr, n, h, w, hr);
+  else return cudaErrorNotSupported;
+  return cudaGetLastError();
+}
+
+}  // namespace sr

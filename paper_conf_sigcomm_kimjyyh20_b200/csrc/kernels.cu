@@ -1,0 +1,206 @@
+// Memory-bound kernels of the hot path: input packing, weight packing, wgrad reduction, fused Adam,
+// recency-weighted sampler + patch gather, integer SSE (PSNR), bilinear-only baseline.
+#include "ptx.cuh"
+#include "sr_internal.h"
+#include "kernels.h"
+
+namespace sr {
+
+// --------------------------------------------------------------- head input: u8 RGB -> bf16 [.., 16]
+// x = v / 255 (reading R3), channels 3..15 zero so the head conv runs with K = 9 x 16.
+__global__ void k_pack_input(const uint8_t* __restrict__ lr, size_t npix, uint4* __restrict__ x) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= npix) return;
+  const uint8_t* p = lr + i * 3;
+  uint4 lo;
+  lo.x = pack_bf16x2(p[0] * (1.f / 255.f), p[1] * (1.f / 255.f));
+  lo.y = pack_bf16x2(p[2] * (1.f / 255.f), 0.f);
+  lo.z = 0u;
+  lo.w = 0u;
+  x[2 * i] = lo;
+  x[2 * i + 1] = make_uint4(0u, 0u, 0u, 0u);
+}
+
+void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st) {
+  int th = 256;
+  k_pack_input<<<(unsigned)((npix + th - 1) / th), th, 0, st>>>(lr, npix, reinterpret_cast<uint4*>(x));
+}
+
+// --------------------------------------------------------------- weight packing
+// fwd:   Wf[t][ci/8][co][ci%8]   = W[co][ci][ky][kx],        t = 3 ky + kx    (B operand, K-major, no swizzle)
+// dgrad: Wd[t'][co/8][ci][co%8]  = W[co][ci][2-ky'][2-kx'],  t' = 3 ky' + kx' (180-degree rotation, Cin<->Cout)
+__global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc* __restrict__ convs, int nconv,
+                               bf16* __restrict__ wf, bf16* __restrict__ wd, float* __restrict__ bias) {
+  const int c = blockIdx.y;
+  if (c >= nconv) return;
+  const ConvDesc d = convs[c];
+  const float* W = params + d.w_off;
+  const int tot = 9 * d.cinp * d.coutp;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < tot; i += gridDim.x * blockDim.x) {
+    {  // fwd element i = ((t * cinp/8 + j) * coutp + co) * 8 + e
+      int e = i & 7, r = i >> 3;
+      int co = r % d.coutp; r /= d.coutp;
+      int j = r % (d.cinp / 8), t = r / (d.cinp / 8);
+      int ci = 8 * j + e;
+      float v = (ci < d.cin && co < d.cout) ? W[((co * d.cin + ci) * 3 + t / 3) * 3 + t % 3] : 0.f;
+      wf[d.pk_off + i] = __float2bfloat16_rn(v);
+    }
+    if (wd) {  // dgrad element i = ((t' * coutp/8 + j') * cinp + co') * 8 + e'; ci' = fwd co, co' = fwd ci
+      int e = i & 7, r = i >> 3;
+      int cop = r % d.cinp; r /= d.cinp;
+      int j = r % (d.coutp / 8), t = r / (d.coutp / 8);
+      int cip = 8 * j + e;
+      int ky = 2 - t / 3, kx = 2 - t % 3;
+      float v = (cip < d.cout && cop < d.cin) ? W[((cip * d.cin + cop) * 3 + ky) * 3 + kx] : 0.f;
+      wd[d.pk_off + i] = __float2bfloat16_rn(v);
+    }
+  }
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < d.coutp; i += gridDim.x * blockDim.x)
+    bias[d.b_off + i] = i < d.cout ? params[d.w_off + (size_t)d.cout * d.cin * 9 + i] : 0.f;
+}
+
+void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
+                         bf16* wd, float* bias, cudaStream_t st) {
+  dim3 grid((max_elems + 255) / 256, nconv);
+  k_pack_weights<<<grid, 256, 0, st>>>(params, convs_dev, nconv, wf, wd, bias);
+}
+
+// --------------------------------------------------------------- wgrad split-K reduction (deterministic)
+// grad W[co][ci][ky][kx] = scale * sum_{cta in order} ws_w[cta][t][ci][co];  grad b[co] = scale * sum ws_b[cta][co]
+__global__ void k_wgrad_reduce(const float* __restrict__ ws_w, const float* __restrict__ ws_b, int nparts,
+                               int cinp, int coutp, int cin, int cout, float scale, float* __restrict__ gW,
+                               float* __restrict__ gb) {
+  const int per = 9 * cinp * coutp;
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < per) {
+    const int co = i % coutp, rest = i / coutp;
+    const int ci = rest % cinp, t = rest / cinp;
+    float s = 0.f;
+    for (int p = 0; p < nparts; ++p) s += ws_w[(size_t)p * per + i];
+    if (co < cout && ci < cin) gW[(co * cin + ci) * 9 + t] = s * scale;
+  } else if (i < per + coutp) {
+    const int co = i - per;
+    float s = 0.f;
+    for (int p = 0; p < nparts; ++p) s += ws_b[(size_t)p * coutp + co];
+    if (co < cout) gb[co] = s * scale;
+  }
+}
+
+void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
+                         float scale, float* gW, float* gb, cudaStream_t st) {
+  int tot = 9 * cinp * coutp + coutp;
+  k_wgrad_reduce<<<(tot + 255) / 256, 256, 0, st>>>(ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
+}
+
+// --------------------------------------------------------------- fused Adam (PyTorch semantics)
+// m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;  p -= (lr / bc1) * m / (sqrt(v) / sqrt(bc2) + eps),  g = s * grad
+__global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
+                       const float* __restrict__ grad, size_t n, float gscale, float lr_bc1, float inv_sqrt_bc2,
+                       float b1, float b2, float eps) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t stride = (size_t)gridDim.x * blockDim.x;
+  for (; i < n; i += stride) {
+    const float g = grad[i] * gscale;
+    const float mi = fmaf(b1, m[i], (1.f - b1) * g);
+    const float vi = fmaf(b2, v[i], (1.f - b2) * g * g);
+    m[i] = mi;
+    v[i] = vi;
+    p[i] -= lr_bc1 * mi / (sqrtf(vi) * inv_sqrt_bc2 + eps);
+  }
+}
+
+void launch_adam(float* p, float* m, float* v, const float* g, size_t n, float gscale, float lr_bc1,
+                 float inv_sqrt_bc2, float b1, float b2, float eps, cudaStream_t st) {
+  int th = 256;
+  int blocks = (int)((n + th - 1) / th);
+  if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
+  k_adam<<<blocks, th, 0, st>>>(p, m, v, g, n, gscale, lr_bc1, inv_sqrt_bc2, b1, b2, eps);
+}
+
+// --------------------------------------------------------------- sampler + gather (reading R10)
+// u_k = mix64(seed + GAMMA * ((((t G + r) << 20) + j) * 4 + k + 1)); K' = min(K, n); W = w K' + n - K';
+// q = umulhi(u_0, W); idx = q < w K' ? n-1-q/w : q - w K'; o = umulhi(u_k, Pp - P + 1).
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+__global__ void k_sample_gather(SampleArgs a) {
+  const int j = blockIdx.x;
+  __shared__ int s_slot, s_oy, s_ox;
+  if (threadIdx.x == 0) {
+    const uint64_t GAMMA = 0x9E3779B97F4A7C15ull;
+    const uint64_t base = ((((uint64_t)a.step * a.world + a.rank) << 20) + (uint64_t)j) * 4ull;
+    const uint64_t u0 = mix64(a.seed + GAMMA * (base + 1));
+    const uint64_t u1 = mix64(a.seed + GAMMA * (base + 2));
+    const uint64_t u2 = mix64(a.seed + GAMMA * (base + 3));
+    const uint64_t n = (uint64_t)a.n_view;
+    const uint64_t kp = n < (uint64_t)a.recent_k ? n : (uint64_t)a.recent_k;
+    const uint64_t Wt = (uint64_t)a.recent_w * kp + (n - kp);
+    const uint64_t q = __umul64hi(u0, Wt);
+    const uint64_t idx = q < (uint64_t)a.recent_w * kp ? n - 1 - q / (uint64_t)a.recent_w : q - (uint64_t)a.recent_w * kp;
+    const uint64_t span = (uint64_t)(a.pp - a.p + 1);
+    s_oy = (int)__umul64hi(u1, span);
+    s_ox = (int)__umul64hi(u2, span);
+    const int64_t arrival = a.view_base + (int64_t)idx;
+    s_slot = (int)(arrival % a.capacity);
+    if (a.idx_out) a.idx_out[j] = (int32_t)idx;
+  }
+  __syncthreads();
+  const int slot = s_slot, oy = s_oy, ox = s_ox;
+  const int p = a.p, pp = a.pp, s = a.scale;
+  // LR crop: p rows of 3p bytes
+  const uint8_t* src = a.lr_pool + (size_t)slot * pp * pp * 3;
+  uint8_t* dst = a.lr_out + (size_t)j * p * p * 3;
+  for (int i = threadIdx.x; i < p * p * 3; i += blockDim.x) {
+    int r = i / (3 * p), c = i - r * 3 * p;
+    dst[i] = src[((size_t)(oy + r) * pp + ox) * 3 + c];
+  }
+  const int sp = s * p, spp = s * pp;
+  const uint8_t* hsrc = a.hr_pool + (size_t)slot * spp * spp * 3;
+  uint8_t* hdst = a.hr_out + (size_t)j * sp * sp * 3;
+  for (int i = threadIdx.x; i < sp * sp * 3; i += blockDim.x) {
+    int r = i / (3 * sp), c = i - r * 3 * sp;
+    hdst[i] = hsrc[((size_t)(s * oy + r) * spp + s * ox) * 3 + c];
+  }
+}
+
+void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st) {
+  k_sample_gather<<<batch, 256, 0, st>>>(a);
+}
+
+// --------------------------------------------------------------- integer SSE per item (warp-shuffle reduction)
+__global__ void k_sse_u8(const uint8_t* __restrict__ a, const uint8_t* __restrict__ b, int64_t elems,
+                         unsigned long long* __restrict__ out) {
+  const uint8_t* pa = a + (size_t)blockIdx.x * elems;
+  const uint8_t* pb = b + (size_t)blockIdx.x * elems;
+  unsigned long long s = 0;
+  for (int64_t i = threadIdx.x; i < elems; i += blockDim.x) {
+    int d = (int)pa[i] - (int)pb[i];
+    s += (unsigned long long)(d * d);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  __shared__ unsigned long long part[32];
+  if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    unsigned long long t = threadIdx.x < (blockDim.x >> 5) ? part[threadIdx.x] : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    if (threadIdx.x == 0) out[blockIdx.x] = t;
+  }
+}
+
+void launch_sse_u8(const uint8_t* a, const uint8_t* b, int n, int64_t elems, unsigned long long* out,
+                   cudaStream_t st) {
+  k_sse_u8<<<n, 256, 0, st>>>(a, b, elems, out);
+}
+
+__global__ void k_loss_finalize(const double* sum, double inv_n, float* out) { *out = (float)(*sum * inv_n); }
+void launch_loss_finalize(const double* sum, double inv_n, float* out, cudaStream_t st) {
+  k_loss_finalize<<<1, 1, 0, st>>>(sum, inv_n, out);
+}
+
+}  // namespace sr

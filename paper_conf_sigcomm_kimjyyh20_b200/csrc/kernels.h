@@ -1,0 +1,41 @@
+// Launchers of the memory-bound kernels (kernels.cu) and of the bilinear-only baseline (conv.cu).
+#pragma once
+#include "sr_internal.h"
+
+namespace sr {
+
+struct ConvDesc {
+  int cin, cout, cinp, coutp;
+  long long w_off;   // float offset of W in the flat canonical parameter vector (b follows W)
+  long long pk_off;  // bf16 element offset in the packed fwd / dgrad buffers
+  long long b_off;   // float offset in the packed bias buffer
+};
+
+struct SampleArgs {
+  uint64_t seed;
+  long long step;
+  int world, rank;
+  long long n_view, view_base, capacity;
+  int recent_k, recent_w;
+  int p, pp, scale;
+  const uint8_t* lr_pool;
+  const uint8_t* hr_pool;
+  uint8_t* lr_out;
+  uint8_t* hr_out;
+  int32_t* idx_out;
+};
+
+void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st);
+void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
+                         bf16* wd, float* bias, cudaStream_t st);
+void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
+                         float scale, float* gW, float* gb, cudaStream_t st);
+void launch_adam(float* p, float* m, float* v, const float* g, size_t n, float gscale, float lr_bc1,
+                 float inv_sqrt_bc2, float b1, float b2, float eps, cudaStream_t st);
+void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st);
+void launch_sse_u8(const uint8_t* a, const uint8_t* b, int n, int64_t elems, unsigned long long* out,
+                   cudaStream_t st);
+void launch_loss_finalize(const double* sum, double inv_n, float* out, cudaStream_t st);
+cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st);
+
+}  // namespace sr

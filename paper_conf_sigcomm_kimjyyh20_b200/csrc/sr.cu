@@ -1,0 +1,833 @@
+// libsr runtime: context, weight snapshots, workspaces, the forward / backward / Adam orchestration and the
+// C ABI declared in include/sr.h.  All arithmetic of the hot path runs in the kernels of conv.cu and
+// kernels.cu; this file only sequences launches on the caller's stream.
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+#include <algorithm>
+#include "sr_internal.h"
+#include "kernels.h"
+
+using namespace sr;
+
+struct Snapshot {
+  bf16* wf = nullptr;    // packed fwd weights (all convs)
+  float* bias = nullptr; // packed fp32 biases
+};
+
+struct sr_ctx {
+  int s = 2, B = 0, C = 0, Cp = 16, OUTP = 16, nconv = 0;
+  sr_options opt{};
+  std::vector<ConvDesc> convs;
+  ConvDesc* convs_dev = nullptr;
+  size_t nparams = 0, pk_total = 0, b_total = 0;
+  int max_pk = 0;
+  float *params = nullptr, *m = nullptr, *v = nullptr, *grad = nullptr;
+  long long t = 0;  // Adam step counter
+  Snapshot snap[4];
+  bf16* wd_train = nullptr;  // dgrad-packed TRAIN weights
+  // inference workspace
+  size_t inf_pix = 0;
+  bf16 *x16 = nullptr, *f0 = nullptr, *fa = nullptr, *fb = nullptr, *tt = nullptr;
+  uint8_t *stage_lr = nullptr, *stage_hr = nullptr;
+  size_t stage_lr_bytes = 0, stage_hr_bytes = 0;
+  // training workspace
+  size_t tr_pix = 0;
+  bf16 *tx16 = nullptr, *tg = nullptr, *tdy = nullptr, *tdg = nullptr, *tdfa = nullptr, *tdfb = nullptr,
+       *tdt = nullptr;
+  std::vector<bf16*> tf, tts;
+  float *ws_w = nullptr, *ws_b = nullptr;
+  size_t ws_w_elems = 0, ws_b_elems = 0;
+  double* loss_sum = nullptr;
+  // patch pool (device ring)
+  uint8_t *pool_lr = nullptr, *pool_hr = nullptr;
+  long long pool_total = 0, pool_cap = 0;
+  int pool_pp = 0;
+  uint8_t *batch_lr = nullptr, *batch_hr = nullptr;
+  size_t batch_bytes_lr = 0, batch_bytes_hr = 0;
+  long long sample_step = 0;
+  // psnr
+  uint8_t *val_a = nullptr, *val_b = nullptr;
+  size_t val_bytes = 0;
+  unsigned long long* sse = nullptr;
+  int sse_n = 0;
+  cudaEvent_t publish_ev = nullptr;
+  unsigned long long launches = 0;
+  // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
+  bool timing = false;
+  struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
+  std::vector<TRec> trec;
+  size_t tnext = 0;
+  std::string err;
+  bool poisoned = false;
+};
+
+// ------------------------------------------------------------------------------------------ helpers
+static sr_status fail(sr_ctx* c, sr_status st, const std::string& msg) {
+  if (c) {
+    c->err = msg;
+    if (st == SR_E_CUDA) c->poisoned = true;
+  }
+  return st;
+}
+#define CK(call)                                                                                       \
+  do {                                                                                                 \
+    cudaError_t e_ = (call);                                                                           \
+    if (e_ != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+#define CKL() CK(cudaGetLastError())
+
+template <class T>
+static cudaError_t dalloc(T** p, size_t count) {
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  if (count == 0) return cudaSuccess;
+  return cudaMalloc(reinterpret_cast<void**>(p), count * sizeof(T));
+}
+static int rup16(int c) { return (c + 15) / 16 * 16; }
+
+static uint64_t mix64h(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st) {
+  launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, ctx->snap[which].wf,
+                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].bias, st);
+  ctx->launches++;
+  CKL();
+  return SR_OK;
+}
+
+// event pair around one launch when timing is enabled (records reused across resets)
+static void tmark_begin(sr_ctx* ctx, const std::string& cls, double flops, double bytes, cudaStream_t st) {
+  if (!ctx->timing) return;
+  if (ctx->tnext == ctx->trec.size()) {
+    sr_ctx::TRec r;
+    cudaEventCreate(&r.a);
+    cudaEventCreate(&r.b);
+    ctx->trec.push_back(r);
+  }
+  auto& r = ctx->trec[ctx->tnext];
+  r.cls = cls;
+  r.flops = flops;
+  r.bytes = bytes;
+  cudaEventRecord(r.a, st);
+}
+static void tmark_end(sr_ctx* ctx, cudaStream_t st) {
+  if (!ctx->timing) return;
+  cudaEventRecord(ctx->trec[ctx->tnext].b, st);
+  ctx->tnext++;
+}
+
+// one conv launch (conv index ci of the network) with given packed weights
+static sr_status conv(sr_ctx* ctx, int cinp, int coutp, int epi, const void* in, const bf16* wpk, int N, int H,
+                      int W, const EpiParams& ep, cudaStream_t st) {
+  size_t smem = 0;
+  ConvGeom g = make_geom(N, H, W, cinp, coutp, &smem);
+  int grid = std::min(g.units, num_sms());
+  if (ctx->timing) {
+    // algorithmic work: 2 * 9 * Cin * Cout FLOP per output pixel (padded channels as launched)
+    const double px = (double)N * H * W;
+    const char* kind = epi == EPI_ACT ? (ep.mask || (!ep.bias && !ep.relu) ? "dgrad" : "fwd") : (epi == EPI_TAIL_U8 ? "tail_u8" : "tail_train");
+    tmark_begin(ctx, std::string("conv_") + kind + "_" + std::to_string(cinp) + "x" + std::to_string(coutp),
+                2.0 * 9 * cinp * coutp * px, px * 2.0 * (cinp + coutp), st);
+  }
+  cudaError_t e = launch_conv(cinp, coutp, epi, in, wpk, g, ep, smem, grid, st);
+  tmark_end(ctx, st);
+  ctx->launches++;
+  if (e != cudaSuccess)
+    return fail(ctx, e == cudaErrorNotSupported ? SR_E_UNSUPPORTED : SR_E_CUDA,
+                std::string("conv launch: ") + cudaGetErrorString(e));
+  return SR_OK;
+}
+
+static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N, int H, int W, float scale,
+                       cudaStream_t st) {
+  const ConvDesc& d = ctx->convs[ci];
+  size_t smem = 0;
+  WgradGeom g = make_wgrad_geom(N, H, W, d.cinp, d.coutp, &smem);
+  int grid = std::min(g.units, num_sms());
+  size_t need_w = (size_t)grid * 9 * d.cinp * d.coutp, need_b = (size_t)grid * d.coutp;
+  if (need_w > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, need_w)); ctx->ws_w_elems = need_w; }
+  if (need_b > ctx->ws_b_elems) { CK(dalloc(&ctx->ws_b, need_b)); ctx->ws_b_elems = need_b; }
+  if (ctx->timing) {
+    const double px = (double)N * H * W;
+    tmark_begin(ctx, "wgrad_" + std::to_string(d.cinp) + "x" + std::to_string(d.coutp),
+                2.0 * 9 * d.cinp * d.coutp * px, px * 2.0 * (d.cinp + d.coutp), st);
+  }
+  cudaError_t e = launch_wgrad(d.cinp, d.coutp, x, dy, g, ctx->ws_w, ctx->ws_b, smem, grid, st);
+  tmark_end(ctx, st);
+  ctx->launches++;
+  if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("wgrad launch: ") + cudaGetErrorString(e));
+  float* gW = ctx->grad + d.w_off;
+  float* gb = gW + (size_t)d.cout * d.cin * 9;
+  launch_wgrad_reduce(ctx->ws_w, ctx->ws_b, grid, d.cinp, d.coutp, d.cin, d.cout, scale, gW, gb, st);
+  ctx->launches++;
+  CKL();
+  return SR_OK;
+}
+
+#define TRY(x)                   \
+  do {                           \
+    sr_status s_ = (x);          \
+    if (s_ != SR_OK) return s_;  \
+  } while (0)
+
+static sr_status ensure_infer_ws(sr_ctx* ctx, size_t pix) {
+  if (pix <= ctx->inf_pix) return SR_OK;
+  CK(dalloc(&ctx->x16, pix * 16));
+  CK(dalloc(&ctx->f0, pix * ctx->Cp));
+  CK(dalloc(&ctx->fa, pix * ctx->Cp));
+  CK(dalloc(&ctx->fb, pix * ctx->Cp));
+  CK(dalloc(&ctx->tt, pix * ctx->Cp));
+  ctx->inf_pix = pix;
+  return SR_OK;
+}
+
+// Inference forward (reading R1): x = v/255; f0 = head(x); f <- f + conv2(relu(conv1(f))) x B;
+// g = f0 + body(f); tail(up(g)) -> u8 with pixel shuffle + bilinear skip + clamp + RNE.
+static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
+                               uint8_t* hr, int row0, int row1, cudaStream_t st) {
+  const size_t pix = (size_t)n * h * w;
+  TRY(ensure_infer_ws(ctx, pix));
+  const int Cp = ctx->Cp;
+  launch_pack_input(lr, pix, ctx->x16, st);
+  ctx->launches++;
+  CKL();
+  auto W = [&](int ci) { return sn.wf + ctx->convs[ci].pk_off; };
+  auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
+  EpiParams ep{};
+  ep.bias = Bv(0);
+  ep.out = ctx->f0;
+  TRY(conv(ctx, 16, Cp, EPI_ACT, ctx->x16, W(0), n, h, w, ep, st));
+  bf16* cur = ctx->f0;
+  for (int b = 0; b < ctx->B; ++b) {
+    EpiParams e1{};
+    e1.bias = Bv(1 + 2 * b);
+    e1.relu = 1;
+    e1.out = ctx->tt;
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, cur, W(1 + 2 * b), n, h, w, e1, st));
+    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+    EpiParams e2{};
+    e2.bias = Bv(2 + 2 * b);
+    e2.res1 = cur;
+    e2.out = nxt;
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tt, W(2 + 2 * b), n, h, w, e2, st));
+    cur = nxt;
+  }
+  const int cb = 1 + 2 * ctx->B, cu = cb + 1;
+  bf16* gbuf = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+  EpiParams eb{};
+  eb.bias = Bv(cb);
+  eb.res1 = ctx->f0;
+  eb.out = gbuf;
+  TRY(conv(ctx, Cp, Cp, EPI_ACT, cur, W(cb), n, h, w, eb, st));
+  EpiParams et{};
+  et.bias = Bv(cu);
+  et.scale = ctx->s;
+  et.lr = lr;
+  et.hr = hr;
+  et.hr_row0 = row0;
+  et.hr_row1 = row1;
+  TRY(conv(ctx, Cp, ctx->OUTP, EPI_TAIL_U8, gbuf, W(cu), n, h, w, et, st));
+  return SR_OK;
+}
+
+static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
+  if (pix <= ctx->tr_pix) return SR_OK;
+  const int Cp = ctx->Cp;
+  CK(dalloc(&ctx->tx16, pix * 16));
+  for (auto& p : ctx->tf) CK(dalloc(&p, pix * Cp));
+  for (auto& p : ctx->tts) CK(dalloc(&p, pix * Cp));
+  CK(dalloc(&ctx->tg, pix * Cp));
+  CK(dalloc(&ctx->tdy, pix * ctx->OUTP));
+  CK(dalloc(&ctx->tdg, pix * Cp));
+  CK(dalloc(&ctx->tdfa, pix * Cp));
+  CK(dalloc(&ctx->tdfb, pix * Cp));
+  CK(dalloc(&ctx->tdt, pix * Cp));
+  ctx->tr_pix = pix;
+  return SR_OK;
+}
+
+// Forward with saved activations, MSE loss + gradient fused into the tail, backward (dgrad = the fwd conv
+// kernel on 180-degree-rotated / transposed weights with ReLU-mask and residual epilogues; wgrad =
+// tcgen05 split-K + deterministic reduce).  grad <- w_r * dL/dtheta.
+static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, int n, int p, float* loss_dev,
+                            cudaStream_t st) {
+  const size_t pix = (size_t)n * p * p;
+  TRY(ensure_train_ws(ctx, pix));
+  const int Cp = ctx->Cp, B = ctx->B, OUTP = ctx->OUTP;
+  const Snapshot& sn = ctx->snap[SR_TRAIN];
+  auto W = [&](int ci) { return sn.wf + ctx->convs[ci].pk_off; };
+  auto WD = [&](int ci) { return ctx->wd_train + ctx->convs[ci].pk_off; };
+  auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
+  launch_pack_input(lr, pix, ctx->tx16, st);
+  ctx->launches++;
+  CK(cudaMemsetAsync(ctx->loss_sum, 0, sizeof(double), st));
+  // ---- forward, saving f_0..f_B and t_1..t_B
+  {
+    EpiParams e{};
+    e.bias = Bv(0);
+    e.out = ctx->tf[0];
+    TRY(conv(ctx, 16, Cp, EPI_ACT, ctx->tx16, W(0), n, p, p, e, st));
+  }
+  for (int b = 0; b < B; ++b) {
+    EpiParams e1{};
+    e1.bias = Bv(1 + 2 * b);
+    e1.relu = 1;
+    e1.out = ctx->tts[b];
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tf[b], W(1 + 2 * b), n, p, p, e1, st));
+    EpiParams e2{};
+    e2.bias = Bv(2 + 2 * b);
+    e2.res1 = ctx->tf[b];
+    e2.out = ctx->tf[b + 1];
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tts[b], W(2 + 2 * b), n, p, p, e2, st));
+  }
+  const int cb = 1 + 2 * B, cu = cb + 1;
+  {
+    EpiParams e{};
+    e.bias = Bv(cb);
+    e.res1 = ctx->tf[0];
+    e.out = ctx->tg;
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tf[B], W(cb), n, p, p, e, st));
+  }
+  {
+    EpiParams e{};
+    e.bias = Bv(cu);
+    e.scale = ctx->s;
+    e.lr = lr;
+    e.hr_ref = hr;
+    e.dy = ctx->tdy;
+    e.loss_sum = ctx->loss_sum;
+    TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, W(cu), n, p, p, e, st));
+  }
+  const double n_el = (double)pix * ctx->s * ctx->s * 3;
+  if (loss_dev) {
+    launch_loss_finalize(ctx->loss_sum, 1.0 / n_el, loss_dev, st);
+    ctx->launches++;
+  }
+  // dy holds 2 (o - t); the mean's 1/n_el and the DP weight are applied once in the wgrad reduction
+  const float gscale = (float)((ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.0f) / n_el);
+  // ---- backward
+  TRY(wgrad(ctx, cu, ctx->tg, ctx->tdy, n, p, p, gscale, st));
+  {
+    EpiParams e{};
+    e.out = ctx->tdg;  // dg = dgrad_up(dy)
+    TRY(conv(ctx, OUTP, Cp, EPI_ACT, ctx->tdy, WD(cu), n, p, p, e, st));
+  }
+  TRY(wgrad(ctx, cb, ctx->tf[B], ctx->tdg, n, p, p, gscale, st));
+  bf16* df = ctx->tdfa;
+  {
+    EpiParams e{};
+    e.out = df;                    // df_B = dgrad_body(dg)   (B == 0: + dg, since f_B = f0)
+    if (B == 0) e.res1 = ctx->tdg;
+    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tdg, WD(cb), n, p, p, e, st));
+  }
+  for (int b = B - 1; b >= 0; --b) {
+    TRY(wgrad(ctx, 2 + 2 * b, ctx->tts[b], df, n, p, p, gscale, st));
+    {
+      EpiParams e{};
+      e.mask = ctx->tts[b];        // ReLU' = 1[t > 0]
+      e.out = ctx->tdt;
+      TRY(conv(ctx, Cp, Cp, EPI_ACT, df, WD(2 + 2 * b), n, p, p, e, st));
+    }
+    TRY(wgrad(ctx, 1 + 2 * b, ctx->tf[b], ctx->tdt, n, p, p, gscale, st));
+    bf16* dfn = (df == ctx->tdfa) ? ctx->tdfb : ctx->tdfa;
+    {
+      EpiParams e{};
+      e.res1 = df;                 // residual path
+      if (b == 0) e.res2 = ctx->tdg;  // global skip into f0
+      e.out = dfn;
+      TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tdt, WD(1 + 2 * b), n, p, p, e, st));
+    }
+    df = dfn;
+  }
+  TRY(wgrad(ctx, 0, ctx->tx16, df, n, p, p, gscale, st));
+  return SR_OK;
+}
+
+static sr_status train_apply(sr_ctx* ctx, float grad_scale, cudaStream_t st) {
+  ctx->t += 1;
+  const double b1 = ctx->opt.beta1, b2 = ctx->opt.beta2;
+  const double bc1 = 1.0 - std::pow(b1, (double)ctx->t), bc2 = 1.0 - std::pow(b2, (double)ctx->t);
+  launch_adam(ctx->params, ctx->m, ctx->v, ctx->grad, ctx->nparams, grad_scale, (float)(ctx->opt.lr / bc1),
+              (float)(1.0 / std::sqrt(bc2)), (float)b1, (float)b2, ctx->opt.eps, st);
+  ctx->launches++;
+  CKL();
+  return repack(ctx, SR_TRAIN, true, st);
+}
+
+static bool valid_model(sr_model m) { return m >= SR_TRAIN && m <= SR_INIT; }
+
+// ------------------------------------------------------------------------------------------ C ABI
+extern "C" {
+
+sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, sr_ctx** out) {
+  if (!out) return SR_E_INVAL;
+  *out = nullptr;
+  if (scale == 4) return SR_E_UNSUPPORTED;
+  if ((scale != 2 && scale != 3) || blocks < 0 || channels < 1 || channels > 64) return SR_E_INVAL;
+  sr_ctx* ctx = new sr_ctx();
+  ctx->s = scale;
+  ctx->B = blocks;
+  ctx->C = channels;
+  ctx->Cp = rup16(channels);
+  if (ctx->Cp == 16 && channels > 16) ctx->Cp = 32;
+  ctx->OUTP = rup16(3 * scale * scale);
+  if (opt) ctx->opt = *opt;
+  if (ctx->opt.lr == 0.f) ctx->opt.lr = 1e-4f;
+  if (ctx->opt.beta1 == 0.f) ctx->opt.beta1 = 0.9f;
+  if (ctx->opt.beta2 == 0.f) ctx->opt.beta2 = 0.999f;
+  if (ctx->opt.eps == 0.f) ctx->opt.eps = 1e-8f;
+  if (ctx->opt.recent_k == 0) ctx->opt.recent_k = 150;
+  if (ctx->opt.recent_w == 0) ctx->opt.recent_w = 4;
+  if (ctx->opt.world <= 0) ctx->opt.world = 1;
+  if (ctx->opt.dp_weight == 0.f) ctx->opt.dp_weight = 1.f;
+  if (ctx->opt.pool_capacity <= 0) ctx->opt.pool_capacity = 8192;
+  if (ctx->opt.rank < 0 || ctx->opt.rank >= ctx->opt.world) { delete ctx; return SR_E_INVAL; }
+  // conv table in canonical order: head, (b.conv1, b.conv2) x B, body, up
+  std::vector<std::pair<int, int>> shp;  // (cout, cin)
+  shp.push_back({channels, 3});
+  for (int b = 0; b < blocks; ++b) { shp.push_back({channels, channels}); shp.push_back({channels, channels}); }
+  shp.push_back({channels, channels});
+  shp.push_back({3 * scale * scale, channels});
+  long long woff = 0, pk = 0, bo = 0;
+  for (auto& sc : shp) {
+    ConvDesc d{};
+    d.cout = sc.first;
+    d.cin = sc.second;
+    d.cinp = d.cin == 3 ? 16 : ctx->Cp;
+    d.coutp = d.cout == 3 * scale * scale ? ctx->OUTP : ctx->Cp;
+    d.w_off = woff;
+    d.pk_off = pk;
+    d.b_off = bo;
+    woff += (long long)d.cout * d.cin * 9 + d.cout;
+    pk += 9LL * d.cinp * d.coutp;
+    bo += d.coutp;
+    ctx->max_pk = std::max(ctx->max_pk, 9 * d.cinp * d.coutp);
+    ctx->convs.push_back(d);
+  }
+  ctx->nconv = (int)ctx->convs.size();
+  ctx->nparams = (size_t)woff;
+  ctx->pk_total = (size_t)pk;
+  ctx->b_total = (size_t)bo;
+  sr_status st = SR_OK;
+  auto al = [&](auto** p, size_t n) {
+    if (st == SR_OK && dalloc(p, n) != cudaSuccess) st = SR_E_NOMEM;
+  };
+  al(&ctx->convs_dev, ctx->convs.size());
+  al(&ctx->params, ctx->nparams);
+  al(&ctx->m, ctx->nparams);
+  al(&ctx->v, ctx->nparams);
+  al(&ctx->grad, ctx->nparams);
+  for (int k = 0; k < 4; ++k) { al(&ctx->snap[k].wf, ctx->pk_total); al(&ctx->snap[k].bias, ctx->b_total); }
+  al(&ctx->wd_train, ctx->pk_total);
+  al(&ctx->loss_sum, 1);
+  ctx->tf.assign(blocks + 1, nullptr);
+  ctx->tts.assign(blocks, nullptr);
+  if (st != SR_OK) { sr_destroy(ctx); return st; }
+  if (cudaMemcpy(ctx->convs_dev, ctx->convs.data(), ctx->convs.size() * sizeof(ConvDesc),
+                 cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ctx->publish_ev, cudaEventDisableTiming) != cudaSuccess) {
+    sr_destroy(ctx);
+    return SR_E_CUDA;
+  }
+  // seeded init: SplitMix64 stream, u = (z >> 40) 2^-24, w = fp32((2u - 1) / sqrt(9 Cin)), per conv W then b
+  std::vector<float> h(ctx->nparams);
+  uint64_t state = ctx->opt.seed;
+  size_t i = 0;
+  for (auto& d : ctx->convs) {
+    const double bound = 1.0 / std::sqrt(9.0 * d.cin);
+    const size_t cnt = (size_t)d.cout * d.cin * 9 + d.cout;
+    for (size_t k = 0; k < cnt; ++k, ++i) {
+      state += 0x9E3779B97F4A7C15ull;
+      const double u = (double)(mix64h(state) >> 40) * (1.0 / 16777216.0);
+      h[i] = (float)((2.0 * u - 1.0) * bound);
+    }
+  }
+  st = sr_set_params(ctx, h.data(), h.size());
+  if (st != SR_OK) { sr_destroy(ctx); return st; }
+  *out = ctx;
+  return SR_OK;
+}
+
+void sr_destroy(sr_ctx* ctx) {
+  if (!ctx) return;
+  cudaDeviceSynchronize();
+  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->x16, ctx->f0,
+                  ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
+                  ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->pool_lr,
+                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->val_b, ctx->sse};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].bias); }
+  for (auto p : ctx->tf) if (p) cudaFree(p);
+  for (auto p : ctx->tts) if (p) cudaFree(p);
+  if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
+  for (auto& r : ctx->trec) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+  delete ctx;
+}
+
+sr_status sr_kernel_timing(sr_ctx* ctx, int enable) {
+  if (!ctx) return SR_E_INVAL;
+  ctx->timing = enable != 0;
+  ctx->tnext = 0;
+  return SR_OK;
+}
+
+int sr_kernel_stats(sr_ctx* ctx, char* buf, size_t cap) {
+  if (!ctx || !buf || cap == 0) return SR_E_INVAL;
+  if (cudaDeviceSynchronize() != cudaSuccess) return SR_E_CUDA;
+  struct Acc { long long n = 0; double ms = 0, flops = 0, bytes = 0; };
+  std::vector<std::pair<std::string, Acc>> acc;
+  for (size_t i = 0; i < ctx->tnext; ++i) {
+    auto& r = ctx->trec[i];
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, r.a, r.b);
+    auto it = std::find_if(acc.begin(), acc.end(), [&](auto& kv) { return kv.first == r.cls; });
+    if (it == acc.end()) { acc.push_back({r.cls, Acc{}}); it = acc.end() - 1; }
+    it->second.n++;
+    it->second.ms += ms;
+    it->second.flops += r.flops;
+    it->second.bytes += r.bytes;
+  }
+  std::string out = "{";
+  for (size_t i = 0; i < acc.size(); ++i) {
+    char tmp[512];
+    snprintf(tmp, sizeof tmp, "%s\"%s\": {\"launches\": %lld, \"ms\": %.6f, \"flops\": %.6e, \"bytes\": %.6e}",
+             i ? ", " : "", acc[i].first.c_str(), acc[i].second.n, acc[i].second.ms, acc[i].second.flops,
+             acc[i].second.bytes);
+    out += tmp;
+  }
+  out += "}";
+  snprintf(buf, cap, "%s", out.c_str());
+  return (int)out.size();
+}
+
+const char* sr_last_error(const sr_ctx* ctx) { return ctx ? ctx->err.c_str() : "null ctx"; }
+size_t sr_num_params(const sr_ctx* ctx) { return ctx ? ctx->nparams : 0; }
+uint64_t sr_launch_count(const sr_ctx* ctx) { return ctx ? ctx->launches : 0; }
+float* sr_grad_buffer(sr_ctx* ctx) { return ctx ? ctx->grad : nullptr; }
+
+#define GUARD()                                                                  \
+  do {                                                                           \
+    if (!ctx) return SR_E_INVAL;                                                 \
+    if (ctx->poisoned) return fail(ctx, SR_E_STATE, "ctx poisoned: " + ctx->err); \
+  } while (0)
+
+sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
+  GUARD();
+  if (!host_in || n != ctx->nparams) return fail(ctx, SR_E_INVAL, "sr_set_params: size mismatch");
+  CK(cudaMemcpy(ctx->params, host_in, n * sizeof(float), cudaMemcpyHostToDevice));
+  CK(cudaMemset(ctx->m, 0, n * sizeof(float)));
+  CK(cudaMemset(ctx->v, 0, n * sizeof(float)));
+  CK(cudaMemset(ctx->grad, 0, n * sizeof(float)));
+  ctx->t = 0;
+  TRY(repack(ctx, SR_TRAIN, true, 0));
+  for (int k = 1; k < 4; ++k) {
+    CK(cudaMemcpy(ctx->snap[k].wf, ctx->snap[SR_TRAIN].wf, ctx->pk_total * sizeof(bf16), cudaMemcpyDeviceToDevice));
+    CK(cudaMemcpy(ctx->snap[k].bias, ctx->snap[SR_TRAIN].bias, ctx->b_total * sizeof(float),
+                  cudaMemcpyDeviceToDevice));
+  }
+  CK(cudaDeviceSynchronize());
+  return SR_OK;
+}
+
+sr_status sr_get_params(sr_ctx* ctx, sr_model which, float* host_out, size_t n) {
+  GUARD();
+  if (!host_out || n != ctx->nparams || !valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_get_params: bad args");
+  CK(cudaDeviceSynchronize());
+  if (which == SR_TRAIN) {
+    CK(cudaMemcpy(host_out, ctx->params, n * sizeof(float), cudaMemcpyDeviceToHost));
+    return SR_OK;
+  }
+  std::vector<bf16> wf(ctx->pk_total);
+  std::vector<float> bias(ctx->b_total);
+  CK(cudaMemcpy(wf.data(), ctx->snap[which].wf, wf.size() * sizeof(bf16), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(bias.data(), ctx->snap[which].bias, bias.size() * sizeof(float), cudaMemcpyDeviceToHost));
+  for (auto& d : ctx->convs) {
+    float* W = host_out + d.w_off;
+    for (int co = 0; co < d.cout; ++co)
+      for (int ci = 0; ci < d.cin; ++ci)
+        for (int t = 0; t < 9; ++t)
+          W[(co * d.cin + ci) * 9 + t] =
+              __bfloat162float(wf[d.pk_off + ((size_t)(t * d.cinp / 8 + ci / 8) * d.coutp + co) * 8 + ci % 8]);
+    for (int co = 0; co < d.cout; ++co) W[(size_t)d.cout * d.cin * 9 + co] = bias[d.b_off + co];
+  }
+  return SR_OK;
+}
+
+sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, int h, int w, uint8_t* hr_dev,
+                   sr_stream stream) {
+  GUARD();
+  if (!lr_dev || !hr_dev || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  if (which == SR_BILINEAR) {
+    cudaError_t e = launch_bilinear_u8(lr_dev, n, h, w, ctx->s, hr_dev, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, cudaGetErrorString(e));
+    return SR_OK;
+  }
+  if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer: bad model");
+  CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
+  return forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st);
+}
+
+sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
+                        uint8_t* hr_host, sr_stream stream) {
+  GUARD();
+  if (!lr_host || !hr_host || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer_host: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t lb = (size_t)n * h * w * 3, hb = lb * ctx->s * ctx->s;
+  if (lb > ctx->stage_lr_bytes) { CK(dalloc(&ctx->stage_lr, lb)); ctx->stage_lr_bytes = lb; }
+  if (hb > ctx->stage_hr_bytes) { CK(dalloc(&ctx->stage_hr, hb)); ctx->stage_hr_bytes = hb; }
+  CK(cudaMemcpyAsync(ctx->stage_lr, lr_host, lb, cudaMemcpyHostToDevice, st));
+  TRY(sr_infer(ctx, which, ctx->stage_lr, n, h, w, ctx->stage_hr, stream));
+  CK(cudaMemcpyAsync(hr_host, ctx->stage_hr, hb, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  return SR_OK;
+}
+
+sr_status sr_infer_rows(sr_ctx* ctx, sr_model which, const uint8_t* lr_full_dev, int h, int w, int row0, int row1,
+                        uint8_t* hr_full_dev, sr_stream stream) {
+  GUARD();
+  if (!lr_full_dev || !hr_full_dev || h < 1 || w < 1 || row0 < 0 || row1 > h || row0 >= row1)
+    return fail(ctx, SR_E_INVAL, "sr_infer_rows: bad args");
+  if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer_rows: bad model");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int halo = 2 * ctx->B + 4;  // receptive field of the 2B+3 convs (+1 margin)
+  const int lo = std::max(0, row0 - halo), hi = std::min(h, row1 + halo);
+  const int s = ctx->s;
+  CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
+  return forward_infer(ctx, ctx->snap[which], lr_full_dev + (size_t)lo * w * 3, 1, hi - lo, w,
+                       hr_full_dev + (size_t)lo * s * (size_t)s * w * 3, row0 - lo, row1 - lo, st);
+}
+
+sr_status sr_train_grad(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
+                        sr_stream stream) {
+  GUARD();
+  if (!lr_dev || !hr_dev || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_grad: bad args");
+  return train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, (cudaStream_t)stream);
+}
+
+sr_status sr_train_apply(sr_ctx* ctx, float grad_scale, sr_stream stream) {
+  GUARD();
+  return train_apply(ctx, grad_scale, (cudaStream_t)stream);
+}
+
+sr_status sr_train_step(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
+                        sr_stream stream) {
+  GUARD();
+  TRY(sr_train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, stream));
+  const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
+  return train_apply(ctx, 1.0f / w, (cudaStream_t)stream);
+}
+
+sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int pp,
+                       const int64_t* arrival_ts, sr_stream stream) {
+  (void)arrival_ts;
+  GUARD();
+  if (!lr_dev || !hr_dev || n < 1 || pp < 1) return fail(ctx, SR_E_INVAL, "sr_pool_push: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int s = ctx->s;
+  if (!ctx->pool_lr) {
+    ctx->pool_pp = pp;
+    ctx->pool_cap = ctx->opt.pool_capacity;
+    CK(dalloc(&ctx->pool_lr, (size_t)ctx->pool_cap * pp * pp * 3));
+    CK(dalloc(&ctx->pool_hr, (size_t)ctx->pool_cap * s * s * pp * pp * 3));
+  } else if (pp != ctx->pool_pp) {
+    return fail(ctx, SR_E_INVAL, "sr_pool_push: patch size differs from the first push");
+  }
+  const size_t lb = (size_t)pp * pp * 3, hb = lb * s * s;
+  for (int i = 0; i < n; ++i) {
+    const long long slot = (ctx->pool_total + i) % ctx->pool_cap;
+    CK(cudaMemcpyAsync(ctx->pool_lr + slot * lb, lr_dev + i * lb, lb, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(ctx->pool_hr + slot * hb, hr_dev + i * hb, hb, cudaMemcpyDeviceToDevice, st));
+  }
+  ctx->pool_total += n;
+  return SR_OK;
+}
+
+size_t sr_pool_size(const sr_ctx* ctx) {
+  if (!ctx) return 0;
+  return (size_t)std::min(ctx->pool_total, ctx->pool_cap);
+}
+
+sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* lr_out_dev, uint8_t* hr_out_dev,
+                          int32_t* idx_out_dev, sr_stream stream) {
+  GUARD();
+  if (!lr_out_dev || !hr_out_dev || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_sample_batch: bad args");
+  if (ctx->pool_total == 0) return fail(ctx, SR_E_STATE, "sr_sample_batch: empty pool");
+  if (p > ctx->pool_pp) return fail(ctx, SR_E_INVAL, "sr_sample_batch: p larger than pool patch");
+  const long long avail = std::min(ctx->pool_total, ctx->pool_cap);
+  const int G = ctx->opt.world, r = ctx->opt.rank;
+  const long long lo = avail * r / G, hi = avail * (r + 1) / G;
+  if (hi <= lo) return fail(ctx, SR_E_STATE, "sr_sample_batch: empty rank view");
+  SampleArgs a{};
+  a.seed = ctx->opt.seed;
+  a.step = step;
+  a.world = G;
+  a.rank = r;
+  a.n_view = hi - lo;
+  a.view_base = ctx->pool_total - avail + lo;
+  a.capacity = ctx->pool_cap;
+  a.recent_k = ctx->opt.recent_k;
+  a.recent_w = ctx->opt.recent_w;
+  a.p = p;
+  a.pp = ctx->pool_pp;
+  a.scale = ctx->s;
+  a.lr_pool = ctx->pool_lr;
+  a.hr_pool = ctx->pool_hr;
+  a.lr_out = lr_out_dev;
+  a.hr_out = hr_out_dev;
+  a.idx_out = idx_out_dev;
+  launch_sample_gather(a, batch, (cudaStream_t)stream);
+  ctx->launches++;
+  CKL();
+  return SR_OK;
+}
+
+sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss_dev, sr_stream stream) {
+  GUARD();
+  if (iters < 1 || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_sampled: bad args");
+  if (ctx->opt.world != 1) return fail(ctx, SR_E_STATE, "sr_train_sampled: world > 1 needs the split API");
+  const size_t lb = (size_t)batch * p * p * 3, hb = lb * ctx->s * ctx->s;
+  if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; }
+  if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; }
+  for (int it = 0; it < iters; ++it) {
+    TRY(sr_sample_batch(ctx, ctx->sample_step++, batch, p, ctx->batch_lr, ctx->batch_hr, nullptr, stream));
+    TRY(sr_train_step(ctx, ctx->batch_lr, ctx->batch_hr, batch, p, loss_dev, stream));
+  }
+  return SR_OK;
+}
+
+sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
+  GUARD();
+  cudaStream_t st = (cudaStream_t)stream;
+  CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wf, ctx->snap[SR_SERVE].wf, ctx->pk_total * sizeof(bf16),
+                     cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ctx->snap[SR_PREV].bias, ctx->snap[SR_SERVE].bias, ctx->b_total * sizeof(float),
+                     cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ctx->snap[SR_SERVE].wf, ctx->snap[SR_TRAIN].wf, ctx->pk_total * sizeof(bf16),
+                     cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ctx->snap[SR_SERVE].bias, ctx->snap[SR_TRAIN].bias, ctx->b_total * sizeof(float),
+                     cudaMemcpyDeviceToDevice, st));
+  CK(cudaEventRecord(ctx->publish_ev, st));
+  return SR_OK;
+}
+
+sr_status sr_sse_u8(const uint8_t* a_dev, const uint8_t* b_dev, int n, int64_t elems, uint64_t* out_dev,
+                    sr_stream stream) {
+  if (!a_dev || !b_dev || !out_dev || n < 1 || elems < 1) return SR_E_INVAL;
+  launch_sse_u8(a_dev, b_dev, n, elems, reinterpret_cast<unsigned long long*>(out_dev), (cudaStream_t)stream);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
+sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
+                       int p, sr_quality* out_host, sr_stream stream) {
+  GUARD();
+  if (!lr_dev || !hr_dev || !out_host || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_psnr_gain: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int s = ctx->s;
+  const size_t per = (size_t)s * p * s * p * 3, tot = per * n;
+  if (tot > ctx->val_bytes) {
+    CK(dalloc(&ctx->val_a, tot));
+    CK(dalloc(&ctx->val_b, tot));
+    ctx->val_bytes = tot;
+  }
+  if (n > ctx->sse_n) { CK(dalloc(&ctx->sse, 2 * (size_t)n)); ctx->sse_n = n; }
+  TRY(sr_infer(ctx, a, lr_dev, n, p, p, ctx->val_a, stream));
+  TRY(sr_infer(ctx, b, lr_dev, n, p, p, ctx->val_b, stream));
+  launch_sse_u8(ctx->val_a, hr_dev, n, (int64_t)per, ctx->sse, st);
+  launch_sse_u8(ctx->val_b, hr_dev, n, (int64_t)per, ctx->sse + n, st);
+  ctx->launches += 2;
+  CKL();
+  std::vector<unsigned long long> h(2 * (size_t)n);
+  CK(cudaMemcpyAsync(h.data(), ctx->sse, h.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  double sa = 0, sb = 0;
+  for (int i = 0; i < n; ++i) {
+    sa += h[i] == 0 ? 100.0 : 10.0 * std::log10(255.0 * 255.0 * (double)per / (double)h[i]);
+    sb += h[n + i] == 0 ? 100.0 : 10.0 * std::log10(255.0 * 255.0 * (double)per / (double)h[n + i]);
+  }
+  out_host->psnr_a = sa / n;
+  out_host->psnr_b = sb / n;
+  out_host->gain = out_host->psnr_a - out_host->psnr_b;
+  return SR_OK;
+}
+
+// ---- test-only exports
+sr_status sr_test_pack_input(const uint8_t* lr_dev, int n, int h, int w, void* x_dev, sr_stream stream) {
+  if (!lr_dev || !x_dev) return SR_E_INVAL;
+  launch_pack_input(lr_dev, (size_t)n * h * w, (bf16*)x_dev, (cudaStream_t)stream);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
+sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout, const float* w_host,
+                       const float* b_host, const void* res_dev, const void* mask_dev, int relu, int dgrad,
+                       void* out_dev, sr_stream stream) {
+  if (!x_dev || !w_host || !out_dev) return SR_E_INVAL;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int cinp = rup16(cin), coutp = rup16(cout);
+  ConvDesc d{};
+  d.cin = cin; d.cout = cout; d.cinp = cinp; d.coutp = coutp;
+  const size_t np = (size_t)cout * cin * 9 + cout;
+  std::vector<float> hp(np, 0.f);
+  memcpy(hp.data(), w_host, (size_t)cout * cin * 9 * sizeof(float));
+  if (b_host) memcpy(hp.data() + (size_t)cout * cin * 9, b_host, cout * sizeof(float));
+  float *pd = nullptr, *bias = nullptr;
+  bf16 *wf = nullptr, *wd = nullptr;
+  ConvDesc* dd = nullptr;
+  const size_t pk = 9 * (size_t)cinp * coutp;
+  if (cudaMalloc(&pd, np * 4) || cudaMalloc(&bias, coutp * 4) || cudaMalloc(&wf, pk * 2) ||
+      cudaMalloc(&wd, pk * 2) || cudaMalloc(&dd, sizeof(ConvDesc)))
+    return SR_E_NOMEM;
+  cudaMemcpy(pd, hp.data(), np * 4, cudaMemcpyHostToDevice);
+  cudaMemcpy(dd, &d, sizeof(ConvDesc), cudaMemcpyHostToDevice);
+  launch_pack_weights(pd, dd, 1, (int)pk, wf, wd, bias, st);
+  EpiParams ep{};
+  ep.bias = (b_host && !dgrad) ? bias : nullptr;
+  ep.res1 = (const bf16*)res_dev;
+  ep.mask = (const bf16*)mask_dev;
+  ep.relu = relu;
+  ep.out = (bf16*)out_dev;
+  size_t smem = 0;
+  const int ci_eff = dgrad ? coutp : cinp, co_eff = dgrad ? cinp : coutp;
+  ConvGeom g = make_geom(n, h, w, ci_eff, co_eff, &smem);
+  int grid = std::min(g.units, num_sms());
+  cudaError_t e = launch_conv(ci_eff, co_eff, EPI_ACT, x_dev, dgrad ? wd : wf, g, ep, smem, grid, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  cudaFree(pd); cudaFree(bias); cudaFree(wf); cudaFree(wd); cudaFree(dd);
+  if (e == cudaErrorNotSupported) return SR_E_UNSUPPORTED;
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
+
+sr_status sr_test_wgrad(const void* x_dev, const void* dy_dev, int n, int h, int w, int cin, int cout,
+                        float* dw_host, float* db_host, sr_stream stream) {
+  if (!x_dev || !dy_dev || !dw_host || !db_host) return SR_E_INVAL;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int cinp = rup16(cin), coutp = rup16(cout);
+  size_t smem = 0;
+  WgradGeom g = make_wgrad_geom(n, h, w, cinp, coutp, &smem);
+  int grid = std::min(g.units, num_sms());
+  float *ws_w = nullptr, *ws_b = nullptr, *gout = nullptr;
+  const size_t np = (size_t)cout * cin * 9 + cout;
+  if (cudaMalloc(&ws_w, (size_t)grid * 9 * cinp * coutp * 4) || cudaMalloc(&ws_b, (size_t)grid * coutp * 4) ||
+      cudaMalloc(&gout, np * 4))
+    return SR_E_NOMEM;
+  cudaError_t e = launch_wgrad(cinp, coutp, (const bf16*)x_dev, (const bf16*)dy_dev, g, ws_w, ws_b, smem, grid, st);
+  launch_wgrad_reduce(ws_w, ws_b, grid, cinp, coutp, cin, cout, 1.0f, gout, gout + (size_t)cout * cin * 9, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  std::vector<float> h_(np);
+  cudaMemcpy(h_.data(), gout, np * 4, cudaMemcpyDeviceToHost);
+  memcpy(dw_host, h_.data(), (size_t)cout * cin * 9 * 4);
+  memcpy(db_host, h_.data() + (size_t)cout * cin * 9, cout * 4);
+  cudaFree(ws_w); cudaFree(ws_b); cudaFree(gout);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
+
+}  // extern "C"

@@ -1,0 +1,129 @@
+// Test-only exports: validate the tcgen05 descriptor encodings and the 5-D TMA layouts the conv kernels
+// rely on, and micro-benchmark tcgen05.mma issue rate at the small N this network has.
+#include "ptx.cuh"
+#include "tmap.h"
+#include "sr_internal.h"
+
+namespace sr {
+
+// One CTA: D[128 x N] = A[128 x K] * B[N x K]^T.  A/B given row-major in global (K contiguous).
+// a_mn: stage A in the MN-major canonical layout instead of K-major (B likewise with b_mn).
+// reps > 0: throughput mode; the MMA thread re-issues the K/16 MMAs `reps` times (accumulating) and
+// reports clock64 cycles; shift != 0 offsets A's start address by 16*(i%3) bytes per MMA (per-tap style).
+__global__ void __launch_bounds__(128, 1)
+k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict__ B, float* __restrict__ D,
+           int N, int K, int a_mn, int b_mn, int reps, int shift, long long* cycles) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tmem_base;
+  const int M = 128;
+  const int MA = M + 8;  // extra rows so shifted reads stay inside the buffer
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + MA * K * 2;
+  // ---- stage A
+  for (int i = threadIdx.x; i < MA * K; i += blockDim.x) {
+    int m = i / K, k = i % K;
+    __nv_bfloat16 v = m < M ? A[m * K + k] : __float2bfloat16(0.f);
+    uint32_t off;
+    if (!a_mn) off = (k / 8) * (MA * 16) + m * 16 + (k % 8) * 2;          // K-major: LBO = MA*16, SBO = 128
+    else off = (m / 8) * (K * 16) + k * 16 + (m % 8) * 2;                  // MN-major: SBO = K*16, LBO = 128
+    *reinterpret_cast<__nv_bfloat16*>(sA + off) = v;
+  }
+  for (int i = threadIdx.x; i < N * K; i += blockDim.x) {
+    int n = i / K, k = i % K;
+    uint32_t off;
+    if (!b_mn) off = (k / 8) * (N * 16) + n * 16 + (k % 8) * 2;
+    else off = (n / 8) * (K * 16) + k * 16 + (n % 8) * 2;
+    *reinterpret_cast<__nv_bfloat16*>(sB + off) = B[i];
+  }
+  fence_proxy_async_smem();
+  if (warp_id() == 0) tmem_alloc<256>(&tmem_base);
+  if (threadIdx.x == 0) { mbar_init(&bar, 1); fence_barrier_init(); }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base;
+  if (threadIdx.x == 0) {
+    const uint32_t idesc = make_idesc(128, N, a_mn, b_mn);
+    const uint32_t a0 = smem_u32(sA), b0 = smem_u32(sB);
+    uint64_t adesc = a_mn ? make_desc(a0, 128, K * 16) : make_desc(a0, MA * 16, 128);
+    uint64_t bdesc = b_mn ? make_desc(b0, 128, K * 16) : make_desc(b0, N * 16, 128);
+    const int ksteps = K / 16;
+    // one K step = 16 elements = 2 chunks: K-major advances by 2*LBO, MN-major by 2 LBO-groups (256 B)
+    const uint32_t a_step = a_mn ? 256 : 2 * MA * 16;
+    const uint32_t b_step = b_mn ? 256 : 2 * N * 16;
+    long long t0 = clock64();
+    int total = reps > 0 ? reps : 1;
+    for (int r = 0; r < total; ++r) {
+      for (int ks = 0; ks < ksteps; ++ks) {
+        uint32_t sh = shift ? 16u * ((r * ksteps + ks) % 3) : 0u;
+        mma_bf16_ss(tmem, desc_add(adesc, ks * a_step + sh), desc_add(bdesc, ks * b_step), idesc,
+                    (r | ks) != 0);
+      }
+    }
+    mma_commit(&bar);
+    mbar_wait(&bar, 0);
+    long long t1 = clock64();
+    if (cycles) cycles[0] = t1 - t0;
+  }
+  __syncthreads();
+  tc_fence_after();
+  // ---- drain: warp w reads lanes 32w..32w+31
+  const int row = warp_id() * 32 + lane_id();
+  for (int c0 = 0; c0 < N; c0 += 16) {
+    float v[16];
+    tmem_ld16(tmem + ((warp_id() * 32u) << 16) + c0, v);
+    tmem_ld_wait();
+    for (int j = 0; j < 16; ++j) D[row * N + c0 + j] = v[j];
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp_id() == 0) tmem_dealloc<256>(tmem);
+}
+
+// Dump what a 5-D TMA box lands in shared memory (to check the chunk-planar layouts and OOB zero fill).
+__global__ void k_test_tma(const __grid_constant__ CUtensorMap tm, uint8_t* out, uint32_t bytes, int c1, int c2,
+                           int c3, int c4) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint64_t bar;
+  if (threadIdx.x == 0) {
+    mbar_init(&bar, 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    mbar_arrive_expect_tx(&bar, bytes);
+    tma_load_5d(smem, &tm, &bar, 0, c1, c2, c3, c4);
+  }
+  mbar_wait(&bar, 0);
+  for (uint32_t i = threadIdx.x; i < bytes; i += blockDim.x) out[i] = smem[i];
+}
+
+}  // namespace sr
+
+using namespace sr;
+
+extern "C" int sr_test_mma(const void* A, const void* B, float* D, int N, int K, int a_mn, int b_mn, int reps,
+                           int shift, long long* cycles_dev, void* stream) {
+  if (N % 16 || N < 16 || N > 256 || K % 16 || K < 16) return SR_E_INVAL;
+  size_t smem = (size_t)(128 + 8) * K * 2 + (size_t)N * K * 2 + 1024;
+  if (smem > 200 * 1024) return SR_E_INVAL;
+  cudaFuncSetAttribute(k_test_mma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_test_mma<<<1, 128, smem, (cudaStream_t)stream>>>((const __nv_bfloat16*)A, (const __nv_bfloat16*)B, D, N, K,
+                                                    a_mn, b_mn, reps, shift, cycles_dev);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
+extern "C" int sr_test_tma(const void* act, int N, int H, int W, int Cp, int box_w, int box_h, int box_chunks,
+                           int order, int x0, int y0, uint8_t* out, void* stream) {
+  CUtensorMap tm;
+  if (make_act_tmap(&tm, act, N, H, W, Cp, box_w, box_h, box_chunks, (TmapOrder)order) != CUDA_SUCCESS)
+    return SR_E_CUDA;
+  uint32_t bytes = (uint32_t)box_w * box_h * box_chunks * 16;
+  cudaFuncSetAttribute(k_test_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (order == CHUNK_ROW_PIX)
+    k_test_tma<<<1, 128, bytes, (cudaStream_t)stream>>>(tm, out, bytes, x0, y0, 0, 0);
+  else
+    k_test_tma<<<1, 128, bytes, (cudaStream_t)stream>>>(tm, out, bytes, x0, 0, y0, 0);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}

@@ -1,0 +1,54 @@
+// Host helpers: TMA tensor-map encoding through the driver entry point (no -lcuda link needed).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+#include <cstdint>
+#include <cstring>
+
+namespace sr {
+
+inline PFN_cuTensorMapEncodeTiled_v12000 get_encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
+// NHWC bf16 activation [N][H][W][Cp] viewed as a 5-D tensor whose innermost dimension is one 8-channel
+// (16-byte) chunk.  `order` selects the smem layout the box lands in (the box is written innermost-first):
+//   CHUNK_ROW_PIX : dims {8, W, H, Cp/8, N}  -> smem [chunk][row][pixel][8]   (fwd conv A operand)
+//   ROW_CHUNK_PIX : dims {8, W, Cp/8, H, N}  -> smem [row][chunk][pixel][8]   (wgrad operands)
+// Out-of-bounds box elements (image border, padding) are zero-filled by the TMA unit.
+enum TmapOrder { CHUNK_ROW_PIX = 0, ROW_CHUNK_PIX = 1 };
+
+inline CUresult make_act_tmap(CUtensorMap* tm, const void* base, int N, int H, int W, int Cp, int box_w,
+                              int box_h, int box_chunks, TmapOrder order) {
+  auto fn = get_encode_fn();
+  if (!fn) return CUDA_ERROR_NOT_SUPPORTED;
+  const uint64_t es = 2;
+  cuuint64_t dims[5];
+  cuuint64_t strides[4];  // bytes, dims 1..4
+  cuuint32_t box[5];
+  cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+  const uint64_t pix = (uint64_t)Cp * es, row = (uint64_t)W * pix, img = (uint64_t)H * row;
+  if (order == CHUNK_ROW_PIX) {
+    dims[0] = 8; dims[1] = W; dims[2] = H; dims[3] = Cp / 8; dims[4] = N;
+    strides[0] = pix; strides[1] = row; strides[2] = 16; strides[3] = img;
+    box[0] = 8; box[1] = box_w; box[2] = box_h; box[3] = box_chunks; box[4] = 1;
+  } else {
+    dims[0] = 8; dims[1] = W; dims[2] = Cp / 8; dims[3] = H; dims[4] = N;
+    strides[0] = pix; strides[1] = 16; strides[2] = row; strides[3] = img;
+    box[0] = 8; box[1] = box_w; box[2] = box_chunks; box[3] = box_h; box[4] = 1;
+  }
+  return fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, const_cast<void*>(base), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+}
+
+}  // namespace sr

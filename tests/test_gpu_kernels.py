@@ -1,0 +1,188 @@
+"""Kernel-level GPU parity through the C ABI's test exports (same kernels sr_infer / sr_train_* launch).
+
+Convs are compared with the fp64 oracle on bf16-pre-rounded operands, so the only differences left are
+the fp32 accumulation order and the final bf16 store (relative 2^-9)."""
+import ctypes as C
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from tests.helpers import bf16_round, from_dev_bf16, rel_l2, rup16, to_dev_bf16
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_sigcomm_kimjyyh20_b200 import load
+    return load()
+
+
+def _p(t):
+    return C.c_void_p(t.data_ptr()) if t is not None else None
+
+
+def _s():
+    return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+
+
+# ------------------------------------------------------------------ tcgen05 descriptor / shape sanity
+@pytest.mark.parametrize("N", [16, 32, 48, 64, 144, 256])
+@pytest.mark.parametrize("K", [16, 64])
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (1, 1), (0, 1), (1, 0)])
+def test_mma_descriptors(lib, N, K, a_mn, b_mn):
+    r = np.random.default_rng(N * 1000 + K + 10 * a_mn + b_mn)
+    A = bf16_round(r.standard_normal((128, K)))
+    B = bf16_round(r.standard_normal((N, K)))
+    At = torch.from_numpy(A.astype(np.float32)).to(torch.bfloat16).cuda()
+    Bt = torch.from_numpy(B.astype(np.float32)).to(torch.bfloat16).cuda()
+    D = torch.zeros((128, N), dtype=torch.float32, device="cuda")
+    assert lib.sr_test_mma(_p(At), _p(Bt), _p(D), N, K, a_mn, b_mn, 0, 0, None, _s()) == 0
+    torch.cuda.synchronize()
+    ref = A @ B.T
+    np.testing.assert_allclose(D.cpu().numpy(), ref, rtol=1e-5, atol=1e-4)
+
+
+# ------------------------------------------------------------------ TMA 5-D box layouts
+@pytest.mark.parametrize("order", [0, 1])
+def test_tma_box_layout(lib, order):
+    N, H, W, Cp = 2, 5, 20, 48
+    ids = (np.arange(N * H * W * Cp) % 251 + 1).astype(np.float32).reshape(N, H, W, Cp)
+    act = torch.from_numpy(ids).to(torch.bfloat16).cuda()
+    bw, bh, bc = 12, 3, Cp // 8
+    x0, y0 = -1, 3  # OOB on the left and below
+    nbytes = bw * bh * bc * 16
+    out = torch.zeros(nbytes, dtype=torch.uint8, device="cuda")
+    assert lib.sr_test_tma(_p(act), N, H, W, Cp, bw, bh, bc, order, x0, y0, _p(out), _s()) == 0
+    torch.cuda.synchronize()
+    got = out.cpu().view(torch.bfloat16).float().numpy()
+    img = 0
+    exp = np.zeros(nbytes // 2, np.float32)
+    for j in range(bc):
+        for rr in range(bh):
+            for p in range(bw):
+                y, x = y0 + rr, x0 + p
+                for e in range(8):
+                    v = ids[img, y, x, 8 * j + e] if (0 <= y < H and 0 <= x < W) else 0.0
+                    idx = ((j * bh + rr) * bw + p) * 8 + e if order == 0 else ((rr * bc + j) * bw + p) * 8 + e
+                    exp[idx] = v
+    np.testing.assert_array_equal(got, exp)
+
+
+# ------------------------------------------------------------------ conv forward / dgrad
+CONV_CASES = [
+    # n, h, w, cin, cout
+    (2, 7, 20, 16, 48),    # narrow tile, head-like input
+    (1, 9, 300, 48, 48),   # wide tiles incl. a ragged last tile
+    (3, 11, 48, 32, 32),   # training-patch geometry
+    (1, 5, 130, 48, 16),   # up-conv width (x2)
+    (1, 6, 64, 48, 32),    # up-conv width (x3)
+    (2, 13, 17, 8, 8),     # padded channels (tiny config)
+    (1, 3, 1, 16, 16),     # degenerate width
+    (40, 48, 48, 48, 48),  # > 148 narrow units: CTAs loop over units, both smem stages + TMEM slot wrap
+    (3, 40, 700, 32, 32),  # > 148 wide units
+]
+
+
+def _conv_case(lib, n, h, w, cin, cout, relu, res, seed):
+    r = np.random.default_rng(seed)
+    x = bf16_round(r.standard_normal((n, h, w, cin)))
+    Wt = bf16_round(r.standard_normal((cout, cin, 3, 3)) / np.sqrt(9 * cin))
+    b = r.standard_normal(cout).astype(np.float32) * 0.1
+    xd = to_dev_bf16(x, rup16(cin))
+    outd = torch.zeros((n, h, w, rup16(cout)), dtype=torch.bfloat16, device="cuda")
+    resv = bf16_round(r.standard_normal((n, h, w, cout))) if res else None
+    resd = to_dev_bf16(resv, rup16(cout)) if res else None
+    Wf = np.ascontiguousarray(Wt, np.float32)
+    st = lib.sr_test_conv(_p(xd), n, h, w, cin, cout, Wf.ctypes.data_as(C.c_void_p),
+                          b.ctypes.data_as(C.c_void_p), _p(resd), None, int(relu), 0, _p(outd), _s())
+    assert st == 0
+    torch.cuda.synchronize()
+    ref = O.conv3x3(x, Wt, b.astype(np.float64))
+    if res:
+        ref = ref + resv
+    if relu:
+        ref = np.maximum(ref, 0)
+    got = from_dev_bf16(outd)
+    assert np.all(got[..., cout:] == 0)
+    return got[..., :cout], ref
+
+
+@pytest.mark.parametrize("case", CONV_CASES)
+def test_conv_fwd_matches_oracle(lib, case):
+    got, ref = _conv_case(lib, *case, relu=False, res=False, seed=1)
+    err = np.abs(got - ref)
+    assert err.max() <= 2 ** -8 * np.abs(ref).max() + 1e-6, err.max()
+    assert rel_l2(got, ref) < 3e-3
+
+
+@pytest.mark.parametrize("case", CONV_CASES[:3])
+def test_conv_fwd_relu_residual(lib, case):
+    got, ref = _conv_case(lib, *case, relu=True, res=True, seed=2)
+    assert rel_l2(got, ref) < 3e-3
+
+
+@pytest.mark.parametrize("case", [(2, 7, 20, 16, 48), (1, 9, 300, 48, 48), (3, 11, 48, 16, 48)])
+def test_conv_dgrad_with_mask(lib, case):
+    n, h, w, cin, cout = case
+    r = np.random.default_rng(3)
+    dy = bf16_round(r.standard_normal((n, h, w, cout)))
+    Wt = bf16_round(r.standard_normal((cout, cin, 3, 3)) / np.sqrt(9 * cin))
+    mask = bf16_round(np.maximum(r.standard_normal((n, h, w, cin)), 0))
+    dyd = to_dev_bf16(dy, rup16(cout))
+    maskd = to_dev_bf16(mask, rup16(cin))
+    outd = torch.zeros((n, h, w, rup16(cin)), dtype=torch.bfloat16, device="cuda")
+    Wf = np.ascontiguousarray(Wt, np.float32)
+    st = lib.sr_test_conv(_p(dyd), n, h, w, cin, cout, Wf.ctypes.data_as(C.c_void_p), None, None, _p(maskd), 0, 1,
+                          _p(outd), _s())
+    assert st == 0
+    torch.cuda.synchronize()
+    ref = O.conv3x3_dgrad(dy, Wt) * (mask > 0)
+    got = from_dev_bf16(outd, cin)
+    assert rel_l2(got, ref) < 3e-3
+
+
+# ------------------------------------------------------------------ wgrad
+@pytest.mark.parametrize("case", [(2, 7, 20, 16, 48), (1, 9, 150, 48, 48), (4, 48, 48, 48, 48),
+                                  (3, 11, 48, 32, 16), (2, 12, 48, 48, 32), (2, 13, 17, 8, 8),
+                                  (48, 48, 48, 48, 48), (2, 90, 300, 16, 48)])
+def test_wgrad_matches_oracle(lib, case):
+    n, h, w, cin, cout = case
+    r = np.random.default_rng(4)
+    x = bf16_round(r.standard_normal((n, h, w, cin)))
+    dy = bf16_round(r.standard_normal((n, h, w, cout)))
+    xd = to_dev_bf16(x, rup16(cin))
+    dyd = to_dev_bf16(dy, rup16(cout))
+    dw = np.zeros((cout, cin, 3, 3), np.float32)
+    db = np.zeros(cout, np.float32)
+    st = lib.sr_test_wgrad(_p(xd), _p(dyd), n, h, w, cin, cout, dw.ctypes.data_as(C.c_void_p),
+                           db.ctypes.data_as(C.c_void_p), _s())
+    assert st == 0
+    rW, rb = O.conv3x3_wgrad(x, dy)
+    assert rel_l2(dw, rW) < 1e-5
+    assert rel_l2(db, rb) < 1e-5
+
+
+# ------------------------------------------------------------------ small kernels
+def test_pack_input_exact(lib):
+    v = torch.randint(0, 256, (2, 5, 7, 3), dtype=torch.uint8, device="cuda")
+    x = torch.empty((2, 5, 7, 16), dtype=torch.bfloat16, device="cuda")
+    assert lib.sr_test_pack_input(_p(v), 2, 5, 7, _p(x), _s()) == 0
+    torch.cuda.synchronize()
+    exp = (v.float() * (1.0 / 255.0)).to(torch.bfloat16)
+    assert torch.equal(x[..., :3], exp)
+    assert torch.all(x[..., 3:] == 0)
+
+
+def test_sse_exact(lib):
+    r = np.random.default_rng(5)
+    a = r.integers(0, 256, (5, 120 * 120 * 3)).astype(np.uint8)
+    b = r.integers(0, 256, (5, 120 * 120 * 3)).astype(np.uint8)
+    out = torch.zeros(5, dtype=torch.int64, device="cuda")
+    assert lib.sr_sse_u8(_p(torch.from_numpy(a).cuda()), _p(torch.from_numpy(b).cuda()), 5, a.shape[1], _p(out),
+                         _s()) == 0
+    torch.cuda.synchronize()
+    exp = ((a.astype(np.int64) - b.astype(np.int64)) ** 2).sum(axis=1)
+    np.testing.assert_array_equal(out.cpu().numpy(), exp)
