@@ -19,7 +19,8 @@
 
 namespace sr {
 
-static constexpr int kConvThreads = 192;
+static constexpr int kConvThreads = 320;   // conv: TMA warp, MMA warp, 2 x 4 epilogue warps
+static constexpr int kWgradThreads = 192;  // wgrad: TMA warp, MMA warp, 4 epilogue warps
 static constexpr int kStages = 2;
 static constexpr int kSmemLimit = 227 * 1024;
 
@@ -102,33 +103,63 @@ __device__ __forceinline__ void store_bf16_row(bf16* p, const float* v) {
   }
 }
 
+// Residual / mask rows of one output pixel, loaded BEFORE the accumulator is waited on so that the global
+// load latency overlaps the MMAs of this M-tile.
 template <int COUTP>
-__device__ __forceinline__ void epi_act(const EpiParams& ep, const float* sbias, size_t pix, float* v) {
+struct EpiPre {
+  uint4 r1[COUTP / 8], r2[COUTP / 8], mk[COUTP / 8];
+};
+
+template <int COUTP>
+__device__ __forceinline__ void epi_prefetch(const EpiParams& ep, size_t pix, EpiPre<COUTP>& pre) {
+#pragma unroll
+  for (int i = 0; i < COUTP / 8; ++i) {
+    if (ep.res1) pre.r1[i] = __ldg(reinterpret_cast<const uint4*>(ep.res1 + pix * COUTP) + i);
+    if (ep.res2) pre.r2[i] = __ldg(reinterpret_cast<const uint4*>(ep.res2 + pix * COUTP) + i);
+    if (ep.mask) pre.mk[i] = __ldg(reinterpret_cast<const uint4*>(ep.mask + pix * COUTP) + i);
+  }
+}
+
+__device__ __forceinline__ void unpack8(const uint4& u, float* f) {
+  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    float2 t = __bfloat1622float2(h[j]);
+    f[2 * j] = t.x;
+    f[2 * j + 1] = t.y;
+  }
+}
+
+// out = [mask>0] * act(acc + bias + res1 + res2)
+template <int COUTP>
+__device__ __forceinline__ void epi_act(const EpiParams& ep, const float* sbias, size_t pix, float* v,
+                                        const EpiPre<COUTP>& pre) {
   if (ep.bias) {
 #pragma unroll
     for (int c = 0; c < COUTP; ++c) v[c] += sbias[c];
   }
-  if (ep.res1) {
-    float r[COUTP];
-    load_bf16_row<COUTP>(ep.res1 + pix * COUTP, r);
 #pragma unroll
-    for (int c = 0; c < COUTP; ++c) v[c] += r[c];
-  }
-  if (ep.res2) {
-    float r[COUTP];
-    load_bf16_row<COUTP>(ep.res2 + pix * COUTP, r);
+  for (int i = 0; i < COUTP / 8; ++i) {
+    float f[8];
+    if (ep.res1) {
+      unpack8(pre.r1[i], f);
 #pragma unroll
-    for (int c = 0; c < COUTP; ++c) v[c] += r[c];
-  }
-  if (ep.relu) {
+      for (int j = 0; j < 8; ++j) v[8 * i + j] += f[j];
+    }
+    if (ep.res2) {
+      unpack8(pre.r2[i], f);
 #pragma unroll
-    for (int c = 0; c < COUTP; ++c) v[c] = fmaxf(v[c], 0.f);
-  }
-  if (ep.mask) {
-    float r[COUTP];
-    load_bf16_row<COUTP>(ep.mask + pix * COUTP, r);
+      for (int j = 0; j < 8; ++j) v[8 * i + j] += f[j];
+    }
+    if (ep.relu) {
 #pragma unroll
-    for (int c = 0; c < COUTP; ++c) v[c] = r[c] > 0.f ? v[c] : 0.f;
+      for (int j = 0; j < 8; ++j) v[8 * i + j] = fmaxf(v[8 * i + j], 0.f);
+    }
+    if (ep.mask) {
+      unpack8(pre.mk[i], f);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[8 * i + j] = f[j] > 0.f ? v[8 * i + j] : 0.f;
+    }
   }
   store_bf16_row<COUTP>(ep.out + pix * COUTP, v);
 }
@@ -302,17 +333,28 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
     }
     __syncwarp();
   } else {
-    // ===================== epilogue (warps 2..5) =====================
-    const int quarter = warp & 3;  // TMEM lane quarter this warp may access
+    // ===================== epilogue (warps 2..9: two groups of 4 alternate M-tiles) =====================
+    const int quarter = warp & 3;            // TMEM lane quarter this warp may access
+    const int grp = (warp - 2) >> 2;         // M-tile k is drained by group k % 2
     const int row = quarter * 32 + lane_id();
-    int slot = 0;
-    uint32_t tph = 0;
     float lsum = 0.f;
+    int k = 0;                               // running M-tile index (same sequence as the MMA issuer)
     for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
       const int n = u / tiles_xy, rem = u - n * tiles_xy;
       const int ty = rem / g.tiles_x, tx = rem - ty * g.tiles_x;
       const int y0 = ty * g.R, x0 = tx * g.TW;
-      for (int mt = 0; mt < g.n_mt; ++mt) {
+      for (int mt = 0; mt < g.n_mt; ++mt, ++k) {
+        if ((k & 1) != grp) continue;
+        const int slot = k % NSLOT;
+        const uint32_t tph = (uint32_t)(k / NSLOT) & 1u;
+        int r, x;
+        if (g.wide) { r = mt; x = row; }
+        else { const int q = mt * 128 + row; r = q / P; x = q - r * P; }
+        const int Y = y0 + r, X = x0 + x;
+        const bool valid = x < g.TW && r < g.R && Y < g.H && X < g.W;
+        const size_t pix = ((size_t)n * g.H + Y) * g.W + X;
+        EpiPre<COUTP> pre;
+        if (EPI == EPI_ACT && valid && ep.dbg == 0) epi_prefetch<COUTP>(ep, pix, pre);
         mbar_wait(&tfull_bar[slot], tph);
         tc_fence_after();
         float v[COUTP];
@@ -323,15 +365,11 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
         tc_fence_before();
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&tempty_bar[slot]);
-        if (++slot == NSLOT) { slot = 0; tph ^= 1; }
-        int r, x;
-        if (g.wide) { r = mt; x = row; }
-        else { const int q = mt * 128 + row; r = q / P; x = q - r * P; }
-        const int Y = y0 + r, X = x0 + x;
-        const bool valid = x < g.TW && r < g.R && Y < g.H && X < g.W;
-        if (!valid) continue;
-        if (EPI == EPI_ACT) {
-          epi_act<COUTP>(ep, sbias, ((size_t)n * g.H + Y) * g.W + X, v);
+        if (!valid || ep.dbg == 1) continue;
+        if (EPI == EPI_ACT && ep.dbg == 2) {
+          store_bf16_row<COUTP>(ep.out + pix * COUTP, v);
+        } else if (EPI == EPI_ACT) {
+          epi_act<COUTP>(ep, sbias, pix, v, pre);
         } else if (EPI == EPI_TAIL_U8) {
           if (Y >= ep.hr_row0 && Y < ep.hr_row1) epi_tail<S, COUTP, false>(ep, sbias, n, Y, X, g.H, g.W, v, lsum);
         } else {
@@ -423,7 +461,7 @@ WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem
 }
 
 template <int CINP, int COUTP>
-__global__ void __launch_bounds__(kConvThreads, 1)
+__global__ void __launch_bounds__(kWgradThreads, 1)
 k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_dy, const WgradGeom g,
         float* __restrict__ ws_w, float* __restrict__ ws_b) {
   constexpr int CCH = CINP / 8, OCH = COUTP / 8;
@@ -580,7 +618,7 @@ static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, 
     if (e != cudaSuccess) return e;
     configured = smem;
   }
-  kern<<<grid, kConvThreads, smem, st>>>(tx, ty, g, ws_w, ws_b);
+  kern<<<grid, kWgradThreads, smem, st>>>(tx, ty, g, ws_w, ws_b);
   return cudaGetLastError();
 }
 

@@ -29,8 +29,10 @@ void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st)
 // --------------------------------------------------------------- weight packing
 // fwd:   Wf[t][ci/8][co][ci%8]   = W[co][ci][ky][kx],        t = 3 ky + kx    (B operand, K-major, no swizzle)
 // dgrad: Wd[t'][co/8][ci][co%8]  = W[co][ci][2-ky'][2-kx'],  t' = 3 ky' + kx' (180-degree rotation, Cin<->Cout)
+// fold:  Wo[kx][ci/8][ky*coutp + co][ci%8] = W[co][ci][ky][kx]  (N = 3 coutp: the rolling dy-fold conv, conv_roll.cu)
 __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc* __restrict__ convs, int nconv,
-                               bf16* __restrict__ wf, bf16* __restrict__ wd, float* __restrict__ bias) {
+                               bf16* __restrict__ wf, bf16* __restrict__ wd, bf16* __restrict__ wo,
+                               float* __restrict__ bias) {
   const int c = blockIdx.y;
   if (c >= nconv) return;
   const ConvDesc d = convs[c];
@@ -54,15 +56,24 @@ __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc*
       float v = (cip < d.cout && cop < d.cin) ? W[((cip * d.cin + cop) * 3 + ky) * 3 + kx] : 0.f;
       wd[d.pk_off + i] = __float2bfloat16_rn(v);
     }
+    if (wo) {  // fold element i = ((kx * cinp/8 + j) * 3 coutp + ky * coutp + co) * 8 + e
+      int e = i & 7, r = i >> 3;
+      int n = r % (3 * d.coutp); r /= 3 * d.coutp;
+      int j = r % (d.cinp / 8), kx = r / (d.cinp / 8);
+      int ky = n / d.coutp, co = n % d.coutp;
+      int ci = 8 * j + e;
+      float v = (ci < d.cin && co < d.cout) ? W[((co * d.cin + ci) * 3 + ky) * 3 + kx] : 0.f;
+      wo[d.pk_off + i] = __float2bfloat16_rn(v);
+    }
   }
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < d.coutp; i += gridDim.x * blockDim.x)
     bias[d.b_off + i] = i < d.cout ? params[d.w_off + (size_t)d.cout * d.cin * 9 + i] : 0.f;
 }
 
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, float* bias, cudaStream_t st) {
+                         bf16* wd, bf16* wo, float* bias, cudaStream_t st) {
   dim3 grid((max_elems + 255) / 256, nconv);
-  k_pack_weights<<<grid, 256, 0, st>>>(params, convs_dev, nconv, wf, wd, bias);
+  k_pack_weights<<<grid, 256, 0, st>>>(params, convs_dev, nconv, wf, wd, wo, bias);
 }
 
 // --------------------------------------------------------------- wgrad split-K reduction (deterministic)
@@ -70,26 +81,39 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 __global__ void k_wgrad_reduce(const float* __restrict__ ws_w, const float* __restrict__ ws_b, int nparts,
                                int cinp, int coutp, int cin, int cout, float scale, float* __restrict__ gW,
                                float* __restrict__ gb) {
+  // block = 32 outputs x 8 partial groups; group gi sums partials gi, gi+8, ... (fixed order), then the 8 group
+  // sums are added in order 0..7 -> deterministic.
+  __shared__ float part[8][33];
   const int per = 9 * cinp * coutp;
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int i = blockIdx.x * 32 + threadIdx.x;
+  const int gi = threadIdx.y;
+  float s = 0.f;
   if (i < per) {
-    const int co = i % coutp, rest = i / coutp;
-    const int ci = rest % cinp, t = rest / cinp;
-    float s = 0.f;
-    for (int p = 0; p < nparts; ++p) s += ws_w[(size_t)p * per + i];
-    if (co < cout && ci < cin) gW[(co * cin + ci) * 9 + t] = s * scale;
+    for (int p = gi; p < nparts; p += 8) s += ws_w[(size_t)p * per + i];
   } else if (i < per + coutp) {
-    const int co = i - per;
-    float s = 0.f;
-    for (int p = 0; p < nparts; ++p) s += ws_b[(size_t)p * coutp + co];
-    if (co < cout) gb[co] = s * scale;
+    for (int p = gi; p < nparts; p += 8) s += ws_b[(size_t)p * coutp + (i - per)];
+  }
+  part[gi][threadIdx.x] = s;
+  __syncthreads();
+  if (gi == 0) {
+    float t = 0.f;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) t += part[q][threadIdx.x];
+    if (i < per) {
+      const int co = i % coutp, rest = i / coutp;
+      const int ci = rest % cinp, tap = rest / cinp;
+      if (co < cout && ci < cin) gW[(co * cin + ci) * 9 + tap] = t * scale;
+    } else if (i < per + coutp) {
+      const int co = i - per;
+      if (co < cout) gb[co] = t * scale;
+    }
   }
 }
 
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st) {
   int tot = 9 * cinp * coutp + coutp;
-  k_wgrad_reduce<<<(tot + 255) / 256, 256, 0, st>>>(ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
+  k_wgrad_reduce<<<(tot + 31) / 32, dim3(32, 8), 0, st>>>(ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
 }
 
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
@@ -127,6 +151,8 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
 }
 
 __global__ void k_sample_gather(SampleArgs a) {
+  // grid (batch, kGatherSplit): block (j, part) computes draw j (cheap, redundant per part) and copies the crop
+  // rows r = part, part + kGatherSplit, ...
   const int j = blockIdx.x;
   __shared__ int s_slot, s_oy, s_ox;
   if (threadIdx.x == 0) {
@@ -145,29 +171,27 @@ __global__ void k_sample_gather(SampleArgs a) {
     s_ox = (int)__umul64hi(u2, span);
     const int64_t arrival = a.view_base + (int64_t)idx;
     s_slot = (int)(arrival % a.capacity);
-    if (a.idx_out) a.idx_out[j] = (int32_t)idx;
+    if (a.idx_out && blockIdx.y == 0) a.idx_out[j] = (int32_t)idx;
   }
   __syncthreads();
   const int slot = s_slot, oy = s_oy, ox = s_ox;
   const int p = a.p, pp = a.pp, s = a.scale;
-  // LR crop: p rows of 3p bytes
+  const int rb = 3 * p;  // bytes per LR crop row
   const uint8_t* src = a.lr_pool + (size_t)slot * pp * pp * 3;
   uint8_t* dst = a.lr_out + (size_t)j * p * p * 3;
-  for (int i = threadIdx.x; i < p * p * 3; i += blockDim.x) {
-    int r = i / (3 * p), c = i - r * 3 * p;
-    dst[i] = src[((size_t)(oy + r) * pp + ox) * 3 + c];
-  }
-  const int sp = s * p, spp = s * pp;
+  for (int r = blockIdx.y; r < p; r += gridDim.y)
+    for (int c = threadIdx.x; c < rb; c += blockDim.x)
+      dst[r * rb + c] = src[((size_t)(oy + r) * pp + ox) * 3 + c];
+  const int sp = s * p, spp = s * pp, hb = 3 * sp;
   const uint8_t* hsrc = a.hr_pool + (size_t)slot * spp * spp * 3;
   uint8_t* hdst = a.hr_out + (size_t)j * sp * sp * 3;
-  for (int i = threadIdx.x; i < sp * sp * 3; i += blockDim.x) {
-    int r = i / (3 * sp), c = i - r * 3 * sp;
-    hdst[i] = hsrc[((size_t)(s * oy + r) * spp + s * ox) * 3 + c];
-  }
+  for (int r = blockIdx.y; r < sp; r += gridDim.y)
+    for (int c = threadIdx.x; c < hb; c += blockDim.x)
+      hdst[r * hb + c] = hsrc[((size_t)(s * oy + r) * spp + s * ox) * 3 + c];
 }
 
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st) {
-  k_sample_gather<<<batch, 256, 0, st>>>(a);
+  k_sample_gather<<<dim3(batch, 16), 128, 0, st>>>(a);
 }
 
 // --------------------------------------------------------------- integer SSE per item (warp-shuffle reduction)

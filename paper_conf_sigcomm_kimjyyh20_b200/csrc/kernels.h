@@ -27,7 +27,10 @@ struct SampleArgs {
 
 void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st);
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, float* bias, cudaStream_t st);
+                         bf16* wd, bf16* wo, float* bias, cudaStream_t st);
+bool roll_supported(int cinp, int coutp, int W);
+cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
+                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st);
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st);
 void launch_adam(float* p, float* m, float* v, const float* g, size_t n, float gscale, float lr_bc1,

@@ -14,6 +14,7 @@ using namespace sr;
 
 struct Snapshot {
   bf16* wf = nullptr;    // packed fwd weights (all convs)
+  bf16* wo = nullptr;    // packed dy-fold weights (rolling conv for wide frames)
   float* bias = nullptr; // packed fp32 biases
 };
 
@@ -96,7 +97,7 @@ static uint64_t mix64h(uint64_t z) {
 
 static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st) {
   launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, ctx->snap[which].wf,
-                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].bias, st);
+                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].wo, ctx->snap[which].bias, st);
   ctx->launches++;
   CKL();
   return SR_OK;
@@ -143,6 +144,26 @@ static sr_status conv(sr_ctx* ctx, int cinp, int coutp, int epi, const void* in,
     return fail(ctx, e == cudaErrorNotSupported ? SR_E_UNSUPPORTED : SR_E_CUDA,
                 std::string("conv launch: ") + cudaGetErrorString(e));
   return SR_OK;
+}
+
+// forward conv with the fastest kernel for the shape: the rolling dy-fold kernel for wide frames (EPI_ACT
+// without mask / second residual), otherwise the general tiled kernel.
+static sr_status conv_fwd(sr_ctx* ctx, int cinp, int coutp, const void* in, const Snapshot& sn, int ci, int N, int H,
+                          int W, const EpiParams& ep, cudaStream_t st) {
+  if (roll_supported(cinp, coutp, W) && !ep.mask && !ep.res2) {
+    if (ctx->timing) {
+      const double px = (double)N * H * W;
+      tmark_begin(ctx, std::string("conv_roll_") + std::to_string(cinp) + "x" + std::to_string(coutp),
+                  2.0 * 9 * cinp * coutp * px, px * 2.0 * (cinp + coutp), st);
+    }
+    cudaError_t e = launch_conv_roll(cinp, coutp, in, sn.wo + ctx->convs[ci].pk_off, ep.bias, ep.res1, ep.relu,
+                                     ep.out, N, H, W, st);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("conv_roll launch: ") + cudaGetErrorString(e));
+    return SR_OK;
+  }
+  return conv(ctx, cinp, coutp, EPI_ACT, in, sn.wf + ctx->convs[ci].pk_off, N, H, W, ep, st);
 }
 
 static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N, int H, int W, float scale,
@@ -203,20 +224,20 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   EpiParams ep{};
   ep.bias = Bv(0);
   ep.out = ctx->f0;
-  TRY(conv(ctx, 16, Cp, EPI_ACT, ctx->x16, W(0), n, h, w, ep, st));
+  TRY(conv_fwd(ctx, 16, Cp, ctx->x16, sn, 0, n, h, w, ep, st));
   bf16* cur = ctx->f0;
   for (int b = 0; b < ctx->B; ++b) {
     EpiParams e1{};
     e1.bias = Bv(1 + 2 * b);
     e1.relu = 1;
     e1.out = ctx->tt;
-    TRY(conv(ctx, Cp, Cp, EPI_ACT, cur, W(1 + 2 * b), n, h, w, e1, st));
+    TRY(conv_fwd(ctx, Cp, Cp, cur, sn, 1 + 2 * b, n, h, w, e1, st));
     bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
     EpiParams e2{};
     e2.bias = Bv(2 + 2 * b);
     e2.res1 = cur;
     e2.out = nxt;
-    TRY(conv(ctx, Cp, Cp, EPI_ACT, ctx->tt, W(2 + 2 * b), n, h, w, e2, st));
+    TRY(conv_fwd(ctx, Cp, Cp, ctx->tt, sn, 2 + 2 * b, n, h, w, e2, st));
     cur = nxt;
   }
   const int cb = 1 + 2 * ctx->B, cu = cb + 1;
@@ -225,7 +246,7 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   eb.bias = Bv(cb);
   eb.res1 = ctx->f0;
   eb.out = gbuf;
-  TRY(conv(ctx, Cp, Cp, EPI_ACT, cur, W(cb), n, h, w, eb, st));
+  TRY(conv_fwd(ctx, Cp, Cp, cur, sn, cb, n, h, w, eb, st));
   EpiParams et{};
   et.bias = Bv(cu);
   et.scale = ctx->s;
@@ -424,7 +445,11 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->m, ctx->nparams);
   al(&ctx->v, ctx->nparams);
   al(&ctx->grad, ctx->nparams);
-  for (int k = 0; k < 4; ++k) { al(&ctx->snap[k].wf, ctx->pk_total); al(&ctx->snap[k].bias, ctx->b_total); }
+  for (int k = 0; k < 4; ++k) {
+    al(&ctx->snap[k].wf, ctx->pk_total);
+    al(&ctx->snap[k].wo, ctx->pk_total);
+    al(&ctx->snap[k].bias, ctx->b_total);
+  }
   al(&ctx->wd_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
   ctx->tf.assign(blocks + 1, nullptr);
@@ -464,7 +489,7 @@ void sr_destroy(sr_ctx* ctx) {
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->val_b, ctx->sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
-  for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].bias); }
+  for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].wo); cudaFree(ctx->snap[k].bias); }
   for (auto p : ctx->tf) if (p) cudaFree(p);
   for (auto p : ctx->tts) if (p) cudaFree(p);
   if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
@@ -530,6 +555,7 @@ sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
   TRY(repack(ctx, SR_TRAIN, true, 0));
   for (int k = 1; k < 4; ++k) {
     CK(cudaMemcpy(ctx->snap[k].wf, ctx->snap[SR_TRAIN].wf, ctx->pk_total * sizeof(bf16), cudaMemcpyDeviceToDevice));
+    CK(cudaMemcpy(ctx->snap[k].wo, ctx->snap[SR_TRAIN].wo, ctx->pk_total * sizeof(bf16), cudaMemcpyDeviceToDevice));
     CK(cudaMemcpy(ctx->snap[k].bias, ctx->snap[SR_TRAIN].bias, ctx->b_total * sizeof(float),
                   cudaMemcpyDeviceToDevice));
   }
@@ -712,6 +738,10 @@ sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
                      cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].bias, ctx->snap[SR_SERVE].bias, ctx->b_total * sizeof(float),
                      cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wo, ctx->snap[SR_SERVE].wo, ctx->pk_total * sizeof(bf16),
+                     cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ctx->snap[SR_SERVE].wo, ctx->snap[SR_TRAIN].wo, ctx->pk_total * sizeof(bf16),
+                     cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_SERVE].wf, ctx->snap[SR_TRAIN].wf, ctx->pk_total * sizeof(bf16),
                      cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_SERVE].bias, ctx->snap[SR_TRAIN].bias, ctx->b_total * sizeof(float),
@@ -788,7 +818,9 @@ sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout
     return SR_E_NOMEM;
   cudaMemcpy(pd, hp.data(), np * 4, cudaMemcpyHostToDevice);
   cudaMemcpy(dd, &d, sizeof(ConvDesc), cudaMemcpyHostToDevice);
-  launch_pack_weights(pd, dd, 1, (int)pk, wf, wd, bias, st);
+  bf16* wo = nullptr;
+  if (cudaMalloc(&wo, pk * 2)) return SR_E_NOMEM;
+  launch_pack_weights(pd, dd, 1, (int)pk, wf, wd, wo, bias, st);
   EpiParams ep{};
   ep.bias = (b_host && !dgrad) ? bias : nullptr;
   ep.res1 = (const bf16*)res_dev;
@@ -799,9 +831,13 @@ sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout
   const int ci_eff = dgrad ? coutp : cinp, co_eff = dgrad ? cinp : coutp;
   ConvGeom g = make_geom(n, h, w, ci_eff, co_eff, &smem);
   int grid = std::min(g.units, num_sms());
-  cudaError_t e = launch_conv(ci_eff, co_eff, EPI_ACT, x_dev, dgrad ? wd : wf, g, ep, smem, grid, st);
+  cudaError_t e;
+  if (!dgrad && !mask_dev && roll_supported(cinp, coutp, w))
+    e = launch_conv_roll(cinp, coutp, x_dev, wo, ep.bias, ep.res1, relu, (bf16*)out_dev, n, h, w, st);
+  else
+    e = launch_conv(ci_eff, co_eff, EPI_ACT, x_dev, dgrad ? wd : wf, g, ep, smem, grid, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
-  cudaFree(pd); cudaFree(bias); cudaFree(wf); cudaFree(wd); cudaFree(dd);
+  cudaFree(pd); cudaFree(bias); cudaFree(wf); cudaFree(wd); cudaFree(wo); cudaFree(dd);
   if (e == cudaErrorNotSupported) return SR_E_UNSUPPORTED;
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }

@@ -42,6 +42,7 @@ struct EpiParams {
   const uint8_t* hr_ref;  // EPI_TAIL_TRAIN: target [N, sH, sW, 3]
   bf16* dy;            // EPI_TAIL_TRAIN: 2*(o - t) in pixel-unshuffled layout [N,H,W,COUTP]
   double* loss_sum;    // EPI_TAIL_TRAIN: += sum (o - t)^2
+  int dbg;             // benchmarking only: 1 = drain TMEM and skip the epilogue, 2 = plain store (no bias/res)
 };
 
 ConvGeom make_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes);

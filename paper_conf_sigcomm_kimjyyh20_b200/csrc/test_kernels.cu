@@ -3,6 +3,7 @@
 #include "ptx.cuh"
 #include "tmap.h"
 #include "sr_internal.h"
+#include "kernels.h"
 
 namespace sr {
 
@@ -53,12 +54,29 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
     const uint32_t a_step = a_mn ? 256 : 2 * MA * 16;
     const uint32_t b_step = b_mn ? 256 : 2 * N * 16;
     long long t0 = clock64();
-    int total = reps > 0 ? reps : 1;
-    for (int r = 0; r < total; ++r) {
-      for (int ks = 0; ks < ksteps; ++ks) {
-        uint32_t sh = shift ? 16u * ((r * ksteps + ks) % 3) : 0u;
-        mma_bf16_ss(tmem, desc_add(adesc, ks * a_step + sh), desc_add(bdesc, ks * b_step), idesc,
-                    (r | ks) != 0);
+    if (reps > 0 && ksteps == 4) {
+      // throughput mode: descriptors precomputed, 4 MMAs per iteration fully unrolled; shift=2 alternates
+      // between two TMEM accumulators (independent D) to separate accumulate-dependency from issue rate
+      uint64_t ad[4], bd[4];
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) {
+        ad[ks] = desc_add(adesc, ks * a_step + (shift == 1 ? 16u * (ks % 3) : 0u));
+        bd[ks] = desc_add(bdesc, ks * b_step);
+      }
+      const uint32_t d1 = shift == 2 ? tmem + 256 - N : tmem;
+      mma_bf16_ss(tmem, ad[0], bd[0], idesc, 0u);
+      for (int r = 0; r < reps; ++r) {
+#pragma unroll
+        for (int ks = 0; ks < 4; ++ks) mma_bf16_ss((ks & 1) ? d1 : tmem, ad[ks], bd[ks], idesc, 1u);
+      }
+    } else {
+      int total = reps > 0 ? reps : 1;
+      for (int r = 0; r < total; ++r) {
+        for (int ks = 0; ks < ksteps; ++ks) {
+          uint32_t sh = shift ? 16u * ((r * ksteps + ks) % 3) : 0u;
+          mma_bf16_ss(tmem, desc_add(adesc, ks * a_step + sh), desc_add(bdesc, ks * b_step), idesc,
+                      (r | ks) != 0);
+        }
       }
     }
     mma_commit(&bar);
@@ -126,4 +144,51 @@ extern "C" int sr_test_tma(const void* act, int N, int H, int W, int Cp, int box
   else
     k_test_tma<<<1, 128, bytes, (cudaStream_t)stream>>>(tm, out, bytes, x0, 0, y0, 0);
   return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
+// Kernel-level timing of one conv launch configuration on device-resident random data (benchmarking only).
+// mode: 0 = fwd + bias + ReLU, 1 = fwd + bias + residual, 2 = plain store, 3 = skip epilogue.
+extern "C" int sr_bench_conv(int cinp, int coutp, int n, int h, int w, int mode, int iters, float* ms_out,
+                             void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t pix = (size_t)n * h * w;
+  bf16 *x = nullptr, *y = nullptr, *res = nullptr, *wpk = nullptr;
+  float* bias = nullptr;
+  if (cudaMalloc(&x, pix * cinp * 2) || cudaMalloc(&y, pix * coutp * 2) || cudaMalloc(&res, pix * coutp * 2) ||
+      cudaMalloc(&wpk, 9 * cinp * coutp * 2) || cudaMalloc(&bias, coutp * 4))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(x, 0x3c, pix * cinp * 2, st);
+  cudaMemsetAsync(res, 0x3c, pix * coutp * 2, st);
+  cudaMemsetAsync(wpk, 0x1c, 9 * cinp * coutp * 2, st);
+  cudaMemsetAsync(bias, 0, coutp * 4, st);
+  const bool roll = mode >= 10;
+  if (roll) mode -= 10;
+  EpiParams ep{};
+  ep.bias = bias;
+  ep.out = y;
+  ep.relu = mode == 0;
+  ep.res1 = mode == 1 ? res : nullptr;
+  ep.dbg = mode == 2 ? 2 : (mode == 3 ? 1 : 0);
+  size_t smem = 0;
+  ConvGeom g = make_geom(n, h, w, cinp, coutp, &smem);
+  int grid = g.units < num_sms() ? g.units : num_sms();
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  auto run = [&]() {
+    return roll ? launch_conv_roll(cinp, coutp, x, wpk, bias, ep.res1, ep.relu, y, n, h, w, st)
+                : launch_conv(cinp, coutp, EPI_ACT, x, wpk, g, ep, smem, grid, st);
+  };
+  cudaError_t e = run();  // warm-up
+  cudaEventRecord(a, st);
+  for (int i = 0; i < iters && e == cudaSuccess; ++i) e = run();
+  cudaEventRecord(b, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, a, b);
+  *ms_out = ms / (iters > 0 ? iters : 1);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(x); cudaFree(y); cudaFree(res); cudaFree(wpk); cudaFree(bias);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }

@@ -51,4 +51,18 @@ inline CUresult make_act_tmap(CUtensorMap* tm, const void* base, int N, int H, i
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+// NHWC bf16 [N][H][W][Cp] as a 4-D tensor {Cp, W, H, N}; box {box_c, box_w, 1, 1} = (part of the channels of)
+// one row segment, smem layout [pixel][box_c] (residual rows; per-warp output slices for the TMA store).
+inline CUresult make_row_tmap(CUtensorMap* tm, const void* base, int N, int H, int W, int Cp, int box_w, int box_c) {
+  auto fn = get_encode_fn();
+  if (!fn) return CUDA_ERROR_NOT_SUPPORTED;
+  cuuint64_t dims[4] = {(cuuint64_t)Cp, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[3] = {(cuuint64_t)Cp * 2, (cuuint64_t)W * Cp * 2, (cuuint64_t)H * W * Cp * 2};
+  cuuint32_t box[4] = {(cuuint32_t)box_c, (cuuint32_t)box_w, 1, 1};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  return fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+}
+
 }  // namespace sr
