@@ -96,6 +96,7 @@ def run_ours(args):
     import torch
     import torch.distributed as dist
     from paper_conf_sigcomm_kimjyyh20_b200 import SRContext
+    from paper_conf_sigcomm_kimjyyh20_b200.parallel import dp_allreduce_grad, max_over_ranks
     from synth import synth_frames, synth_patch_pool
 
     world, rank, local = dist_env()
@@ -124,10 +125,9 @@ def run_ours(args):
         for _ in range(args.iters):
             ctx.sample_batch(state["step"], BATCH, PATCH, out=(blr, bhr, bidx))
             state["step"] += 1
-            ctx.train_grad(blr, bhr, loss)
-            if world > 1:
-                dist.all_reduce(grad)           # NCCL over NVLink: sum_r w_r g_r
-            ctx.train_apply(1.0 / world)        # / sum_r w_r  (w_r = 1)
+            ctx.train_grad(blr, bhr, loss)      # grad <- w_r g_r
+            scale = dp_allreduce_grad(grad)     # NCCL over NVLink (world > 1): sum_r w_r g_r; 1 / sum_r w_r
+            ctx.train_apply(scale)
         ctx.publish()
 
     def step():
@@ -159,10 +159,7 @@ def run_ours(args):
     stats = ctx.kernel_stats()
     ctx.kernel_timing(False)
     clocks = clk.stop()
-    if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = max_over_ranks(ms, device=dev)
 
     # ---- end-to-end: host (pinned) frames in, host frames out, through the C ABI (sr_infer_host)
     lr_host = torch.from_numpy(lr_np).pin_memory()
@@ -183,11 +180,7 @@ def run_ours(args):
         step_e2e()
     e3.record()
     barrier()
-    ms_e2e = e2.elapsed_time(e3)
-    if world > 1:
-        t = torch.tensor([ms_e2e], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_e2e = float(t.item())
+    ms_e2e = max_over_ranks(e2.elapsed_time(e3), device=dev)
 
     if rank == 0:
         pk = peaks()
@@ -199,7 +192,6 @@ def run_ours(args):
         total_frames = frames * args.steps * world
         fps = total_frames / (ms * 1e-3)
         fps_e2e = total_frames / (ms_e2e * 1e-3)
-        tflop_step = FLOP_PER_LR_PX * LR_H * LR_W * frames + args.iters * 3.0 * 0  # inference part only
         conv_flops = sum(v["flops"] for v in stats.values())
         line = {
             "metric": "4K SR frames/s (720p->2160p x3, 8x48) with online training at the paper's cadence",
