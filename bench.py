@@ -34,6 +34,8 @@ BATCH, PATCH = 64, 48
 POOL_N, POOL_LR = 512, 60           # pool entries: 60x60 LR / 180x180 HR (crop offsets span 0..12)
 VAL_N = 64
 FLOP_PER_LR_PX = 2 * 9 * (3 * CH + 2 * BLOCKS * CH * CH + CH * CH + CH * 3 * S * S)
+# one training iteration: forward + data-grad (no input grad for the head) + weight-grad
+TRAIN_FLOP = BATCH * PATCH * PATCH * (3 * FLOP_PER_LR_PX - 2 * 9 * 3 * CH)
 
 
 def peaks():
@@ -96,7 +98,7 @@ def run_ours(args):
     import torch
     import torch.distributed as dist
     from paper_conf_sigcomm_kimjyyh20_b200 import SRContext
-    from paper_conf_sigcomm_kimjyyh20_b200.parallel import dp_allreduce_grad, max_over_ranks
+    from paper_conf_sigcomm_kimjyyh20_b200.parallel import dp_allreduce_grad_dev, max_over_ranks
     from synth import synth_frames, synth_patch_pool
 
     world, rank, local = dist_env()
@@ -119,15 +121,34 @@ def run_ours(args):
     bidx = torch.empty(BATCH, dtype=torch.int32, device=dev)
     loss = torch.zeros(1, dtype=torch.float32, device=dev)
     grad = ctx.grad_buffer()
-    state = {"step": 0, "q": None}
+    state = {"q": None}
+
+    wdev = torch.ones(1, dtype=torch.float32, device=dev)  # this rank's gradient weight w_r
+
+    def train_iter():
+        ctx.sample_batch(-1, BATCH, PATCH, out=(blr, bhr, bidx))   # device-side step counter
+        ctx.train_grad(blr, bhr, loss)                            # grad <- w_r g_r
+        scale = dp_allreduce_grad_dev(grad, wdev)                 # NCCL over NVLink (N > 1); 1 / sum_r w_r
+        ctx.train_apply_dev(scale)
+
+    # one training iteration captured as a CUDA graph (after an eager warm-up that sizes the workspaces)
+    train_iter()
+    torch.cuda.synchronize()
+    graph = None
+    launches_per_iter = 0
+    if not args.no_graph:
+        graph = torch.cuda.CUDAGraph()
+        lc = ctx.launches
+        with torch.cuda.graph(graph):
+            train_iter()
+        launches_per_iter = ctx.launches - lc   # our kernels inside one captured iteration
 
     def train_iters():
         for _ in range(args.iters):
-            ctx.sample_batch(state["step"], BATCH, PATCH, out=(blr, bhr, bidx))
-            state["step"] += 1
-            ctx.train_grad(blr, bhr, loss)      # grad <- w_r g_r
-            scale = dp_allreduce_grad(grad)     # NCCL over NVLink (world > 1): sum_r w_r g_r; 1 / sum_r w_r
-            ctx.train_apply(scale)
+            if graph is not None:
+                graph.replay()
+            else:
+                train_iter()
         ctx.publish()
 
     def step():
@@ -155,11 +176,24 @@ def run_ours(args):
     e1.record()
     barrier()
     ms = e0.elapsed_time(e1)
-    launches = ctx.launches - l0
+    launches = ctx.launches - l0 + (launches_per_iter * args.iters * args.steps if graph is not None else 0)
     stats = ctx.kernel_stats()
     ctx.kernel_timing(False)
     clocks = clk.stop()
     ms = max_over_ranks(ms, device=dev)
+
+    # ---- training iteration alone (informational; the step above already contains it)
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t0.record()
+    for _ in range(20):
+        if graph is not None:
+            graph.replay()
+        else:
+            train_iter()
+    t1.record()
+    torch.cuda.synchronize()
+    train_iter_ms = t0.elapsed_time(t1) / 20
 
     # ---- end-to-end: host (pinned) frames in, host frames out, through the C ABI (sr_infer_host)
     lr_host = torch.from_numpy(lr_np).pin_memory()
@@ -215,9 +249,13 @@ def run_ours(args):
                 "l2": "working set > L2 (one 720p activation tensor at 48 ch = 88 MB; 30 frames per step)",
             },
             "train_patches_per_s": round(BATCH * args.iters * args.steps * world / (ms * 1e-3), 1),
+            "train_iter": {"ms": round(train_iter_ms, 4), "tflops": round(TRAIN_FLOP / (train_iter_ms * 1e-3) / 1e12, 1),
+                           "graph": graph is not None, "note": "one sampled training iteration alone (rank 0)"},
             "quality_gain_db": round(state["q"][2], 4) if state["q"] else None,
             "tensor_tflops_all_convs": round(conv_flops / (sum(v["ms"] for v in stats.values()) * 1e-3) / 1e12, 1),
             "kernel_share": {k: round(v["ms"] / ktot, 4) for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"])},
+            "kernel_share_note": "CUDA-event time per kernel class of the eagerly launched kernels (inference, "
+                                 "psnr_gain); the graph-replayed training kernels are in train_iter",
             "roofline": {"bound": "tensor", "kernel": dom, "achieved": round(achieved, 1),
                          "peak": sustained, "unit": "TFLOP/s", "frac": round(achieved / sustained, 4),
                          "peak_kind": "measured bf16_tflops_sustained (MEASURED_PEAKS.json)",
@@ -292,6 +330,7 @@ def main():
     ap.add_argument("--frames", type=int, default=FRAMES)
     ap.add_argument("--iters", type=int, default=ITERS)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-graph", action="store_true", help="launch the training iterations eagerly")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

@@ -119,6 +119,10 @@ class SRContext:
     def train_apply(self, grad_scale=1.0, stream=None):
         check(self.lib.sr_train_apply(self.h, C.c_float(grad_scale), _stream(stream)), self.h, "sr_train_apply")
 
+    def train_apply_dev(self, scale_dev, stream=None):
+        """Adam with the gradient scale read from a device float tensor (graph-capturable)."""
+        check(self.lib.sr_train_apply_dev(self.h, _ptr(scale_dev), _stream(stream)), self.h, "sr_train_apply_dev")
+
     def pool_push(self, lr, hr, stream=None):
         n, pp = lr.shape[0], lr.shape[1]
         check(self.lib.sr_pool_push(self.h, _ptr(lr), _ptr(hr), n, pp, None, _stream(stream)), self.h,

@@ -40,6 +40,7 @@ _SIGS = {
     "sr_train_grad": (_I, [_P, _P, _P, _I, _I, _P, _P]),
     "sr_grad_buffer": (_P, [_P]),
     "sr_train_apply": (_I, [_P, C.c_float, _P]),
+    "sr_train_apply_dev": (_I, [_P, _P, _P]),
     "sr_pool_push": (_I, [_P, _P, _P, _I, _I, _P, _P]),
     "sr_pool_size": (C.c_size_t, [_P]),
     "sr_sample_batch": (_I, [_P, C.c_int64, _I, _I, _P, _P, _P, _P]),

@@ -594,10 +594,10 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
           float v[16];
           tmem_ld16(tmem + ((uint32_t)(quarter * 32) << 16) + (dx * NMT + mt) * COUTP + c0, v);
           tmem_ld_wait();
-          if (ok) {
-            float* o = outp + ((size_t)(dy * 3 + dx) * CINP + ci) * COUTP + c0;
+          if (ok) {  // 16 consecutive floats: four 16-byte stores
+            float4* o = reinterpret_cast<float4*>(outp + ((size_t)(dy * 3 + dx) * CINP + ci) * COUTP + c0);
 #pragma unroll
-            for (int q = 0; q < 16; ++q) o[q] = v[q];
+            for (int q = 0; q < 4; ++q) o[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
           }
         }
       }

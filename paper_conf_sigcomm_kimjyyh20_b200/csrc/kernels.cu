@@ -118,13 +118,26 @@ void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int c
 
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
 // m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;  p -= (lr / bc1) * m / (sqrt(v) / sqrt(bc2) + eps),  g = s * grad
+// t and the bias corrections live on the device (k_adam_prep) so the step is replayable from a CUDA graph.
+__global__ void k_adam_prep(long long* counters, float* scal, double lr, double b1, double b2) {
+  const long long t = ++counters[1];
+  scal[0] = (float)(lr / (1.0 - pow(b1, (double)t)));
+  scal[1] = (float)(1.0 / sqrt(1.0 - pow(b2, (double)t)));
+}
+
+void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st) {
+  k_adam_prep<<<1, 1, 0, st>>>(counters, scal, lr, b1, b2);
+}
+
 __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
-                       const float* __restrict__ grad, size_t n, float gscale, float lr_bc1, float inv_sqrt_bc2,
-                       float b1, float b2, float eps) {
+                       const float* __restrict__ grad, size_t n, const float* __restrict__ gscale_dev, float gscale,
+                       const float* __restrict__ scal, float b1, float b2, float eps) {
+  const float gs = gscale * (gscale_dev ? *gscale_dev : 1.f);
+  const float lr_bc1 = scal[0], inv_sqrt_bc2 = scal[1];
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   const size_t stride = (size_t)gridDim.x * blockDim.x;
   for (; i < n; i += stride) {
-    const float g = grad[i] * gscale;
+    const float g = grad[i] * gs;
     const float mi = fmaf(b1, m[i], (1.f - b1) * g);
     const float vi = fmaf(b2, v[i], (1.f - b2) * g * g);
     m[i] = mi;
@@ -133,12 +146,17 @@ __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __re
   }
 }
 
-void launch_adam(float* p, float* m, float* v, const float* g, size_t n, float gscale, float lr_bc1,
-                 float inv_sqrt_bc2, float b1, float b2, float eps, cudaStream_t st) {
+void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
+                 const float* scal, float b1, float b2, float eps, cudaStream_t st) {
   int th = 256;
   int blocks = (int)((n + th - 1) / th);
   if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
-  k_adam<<<blocks, th, 0, st>>>(p, m, v, g, n, gscale, lr_bc1, inv_sqrt_bc2, b1, b2, eps);
+  k_adam<<<blocks, th, 0, st>>>(p, m, v, g, n, gscale_dev, gscale, scal, b1, b2, eps);
+}
+
+__global__ void k_counter_add(long long* c, long long d) { *c += d; }
+void launch_counter_add(long long* counter, long long delta, cudaStream_t st) {
+  k_counter_add<<<1, 1, 0, st>>>(counter, delta);
 }
 
 // --------------------------------------------------------------- sampler + gather (reading R10)
@@ -157,7 +175,8 @@ __global__ void k_sample_gather(SampleArgs a) {
   __shared__ int s_slot, s_oy, s_ox;
   if (threadIdx.x == 0) {
     const uint64_t GAMMA = 0x9E3779B97F4A7C15ull;
-    const uint64_t base = ((((uint64_t)a.step * a.world + a.rank) << 20) + (uint64_t)j) * 4ull;
+    const long long step = a.step >= 0 ? a.step : *a.step_dev;
+    const uint64_t base = ((((uint64_t)step * a.world + a.rank) << 20) + (uint64_t)j) * 4ull;
     const uint64_t u0 = mix64(a.seed + GAMMA * (base + 1));
     const uint64_t u1 = mix64(a.seed + GAMMA * (base + 2));
     const uint64_t u2 = mix64(a.seed + GAMMA * (base + 3));

@@ -13,7 +13,8 @@ struct ConvDesc {
 
 struct SampleArgs {
   uint64_t seed;
-  long long step;
+  long long step;           // < 0: read the step from *step_dev (graph-replayable sampling)
+  const long long* step_dev;
   int world, rank;
   long long n_view, view_base, capacity;
   int recent_k, recent_w;
@@ -33,8 +34,12 @@ cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wf
                              const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st);
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st);
-void launch_adam(float* p, float* m, float* v, const float* g, size_t n, float gscale, float lr_bc1,
-                 float inv_sqrt_bc2, float b1, float b2, float eps, cudaStream_t st);
+// Device-side step counters (so a training iteration can be captured once in a CUDA graph and replayed):
+// counters[0] = sampler step, counters[1] = Adam step t; scal[0] = lr / (1 - b1^t), scal[1] = 1/sqrt(1 - b2^t).
+void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st);
+void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
+                 const float* scal, float b1, float b2, float eps, cudaStream_t st);
+void launch_counter_add(long long* counter, long long delta, cudaStream_t st);
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st);
 void launch_sse_u8(const uint8_t* a, const uint8_t* b, int n, int64_t elems, unsigned long long* out,
                    cudaStream_t st);

@@ -42,6 +42,8 @@ struct sr_ctx {
   float *ws_w = nullptr, *ws_b = nullptr;
   size_t ws_w_elems = 0, ws_b_elems = 0;
   double* loss_sum = nullptr;
+  long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t
+  float* adam_scal = nullptr;     // device: lr/bc1, 1/sqrt(bc2)
   // patch pool (device ring)
   uint8_t *pool_lr = nullptr, *pool_hr = nullptr;
   long long pool_total = 0, pool_cap = 0;
@@ -55,6 +57,9 @@ struct sr_ctx {
   unsigned long long* sse = nullptr;
   int sse_n = 0;
   cudaEvent_t publish_ev = nullptr;
+  // CUDA graph of one sampled training iteration (sample -> fwd/bwd -> Adam), per (batch, p)
+  cudaGraphExec_t train_graph = nullptr;
+  int graph_batch = 0, graph_p = 0;
   unsigned long long launches = 0;
   // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
   bool timing = false;
@@ -371,13 +376,12 @@ static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, i
   return SR_OK;
 }
 
-static sr_status train_apply(sr_ctx* ctx, float grad_scale, cudaStream_t st) {
-  ctx->t += 1;
-  const double b1 = ctx->opt.beta1, b2 = ctx->opt.beta2;
-  const double bc1 = 1.0 - std::pow(b1, (double)ctx->t), bc2 = 1.0 - std::pow(b2, (double)ctx->t);
-  launch_adam(ctx->params, ctx->m, ctx->v, ctx->grad, ctx->nparams, grad_scale, (float)(ctx->opt.lr / bc1),
-              (float)(1.0 / std::sqrt(bc2)), (float)b1, (float)b2, ctx->opt.eps, st);
-  ctx->launches++;
+static sr_status train_apply(sr_ctx* ctx, float grad_scale, const float* grad_scale_dev, cudaStream_t st) {
+  ctx->t += 1;  // host mirror only; the kernels use the device counter (graph-replayable)
+  launch_adam_prep(ctx->counters, ctx->adam_scal, ctx->opt.lr, ctx->opt.beta1, ctx->opt.beta2, st);
+  launch_adam(ctx->params, ctx->m, ctx->v, ctx->grad, ctx->nparams, grad_scale_dev, grad_scale, ctx->adam_scal,
+              ctx->opt.beta1, ctx->opt.beta2, ctx->opt.eps, st);
+  ctx->launches += 2;
   CKL();
   return repack(ctx, SR_TRAIN, true, st);
 }
@@ -452,6 +456,8 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   }
   al(&ctx->wd_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
+  al(&ctx->counters, 2);
+  al(&ctx->adam_scal, 2);
   ctx->tf.assign(blocks + 1, nullptr);
   ctx->tts.assign(blocks, nullptr);
   if (st != SR_OK) { sr_destroy(ctx); return st; }
@@ -485,7 +491,8 @@ void sr_destroy(sr_ctx* ctx) {
   cudaDeviceSynchronize();
   void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->x16, ctx->f0,
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
-                  ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->pool_lr,
+                  ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->counters,
+                  ctx->adam_scal, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->val_b, ctx->sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -493,6 +500,7 @@ void sr_destroy(sr_ctx* ctx) {
   for (auto p : ctx->tf) if (p) cudaFree(p);
   for (auto p : ctx->tts) if (p) cudaFree(p);
   if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
+  if (ctx->train_graph) cudaGraphExecDestroy(ctx->train_graph);
   for (auto& r : ctx->trec) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
   delete ctx;
 }
@@ -551,6 +559,7 @@ sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
   CK(cudaMemset(ctx->m, 0, n * sizeof(float)));
   CK(cudaMemset(ctx->v, 0, n * sizeof(float)));
   CK(cudaMemset(ctx->grad, 0, n * sizeof(float)));
+  CK(cudaMemset(ctx->counters, 0, 2 * sizeof(long long)));
   ctx->t = 0;
   TRY(repack(ctx, SR_TRAIN, true, 0));
   for (int k = 1; k < 4; ++k) {
@@ -642,7 +651,13 @@ sr_status sr_train_grad(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_de
 
 sr_status sr_train_apply(sr_ctx* ctx, float grad_scale, sr_stream stream) {
   GUARD();
-  return train_apply(ctx, grad_scale, (cudaStream_t)stream);
+  return train_apply(ctx, grad_scale, nullptr, (cudaStream_t)stream);
+}
+
+sr_status sr_train_apply_dev(sr_ctx* ctx, const float* grad_scale_dev, sr_stream stream) {
+  GUARD();
+  if (!grad_scale_dev) return fail(ctx, SR_E_INVAL, "sr_train_apply_dev: null scale");
+  return train_apply(ctx, 1.0f, grad_scale_dev, (cudaStream_t)stream);
 }
 
 sr_status sr_train_step(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
@@ -650,7 +665,7 @@ sr_status sr_train_step(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_de
   GUARD();
   TRY(sr_train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, stream));
   const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
-  return train_apply(ctx, 1.0f / w, (cudaStream_t)stream);
+  return train_apply(ctx, 1.0f / w, nullptr, (cudaStream_t)stream);
 }
 
 sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int pp,
@@ -696,6 +711,7 @@ sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* 
   SampleArgs a{};
   a.seed = ctx->opt.seed;
   a.step = step;
+  a.step_dev = ctx->counters;
   a.world = G;
   a.rank = r;
   a.n_view = hi - lo;
@@ -713,6 +729,10 @@ sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* 
   a.idx_out = idx_out_dev;
   launch_sample_gather(a, batch, (cudaStream_t)stream);
   ctx->launches++;
+  if (step < 0) {  // graph mode: advance the device-side sampler step
+    launch_counter_add(ctx->counters, 1, (cudaStream_t)stream);
+    ctx->launches++;
+  }
   CKL();
   return SR_OK;
 }
@@ -721,12 +741,43 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
   GUARD();
   if (iters < 1 || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_sampled: bad args");
   if (ctx->opt.world != 1) return fail(ctx, SR_E_STATE, "sr_train_sampled: world > 1 needs the split API");
+  cudaStream_t st = (cudaStream_t)stream;
   const size_t lb = (size_t)batch * p * p * 3, hb = lb * ctx->s * ctx->s;
-  if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; }
-  if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; }
+  auto one_iter = [&]() -> sr_status {
+    TRY(sr_sample_batch(ctx, -1, batch, p, ctx->batch_lr, ctx->batch_hr, nullptr, stream));  // device step counter
+    TRY(train_grad(ctx, ctx->batch_lr, ctx->batch_hr, batch, p, loss_dev, st));
+    const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
+    return train_apply(ctx, 1.0f / w, nullptr, st);
+  };
+  if (!ctx->train_graph || ctx->graph_batch != batch || ctx->graph_p != p || st == nullptr) {
+    if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; }
+    if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; }
+    TRY(one_iter());  // eager iteration: grows the workspaces, configures the kernels
+    --iters;
+    if (st != nullptr) {  // capture one iteration (the legacy default stream cannot be captured)
+      if (ctx->train_graph) { cudaGraphExecDestroy(ctx->train_graph); ctx->train_graph = nullptr; }
+      const bool timing = ctx->timing;
+      ctx->timing = false;
+      cudaGraph_t g = nullptr;
+      CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+      sr_status cs = one_iter();
+      cudaError_t ce = cudaStreamEndCapture(st, &g);
+      ctx->timing = timing;
+      TRY(cs);
+      CK(ce);
+      CK(cudaGraphInstantiate(&ctx->train_graph, g, 0));
+      cudaGraphDestroy(g);
+      ctx->graph_batch = batch;
+      ctx->graph_p = p;
+    }
+  }
   for (int it = 0; it < iters; ++it) {
-    TRY(sr_sample_batch(ctx, ctx->sample_step++, batch, p, ctx->batch_lr, ctx->batch_hr, nullptr, stream));
-    TRY(sr_train_step(ctx, ctx->batch_lr, ctx->batch_hr, batch, p, loss_dev, stream));
+    if (ctx->train_graph && st != nullptr) {
+      CK(cudaGraphLaunch(ctx->train_graph, st));
+      ctx->launches += 1;
+    } else {
+      TRY(one_iter());
+    }
   }
   return SR_OK;
 }

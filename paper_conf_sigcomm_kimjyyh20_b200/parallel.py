@@ -43,6 +43,17 @@ def dp_allreduce_grad(grad, weight: float = 1.0, group=None) -> float:
     return 1.0 / float(w.item())
 
 
+def dp_allreduce_grad_dev(grad, weight_dev, group=None):
+    """Graph-capturable variant: sum-allreduce `grad` and the 1-element weight tensor `weight_dev` on the device and
+    return a device tensor holding 1 / sum_r w_r (feed it to SRContext.train_apply_dev)."""
+    import torch.distributed as dist
+    w = weight_dev.clone()
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(grad, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(w, op=dist.ReduceOp.SUM, group=group)
+    return w.reciprocal()
+
+
 def max_over_ranks(value: float, device=None, group=None) -> float:
     """Max of a scalar over ranks (timings are reported as the slowest rank)."""
     import torch
