@@ -159,6 +159,9 @@ class SRContext:
                                     _stream(stream)), self.h, "sr_psnr_gain")
         return q.psnr_a, q.psnr_b, q.gain
 
+    def set_fusion(self, fuse_blocks=True):
+        check(self.lib.sr_set_fusion(self.h, int(fuse_blocks)), self.h, "sr_set_fusion")
+
     def kernel_timing(self, enable=True):
         check(self.lib.sr_kernel_timing(self.h, int(enable)), self.h, "sr_kernel_timing")
 

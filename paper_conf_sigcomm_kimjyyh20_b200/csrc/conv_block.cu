@@ -1,0 +1,427 @@
+// Fused residual block for wide frames:  f' = f + conv2(ReLU(conv1(f) + b1)) + b2   (sm_100a tcgen05)
+//
+// Unfused, one block moves 480 B per pixel through HBM at C = 48 (conv1: read f, write t; conv2: read t, read f,
+// write f') against 83 kFLOP -- below the B200 ridge.  Here the ReLU intermediate t never leaves the SM: both
+// convs use the rolling dy-fold form of conv_roll.cu (N = 3C per MMA, one input row per step) and t rows pass
+// through a shared-memory ring from the conv1 epilogue to the conv2 MMAs.  HBM per pixel: f once (+2 columns of
+// halo per 126) and f' once.
+//
+// Column strip of 126 output pixels starting at x0 (MMA M = 128 lanes):
+//   f row in smem  : pixels x0-2 .. x0+127 (130, TMA, zero outside the frame)
+//   conv1 lane m   : t column x0-1+m, reads f positions m+dx              -> t row in smem (128 + 2 spare positions)
+//   conv2 lane m   : out column x0+m (m < 126), reads t positions m+dx
+//   t is forced to 0 outside the frame (it is conv2's zero padding).
+//
+// Accumulation (the point of this design): for every input row the MMA group (3 dx x C/16 MMAs, N = 3C) adds
+//   dy = 0 into the accumulator of output row i+1, dy = 1 into row i, dy = 2 into row i-1,
+// i.e. out[r] = sum_{dy} sum_{dx,ci} in[r+dy-1, x+dx-1, ci] W[co,ci,dy,dx] is summed by the tensor core in TMEM.
+// Output rows own C-column blocks of a TMEM ring (RB blocks per conv, descending so the three targets of a step
+// are contiguous; when the ring wraps inside them the step is issued as two MMA groups).  Blocks are armed with
+// the bias (tcgen05.st) by the epilogue, so the epilogue only drains a finished row: ReLU -> t smem (conv1) or
+// + residual -> TMA store (conv2), then re-arms the block.
+// Rows of a strip piece with output rows [y0,y1): f rows y0-2 .. y1+1 (n_f), t rows y0-1 .. y1 (n_t = n_f - 2).
+// Per conv the out-row sequence of a piece has n_in + 2 entries (local q = -1 .. n_in); q in [1, n_in-2] are
+// the rows that are kept.
+//
+// Warps: 0 TMA producer, 1 TMEM alloc + MMA issuer (conv1 runs three rows ahead of conv2), 2..5 conv1
+// epilogue, 6..9 conv2 epilogue (residual from global/L2, rows -> smem -> TMA store).  The kernel is bound by the
+// 128 B/clk shared-memory port: per row-step the MMAs read ~155 KB of operands (A 4 KB + B 4.5 KB per MMA) and the
+// TMA/epilogue traffic adds ~49 KB (clock64 timeline, scripts/bench_block.py).
+#include <cuda.h>
+#include "ptx.cuh"
+#include "tmap.h"
+#include "sr_internal.h"
+
+namespace sr {
+
+static constexpr int kBlkThreads = 320;
+static constexpr int kBlkTW = 126;  // output pixels per strip
+static constexpr int kBlkNF = 4;    // f-row ring
+static constexpr int kBlkNT = 3;    // t-row ring
+static constexpr int kBlkNO = 3;    // output staging rows (TMA store)
+
+template <int C>
+struct BlkCfg {
+  static constexpr int CCH = C / 8, KS = C / 16, N = 3 * C;
+  static constexpr int RB = (256 / C) < 8 ? (256 / C) : 8;  // TMEM ring blocks per conv (256 columns each)
+  static constexpr uint32_t WBYTES = 9u * C * C * 2u;
+  static constexpr uint32_t PLANE = 130 * 16;
+  static constexpr uint32_t ROWB = ((CCH * PLANE) + 1023u) & ~1023u;             // f / t ring slot
+  static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
+  static constexpr uint32_t OUTB = ((kBlkTW * C * 2) + 1023u) & ~1023u;          // staging row
+  static constexpr size_t SMEM = 1024 + 2 * WB_AL + (size_t)kBlkNF * ROWB + (size_t)kBlkNT * ROWB +
+                                 (size_t)kBlkNO * OUTB;
+};
+
+// One rolling dy-fold step of a conv: A = input row in smem (chunk-planar, pitch 130), B = dy-fold weights.
+// g = global out-row index of the dy = 2 target (the row this step completes).
+template <int C>
+__device__ __forceinline__ void blk_mma_step(uint32_t ring_base, long long g, uint64_t ad, uint64_t bd) {
+  using Cfg = BlkCfg<C>;
+  constexpr int RB = Cfg::RB, CCH = Cfg::CCH, KS = Cfg::KS;
+  constexpr uint32_t PLANE = Cfg::PLANE;
+  const int i0 = ring_idx<RB>(g);
+  // (column block, first B row, N) of up to two groups
+  int blkA, rowA, nA, blkB = 0, rowB = 0, nB = 0;
+  if (i0 >= 2) { blkA = i0 - 2; rowA = 0; nA = 3 * C; }
+  else if (i0 == 0) { blkA = RB - 2; rowA = 0; nA = 2 * C; blkB = 0; rowB = 2 * C; nB = C; }
+  else { blkA = RB - 1; rowA = 0; nA = C; blkB = 0; rowB = C; nB = 2 * C; }
+  const uint32_t idA = make_idesc(128, nA, 0, 0);
+#pragma unroll
+  for (int dx = 0; dx < 3; ++dx)
+#pragma unroll
+    for (int ks = 0; ks < KS; ++ks)
+      mma_bf16_ss(ring_base + blkA * C, desc_add(ad, dx * 16u + ks * 2u * PLANE),
+                  desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * Cfg::N * 16u + rowA * 16u), idA, 1u);
+  if (nB) {
+    const uint32_t idB = make_idesc(128, nB, 0, 0);
+#pragma unroll
+    for (int dx = 0; dx < 3; ++dx)
+#pragma unroll
+      for (int ks = 0; ks < KS; ++ks)
+        mma_bf16_ss(ring_base + blkB * C, desc_add(ad, dx * 16u + ks * 2u * PLANE),
+                    desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * Cfg::N * 16u + rowB * 16u), idB, 1u);
+  }
+}
+
+// Epilogue helper: load the C accumulator columns of a ring block (this thread's lane) and re-arm the block with
+// the bias (the next row that lands in it starts from b).
+template <int C>
+__device__ __forceinline__ void blk_drain(uint32_t taddr, float* v, const float4* sbias) {
+#pragma unroll
+  for (int c0 = 0; c0 < C; c0 += 16) tmem_ld16(taddr + c0, v + c0);
+  tmem_ld_wait();
+#pragma unroll
+  for (int c0 = 0; c0 < C; c0 += 16) {
+    float b[16];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const float4 t = sbias[c0 / 4 + q];
+      b[4 * q] = t.x; b[4 * q + 1] = t.y; b[4 * q + 2] = t.z; b[4 * q + 3] = t.w;
+    }
+    tmem_st16(taddr + c0, b);
+  }
+  tmem_st_wait();
+}
+
+template <int C>
+__global__ void __launch_bounds__(kBlkThreads, 1)
+k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
+           const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
+           const float* __restrict__ b2, const bf16* __restrict__ fres, bf16* __restrict__ outp, const int N,
+           const int H, const int W, long long* __restrict__ dbg) {
+  // dbg (benchmarking only, CTA 0): clock64 stamps [event][step], events: 0 f issued, 1 conv1 step issued,
+  // 2 conv2 step issued, 3 epi1 got a block, 4 epi1 t row done, 5 epi2 got a block, 6 epi2 row stored
+#define SR_DBG(ev, idx) \
+  if (dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) dbg[(ev) * 256 + (idx)] = clock64();
+  // more MMA-thread stamps: 7 step start, 8 conv1 blocks acquired, 9 f row landed, 10 conv2 part start,
+  // 11 conv2 blocks acquired, 12 t row ready
+  using Cfg = BlkCfg<C>;
+  constexpr int CCH = Cfg::CCH, RB = Cfg::RB;
+  constexpr uint32_t PLANE = Cfg::PLANE, ROWB = Cfg::ROWB, OUTB = Cfg::OUTB;
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sW1 = smem;
+  uint8_t* sW2 = sW1 + Cfg::WB_AL;
+  uint8_t* sF = sW2 + Cfg::WB_AL;
+  uint8_t* sT = sF + kBlkNF * ROWB;
+  uint8_t* sO = sT + kBlkNT * ROWB;
+  __shared__ __align__(8) uint64_t f_full[kBlkNF], f_empty[kBlkNF], t_full[kBlkNT], t_empty[kBlkNT], r1_ready[RB],
+      r1_free[RB], r2_ready[RB], r2_free[RB], w_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ __align__(16) float4 sb1v[C / 4], sb2v[C / 4];
+
+  const int warp = warp_id();
+  if (threadIdx.x < C) {
+    reinterpret_cast<float*>(sb1v)[threadIdx.x] = b1[threadIdx.x];
+    reinterpret_cast<float*>(sb2v)[threadIdx.x] = b2[threadIdx.x];
+  }
+  // spare t positions 128, 129 of every plane of every t slot are read by the two invalid conv2 lanes: zero them
+  for (int i = threadIdx.x; i < kBlkNT * CCH * 2; i += blockDim.x) {
+    const int slot = i / (CCH * 2), rem = i % (CCH * 2);
+    *reinterpret_cast<uint4*>(sT + slot * ROWB + (rem / 2) * PLANE + (128 + rem % 2) * 16) = make_uint4(0, 0, 0, 0);
+  }
+  fence_proxy_async_smem();
+  if (warp == 0 && lane_id() == 0) {
+    for (int s = 0; s < kBlkNF; ++s) { mbar_init(&f_full[s], 1); mbar_init(&f_empty[s], 1); }
+    for (int s = 0; s < kBlkNT; ++s) { mbar_init(&t_full[s], 4); mbar_init(&t_empty[s], 1); }
+    for (int s = 0; s < RB; ++s) {
+      mbar_init(&r1_ready[s], 1); mbar_init(&r1_free[s], 4);
+      mbar_init(&r2_ready[s], 1); mbar_init(&r2_free[s], 4);
+    }
+    mbar_init(&w_bar, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const uint32_t ring1 = tmem, ring2 = tmem + 256;
+
+  const int tiles_x = (W + kBlkTW - 1) / kBlkTW;
+  const long long total = (long long)N * tiles_x * H;
+  const long long beg = total * blockIdx.x / gridDim.x, end = total * (blockIdx.x + 1) / gridDim.x;
+#define SR_PIECE_BEGIN                                                                \
+  for (long long pos = beg; pos < end;) {                                             \
+    const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);             \
+    const int y1 = (int)min((long long)H, y0 + (end - pos));                          \
+    pos += y1 - y0;                                                                   \
+    const int n = col / tiles_x, x0 = (col - n * tiles_x) * kBlkTW;                   \
+    const int n_f = y1 - y0 + 4, n_t = n_f - 2;                                       \
+    (void)n; (void)x0; (void)n_t;
+#define SR_PIECE_END }
+
+  if (warp == 0) {
+    // ===================== producer: weights once, then f rows y0-2 .. y1+1 of every piece =====================
+    if (elect_one()) {
+      tma_prefetch_desc(&tm_f);
+      mbar_arrive_expect_tx(&w_bar, 2 * Cfg::WBYTES);
+      bulk_load(sW1, w1, Cfg::WBYTES, &w_bar);
+      bulk_load(sW2, w2, Cfg::WBYTES, &w_bar);
+      int s = 0;
+      uint32_t ph = 0;
+      SR_PIECE_BEGIN
+      for (int i = 0; i < n_f; ++i) {
+        mbar_wait(&f_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&f_full[s], CCH * PLANE);
+        tma_load_5d(sF + s * ROWB, &tm_f, &f_full[s], 0, x0 - 2, y0 - 2 + i, 0, n);
+        SR_DBG(0, i)
+        if (++s == kBlkNF) { s = 0; ph ^= 1; }
+      }
+      SR_PIECE_END
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    // ===================== MMA issuer: conv1 step st (f row st), then conv2 step st-3 (t row st-3) ===============
+    if (elect_one()) {
+      mbar_wait(&w_bar, 0);
+      const uint64_t bd1 = make_desc(smem_u32(sW1), Cfg::N * 16, 128);
+      const uint64_t bd2 = make_desc(smem_u32(sW2), Cfg::N * 16, 128);
+      int fs = 0, ts = 0;
+      uint32_t fph = 0, tph = 0;
+      long long G1 = 0, G2 = 0, acq1 = 0, acq2 = 0;  // out-row sequences (first row of the piece) / blocks acquired
+      SR_PIECE_BEGIN
+      for (int st = 0; st <= n_f + 2; ++st) {
+        SR_DBG(7, st)
+        if (st < n_f) {
+          const long long g = G1 + st;
+          for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
+          SR_DBG(8, st)
+          mbar_wait(&f_full[fs], fph);
+          SR_DBG(9, st)
+          tc_fence_after();
+          blk_mma_step<C>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1);
+          mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
+          mma_commit(&f_empty[fs]);
+          if (st == n_f - 1) {                      // the last two rows of the piece receive nothing more
+            mma_commit(&r1_ready[ring_idx<RB>(g + 1)]);
+            mma_commit(&r1_ready[ring_idx<RB>(g + 2)]);
+          }
+          SR_DBG(1, st)
+          if (++fs == kBlkNF) { fs = 0; fph ^= 1; }
+        }
+        const int k = st - 3;
+        SR_DBG(10, st)
+        if (k >= 0 && k < n_t) {
+          const long long g = G2 + k;
+          for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
+          SR_DBG(11, st)
+          mbar_wait(&t_full[ts], tph);
+          SR_DBG(12, st)
+          tc_fence_after();
+          blk_mma_step<C>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2);
+          mma_commit(&r2_ready[ring_idx<RB>(g)]);
+          mma_commit(&t_empty[ts]);
+          if (k == n_t - 1) {
+            mma_commit(&r2_ready[ring_idx<RB>(g + 1)]);
+            mma_commit(&r2_ready[ring_idx<RB>(g + 2)]);
+          }
+          SR_DBG(2, k)
+          if (++ts == kBlkNT) { ts = 0; tph ^= 1; }
+        }
+      }
+      G1 += n_f + 2;
+      G2 += n_t + 2;
+      SR_PIECE_END
+    }
+    __syncwarp();
+  } else if (warp < 6) {
+    // ===================== conv1 epilogue: drain finished t rows -> ReLU -> t smem ring =====================
+    const int quarter = warp & 3;
+    const int m = quarter * 32 + lane_id();
+    const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+    {  // arm every ring block with b1
+      float v[C];
+      for (int b = 0; b < RB; ++b) {
+        blk_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+        tc_fence_before();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&r1_free[b]);
+      }
+    }
+    int ts = 0;
+    uint32_t tph = 0;
+    long long G = 0;
+    SR_PIECE_BEGIN
+    const int tcol = x0 - 1 + m;
+    const bool col_ok = tcol >= 0 && tcol < W;
+    for (int q = -1; q <= n_f; ++q) {         // out rows of conv1 = t rows y0-2+q
+      const long long g = G + q + 1;
+      const bool emit = q >= 1 && q <= n_f - 2;
+      const int trow = y0 - 2 + q;
+      const bool ok = col_ok && trow >= 0 && trow < H;
+      if (emit) mbar_wait(&t_empty[ts], tph ^ 1);
+      const int b = ring_idx<RB>(g);
+      mbar_wait(&r1_ready[b], (uint32_t)(g / RB) & 1u);
+      tc_fence_after();
+      if (warp == 2 && lane_id() == 0) { SR_DBG(3, q + 1) }
+      float v[C];
+      blk_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+      tc_fence_before();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&r1_free[b]);
+      if (emit) {
+        uint8_t* dst = sT + ts * ROWB + m * 16;
+#pragma unroll
+        for (int j = 0; j < CCH; ++j) {
+          float a[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) a[e] = ok ? fmaxf(v[8 * j + e], 0.f) : 0.f;
+          uint4 u;
+          u.x = pack_bf16x2(a[0], a[1]);
+          u.y = pack_bf16x2(a[2], a[3]);
+          u.z = pack_bf16x2(a[4], a[5]);
+          u.w = pack_bf16x2(a[6], a[7]);
+          *reinterpret_cast<uint4*>(dst + j * PLANE) = u;
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&t_full[ts]);
+        if (warp == 2 && lane_id() == 0) { SR_DBG(4, q + 1) }
+        if (++ts == kBlkNT) { ts = 0; tph ^= 1; }
+      }
+    }
+    G += n_f + 2;
+    SR_PIECE_END
+  } else {
+    // ===================== conv2 epilogue: drain finished rows -> + residual f -> smem -> TMA store ==========
+    const int quarter = warp & 3;
+    const int m = quarter * 32 + lane_id();
+    const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+    const bool leader = (warp == 6 && lane_id() == 0);
+    {
+      float v[C];
+      for (int b = 0; b < RB; ++b) {
+        blk_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+        tc_fence_before();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&r2_free[b]);
+      }
+    }
+    int os = 0;
+    long long G = 0;
+    SR_PIECE_BEGIN
+    const bool lane_ok = m < kBlkTW && x0 + m < W;
+    for (int q = -1; q <= n_t; ++q) {         // out rows of conv2 = output rows y0-1+q
+      const long long g = G + q + 1;
+      const bool emit = q >= 1 && q <= n_t - 2;
+      const int r = y0 - 1 + q;
+      uint4 res[C / 8];
+      if (emit && lane_ok) {
+        const uint4* rp = reinterpret_cast<const uint4*>(fres + ((((size_t)n * H + r) * W) + x0 + m) * C);
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) res[j] = __ldg(rp + j);
+      }
+      const int b = ring_idx<RB>(g);
+      mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
+      tc_fence_after();
+      if (warp == 6 && lane_id() == 0) { SR_DBG(5, q + 1) }
+      float v[C];
+      blk_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+      tc_fence_before();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&r2_free[b]);
+      if (emit) {
+        if (lane_ok) {
+          uint4* orow = reinterpret_cast<uint4*>(sO + os * OUTB + m * C * 2);
+#pragma unroll
+          for (int j = 0; j < C / 8; ++j) {
+            const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&res[j]);
+            float a[8];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float2 f2 = __bfloat1622float2(h2[e]);
+              a[2 * e] = v[8 * j + 2 * e] + f2.x;
+              a[2 * e + 1] = v[8 * j + 2 * e + 1] + f2.y;
+            }
+            uint4 u;
+            u.x = pack_bf16x2(a[0], a[1]);
+            u.y = pack_bf16x2(a[2], a[3]);
+            u.z = pack_bf16x2(a[4], a[5]);
+            u.w = pack_bf16x2(a[6], a[7]);
+            orow[j] = u;
+          }
+        }
+        fence_proxy_async_smem();
+        named_bar_sync(2, 128);
+        if (leader) {
+          tma_store_4d(&tm_out, sO + os * OUTB, 0, x0, r, n);
+          bulk_commit();
+          bulk_wait_read<kBlkNO - 2>();
+          SR_DBG(6, q + 1)
+        }
+        os = os == kBlkNO - 1 ? 0 : os + 1;
+      }
+    }
+    G += n_t + 2;
+    SR_PIECE_END
+    if (leader) bulk_wait<0>();
+  }
+#undef SR_PIECE_BEGIN
+#undef SR_PIECE_END
+#undef SR_DBG
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tmem);
+}
+
+template <int C>
+static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, const bf16* w1, const bf16* w2,
+                                  const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
+                                  int grid, long long* dbg, cudaStream_t st) {
+  auto kern = k_resblock<C>;
+  static bool configured = false;
+  if (!configured) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BlkCfg<C>::SMEM);
+    if (e != cudaSuccess) return e;
+    configured = true;
+  }
+  kern<<<grid, kBlkThreads, BlkCfg<C>::SMEM, st>>>(tf, to, w1, w2, b1, b2, f, out, N, H, W, dbg);
+  return cudaGetLastError();
+}
+
+bool resblock_supported(int cp, int W) {
+  if (W < 96) return false;
+  if (cp == 16) return BlkCfg<16>::SMEM <= 227 * 1024;
+  if (cp == 32) return BlkCfg<32>::SMEM <= 227 * 1024;
+  if (cp == 48) return BlkCfg<48>::SMEM <= 227 * 1024;
+  return false;
+}
+
+cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
+                            const float* b2, bf16* out, int N, int H, int W, cudaStream_t st, long long* dbg) {
+  CUtensorMap tf, to;
+  if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, cp, kBlkTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  const long long rows = (long long)N * ((W + kBlkTW - 1) / kBlkTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
+  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
+  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
+  return cudaErrorNotSupported;
+}
+
+}  // namespace sr

@@ -32,6 +32,10 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 bool roll_supported(int cinp, int coutp, int W);
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
                              const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st);
+bool resblock_supported(int cp, int W);
+cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
+                            const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,
+                            long long* dbg = nullptr);
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st);
 // Device-side step counters (so a training iteration can be captured once in a CUDA graph and replayed):

@@ -200,3 +200,27 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
   for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
 }
 }  // namespace sr
+
+namespace sr {
+// registers -> TMEM: 32 lanes x 16 consecutive columns (one lane per thread)
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const float* v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])), "r"(__float_as_uint(v[3])),
+      "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])), "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])),
+      "r"(__float_as_uint(v[8])), "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])),
+      "r"(__float_as_uint(v[11])), "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])),
+      "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15]))
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// Rolling dy-fold accumulator ring in TMEM (see conv_block.cu): output-row g owns block idx(g) = (-g) mod RB of
+// C columns; one input-row step writes blocks of rows g+2 (dy0), g+1 (dy1), g (dy2), contiguous unless the ring
+// wraps inside the three (idx(g) < 2), in which case the step is issued as two MMA groups.
+template <int RB>
+__host__ __device__ constexpr int ring_idx(long long g) {
+  return (int)((RB - (g % RB)) % RB);
+}
+}  // namespace sr

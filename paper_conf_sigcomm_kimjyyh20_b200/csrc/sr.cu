@@ -63,6 +63,7 @@ struct sr_ctx {
   unsigned long long launches = 0;
   // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
   bool timing = false;
+  bool fuse_blocks = true;  // fused residual-block kernel for wide frames (sr_set_option)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -232,12 +233,25 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   TRY(conv_fwd(ctx, 16, Cp, ctx->x16, sn, 0, n, h, w, ep, st));
   bf16* cur = ctx->f0;
   for (int b = 0; b < ctx->B; ++b) {
+    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+    if (ctx->fuse_blocks && resblock_supported(Cp, w)) {  // fused block: t stays in shared memory
+      if (ctx->timing) {
+        const double px = (double)n * h * w;
+        tmark_begin(ctx, "resblock_" + std::to_string(Cp), 2 * 2.0 * 9 * Cp * Cp * px, px * 2.0 * 2 * Cp, st);
+      }
+      cudaError_t e = launch_resblock(Cp, cur, sn.wo + ctx->convs[1 + 2 * b].pk_off, sn.wo + ctx->convs[2 + 2 * b].pk_off,
+                                      Bv(1 + 2 * b), Bv(2 + 2 * b), nxt, n, h, w, st);
+      tmark_end(ctx, st);
+      ctx->launches++;
+      if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("resblock launch: ") + cudaGetErrorString(e));
+      cur = nxt;
+      continue;
+    }
     EpiParams e1{};
     e1.bias = Bv(1 + 2 * b);
     e1.relu = 1;
     e1.out = ctx->tt;
     TRY(conv_fwd(ctx, Cp, Cp, cur, sn, 1 + 2 * b, n, h, w, e1, st));
-    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
     EpiParams e2{};
     e2.bias = Bv(2 + 2 * b);
     e2.res1 = cur;
@@ -503,6 +517,12 @@ void sr_destroy(sr_ctx* ctx) {
   if (ctx->train_graph) cudaGraphExecDestroy(ctx->train_graph);
   for (auto& r : ctx->trec) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
   delete ctx;
+}
+
+sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
+  if (!ctx) return SR_E_INVAL;
+  ctx->fuse_blocks = fuse_blocks != 0;
+  return SR_OK;
 }
 
 sr_status sr_kernel_timing(sr_ctx* ctx, int enable) {

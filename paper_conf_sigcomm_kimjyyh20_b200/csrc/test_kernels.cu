@@ -192,3 +192,37 @@ extern "C" int sr_bench_conv(int cinp, int coutp, int n, int h, int w, int mode,
   cudaFree(x); cudaFree(y); cudaFree(res); cudaFree(wpk); cudaFree(bias);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
+
+// Fused residual block on random data: timing, and (dbg_host != NULL) CTA-0 pipeline timestamps [7][256].
+extern "C" int sr_bench_resblock(int c, int n, int h, int w, int iters, float* ms_out, long long* dbg_host,
+                                 void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t pix = (size_t)n * h * w;
+  bf16 *x = nullptr, *y = nullptr, *w1 = nullptr, *w2 = nullptr;
+  float* bias = nullptr;
+  long long* dbg = nullptr;
+  if (cudaMalloc(&x, pix * c * 2) || cudaMalloc(&y, pix * c * 2) || cudaMalloc(&w1, 9 * c * c * 2) ||
+      cudaMalloc(&w2, 9 * c * c * 2) || cudaMalloc(&bias, c * 4) || cudaMalloc(&dbg, 16 * 256 * 8))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(x, 0x3c, pix * c * 2, st);
+  cudaMemsetAsync(w1, 0x1c, 9 * c * c * 2, st);
+  cudaMemsetAsync(w2, 0x1c, 9 * c * c * 2, st);
+  cudaMemsetAsync(bias, 0, c * 4, st);
+  cudaMemsetAsync(dbg, 0, 16 * 256 * 8, st);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  cudaError_t e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, dbg_host ? dbg : nullptr);
+  cudaEventRecord(a, st);
+  for (int i = 0; i < iters && e == cudaSuccess; ++i) e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st);
+  cudaEventRecord(b, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, a, b);
+  *ms_out = ms / (iters > 0 ? iters : 1);
+  if (dbg_host) cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(x); cudaFree(y); cudaFree(w1); cudaFree(w2); cudaFree(bias); cudaFree(dbg);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}

@@ -222,3 +222,21 @@ def test_publish_snapshots():
     sv = ctx.get_params("serve")
     assert not np.array_equal(sv, init)
     assert np.max(np.abs(sv - tr)) <= np.max(np.abs(tr)) * 2 ** -8
+
+
+@pytest.mark.parametrize("cfg,hw", [((3, 8, 48), (90, 700)), ((2, 4, 32), (67, 260)), ((2, 2, 16), (33, 130))])
+def test_fused_block_equals_unfused(cfg, hw):
+    """Fused residual block (tensor-core accumulation of the three dy partials in TMEM, bias-seeded) vs the two
+    separate rolling convs: same math, different fp32 summation order -> u8 frames within 1 LSB, and both within
+    the oracle bar."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=12)
+    lr = torch.from_numpy(synth_frames(2, hw[0], hw[1], seed=13)).cuda()
+    a = ctx.infer(lr, "serve").clone()
+    ctx.set_fusion(False)
+    b = ctx.infer(lr, "serve")
+    torch.cuda.synchronize()
+    assert (a.int() - b.int()).abs().max().item() <= 1
+    ref = O.infer_u8(ctx.get_params("serve"), lr.cpu().numpy(), s, B, C)
+    _check_frames(a.cpu().numpy(), ref)
+    _check_frames(b.cpu().numpy(), ref)
