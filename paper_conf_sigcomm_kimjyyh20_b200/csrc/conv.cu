@@ -476,7 +476,7 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], done_bar;
   __shared__ uint32_t tmem_base_sh;
-  __shared__ float sdb[8][COUTP];
+  __shared__ float sdb[128 / OCH][COUTP];
 
   const int TW = g.TW, P = g.P, R = g.R;
   const uint32_t xbox = (uint32_t)(R + 2) * CCH * P * 16, ybox = (uint32_t)R * OCH * TW * 16;  // TMA box bytes
@@ -547,32 +547,45 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
     }
     __syncwarp();
   } else {
-    // epilogue warps: bias gradient from the dY tiles while the MMAs run, then drain the accumulators
+    // epilogue warps: bias gradient from the dY tiles while the MMAs run, then drain the accumulators.
+    // Thread et owns 8-channel chunk j = et % OCH and pixel subset grp = et / OCH (fixed order -> deterministic).
     const int et = threadIdx.x - 64;  // 0..127
-    const int c = et % COUTP;
-    const int part = et / COUTP;      // thread groups summing disjoint pixel subsets
-    const int nparts = 128 / COUTP;
-    float dbsum = 0.f;
+    constexpr int NG = 128 / OCH;
+    const int j = et % OCH, grp = et / OCH;
+    float acc8[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc8[e] = 0.f;
     int s = 0;
     uint32_t ph = 0;
     for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
       mbar_wait(&full_bar[s], ph);
-      if (part < nparts) {
-        const bf16* yt = reinterpret_cast<const bf16*>(smem + s * stage_bytes + xbytes);
-        for (int q = part; q < R * TW; q += nparts) {
-          const int r = q / TW, p = q - r * TW;
-          dbsum += __bfloat162float(yt[((size_t)(r * OCH + c / 8) * TW + p) * 8 + (c % 8)]);
+      if (grp < NG) {
+        const uint8_t* yt = smem + s * stage_bytes + xbytes;
+        for (int r = 0; r < R; ++r) {
+          for (int p = grp; p < TW; p += NG) {
+            const uint4 q = *reinterpret_cast<const uint4*>(yt + ((size_t)(r * OCH + j) * TW + p) * 16);
+            const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float2 f2 = __bfloat1622float2(h2[e]);
+              acc8[2 * e] += f2.x;
+              acc8[2 * e + 1] += f2.y;
+            }
+          }
         }
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
       if (et == 0) mbar_arrive(&empty_bar[s]);
       if (++s == kStages) { s = 0; ph ^= 1; }
     }
-    if (part < nparts) sdb[part][c] = dbsum;
+    if (grp < NG) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) sdb[grp][j * 8 + e] = acc8[e];
+    }
     asm volatile("bar.sync 1, 128;" ::: "memory");
     if (et < COUTP) {
       float t = 0.f;
-      for (int p2 = 0; p2 < nparts; ++p2) t += sdb[p2][et];
+      for (int p2 = 0; p2 < NG; ++p2) t += sdb[p2][et];
       ws_b[(size_t)blockIdx.x * COUTP + et] = t;
     }
     // drain: lane m of M-tile mt = row (16*mt + m/8 -> (dy, j)), ci = 8 j + m % 8

@@ -31,6 +31,7 @@
 #include "ptx.cuh"
 #include "tmap.h"
 #include "sr_internal.h"
+#include "ring.cuh"
 
 namespace sr {
 
@@ -52,57 +53,6 @@ struct BlkCfg {
   static constexpr size_t SMEM = 1024 + 2 * WB_AL + (size_t)kBlkNF * ROWB + (size_t)kBlkNT * ROWB +
                                  (size_t)kBlkNO * OUTB;
 };
-
-// One rolling dy-fold step of a conv: A = input row in smem (chunk-planar, pitch 130), B = dy-fold weights.
-// g = global out-row index of the dy = 2 target (the row this step completes).
-template <int C>
-__device__ __forceinline__ void blk_mma_step(uint32_t ring_base, long long g, uint64_t ad, uint64_t bd) {
-  using Cfg = BlkCfg<C>;
-  constexpr int RB = Cfg::RB, CCH = Cfg::CCH, KS = Cfg::KS;
-  constexpr uint32_t PLANE = Cfg::PLANE;
-  const int i0 = ring_idx<RB>(g);
-  // (column block, first B row, N) of up to two groups
-  int blkA, rowA, nA, blkB = 0, rowB = 0, nB = 0;
-  if (i0 >= 2) { blkA = i0 - 2; rowA = 0; nA = 3 * C; }
-  else if (i0 == 0) { blkA = RB - 2; rowA = 0; nA = 2 * C; blkB = 0; rowB = 2 * C; nB = C; }
-  else { blkA = RB - 1; rowA = 0; nA = C; blkB = 0; rowB = C; nB = 2 * C; }
-  const uint32_t idA = make_idesc(128, nA, 0, 0);
-#pragma unroll
-  for (int dx = 0; dx < 3; ++dx)
-#pragma unroll
-    for (int ks = 0; ks < KS; ++ks)
-      mma_bf16_ss(ring_base + blkA * C, desc_add(ad, dx * 16u + ks * 2u * PLANE),
-                  desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * Cfg::N * 16u + rowA * 16u), idA, 1u);
-  if (nB) {
-    const uint32_t idB = make_idesc(128, nB, 0, 0);
-#pragma unroll
-    for (int dx = 0; dx < 3; ++dx)
-#pragma unroll
-      for (int ks = 0; ks < KS; ++ks)
-        mma_bf16_ss(ring_base + blkB * C, desc_add(ad, dx * 16u + ks * 2u * PLANE),
-                    desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * Cfg::N * 16u + rowB * 16u), idB, 1u);
-  }
-}
-
-// Epilogue helper: load the C accumulator columns of a ring block (this thread's lane) and re-arm the block with
-// the bias (the next row that lands in it starts from b).
-template <int C>
-__device__ __forceinline__ void blk_drain(uint32_t taddr, float* v, const float4* sbias) {
-#pragma unroll
-  for (int c0 = 0; c0 < C; c0 += 16) tmem_ld16(taddr + c0, v + c0);
-  tmem_ld_wait();
-#pragma unroll
-  for (int c0 = 0; c0 < C; c0 += 16) {
-    float b[16];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const float4 t = sbias[c0 / 4 + q];
-      b[4 * q] = t.x; b[4 * q + 1] = t.y; b[4 * q + 2] = t.z; b[4 * q + 3] = t.w;
-    }
-    tmem_st16(taddr + c0, b);
-  }
-  tmem_st_wait();
-}
 
 template <int C>
 __global__ void __launch_bounds__(kBlkThreads, 1)
@@ -212,7 +162,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           mbar_wait(&f_full[fs], fph);
           SR_DBG(9, st)
           tc_fence_after();
-          blk_mma_step<C>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1);
+          ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, PLANE);
           mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
           mma_commit(&f_empty[fs]);
           if (st == n_f - 1) {                      // the last two rows of the piece receive nothing more
@@ -231,7 +181,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           mbar_wait(&t_full[ts], tph);
           SR_DBG(12, st)
           tc_fence_after();
-          blk_mma_step<C>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2);
+          ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, PLANE);
           mma_commit(&r2_ready[ring_idx<RB>(g)]);
           mma_commit(&t_empty[ts]);
           if (k == n_t - 1) {
@@ -255,7 +205,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     {  // arm every ring block with b1
       float v[C];
       for (int b = 0; b < RB; ++b) {
-        blk_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+        ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
         tc_fence_before();
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&r1_free[b]);
@@ -278,7 +228,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       tc_fence_after();
       if (warp == 2 && lane_id() == 0) { SR_DBG(3, q + 1) }
       float v[C];
-      blk_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+      ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
       tc_fence_before();
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&r1_free[b]);
@@ -314,7 +264,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     {
       float v[C];
       for (int b = 0; b < RB; ++b) {
-        blk_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+        ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
         tc_fence_before();
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&r2_free[b]);
@@ -339,7 +289,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       tc_fence_after();
       if (warp == 6 && lane_id() == 0) { SR_DBG(5, q + 1) }
       float v[C];
-      blk_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+      ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
       tc_fence_before();
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&r2_free[b]);

@@ -1,306 +1,362 @@
-// Forward 3x3 conv for wide frames, "rolling dy-fold" form (sm_100a tcgen05).
+// One 3x3 conv over wide images, rolling dy-fold form with tensor-core accumulation in a TMEM ring (sm_100a).
 //
-// Why: with N = Cout = 32/48 a tcgen05.mma (M=128, K=16, both operands in smem) is limited by the 128 B/clk
+// Why: with N = Cout = 32/48 a tcgen05.mma (M=128, K=16, operands in smem) is limited by the 128 B/clk
 // shared-memory read port: A (4 KB) + B (1.5 KB) per MMA -> 44.6 cycles instead of the 24-cycle tensor floor
-// (measured, scripts/mma_rate.py).  Folding the three vertical taps into N (N = 3 Cout = 144 at C = 48) keeps
-// A traffic the same while tripling the work per MMA: 72 cycles at the floor, 121 B/clk of smem.
+// (measured, scripts/mma_rate.py).  Folding the three vertical taps into N (N = 3 Cout) keeps A traffic the same
+// while tripling the work per MMA (72 cycles at the floor for N = 144).  The three dy partials of an output row are
+// summed by the tensor core itself: each output row owns a bias-armed block of a TMEM ring (ring.cuh).
 //
-//   For every input row i of a column strip (one 128-pixel segment + 1-pixel halo, TMA-loaded once):
-//     E_i[x, (dy, co)] = sum_{dx, ci} in[i, x + dx - 1, ci] * W[co, ci, dy, dx]      (3 dx x Cin/16 MMAs, N = 3 Cout)
-//   and the output row r needs the dy-blocks of three consecutive E at the SAME lane x:
-//     out[r, x, co] = E_{r-1}[x, (0, co)] + E_r[x, (1, co)] + E_{r+1}[x, (2, co)]   (+ bias, + residual, ReLU)
-//   (out[y,x] = b + sum_{ky,kx,ci} W[co,ci,ky,kx] in[y+ky-1, x+kx-1, ci]: with i = y + ky - 1, ky = dy.)
-//   The epilogue keeps the two partial output rows in registers, so every E_i is drained once and its TMEM
-//   slot recycled immediately.  Each CTA takes a contiguous range of (column strip, row) work so all CTAs get
-//   the same number of rows; input rows are read once per strip piece (+2 halo rows per piece).
+//   out[y, x, co] = b[co] + sum_{ky,kx,ci} W[co,ci,ky,kx] in[y+ky-1, x+kx-1, ci]            (zero padding)
+//   step for input row i:  block(i+1) += in_i (x) Wo[dy=0],  block(i) += .. [dy=1],  block(i-1) += .. [dy=2]
 //
-// Warp roles (320 threads): warp 0 TMA producer (input rows, residual rows), warp 1 TMEM alloc + MMA issuer,
-// warps 2..9 epilogue (group g = channels [g*Cout/2, (g+1)*Cout/2)); output rows leave through smem + TMA store.
+// Epilogue (per finished row): optional ReLU, + res1 + res2, x 1[mask > 0] (ReLU' for the data gradient), and
+// zero-forced "separator" columns (col % sep in {0, sep-1}) for the virtual wide training batch.
+// Each CTA takes a contiguous range of (column strip, row) work (equal rows per CTA); input rows are read once
+// per strip piece (+2 halo rows per piece).  Strips are 128 output pixels (= MMA M).
+//
+// Warp roles (352 threads): warp 0 TMA producer, warp 1 TMEM alloc + MMA issuer, warps 2..9 epilogue in two groups
+// of 4 that take alternate output rows (all channels) and hand finished rows to warp 10, which issues the TMA
+// stores.  The per-row epilogue chain (drain, re-arm, residual, stage) is latency-bound: two rows in flight and no
+// barrier or store wait on it.
 #include <cuda.h>
 #include "ptx.cuh"
+#include "ring.cuh"
 #include "tmap.h"
 #include "sr_internal.h"
+#include "kernels.h"
 
 namespace sr {
 
-static constexpr int kRollThreads = 320;
-static constexpr int kRollIn = 6;    // input-row ring slots
-static constexpr int kRollRes = 4;   // residual-row ring slots
+static constexpr int kRollThreads = 352;  // + warp 10: TMA-store warp
+static constexpr int kRollNO = 3;    // output staging rows per epilogue group
 static constexpr int kRollTW = 128;  // output pixels per strip (= MMA M)
 
-template <int COUTP>
+template <int CINP, int COUTP>
 struct RollCfg {
-  static constexpr int N = 3 * COUTP;
-  static constexpr int ESTRIDE = ((N + 31) / 32) * 32;
-  static constexpr int NE = (512 / ESTRIDE) < 4 ? (512 / ESTRIDE) : 4;
-  static constexpr uint32_t TMEM_COLS = 512;
-  static constexpr int HALF = COUTP / 2;
+  static constexpr int RB = (512 / COUTP) < 8 ? (512 / COUTP) : 8;
+  static constexpr uint32_t WBYTES = 9u * CINP * COUTP * 2u;
+  static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
+  static constexpr uint32_t PLANE = (kRollTW + 2) * 16;
+  static constexpr uint32_t IN_BOX = (CINP / 8) * PLANE;
+  static constexpr uint32_t IN_STRIDE = (IN_BOX + 1023u) & ~1023u;
+  static constexpr uint32_t ROWB = ((kRollTW * COUTP * 2) + 1023u) & ~1023u;
+  static constexpr int NAUX = 4;  // residual / mask rows (TMA)
+  static constexpr size_t BASE = 1024 + WB_AL + (size_t)2 * kRollNO * ROWB + (size_t)NAUX * ROWB;
+  static constexpr int NIN = (BASE + 4 * IN_STRIDE <= 227 * 1024) ? 4 : 3;  // input-row ring slots
+  static constexpr size_t SMEM = BASE + (size_t)NIN * IN_STRIDE;
 };
 
-size_t roll_smem(int cinp, int coutp) {
-  size_t w = (size_t)9 * cinp * coutp * 2;
-  size_t in = ((size_t)(cinp / 8) * (kRollTW + 2) * 16 + 1023) / 1024 * 1024;
-  size_t row = ((size_t)kRollTW * coutp * 2 + 1023) / 1024 * 1024;
-  return 1024 + ((w + 1023) / 1024 * 1024) + kRollIn * in + kRollRes * row + 3 * row;
-}
+struct RollArgs {
+  const float* bias;
+  const bf16* res1;
+  const bf16* res2;
+  const bf16* mask;
+  int relu;
+  int sep;  // > 0: output columns with col % sep in {0, sep-1} are forced to 0
+  int N, H, W;
+  long long* dbg;  // benchmarking only: CTA-0 clock64 stamps [event][step]
+};
+#define SR_RDBG(ev, idx) \
+  if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
 
-template <int HALF>
-__device__ __forceinline__ void tmem_ld_half(uint32_t taddr, float* v) {
-  static_assert(HALF % 8 == 0, "channel half must be a multiple of 8");
-  int c = 0;
+template <int CH>
+__device__ __forceinline__ void ld_row(const bf16* base, uint4* dst) {
+  const uint4* p = reinterpret_cast<const uint4*>(base);
 #pragma unroll
-  for (; c + 16 <= HALF; c += 16) tmem_ld16(taddr + c, v + c);
-  if (HALF % 16) tmem_ld8(taddr + c, v + c);
+  for (int q = 0; q < CH / 8; ++q) dst[q] = __ldg(p + q);
 }
 
 template <int CINP, int COUTP>
 __global__ void __launch_bounds__(kRollThreads, 1)
-k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_res,
-            const __grid_constant__ CUtensorMap tm_out, const bf16* __restrict__ wfold, const int N, const int H,
-            const int W, const float* __restrict__ bias, const int relu, const int has_res) {
-  using Cfg = RollCfg<COUTP>;
-  constexpr int CCH = CINP / 8, KS = CINP / 16, HALF = Cfg::HALF, NE = Cfg::NE, ESTRIDE = Cfg::ESTRIDE;
-  constexpr uint32_t WBYTES = 9u * CINP * COUTP * 2u;
-  constexpr uint32_t PLANE = (kRollTW + 2) * 16;                  // one 8-channel chunk of an input row
-  constexpr uint32_t IN_BOX = CCH * PLANE;
-  constexpr uint32_t IN_STRIDE = (IN_BOX + 1023u) & ~1023u;
-  constexpr uint32_t ROW_BOX = kRollTW * COUTP * 2;
-  constexpr uint32_t ROW_STRIDE = (ROW_BOX + 1023u) & ~1023u;
-  constexpr uint32_t IDESC = make_idesc(128, Cfg::N, 0, 0);
+k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
+            const __grid_constant__ CUtensorMap tm_aux, const bf16* __restrict__ wfold, const RollArgs a) {
+  using Cfg = RollCfg<CINP, COUTP>;
+  constexpr int RB = Cfg::RB, kRollIn = Cfg::NIN, NAUX = Cfg::NAUX;
+  constexpr uint32_t PLANE = Cfg::PLANE, IN_STRIDE = Cfg::IN_STRIDE, ROWB = Cfg::ROWB;
 
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sW = smem;
-  uint8_t* sIn = sW + ((WBYTES + 1023u) & ~1023u);
-  uint8_t* sRes = sIn + kRollIn * IN_STRIDE;
-  uint8_t* sOut = sRes + kRollRes * ROW_STRIDE;  // 3 x [128 px][COUTP] staging rows for the TMA store
-  __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], res_full[kRollRes], res_empty[kRollRes],
-      e_full[NE], e_empty[NE], w_bar;
+  uint8_t* sIn = sW + Cfg::WB_AL;
+  uint8_t* sO = sIn + kRollIn * IN_STRIDE;
+  uint8_t* sA = sO + 2 * kRollNO * ROWB;
+  __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
+      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar;
+  // the aux row (res1 or mask) travels by TMA; res2 (used once per backward pass) by plain loads
+  const bool has_aux = a.res1 != nullptr || a.mask != nullptr;
   __shared__ uint32_t tmem_base_sh;
+  __shared__ __align__(16) float4 sbv[COUTP / 4];
 
+  const int N = a.N, H = a.H, W = a.W;
   const int warp = warp_id();
+  if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
   if (warp == 0 && lane_id() == 0) {
     for (int s = 0; s < kRollIn; ++s) { mbar_init(&in_full[s], 1); mbar_init(&in_empty[s], 1); }
-    for (int s = 0; s < kRollRes; ++s) { mbar_init(&res_full[s], 1); mbar_init(&res_empty[s], 8); }
-    for (int s = 0; s < NE; ++s) { mbar_init(&e_full[s], 1); mbar_init(&e_empty[s], 8); }
+    for (int s = 0; s < RB; ++s) { mbar_init(&r_ready[s], 1); mbar_init(&r_free[s], 4); }
+    for (int s = 0; s < NAUX; ++s) { mbar_init(&x_full[s], 1); mbar_init(&x_empty[s], 4); }
+    for (int s = 0; s < 2 * kRollNO; ++s) { mbar_init(&o_full[s], 4); mbar_init(&o_free[s], 1); }
     mbar_init(&w_bar, 1);
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(&tmem_base_sh);
+  if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
 
-  // balanced contiguous range of (column strip, row) work for this CTA
   const int tiles_x = (W + kRollTW - 1) / kRollTW;
   const long long total = (long long)N * tiles_x * H;
   const long long beg = total * blockIdx.x / gridDim.x, end = total * (blockIdx.x + 1) / gridDim.x;
+#define SR_PIECE_BEGIN                                                                \
+  for (long long pos = beg; pos < end;) {                                             \
+    const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);             \
+    const int y1 = (int)min((long long)H, y0 + (end - pos));                          \
+    pos += y1 - y0;                                                                   \
+    const int n = col / tiles_x, x0 = (col - n * tiles_x) * kRollTW;                  \
+    const int n_in = y1 - y0 + 2;                                                     \
+    (void)n; (void)x0;
+#define SR_PIECE_END }
 
   if (warp == 0) {
-    // ===================== TMA producer =====================
+    // ===================== TMA producer: weights, then input rows y0-1 .. y1 of each piece =====================
     if (elect_one()) {
       tma_prefetch_desc(&tm_in);
-      if (has_res) tma_prefetch_desc(&tm_res);
-      mbar_arrive_expect_tx(&w_bar, WBYTES);
-      bulk_load(sW, wfold, WBYTES, &w_bar);
-      int s = 0, rs = 0;
-      uint32_t ph = 0, rph = 0;
-      for (long long pos = beg; pos < end;) {
-        const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);
-        const int y1 = (int)min((long long)H, y0 + (end - pos));
-        pos += y1 - y0;
-        const int n = col / tiles_x, x0 = (col - n * tiles_x) * kRollTW;
-        const int n_in = y1 - y0 + 2;
-        for (int i = 0; i < n_in; ++i) {
-          mbar_wait(&in_empty[s], ph ^ 1);
-          mbar_arrive_expect_tx(&in_full[s], IN_BOX);
-          tma_load_5d(sIn + s * IN_STRIDE, &tm_in, &in_full[s], 0, x0 - 1, y0 - 1 + i, 0, n);
-          if (++s == kRollIn) { s = 0; ph ^= 1; }
-          if (has_res && i >= 1 && i - 1 < y1 - y0) {  // residual of output row y0+i-1, consumed at step i+1
-            mbar_wait(&res_empty[rs], rph ^ 1);
-            mbar_arrive_expect_tx(&res_full[rs], ROW_BOX);
-            tma_load_4d(sRes + rs * ROW_STRIDE, &tm_res, &res_full[rs], 0, x0, y0 + i - 1, n);
-            if (++rs == kRollRes) { rs = 0; rph ^= 1; }
-          }
+      mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
+      bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
+      int s = 0, xs = 0;
+      uint32_t ph = 0, xph = 0;
+      SR_PIECE_BEGIN
+      for (int i = 0; i < n_in; ++i) {
+        mbar_wait(&in_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&in_full[s], Cfg::IN_BOX);
+        tma_load_5d(sIn + s * IN_STRIDE, &tm_in, &in_full[s], 0, x0 - 1, y0 - 1 + i, 0, n);
+        SR_RDBG(0, i)
+        if (++s == kRollIn) { s = 0; ph ^= 1; }
+        if (has_aux && i >= 1 && i - 1 < y1 - y0) {  // aux row of output row y0+i-1 (needed after input row y0+i)
+          mbar_wait(&x_empty[xs], xph ^ 1);
+          mbar_arrive_expect_tx(&x_full[xs], kRollTW * COUTP * 2);
+          tma_load_4d(sA + xs * ROWB, &tm_aux, &x_full[xs], 0, x0, y0 + i - 1, n);
+          if (++xs == NAUX) { xs = 0; xph ^= 1; }
         }
       }
+      SR_PIECE_END
     }
     __syncwarp();
   } else if (warp == 1) {
     // ===================== MMA issuer =====================
     if (elect_one()) {
       mbar_wait(&w_bar, 0);
-      const uint64_t bdesc0 = make_desc(smem_u32(sW), Cfg::N * 16, 128);
-      int s = 0, es = 0;
-      uint32_t ph = 0, eph = 0;
-      for (long long pos = beg; pos < end;) {
-        const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);
-        const int y1 = (int)min((long long)H, y0 + (end - pos));
-        pos += y1 - y0;
-        (void)col;
-        const int n_in = y1 - y0 + 2;
-        for (int i = 0; i < n_in; ++i) {
-          mbar_wait(&in_full[s], ph);
-          mbar_wait(&e_empty[es], eph ^ 1);
-          tc_fence_after();
-          const uint64_t adesc0 = make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128);
-          const uint32_t d = tmem + es * ESTRIDE;
-#pragma unroll
-          for (int dx = 0; dx < 3; ++dx) {
-#pragma unroll
-            for (int ks = 0; ks < KS; ++ks) {
-              mma_bf16_ss(d, desc_add(adesc0, dx * 16u + ks * 2u * PLANE),
-                          desc_add(bdesc0, (uint32_t)(dx * CCH + 2 * ks) * Cfg::N * 16u), IDESC, (dx | ks) != 0);
-            }
-          }
-          mma_commit(&e_full[es]);
-          mma_commit(&in_empty[s]);
-          if (++s == kRollIn) { s = 0; ph ^= 1; }
-          if (++es == NE) { es = 0; eph ^= 1; }
+      const uint64_t bd = make_desc(smem_u32(sW), 3 * COUTP * 16, 128);
+      int s = 0;
+      uint32_t ph = 0;
+      long long G = 0, acq = 0;
+      SR_PIECE_BEGIN
+      for (int i = 0; i < n_in; ++i) {
+        const long long g = G + i;  // out row completed by this step (dy = 2 target)
+        SR_RDBG(1, i)
+        for (; acq < g + 3; ++acq) mbar_wait(&r_free[ring_idx<RB>(acq)], (uint32_t)(acq / RB) & 1u);
+        SR_RDBG(2, i)
+        mbar_wait(&in_full[s], ph);
+        SR_RDBG(3, i)
+        tc_fence_after();
+        ring_mma_step<CINP, COUTP, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, PLANE);
+        mma_commit(&r_ready[ring_idx<RB>(g)]);
+        mma_commit(&in_empty[s]);
+        SR_RDBG(4, i)
+        if (i == n_in - 1) {
+          mma_commit(&r_ready[ring_idx<RB>(g + 1)]);
+          mma_commit(&r_ready[ring_idx<RB>(g + 2)]);
         }
+        if (++s == kRollIn) { s = 0; ph ^= 1; }
       }
+      G += n_in + 2;
+      SR_PIECE_END
+    }
+    __syncwarp();
+  } else if (warp == 10) {
+    // ===================== store warp: TMA-store finished rows in emission order =====================
+    if (elect_one()) {
+      tma_prefetch_desc(&tm_out);
+      int os[2] = {0, 0};
+      uint32_t oph[2] = {0, 0};
+      int pend_b = -1;  // staging slot (global index) of the previously issued store
+      long long G = 0;
+      SR_PIECE_BEGIN
+      for (int q = 1; q <= n_in - 2; ++q) {
+        const long long g = G + q + 1;
+        const int grp = (int)(g & 1);
+        const int b = grp * kRollNO + os[grp];
+        mbar_wait(&o_full[b], oph[grp]);
+        tma_store_4d(&tm_out, sO + b * ROWB, 0, x0, y0 - 1 + q, n);
+        bulk_commit();
+        bulk_wait_read<1>();        // the previous store has read its staging row
+        if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
+        pend_b = b;
+        if (++os[grp] == kRollNO) { os[grp] = 0; oph[grp] ^= 1; }
+      }
+      G += n_in + 2;
+      SR_PIECE_END
+      bulk_wait<0>();
     }
     __syncwarp();
   } else {
-    // ===================== epilogue: 2 groups x 4 warps, group g owns channels [g*HALF, (g+1)*HALF) ==========
+    // ===================== epilogue: 2 groups x 4 warps, group g drains the rows with sequence index % 2 == g ======
     const int quarter = warp & 3;
     const int grp = (warp - 2) >> 2;
-    const int px = quarter * 32 + lane_id();
-    const int c0 = grp * HALF;
-    const bool leader = (warp == 2 && lane_id() == 0);
-    float bv[HALF];
+    const int m = quarter * 32 + lane_id();
+    const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+    uint8_t* stage = sO + grp * kRollNO * ROWB;
+    uint32_t ophase = 0;
+    for (int b = grp; b < RB; b += 2) {  // arm this group's ring blocks with the bias (RB is even)
+      float v[COUTP];
+      ring_drain<COUTP>(tmem + lane_off + b * COUTP, v, sbv);
+      tc_fence_before();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&r_free[b]);
+    }
+    int os = 0;
+    long long G = 0, emitted = 0;  // emitted: output rows of both groups so far (aux ring order)
+    SR_PIECE_BEGIN
+    const int xc = x0 + m;
+    const bool lane_ok = xc < W;
+    const bool sep0 = a.sep > 0 && ((xc % a.sep) == 0 || (xc % a.sep) == a.sep - 1);
+    for (int q = -1; q <= n_in; ++q) {
+      const long long g = G + q + 1;
+      const bool emit = q >= 1 && q <= n_in - 2;
+      const long long xi = emitted;  // aux ring index of this row (if emitted)
+      emitted += emit;
+      if ((int)(g & 1) != grp) continue;
+      const int r = y0 - 1 + q;
+      const size_t pix = (((size_t)n * H + r) * W) + xc;
+      uint4 r2[COUTP / 8];
+      if (emit && lane_ok && a.res2) ld_row<COUTP>(a.res2 + pix * COUTP, r2);
+      const int b = ring_idx<RB>(g);
+      mbar_wait(&r_ready[b], (uint32_t)(g / RB) & 1u);
+      tc_fence_after();
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(5, q + 1) }
+      float v[COUTP];
+      ring_drain<COUTP>(tmem + lane_off + b * COUTP, v, sbv);
+      tc_fence_before();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&r_free[b]);
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(6, q + 1) }
+      if (!emit) continue;
+      const uint4* aux = reinterpret_cast<const uint4*>(sA + (int)(xi % NAUX) * ROWB + m * COUTP * 2);
+      if (has_aux) mbar_wait(&x_full[xi % NAUX], (uint32_t)(xi / NAUX) & 1u);
+      mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);  // the store warp has read this staging row
+      if (lane_ok) {
+        uint4* orow = reinterpret_cast<uint4*>(stage + os * ROWB + m * COUTP * 2);
 #pragma unroll
-    for (int c = 0; c < HALF; ++c) bv[c] = bias ? __ldg(bias + c0 + c) : 0.f;
-    int es = 0, rs = 0, os = 0;
-    uint32_t eph = 0, rph = 0;
-    float pa[HALF], pb[HALF];  // partial sums of output rows i-1 and i (relative to input row i)
-    for (long long pos = beg; pos < end;) {
-      const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);
-      const int y1 = (int)min((long long)H, y0 + (end - pos));
-      pos += y1 - y0;
-      const int n = col / tiles_x, x0 = (col - n * tiles_x) * kRollTW;
-      const int n_in = y1 - y0 + 2;
-      for (int i = 0; i < n_in; ++i) {
-        float e0[HALF], e1[HALF], e2[HALF];
-        mbar_wait(&e_full[es], eph);
-        tc_fence_after();
-        const uint32_t ta = tmem + ((uint32_t)(quarter * 32) << 16) + es * ESTRIDE + c0;
-        tmem_ld_half<HALF>(ta, e0);
-        tmem_ld_half<HALF>(ta + COUTP, e1);
-        tmem_ld_half<HALF>(ta + 2 * COUTP, e2);
-        tmem_ld_wait();
-        tc_fence_before();
-        __syncwarp();
-        if (lane_id() == 0) mbar_arrive(&e_empty[es]);
-        if (++es == NE) { es = 0; eph ^= 1; }
-        if (i >= 2) {
-          // output row r = y0 + i - 2 is complete: pa + E_i dy=2 block
-          const int r = y0 + i - 2;
-          float v[HALF];
+        for (int j = 0; j < COUTP / 8; ++j) {
+          float o[8];
 #pragma unroll
-          for (int c = 0; c < HALF; ++c) v[c] = pa[c] + e2[c] + bv[c];
-          if (has_res) {
-            mbar_wait(&res_full[rs], rph);
-            const uint4* rr = reinterpret_cast<const uint4*>(sRes + rs * ROW_STRIDE + (px * COUTP + c0) * 2);
+          for (int e = 0; e < 8; ++e) o[e] = v[8 * j + e];
+          if (a.res1) {
+            const uint4 t = aux[j];
+            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
 #pragma unroll
-            for (int q = 0; q < HALF / 8; ++q) {
-              uint4 u = rr[q];
-              const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&u);
+            for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
+          }
+          if (a.res2) {
+            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&r2[j]);
 #pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                float2 f = __bfloat1622float2(h2[j]);
-                v[8 * q + 2 * j] += f.x;
-                v[8 * q + 2 * j + 1] += f.y;
-              }
+            for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
+          }
+          if (a.relu) {
+#pragma unroll
+            for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
+          }
+          if (a.mask) {
+            const uint4 t = aux[j];
+            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float2 f = __bfloat1622float2(h[e]);
+              o[2 * e] = f.x > 0.f ? o[2 * e] : 0.f;
+              o[2 * e + 1] = f.y > 0.f ? o[2 * e + 1] : 0.f;
             }
-            __syncwarp();
-            if (lane_id() == 0) mbar_arrive(&res_empty[rs]);
-            if (++rs == kRollRes) { rs = 0; rph ^= 1; }
           }
-          if (relu) {
+          if (sep0) {
 #pragma unroll
-            for (int c = 0; c < HALF; ++c) v[c] = fmaxf(v[c], 0.f);
+            for (int e = 0; e < 8; ++e) o[e] = 0.f;
           }
-          // stage the row in smem (3 buffers), one barrier, one thread TMA-stores it (clipped at the frame edge).
-          // Buffer k%3 was last read by the store of row k-3, which the leader waited for (wait_read<1> after
-          // issuing row k-2's store) before it reached the barrier of row k-1.
-          uint4* orow = reinterpret_cast<uint4*>(sOut + os * ROW_STRIDE + (px * COUTP + c0) * 2);
-#pragma unroll
-          for (int q = 0; q < HALF / 8; ++q) {
-            uint4 u;
-            u.x = pack_bf16x2(v[8 * q + 0], v[8 * q + 1]);
-            u.y = pack_bf16x2(v[8 * q + 2], v[8 * q + 3]);
-            u.z = pack_bf16x2(v[8 * q + 4], v[8 * q + 5]);
-            u.w = pack_bf16x2(v[8 * q + 6], v[8 * q + 7]);
-            orow[q] = u;
-          }
-          fence_proxy_async_smem();
-          named_bar_sync(1, 256);
-          if (leader) {
-            tma_store_4d(&tm_out, sOut + os * ROW_STRIDE, 0, x0, r, n);
-            bulk_commit();
-            bulk_wait_read<1>();
-          }
-          os = os == 2 ? 0 : os + 1;
-        }
-#pragma unroll
-        for (int c = 0; c < HALF; ++c) {
-          pa[c] = pb[c] + e1[c];
-          pb[c] = e0[c];
+          uint4 u;
+          u.x = pack_bf16x2(o[0], o[1]);
+          u.y = pack_bf16x2(o[2], o[3]);
+          u.z = pack_bf16x2(o[4], o[5]);
+          u.w = pack_bf16x2(o[6], o[7]);
+          orow[j] = u;
         }
       }
+      if (has_aux) {
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&x_empty[xi % NAUX]);
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&o_full[grp * kRollNO + os]);
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(7, q + 1) }
+      if (++os == kRollNO) { os = 0; ophase ^= 1; }
     }
-    if (leader) bulk_wait<0>();
+    G += n_in + 2;
+    SR_PIECE_END
   }
+#undef SR_PIECE_BEGIN
+#undef SR_PIECE_END
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) tmem_dealloc<RollCfg<COUTP>::TMEM_COLS>(tmem);
+  if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
 template <int CINP, int COUTP>
-static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& tr, const CUtensorMap& to,
-                                 const bf16* wfold, int N, int H, int W, const float* bias, int relu, int has_res,
-                                 int grid, cudaStream_t st) {
+static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, const CUtensorMap& tx,
+                                 const bf16* wfold, const RollArgs& a, int grid, cudaStream_t st) {
   auto kern = k_conv_roll<CINP, COUTP>;
-  const size_t smem = roll_smem(CINP, COUTP);
+  constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
   static bool configured = false;
   if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     configured = true;
   }
-  kern<<<grid, kRollThreads, smem, st>>>(ti, tr, to, wfold, N, H, W, bias, relu, has_res);
+  kern<<<grid, kRollThreads, smem, st>>>(ti, to, tx, wfold, a);
   return cudaGetLastError();
 }
 
+static bool ch_ok(int c) { return c == 16 || c == 32 || c == 48 || c == 64; }
+
 bool roll_supported(int cinp, int coutp, int W) {
-  if (W < 96) return false;
-  const bool ci = cinp == 16 || cinp == 32 || cinp == 48 || cinp == 64;
-  const bool co = coutp == 16 || coutp == 32 || coutp == 48 || coutp == 64;
-  return ci && co && roll_smem(cinp, coutp) <= 227 * 1024;
+  return W >= 96 && ch_ok(cinp) && (coutp == 16 || coutp == 32 || coutp == 48);
 }
 
 #define SR_ROLL_CASE(CI, CO) \
-  if (cinp == CI && coutp == CO) return launch_roll_t<CI, CO>(ti, tr, to, wfold, N, H, W, bias, relu, has_res, grid, st);
+  if (cinp == CI && coutp == CO) return launch_roll_t<CI, CO>(ti, to, tx, wfold, a, grid, st);
 
-cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
-                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st) {
-  CUtensorMap ti, tr, to;
+cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
+                                const bf16* res1, const bf16* res2, const bf16* mask, int relu, int sep, bf16* out,
+                                int N, int H, int W, cudaStream_t st, long long* dbg) {
+  CUtensorMap ti, to;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
   if (make_row_tmap(&to, out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  if (make_row_tmap(&tr, res ? (const void*)res : (const void*)out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
-  const int has_res = res != nullptr;
+  CUtensorMap tx;
+  const void* auxp = res1 ? (const void*)res1 : (mask ? (const void*)mask : (const void*)out);
+  if (make_row_tmap(&tx, auxp, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (res1 && mask) return cudaErrorNotSupported;  // one TMA aux stream per launch
+  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
-  SR_ROLL_CASE(16, 16) SR_ROLL_CASE(16, 32) SR_ROLL_CASE(16, 48) SR_ROLL_CASE(16, 64)
-  SR_ROLL_CASE(32, 16) SR_ROLL_CASE(32, 32) SR_ROLL_CASE(32, 48) SR_ROLL_CASE(32, 64)
+  SR_ROLL_CASE(16, 16) SR_ROLL_CASE(16, 32) SR_ROLL_CASE(16, 48)
+  SR_ROLL_CASE(32, 16) SR_ROLL_CASE(32, 32) SR_ROLL_CASE(32, 48)
   SR_ROLL_CASE(48, 16) SR_ROLL_CASE(48, 32) SR_ROLL_CASE(48, 48)
-  SR_ROLL_CASE(64, 16) SR_ROLL_CASE(64, 32) SR_ROLL_CASE(64, 64)
+  SR_ROLL_CASE(64, 16) SR_ROLL_CASE(64, 32) SR_ROLL_CASE(64, 48)
   return cudaErrorNotSupported;
+}
+
+cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
+                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st) {
+  return launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res, nullptr, nullptr, relu, 0, out, N, H, W, st);
 }
 
 }  // namespace sr

@@ -226,3 +226,33 @@ extern "C" int sr_bench_resblock(int c, int n, int h, int w, int iters, float* m
   cudaFree(x); cudaFree(y); cudaFree(w1); cudaFree(w2); cudaFree(bias); cudaFree(dbg);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
+
+// Rolling conv on random data with CTA-0 pipeline timestamps [16][256] (benchmarking only).
+extern "C" int sr_bench_roll_dbg(int cinp, int coutp, int n, int h, int w, int res, long long* dbg_host, float* ms_out,
+                                 void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t pix = (size_t)n * h * w;
+  bf16 *x = nullptr, *y = nullptr, *r = nullptr, *wt = nullptr;
+  float* bias = nullptr;
+  long long* dbg = nullptr;
+  if (cudaMalloc(&x, pix * cinp * 2) || cudaMalloc(&y, pix * coutp * 2) || cudaMalloc(&r, pix * coutp * 2) ||
+      cudaMalloc(&wt, 9 * cinp * coutp * 2) || cudaMalloc(&bias, coutp * 4) || cudaMalloc(&dbg, 16 * 256 * 8))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(x, 0x3c, pix * cinp * 2, st);
+  cudaMemsetAsync(r, 0x3c, pix * coutp * 2, st);
+  cudaMemsetAsync(wt, 0x1c, 9 * cinp * coutp * 2, st);
+  cudaMemsetAsync(bias, 0, coutp * 4, st);
+  cudaMemsetAsync(dbg, 0, 16 * 256 * 8, st);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  cudaEventRecord(a, st);
+  cudaError_t e = launch_conv_roll_ex(cinp, coutp, x, wt, bias, res ? r : nullptr, nullptr, nullptr, !res, 0, y, n, h,
+                                      w, st, dbg);
+  cudaEventRecord(b, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  cudaEventElapsedTime(ms_out, a, b);
+  cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
+  cudaFree(x); cudaFree(y); cudaFree(r); cudaFree(wt); cudaFree(bias); cudaFree(dbg);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
