@@ -16,6 +16,7 @@
 #include "tmap.h"
 #include "sr_internal.h"
 #include "kernels.h"
+#include "launch.cuh"
 
 namespace sr {
 
@@ -184,9 +185,11 @@ __device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp)
 // Tail: y = acc + b (3 s^2 channels, index c*s^2 + i*s + j = pixel-shuffle phase (i,j) of colour c);
 // skip = bilinear_s(v) at HR (sY+i, sX+j).  Inference: u8 = RNE(clamp(255 y + skip, 0, 255)).
 // Training: o = y + skip/255, d = o - hr/255 -> loss += d^2, dy[c s^2 + i s + j] = 2 d.
+// (n, Y, X) addresses the LR image / HR target (n-th image of size H x W); dy_pix is the pixel index of this
+// output in the conv's own layout (equal to ((n H + Y) W + X) except for the virtual training batch).
 template <int S, int COUTP, bool TRAIN>
 __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias, int n, int Y, int X, int H,
-                                         int W, float* v, float& lsum) {
+                                         int W, float* v, float& lsum, size_t dy_pix) {
   const uint8_t* lr = ep.lr + (size_t)n * H * W * 3;
   float nb[3][3][3];  // [dy][dx][c] neighbourhood of LR pixel (Y,X), clamped (edge replicate)
 #pragma unroll
@@ -236,7 +239,7 @@ __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias
       }
     }
   }
-  if (TRAIN) store_bf16_row<COUTP>(ep.dy + (((size_t)n * H + Y) * W + X) * COUTP, dyv);
+  if (TRAIN) store_bf16_row<COUTP>(ep.dy + dy_pix * COUTP, dyv);
 }
 
 // ------------------------------------------------------------------------------------------ conv kernel
@@ -267,7 +270,6 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
   uint8_t* sStage = smem + WBYTES;
 
   const int warp = warp_id();
-  if (threadIdx.x < COUTP) sbias[threadIdx.x] = ep.bias ? ep.bias[threadIdx.x] : 0.f;
   if (warp == 0 && lane_id() == 0) {
     for (int s = 0; s < kStages; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
     for (int s = 0; s < NSLOT; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4); }
@@ -276,6 +278,9 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
   }
   if (warp == 1) tmem_alloc<TMEM_COLS>(&tmem_base_sh);
   tc_fence_before();
+  __syncthreads();
+  pdl_enter();
+  if (threadIdx.x < COUTP) sbias[threadIdx.x] = ep.bias ? ep.bias[threadIdx.x] : 0.f;
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
@@ -371,9 +376,23 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
         } else if (EPI == EPI_ACT) {
           epi_act<COUTP>(ep, sbias, pix, v, pre);
         } else if (EPI == EPI_TAIL_U8) {
-          if (Y >= ep.hr_row0 && Y < ep.hr_row1) epi_tail<S, COUTP, false>(ep, sbias, n, Y, X, g.H, g.W, v, lsum);
+          if (Y >= ep.hr_row0 && Y < ep.hr_row1)
+            epi_tail<S, COUTP, false>(ep, sbias, n, Y, X, g.H, g.W, v, lsum, ((size_t)n * g.H + Y) * g.W + X);
         } else {
-          epi_tail<S, COUTP, true>(ep, sbias, n, Y, X, g.H, g.W, v, lsum);
+          const size_t vp = ((size_t)n * g.H + Y) * g.W + X;
+          if (ep.vsep > 0) {  // virtual training batch: patch j at columns [j*vsep + 1, j*vsep + 1 + p)
+            const int j = X / ep.vsep, x = X - j * ep.vsep - 1;
+            if (x < 0 || x >= ep.vp) {  // separator column: no loss, zero gradient
+              float z[COUTP];
+#pragma unroll
+              for (int k = 0; k < COUTP; ++k) z[k] = 0.f;
+              store_bf16_row<COUTP>(ep.dy + vp * COUTP, z);
+            } else {
+              epi_tail<S, COUTP, true>(ep, sbias, j, Y, x, ep.vp, ep.vp, v, lsum, vp);
+            }
+          } else {
+            epi_tail<S, COUTP, true>(ep, sbias, n, Y, X, g.H, g.W, v, lsum, vp);
+          }
         }
       }
     }
@@ -398,8 +417,7 @@ static cudaError_t launch_conv_t(const CUtensorMap& tm, const bf16* wpk, const C
     if (e != cudaSuccess) return e;
     configured = smem;
   }
-  kern<<<grid, kConvThreads, smem, st>>>(tm, wpk, g, ep);
-  return cudaGetLastError();
+  return launch_k(kern, dim3(grid), dim3(kConvThreads), smem, st, tm, wpk, g, ep);
 }
 
 #define SR_CONV_CASE(CI, CO)                                                                 \
@@ -492,6 +510,7 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
   if (warp == 1) tmem_alloc<TMEM_COLS>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
+  pdl_enter();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
   const int tiles_xy = g.tiles_x * g.tiles_y;
@@ -631,8 +650,7 @@ static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, 
     if (e != cudaSuccess) return e;
     configured = smem;
   }
-  kern<<<grid, kWgradThreads, smem, st>>>(tx, ty, g, ws_w, ws_b);
-  return cudaGetLastError();
+  return launch_k(kern, dim3(grid), dim3(kWgradThreads), smem, st, tx, ty, g, ws_w, ws_b);
 }
 
 #define SR_WG_CASE(CI, CO) \
@@ -656,6 +674,7 @@ cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, con
 // SR_BILINEAR "model" (the WebRTC baseline): the tail with y = 0.
 template <int S>
 __global__ void k_bilinear_u8(const uint8_t* __restrict__ lr, int n, int h, int w, uint8_t* __restrict__ hr) {
+  pdl_enter();
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= (long long)n * h * w) return;
   const int X = (int)(i % w);
@@ -669,16 +688,15 @@ __global__ void k_bilinear_u8(const uint8_t* __restrict__ lr, int n, int h, int 
   for (int k = 0; k < 32; ++k) v[k] = 0.f;
   const float zb[32] = {0.f};
   float ls = 0.f;
-  epi_tail<S, 32, false>(ep, zb, img, Y, X, h, w, v, ls);
+  epi_tail<S, 32, false>(ep, zb, img, Y, X, h, w, v, ls, 0);
 }
 
 cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st) {
   long long tot = (long long)n * h * w;
   unsigned blocks = (unsigned)((tot + 255) / 256);
-  if (s == 2) k_bilinear_u8<2><<<blocks, 256, 0, st>>>(lr, n, h, w, hr);
-  else if (s == 3) k_bilinear_u8<3><<<blocks, 256, 0, st>>>(lr, n, h, w, hr);
-  else return cudaErrorNotSupported;
-  return cudaGetLastError();
+  if (s == 2) return launch_k(k_bilinear_u8<2>, dim3(blocks), dim3(256), 0, st, lr, n, h, w, hr);
+  if (s == 3) return launch_k(k_bilinear_u8<3>, dim3(blocks), dim3(256), 0, st, lr, n, h, w, hr);
+  return cudaErrorNotSupported;
 }
 
 }  // namespace sr

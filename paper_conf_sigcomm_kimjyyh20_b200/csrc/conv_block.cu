@@ -32,6 +32,7 @@
 #include "tmap.h"
 #include "sr_internal.h"
 #include "ring.cuh"
+#include "launch.cuh"
 
 namespace sr {
 
@@ -83,10 +84,6 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   __shared__ __align__(16) float4 sb1v[C / 4], sb2v[C / 4];
 
   const int warp = warp_id();
-  if (threadIdx.x < C) {
-    reinterpret_cast<float*>(sb1v)[threadIdx.x] = b1[threadIdx.x];
-    reinterpret_cast<float*>(sb2v)[threadIdx.x] = b2[threadIdx.x];
-  }
   // spare t positions 128, 129 of every plane of every t slot are read by the two invalid conv2 lanes: zero them
   for (int i = threadIdx.x; i < kBlkNT * CCH * 2; i += blockDim.x) {
     const int slot = i / (CCH * 2), rem = i % (CCH * 2);
@@ -105,6 +102,12 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   }
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
+  __syncthreads();
+  pdl_enter();
+  if (threadIdx.x < C) {
+    reinterpret_cast<float*>(sb1v)[threadIdx.x] = b1[threadIdx.x];
+    reinterpret_cast<float*>(sb2v)[threadIdx.x] = b2[threadIdx.x];
+  }
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
@@ -348,8 +351,8 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
     if (e != cudaSuccess) return e;
     configured = true;
   }
-  kern<<<grid, kBlkThreads, BlkCfg<C>::SMEM, st>>>(tf, to, w1, w2, b1, b2, f, out, N, H, W, dbg);
-  return cudaGetLastError();
+  return launch_k(kern, dim3(grid), dim3(kBlkThreads), BlkCfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, out, N, H, W,
+                  dbg);
 }
 
 bool resblock_supported(int cp, int W) {

@@ -24,6 +24,7 @@
 #include "tmap.h"
 #include "sr_internal.h"
 #include "kernels.h"
+#include "launch.cuh"
 
 namespace sr {
 
@@ -89,7 +90,6 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
 
   const int N = a.N, H = a.H, W = a.W;
   const int warp = warp_id();
-  if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
   if (warp == 0 && lane_id() == 0) {
     for (int s = 0; s < kRollIn; ++s) { mbar_init(&in_full[s], 1); mbar_init(&in_empty[s], 1); }
     for (int s = 0; s < RB; ++s) { mbar_init(&r_ready[s], 1); mbar_init(&r_free[s], 4); }
@@ -100,6 +100,9 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   }
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
+  __syncthreads();
+  pdl_enter();  // predecessor complete: global inputs are valid from here on
+  if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
@@ -319,7 +322,7 @@ static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, c
     if (e != cudaSuccess) return e;
     configured = true;
   }
-  kern<<<grid, kRollThreads, smem, st>>>(ti, to, tx, wfold, a);
+  return launch_k(kern, dim3(grid), dim3(kRollThreads), smem, st, ti, to, tx, wfold, a);
   return cudaGetLastError();
 }
 

@@ -3,12 +3,14 @@
 #include "ptx.cuh"
 #include "sr_internal.h"
 #include "kernels.h"
+#include "launch.cuh"
 
 namespace sr {
 
 // --------------------------------------------------------------- head input: u8 RGB -> bf16 [.., 16]
 // x = v / 255 (reading R3), channels 3..15 zero so the head conv runs with K = 9 x 16.
 __global__ void k_pack_input(const uint8_t* __restrict__ lr, size_t npix, uint4* __restrict__ x) {
+  pdl_enter();
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= npix) return;
   const uint8_t* p = lr + i * 3;
@@ -23,16 +25,43 @@ __global__ void k_pack_input(const uint8_t* __restrict__ lr, size_t npix, uint4*
 
 void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st) {
   int th = 256;
-  k_pack_input<<<(unsigned)((npix + th - 1) / th), th, 0, st>>>(lr, npix, reinterpret_cast<uint4*>(x));
+  launch_k(k_pack_input, dim3((unsigned)((npix + th - 1) / th)), dim3(th), 0, st, lr, npix, reinterpret_cast<uint4*>(x));
+}
+
+// Virtual training batch: n patches p x p laid side by side in one p x (n (p+2)) image, patch j at columns
+// [j (p+2) + 1, j (p+2) + 1 + p); the separator columns j (p+2) and j (p+2) + p + 1 are zero and act as every
+// patch's own zero padding for all the 3x3 convs (which re-zero them in their epilogues).
+__global__ void k_pack_input_virtual(const uint8_t* __restrict__ lr, int n, int p, uint4* __restrict__ x) {
+  pdl_enter();
+  const int Wv = n * (p + 2);
+  const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (size_t)p * Wv) return;
+  const int y = (int)(i / Wv), X = (int)(i % Wv);
+  const int j = X / (p + 2), xx = X - j * (p + 2) - 1;
+  uint4 lo = make_uint4(0u, 0u, 0u, 0u);
+  if (xx >= 0 && xx < p) {
+    const uint8_t* q = lr + (((size_t)j * p + y) * p + xx) * 3;
+    lo.x = pack_bf16x2(q[0] * (1.f / 255.f), q[1] * (1.f / 255.f));
+    lo.y = pack_bf16x2(q[2] * (1.f / 255.f), 0.f);
+  }
+  x[2 * i] = lo;
+  x[2 * i + 1] = make_uint4(0u, 0u, 0u, 0u);
+}
+
+void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStream_t st) {
+  const size_t tot = (size_t)p * n * (p + 2);
+  launch_k(k_pack_input_virtual, dim3((unsigned)((tot + 255) / 256)), dim3(256), 0, st, lr, n, p, reinterpret_cast<uint4*>(x));
 }
 
 // --------------------------------------------------------------- weight packing
 // fwd:   Wf[t][ci/8][co][ci%8]   = W[co][ci][ky][kx],        t = 3 ky + kx    (B operand, K-major, no swizzle)
 // dgrad: Wd[t'][co/8][ci][co%8]  = W[co][ci][2-ky'][2-kx'],  t' = 3 ky' + kx' (180-degree rotation, Cin<->Cout)
 // fold:  Wo[kx][ci/8][ky*coutp + co][ci%8] = W[co][ci][ky][kx]  (N = 3 coutp: the rolling dy-fold conv, conv_roll.cu)
+// dfold: Wdo[kx'][co/8][ky' cinp + ci][co%8] = W[co][ci][2-ky'][2-kx']  (dy-fold weights of the data-grad conv)
 __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc* __restrict__ convs, int nconv,
                                bf16* __restrict__ wf, bf16* __restrict__ wd, bf16* __restrict__ wo,
-                               float* __restrict__ bias) {
+                               bf16* __restrict__ wdo, float* __restrict__ bias) {
+  pdl_enter();
   const int c = blockIdx.y;
   if (c >= nconv) return;
   const ConvDesc d = convs[c];
@@ -65,15 +94,24 @@ __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc*
       float v = (ci < d.cin && co < d.cout) ? W[((co * d.cin + ci) * 3 + ky) * 3 + kx] : 0.f;
       wo[d.pk_off + i] = __float2bfloat16_rn(v);
     }
+    if (wdo) {  // dgrad fold element i = ((kx' * coutp/8 + j') * 3 cinp + ky' * cinp + co') * 8 + e'
+      int e = i & 7, r = i >> 3;
+      int nn = r % (3 * d.cinp); r /= 3 * d.cinp;
+      int j = r % (d.coutp / 8), kxp = r / (d.coutp / 8);
+      int kyp = nn / d.cinp, cop = nn % d.cinp;  // cop = fwd input channel
+      int cip = 8 * j + e;                         // cip = fwd output channel
+      float v = (cip < d.cout && cop < d.cin) ? W[((cip * d.cin + cop) * 3 + (2 - kyp)) * 3 + (2 - kxp)] : 0.f;
+      wdo[d.pk_off + i] = __float2bfloat16_rn(v);
+    }
   }
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < d.coutp; i += gridDim.x * blockDim.x)
     bias[d.b_off + i] = i < d.cout ? params[d.w_off + (size_t)d.cout * d.cin * 9 + i] : 0.f;
 }
 
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, bf16* wo, float* bias, cudaStream_t st) {
+                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st) {
   dim3 grid((max_elems + 255) / 256, nconv);
-  k_pack_weights<<<grid, 256, 0, st>>>(params, convs_dev, nconv, wf, wd, wo, bias);
+  launch_k(k_pack_weights, grid, dim3(256), 0, st, params, convs_dev, nconv, wf, wd, wo, wdo, bias);
 }
 
 // --------------------------------------------------------------- wgrad split-K reduction (deterministic)
@@ -81,6 +119,7 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 __global__ void k_wgrad_reduce(const float* __restrict__ ws_w, const float* __restrict__ ws_b, int nparts,
                                int cinp, int coutp, int cin, int cout, float scale, float* __restrict__ gW,
                                float* __restrict__ gb) {
+  pdl_enter();
   // block = 32 outputs x 8 partial groups; group gi sums partials gi, gi+8, ... (fixed order), then the 8 group
   // sums are added in order 0..7 -> deterministic.
   __shared__ float part[8][33];
@@ -113,25 +152,27 @@ __global__ void k_wgrad_reduce(const float* __restrict__ ws_w, const float* __re
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st) {
   int tot = 9 * cinp * coutp + coutp;
-  k_wgrad_reduce<<<(tot + 31) / 32, dim3(32, 8), 0, st>>>(ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
+  launch_k(k_wgrad_reduce, dim3((tot + 31) / 32), dim3(32, 8), 0, st, ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
 }
 
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
 // m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;  p -= (lr / bc1) * m / (sqrt(v) / sqrt(bc2) + eps),  g = s * grad
 // t and the bias corrections live on the device (k_adam_prep) so the step is replayable from a CUDA graph.
 __global__ void k_adam_prep(long long* counters, float* scal, double lr, double b1, double b2) {
+  pdl_enter();
   const long long t = ++counters[1];
   scal[0] = (float)(lr / (1.0 - pow(b1, (double)t)));
   scal[1] = (float)(1.0 / sqrt(1.0 - pow(b2, (double)t)));
 }
 
 void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st) {
-  k_adam_prep<<<1, 1, 0, st>>>(counters, scal, lr, b1, b2);
+  launch_k(k_adam_prep, dim3(1), dim3(1), 0, st, counters, scal, lr, b1, b2);
 }
 
 __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
                        const float* __restrict__ grad, size_t n, const float* __restrict__ gscale_dev, float gscale,
                        const float* __restrict__ scal, float b1, float b2, float eps) {
+  pdl_enter();
   const float gs = gscale * (gscale_dev ? *gscale_dev : 1.f);
   const float lr_bc1 = scal[0], inv_sqrt_bc2 = scal[1];
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -151,12 +192,15 @@ void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const f
   int th = 256;
   int blocks = (int)((n + th - 1) / th);
   if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
-  k_adam<<<blocks, th, 0, st>>>(p, m, v, g, n, gscale_dev, gscale, scal, b1, b2, eps);
+  launch_k(k_adam, dim3(blocks), dim3(th), 0, st, p, m, v, g, n, gscale_dev, gscale, scal, b1, b2, eps);
 }
 
-__global__ void k_counter_add(long long* c, long long d) { *c += d; }
+__global__ void k_counter_add(long long* c, long long d) {
+  pdl_enter();
+  *c += d;
+}
 void launch_counter_add(long long* counter, long long delta, cudaStream_t st) {
-  k_counter_add<<<1, 1, 0, st>>>(counter, delta);
+  launch_k(k_counter_add, dim3(1), dim3(1), 0, st, counter, delta);
 }
 
 // --------------------------------------------------------------- sampler + gather (reading R10)
@@ -169,6 +213,7 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
 }
 
 __global__ void k_sample_gather(SampleArgs a) {
+  pdl_enter();
   // grid (batch, kGatherSplit): block (j, part) computes draw j (cheap, redundant per part) and copies the crop
   // rows r = part, part + kGatherSplit, ...
   const int j = blockIdx.x;
@@ -210,12 +255,13 @@ __global__ void k_sample_gather(SampleArgs a) {
 }
 
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st) {
-  k_sample_gather<<<dim3(batch, 16), 128, 0, st>>>(a);
+  launch_k(k_sample_gather, dim3(batch, 16), dim3(128), 0, st, a);
 }
 
 // --------------------------------------------------------------- integer SSE per item (warp-shuffle reduction)
 __global__ void k_sse_u8(const uint8_t* __restrict__ a, const uint8_t* __restrict__ b, int64_t elems,
                          unsigned long long* __restrict__ out) {
+  pdl_enter();
   const uint8_t* pa = a + (size_t)blockIdx.x * elems;
   const uint8_t* pb = b + (size_t)blockIdx.x * elems;
   unsigned long long s = 0;
@@ -238,12 +284,15 @@ __global__ void k_sse_u8(const uint8_t* __restrict__ a, const uint8_t* __restric
 
 void launch_sse_u8(const uint8_t* a, const uint8_t* b, int n, int64_t elems, unsigned long long* out,
                    cudaStream_t st) {
-  k_sse_u8<<<n, 256, 0, st>>>(a, b, elems, out);
+  launch_k(k_sse_u8, dim3(n), dim3(256), 0, st, a, b, elems, out);
 }
 
-__global__ void k_loss_finalize(const double* sum, double inv_n, float* out) { *out = (float)(*sum * inv_n); }
+__global__ void k_loss_finalize(const double* sum, double inv_n, float* out) {
+  pdl_enter();
+  *out = (float)(*sum * inv_n);
+}
 void launch_loss_finalize(const double* sum, double inv_n, float* out, cudaStream_t st) {
-  k_loss_finalize<<<1, 1, 0, st>>>(sum, inv_n, out);
+  launch_k(k_loss_finalize, dim3(1), dim3(1), 0, st, sum, inv_n, out);
 }
 
 }  // namespace sr

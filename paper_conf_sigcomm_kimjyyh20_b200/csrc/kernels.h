@@ -28,7 +28,8 @@ struct SampleArgs {
 
 void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st);
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, bf16* wo, float* bias, cudaStream_t st);
+                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st);
+void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStream_t st);
 bool roll_supported(int cinp, int coutp, int W);
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
                              const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st);

@@ -231,3 +231,15 @@ __host__ __device__ constexpr int ring_idx(long long g) {
   return (int)((RB - (g % RB)) % RB);
 }
 }  // namespace sr
+
+namespace sr {
+// Programmatic dependent launch: every kernel of the library is launched with programmatic stream
+// serialization; it does its setup (barriers, TMEM, descriptor prefetch), then waits for its predecessor's
+// completion before touching global data, and immediately lets its own dependent start its setup.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_enter() {
+  pdl_wait();
+  pdl_trigger();
+}
+}  // namespace sr

@@ -29,6 +29,8 @@ struct sr_ctx {
   long long t = 0;  // Adam step counter
   Snapshot snap[4];
   bf16* wd_train = nullptr;  // dgrad-packed TRAIN weights
+  bf16* wdo_train = nullptr; // dgrad weights in dy-fold layout (rolling data-grad convs)
+  bool virtual_train = true; // training on the virtual wide batch with the rolling kernels
   // inference workspace
   size_t inf_pix = 0;
   bf16 *x16 = nullptr, *f0 = nullptr, *fa = nullptr, *fb = nullptr, *tt = nullptr;
@@ -103,7 +105,8 @@ static uint64_t mix64h(uint64_t z) {
 
 static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st) {
   launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, ctx->snap[which].wf,
-                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].wo, ctx->snap[which].bias, st);
+                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].wo,
+                      with_dgrad ? ctx->wdo_train : nullptr, ctx->snap[which].bias, st);
   ctx->launches++;
   CKL();
   return SR_OK;
@@ -170,6 +173,22 @@ static sr_status conv_fwd(sr_ctx* ctx, int cinp, int coutp, const void* in, cons
     return SR_OK;
   }
   return conv(ctx, cinp, coutp, EPI_ACT, in, sn.wf + ctx->convs[ci].pk_off, N, H, W, ep, st);
+}
+
+// general rolling conv launch (training / dgrad variants), timed as one class
+static sr_status roll_ex(sr_ctx* ctx, const char* cls, int cinp, int coutp, const void* in, const bf16* wfold,
+                         const float* bias, const bf16* res1, const bf16* res2, const bf16* mask, int relu, int sep,
+                         bf16* out, int N, int H, int W, cudaStream_t st) {
+  if (ctx->timing) {
+    const double px = (double)N * H * W;
+    tmark_begin(ctx, std::string(cls) + "_" + std::to_string(cinp) + "x" + std::to_string(coutp),
+                2.0 * 9 * cinp * coutp * px, px * 2.0 * (cinp + coutp), st);
+  }
+  cudaError_t e = launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res1, res2, mask, relu, sep, out, N, H, W, st);
+  tmark_end(ctx, st);
+  ctx->launches++;
+  if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll launch: ") + cudaGetErrorString(e));
+  return SR_OK;
 }
 
 static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N, int H, int W, float scale,
@@ -293,11 +312,82 @@ static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
   return SR_OK;
 }
 
+// Training step on the virtual wide batch: the n patches (p x p) sit side by side in one p x n(p+2) image with
+// zero separator columns, so every conv of the forward and of the data-gradient pass runs on the rolling wide
+// kernels (separators re-zeroed in their epilogues = each patch's own zero padding), and wgrad sums over the
+// whole image (separators contribute zero).  Same math as the per-patch path below.
+static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, int n, int p,
+                                    float* loss_dev, cudaStream_t st) {
+  const int Hv = p, Wv = n * (p + 2), sep = p + 2;
+  const size_t pix = (size_t)Hv * Wv;
+  TRY(ensure_train_ws(ctx, pix));
+  const int Cp = ctx->Cp, B = ctx->B, OUTP = ctx->OUTP;
+  const Snapshot& sn = ctx->snap[SR_TRAIN];
+  auto WO = [&](int ci) { return sn.wo + ctx->convs[ci].pk_off; };
+  auto WDO = [&](int ci) { return ctx->wdo_train + ctx->convs[ci].pk_off; };
+  auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
+  launch_pack_input_virtual(lr, n, p, ctx->tx16, st);
+  ctx->launches++;
+  CK(cudaMemsetAsync(ctx->loss_sum, 0, sizeof(double), st));
+  // ---- forward (saving f_0..f_B, t_1..t_B, g)
+  TRY(roll_ex(ctx, "train_fwd", 16, Cp, ctx->tx16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ctx->tf[0], 1,
+              Hv, Wv, st));
+  for (int b = 0; b < B; ++b) {
+    TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tf[b], WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1,
+                sep, ctx->tts[b], 1, Hv, Wv, st));
+    TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tts[b], WO(2 + 2 * b), Bv(2 + 2 * b), ctx->tf[b], nullptr, nullptr, 0,
+                sep, ctx->tf[b + 1], 1, Hv, Wv, st));
+  }
+  const int cb = 1 + 2 * B, cu = cb + 1;
+  TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tf[B], WO(cb), Bv(cb), ctx->tf[0], nullptr, nullptr, 0, sep, ctx->tg, 1,
+              Hv, Wv, st));
+  {
+    EpiParams e{};
+    e.bias = Bv(cu);
+    e.scale = ctx->s;
+    e.lr = lr;
+    e.hr_ref = hr;
+    e.dy = ctx->tdy;
+    e.loss_sum = ctx->loss_sum;
+    e.vsep = sep;
+    e.vp = p;
+    TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, e, st));
+  }
+  const double n_el = (double)n * p * p * ctx->s * ctx->s * 3;
+  if (loss_dev) {
+    launch_loss_finalize(ctx->loss_sum, 1.0 / n_el, loss_dev, st);
+    ctx->launches++;
+  }
+  const float gscale = (float)((ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.0f) / n_el);
+  // ---- backward
+  TRY(wgrad(ctx, cu, ctx->tg, ctx->tdy, 1, Hv, Wv, gscale, st));
+  TRY(roll_ex(ctx, "train_dgrad", OUTP, Cp, ctx->tdy, WDO(cu), nullptr, nullptr, nullptr, nullptr, 0, sep, ctx->tdg, 1,
+              Hv, Wv, st));
+  TRY(wgrad(ctx, cb, ctx->tf[B], ctx->tdg, 1, Hv, Wv, gscale, st));
+  bf16* df = ctx->tdfa;
+  TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdg, WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr,
+              0, sep, df, 1, Hv, Wv, st));
+  for (int b = B - 1; b >= 0; --b) {
+    TRY(wgrad(ctx, 2 + 2 * b, ctx->tts[b], df, 1, Hv, Wv, gscale, st));
+    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, df, WDO(2 + 2 * b), nullptr, nullptr, nullptr, ctx->tts[b], 0, sep,
+                ctx->tdt, 1, Hv, Wv, st));
+    TRY(wgrad(ctx, 1 + 2 * b, ctx->tf[b], ctx->tdt, 1, Hv, Wv, gscale, st));
+    bf16* dfn = (df == ctx->tdfa) ? ctx->tdfb : ctx->tdfa;
+    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdt, WDO(1 + 2 * b), nullptr, df, b == 0 ? ctx->tdg : nullptr,
+                nullptr, 0, sep, dfn, 1, Hv, Wv, st));
+    df = dfn;
+  }
+  TRY(wgrad(ctx, 0, ctx->tx16, df, 1, Hv, Wv, gscale, st));
+  return SR_OK;
+}
+
 // Forward with saved activations, MSE loss + gradient fused into the tail, backward (dgrad = the fwd conv
 // kernel on 180-degree-rotated / transposed weights with ReLU-mask and residual epilogues; wgrad =
 // tcgen05 split-K + deterministic reduce).  grad <- w_r * dL/dtheta.
 static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, int n, int p, float* loss_dev,
                             cudaStream_t st) {
+  if (ctx->virtual_train && roll_supported(ctx->OUTP, ctx->Cp, n * (p + 2)) && roll_supported(16, ctx->Cp, n * (p + 2)))
+    return train_grad_virtual(ctx, lr, hr, n, p, loss_dev, st);
   const size_t pix = (size_t)n * p * p;
   TRY(ensure_train_ws(ctx, pix));
   const int Cp = ctx->Cp, B = ctx->B, OUTP = ctx->OUTP;
@@ -469,6 +559,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
     al(&ctx->snap[k].bias, ctx->b_total);
   }
   al(&ctx->wd_train, ctx->pk_total);
+  al(&ctx->wdo_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
   al(&ctx->counters, 2);
   al(&ctx->adam_scal, 2);
@@ -503,7 +594,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
 void sr_destroy(sr_ctx* ctx) {
   if (!ctx) return;
   cudaDeviceSynchronize();
-  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->x16, ctx->f0,
+  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->x16, ctx->f0,
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->counters,
                   ctx->adam_scal, ctx->pool_lr,
@@ -521,7 +612,8 @@ void sr_destroy(sr_ctx* ctx) {
 
 sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   if (!ctx) return SR_E_INVAL;
-  ctx->fuse_blocks = fuse_blocks != 0;
+  ctx->fuse_blocks = (fuse_blocks & 1) != 0;
+  ctx->virtual_train = (fuse_blocks & 2) == 0;  // bit 1 set: per-patch (narrow tile) training path
   return SR_OK;
 }
 
@@ -889,9 +981,9 @@ sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout
     return SR_E_NOMEM;
   cudaMemcpy(pd, hp.data(), np * 4, cudaMemcpyHostToDevice);
   cudaMemcpy(dd, &d, sizeof(ConvDesc), cudaMemcpyHostToDevice);
-  bf16* wo = nullptr;
-  if (cudaMalloc(&wo, pk * 2)) return SR_E_NOMEM;
-  launch_pack_weights(pd, dd, 1, (int)pk, wf, wd, wo, bias, st);
+  bf16 *wo = nullptr, *wdo = nullptr;
+  if (cudaMalloc(&wo, pk * 2) || cudaMalloc(&wdo, pk * 2)) return SR_E_NOMEM;
+  launch_pack_weights(pd, dd, 1, (int)pk, wf, wd, wo, wdo, bias, st);
   EpiParams ep{};
   ep.bias = (b_host && !dgrad) ? bias : nullptr;
   ep.res1 = (const bf16*)res_dev;
@@ -903,12 +995,13 @@ sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout
   ConvGeom g = make_geom(n, h, w, ci_eff, co_eff, &smem);
   int grid = std::min(g.units, num_sms());
   cudaError_t e;
-  if (!dgrad && !mask_dev && roll_supported(cinp, coutp, w))
-    e = launch_conv_roll(cinp, coutp, x_dev, wo, ep.bias, ep.res1, relu, (bf16*)out_dev, n, h, w, st);
+  if (roll_supported(ci_eff, co_eff, w) && !(res_dev && mask_dev))
+    e = launch_conv_roll_ex(ci_eff, co_eff, x_dev, dgrad ? wdo : wo, ep.bias, ep.res1, nullptr, ep.mask, relu, 0,
+                            (bf16*)out_dev, n, h, w, st);
   else
     e = launch_conv(ci_eff, co_eff, EPI_ACT, x_dev, dgrad ? wd : wf, g, ep, smem, grid, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
-  cudaFree(pd); cudaFree(bias); cudaFree(wf); cudaFree(wd); cudaFree(wo); cudaFree(dd);
+  cudaFree(pd); cudaFree(bias); cudaFree(wf); cudaFree(wd); cudaFree(wo); cudaFree(wdo); cudaFree(dd);
   if (e == cudaErrorNotSupported) return SR_E_UNSUPPORTED;
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }

@@ -43,6 +43,7 @@ struct EpiParams {
   bf16* dy;            // EPI_TAIL_TRAIN: 2*(o - t) in pixel-unshuffled layout [N,H,W,COUTP]
   double* loss_sum;    // EPI_TAIL_TRAIN: += sum (o - t)^2
   int dbg;             // benchmarking only: 1 = drain TMEM and skip the epilogue, 2 = plain store (no bias/res)
+  int vsep, vp;        // EPI_TAIL_TRAIN on the virtual training batch: column pitch p+2 and patch size p (0 = off)
 };
 
 ConvGeom make_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes);
