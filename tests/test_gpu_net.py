@@ -263,3 +263,15 @@ def test_virtual_batch_training_matches_oracle_and_narrow_path(cfg, n, p):
         assert abs(lo - ref_loss) / ref_loss < 1e-2
         assert rel_l2(g, ref_g) < 1e-2, rel_l2(g, ref_g)
     assert rel_l2(grads[0][1], grads[1][1]) < 1e-2
+
+
+def test_infer_host_pipeline_equals_device_path():
+    """sr_infer_host (chunked H2D / compute / D2H pipeline on two streams) == sr_infer on device buffers."""
+    s, B, C = 3, 2, 16
+    ctx = _ctx(s, B, C, seed=31)
+    lr = synth_frames(7, 120, 200, seed=32)
+    dev = ctx.infer(torch.from_numpy(lr).cuda(), "serve").cpu()
+    lr_h = torch.from_numpy(lr).pin_memory()
+    out_h = torch.empty((7, 360, 600, 3), dtype=torch.uint8).pin_memory()
+    ctx.infer_host(lr_h, out_h, "serve")
+    assert torch.equal(out_h, dev)
