@@ -60,7 +60,9 @@ __global__ void __launch_bounds__(kBlkThreads, 1)
 k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
            const float* __restrict__ b2, const bf16* __restrict__ fres, bf16* __restrict__ outp, const int N,
-           const int H, const int W, long long* __restrict__ dbg) {
+           const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg) {
+  // tsave (nullable): also write t = ReLU(conv1(f) + b1) to global (training saves it for the backward pass).
+  // sep > 0: columns with col % sep in {0, sep-1} are separators of the virtual training batch -> t and out = 0.
   // dbg (benchmarking only, CTA 0): clock64 stamps [event][step], events: 0 f issued, 1 conv1 step issued,
   // 2 conv2 step issued, 3 epi1 got a block, 4 epi1 t row done, 5 epi2 got a block, 6 epi2 row stored
 #define SR_DBG(ev, idx) \
@@ -219,7 +221,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     long long G = 0;
     SR_PIECE_BEGIN
     const int tcol = x0 - 1 + m;
-    const bool col_ok = tcol >= 0 && tcol < W;
+    const bool col_ok = tcol >= 0 && tcol < W && !(sep > 0 && ((tcol % sep) == 0 || (tcol % sep) == sep - 1));
+    const bool save_col = tsave != nullptr && m >= 1 && m <= kBlkTW && tcol < W;  // this strip's own columns
     for (int q = -1; q <= n_f; ++q) {         // out rows of conv1 = t rows y0-2+q
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_f - 2;
@@ -248,6 +251,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           u.z = pack_bf16x2(a[4], a[5]);
           u.w = pack_bf16x2(a[6], a[7]);
           *reinterpret_cast<uint4*>(dst + j * PLANE) = u;
+          if (save_col && q >= 2 && q <= n_f - 3)  // t rows y0 .. y1-1 belong to this piece
+            reinterpret_cast<uint4*>(tsave + ((((size_t)n * H + trow) * W) + tcol) * C)[j] = u;
         }
         fence_proxy_async_smem();
         __syncwarp();
@@ -277,6 +282,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     long long G = 0;
     SR_PIECE_BEGIN
     const bool lane_ok = m < kBlkTW && x0 + m < W;
+    const bool sep0 = sep > 0 && (((x0 + m) % sep) == 0 || ((x0 + m) % sep) == sep - 1);
     for (int q = -1; q <= n_t; ++q) {         // out rows of conv2 = output rows y0-1+q
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
@@ -306,8 +312,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
               const float2 f2 = __bfloat1622float2(h2[e]);
-              a[2 * e] = v[8 * j + 2 * e] + f2.x;
-              a[2 * e + 1] = v[8 * j + 2 * e + 1] + f2.y;
+              a[2 * e] = sep0 ? 0.f : v[8 * j + 2 * e] + f2.x;
+              a[2 * e + 1] = sep0 ? 0.f : v[8 * j + 2 * e + 1] + f2.y;
             }
             uint4 u;
             u.x = pack_bf16x2(a[0], a[1]);
@@ -343,7 +349,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 template <int C>
 static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, const bf16* w1, const bf16* w2,
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
-                                  int grid, long long* dbg, cudaStream_t st) {
+                                  int grid, bf16* tsave, int sep, long long* dbg, cudaStream_t st) {
   auto kern = k_resblock<C>;
   static bool configured = false;
   if (!configured) {
@@ -352,7 +358,7 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
     configured = true;
   }
   return launch_k(kern, dim3(grid), dim3(kBlkThreads), BlkCfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, out, N, H, W,
-                  dbg);
+                  tsave, sep, dbg);
 }
 
 bool resblock_supported(int cp, int W) {
@@ -364,16 +370,17 @@ bool resblock_supported(int cp, int W) {
 }
 
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
-                            const float* b2, bf16* out, int N, int H, int W, cudaStream_t st, long long* dbg) {
+                            const float* b2, bf16* out, int N, int H, int W, cudaStream_t st, long long* dbg,
+                            bf16* tsave, int sep) {
   CUtensorMap tf, to;
   if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (make_row_tmap(&to, out, N, H, W, cp, kBlkTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   const long long rows = (long long)N * ((W + kBlkTW - 1) / kBlkTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
-  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
-  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
-  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, dbg, st);
+  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
+  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
+  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
   return cudaErrorNotSupported;
 }
 

@@ -40,7 +40,7 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
 bool resblock_supported(int cp, int W);
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,
-                            long long* dbg = nullptr);
+                            long long* dbg = nullptr, bf16* tsave = nullptr, int sep = 0);
 void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
                          float scale, float* gW, float* gb, cudaStream_t st);
 // Device-side step counters (so a training iteration can be captured once in a CUDA graph and replayed):

@@ -335,6 +335,18 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
   TRY(roll_ex(ctx, "train_fwd", 16, Cp, ctx->tx16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ctx->tf[0], 1,
               Hv, Wv, st));
   for (int b = 0; b < B; ++b) {
+    if (ctx->fuse_blocks && resblock_supported(Cp, Wv)) {  // fused block, t also saved for the backward pass
+      if (ctx->timing) {
+        const double px = (double)Hv * Wv;
+        tmark_begin(ctx, "train_resblock_" + std::to_string(Cp), 2 * 2.0 * 9 * Cp * Cp * px, px * 2.0 * 3 * Cp, st);
+      }
+      cudaError_t e = launch_resblock(Cp, ctx->tf[b], WO(1 + 2 * b), WO(2 + 2 * b), Bv(1 + 2 * b), Bv(2 + 2 * b),
+                                      ctx->tf[b + 1], 1, Hv, Wv, st, nullptr, ctx->tts[b], sep);
+      tmark_end(ctx, st);
+      ctx->launches++;
+      if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("resblock launch: ") + cudaGetErrorString(e));
+      continue;
+    }
     TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tf[b], WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1,
                 sep, ctx->tts[b], 1, Hv, Wv, st));
     TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tts[b], WO(2 + 2 * b), Bv(2 + 2 * b), ctx->tf[b], nullptr, nullptr, 0,
