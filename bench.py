@@ -8,8 +8,11 @@ Workload (BASELINE.json config 3 + config 4): per rank 
            (48x48 LR -> 144x144 HR), forward, MSE, backward, [NCCL allreduce of the gradient over NVLink
            when N > 1], Adam                                                                         [sr_sample_batch,
                                                                                                        sr_train_grad, sr_train_apply]
-  * T7     epoch-end publish (TRAIN -> SERVE)                                                        [sr_publish]
-  * Q1     quality gain of SERVE over bilinear on 64 validation patches                              [sr_psnr_gain]
+  * T7     at each epoch end (every 50 iterations = every 5th step, L1247-1253): publish (TRAIN -> SERVE)
+                                                                                                     [sr_publish]
+  * Q1     and Algorithm 1's epoch-end evaluation on 64 recent patches: PSNR of SERVE, PREV, INIT and bilinear,
+           the saturation diff and Q_DNN (reported; the bench stays in the Training state, whose work is
+           the expensive one, so every epoch does the same work)                                     [sr_controller_step]
 The headline metric is 4K frames/s summed over ranks (weak scaling: frames are sharded, 30 per rank per step);
 training patches/s is reported beside it.  `--impl reference` times the fp64 CPU oracle (the paper has no code).
 """
@@ -30,6 +33,7 @@ S, BLOCKS, CH = 3, 8, 48
 LR_H, LR_W = 720, 1280
 FRAMES = 30
 ITERS = 10
+EPOCH_ITERS = 50  # training iterations per epoch; publish + Algorithm 1 at its end
 BATCH, PATCH = 64, 48
 POOL_N, POOL_LR = 512, 60           # pool entries: 60x60 LR / 180x180 HR (crop offsets span 0..12)
 VAL_N = 64
@@ -97,7 +101,7 @@ def run_ours(args):
     import numpy as np
     import torch
     import torch.distributed as dist
-    from paper_conf_sigcomm_kimjyyh20_b200 import SRContext
+    from paper_conf_sigcomm_kimjyyh20_b200 import Controller, SRContext
     from paper_conf_sigcomm_kimjyyh20_b200.parallel import dp_allreduce_grad_dev, max_over_ranks
     from synth import synth_frames, synth_patch_pool
 
@@ -143,18 +147,31 @@ def run_ours(args):
             train_iter()
         launches_per_iter = ctx.launches - lc   # our kernels inside one captured iteration
 
+    ctrl = Controller(thresh_sat=0.05, count_sat=2, thresh_online=0.5, count_online=2)
+    state["iters"] = 0  # training iterations since the last epoch end
+
+    def epoch_eval():
+        r = ctx.controller_step(ctrl, val_lr, val_hr)
+        if ctrl.state != "training":  # keep the measured work constant (see the docstring)
+            ctrl.c.state, ctrl.c.patience = 0, 0
+        state["q"] = r
+        state["epochs"] = state.get("epochs", 0) + 1
+
     def train_iters():
         for _ in range(args.iters):
             if graph is not None:
                 graph.replay()
             else:
                 train_iter()
-        ctx.publish()
+        state["iters"] += args.iters
+        if state["iters"] >= EPOCH_ITERS:  # epoch end (50 iterations, L1247-1250): publish + Algorithm 1
+            state["iters"] = 0
+            ctx.publish()
+            epoch_eval()
 
     def step():
         ctx.infer(lr, "serve", out=hr)
         train_iters()
-        state["q"] = ctx.psnr_gain(val_lr, val_hr, "serve", "bilinear")
 
     def barrier():
         if world > 1:
@@ -164,6 +181,7 @@ def run_ours(args):
     for _ in range(args.warmup):
         step()
     barrier()
+    state["iters"], state["epochs"] = 0, 0  # the timed region starts at an epoch boundary
     clk = ClockSampler(local)
     clk.start()
     l0 = ctx.launches
@@ -176,6 +194,7 @@ def run_ours(args):
     e1.record()
     barrier()
     ms = e0.elapsed_time(e1)
+    epochs_timed = state["epochs"]
     launches = ctx.launches - l0 + (launches_per_iter * args.iters * args.steps if graph is not None else 0)
     stats = ctx.kernel_stats()
     ctx.kernel_timing(False)
@@ -204,10 +223,10 @@ def run_ours(args):
         ctx.infer_host(lr_host, hr_host, "serve")
         train_iters()
         loss_host.copy_(loss, non_blocking=True)
-        state["q"] = ctx.psnr_gain(val_lr, val_hr, "serve", "bilinear")
 
     step_e2e()
     barrier()
+    state["iters"] = 0
     e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e2.record()
     for _ in range(args.steps):
@@ -242,20 +261,23 @@ def run_ours(args):
             "data": "synthetic (seeded 1/f frames + edges + strokes, pan; random-init weights)",
             "config": {
                 "workload": f"cfg3+cfg4: {frames}x 720p->4K x3 frames + {args.iters} train iters (64x 48->144) "
-                            "+ publish + psnr_gain per rank per step",
+                            "+ publish + Algorithm-1 evaluation at each epoch end (every 50 iterations) per rank",
                 "net": f"x{S}, {BLOCKS} blocks x {CH} ch", "frames_per_rank": frames,
                 "train_iters_per_step": args.iters, "batch": BATCH, "patch_lr": PATCH,
+                "epoch_ends_timed": epochs_timed,
                 "parallelism": f"frames sharded x{world}, DP training (NCCL allreduce)" if world > 1 else "1 GPU",
                 "l2": "working set > L2 (one 720p activation tensor at 48 ch = 88 MB; 30 frames per step)",
             },
             "train_patches_per_s": round(BATCH * args.iters * args.steps * world / (ms * 1e-3), 1),
             "train_iter": {"ms": round(train_iter_ms, 4), "tflops": round(TRAIN_FLOP / (train_iter_ms * 1e-3) / 1e12, 1),
                            "graph": graph is not None, "note": "one sampled training iteration alone (rank 0)"},
-            "quality_gain_db": round(state["q"][2], 4) if state["q"] else None,
+            "quality_gain_db": round(state["q"]["q_dnn"], 4) if state["q"] else None,
+            "alg1_last": {k: (round(v, 4) if isinstance(v, float) else v) for k, v in state["q"].items()}
+            if state["q"] else None,
             "tensor_tflops_all_convs": round(conv_flops / (sum(v["ms"] for v in stats.values()) * 1e-3) / 1e12, 1),
             "kernel_share": {k: round(v["ms"] / ktot, 4) for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"])},
             "kernel_share_note": "CUDA-event time per kernel class of the eagerly launched kernels (inference, "
-                                 "psnr_gain); the graph-replayed training kernels are in train_iter",
+                                 "Algorithm-1 evaluation); the graph-replayed training kernels are in train_iter",
             "roofline": {"bound": "tensor", "kernel": dom, "achieved": round(achieved, 1),
                          "peak": sustained, "unit": "TFLOP/s", "frac": round(achieved / sustained, 4),
                          "peak_kind": "measured bf16_tflops_sustained (MEASURED_PEAKS.json)",

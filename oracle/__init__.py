@@ -9,7 +9,8 @@ the paper is silent.
 Parity pins (tests/test_oracle_pins.py, `-m "not gpu"`): brute-force 7-loop conv, identity/delta
 kernels, pixel shuffle as a permutation, zero-weight net == bilinear skip (bit-exact u8, checked
 against torch.nn.functional.interpolate), finite-difference gradients of the whole net, PSNR closed
-form, Adam step-1 closed form (and torch.optim.Adam), sampler statistics, paper arithmetic facts.
+form, Adam step-1 closed form (and torch.optim.Adam), sampler statistics, paper arithmetic facts,
+Algorithm 1 (oracle/controller.py) against traces worked out by hand from App. A (tests/golden/alg1_traces.json).
 "parity unpinned": none of the functions below; the learning-direction check (loss falls) is a
 sanity check only.
 """
@@ -18,3 +19,4 @@ from .srnet import (  # noqa: F401
     bilinear_up, unpack_params, pack_params, forward, infer_u8, train_loss_and_grad, adam_step,
     dp_aggregate, sample_indices, gather_patches, psnr_u8, psnr_gain, conv_shapes_oracle,
 )
+from .controller import Algorithm1, epoch_report  # noqa: F401

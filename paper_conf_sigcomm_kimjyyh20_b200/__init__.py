@@ -9,8 +9,9 @@ import ctypes as C
 
 from . import _lib
 from ._lib import MODELS, SRError, check, load, sr_options, sr_quality  # noqa: F401
+from ._lib import SR_EV_NONE, SR_EV_RESUME, SR_EV_SUSPEND, SR_SUSPENDED, SR_TRAINING  # noqa: F401
 
-__all__ = ["SRContext", "load", "SRError", "MODELS"]
+__all__ = ["SRContext", "Controller", "load", "SRError", "MODELS"]
 
 
 def _ptr(t):
@@ -25,6 +26,35 @@ def _stream(stream):
 
 def _model(m):
     return MODELS[m] if isinstance(m, str) else int(m)
+
+
+class Controller:
+    """Algorithm 1's Training/Suspended state machine (App. A), held in the library's sr_controller
+    struct.  `update(diff)` is one training epoch (Training) or one validation period (Suspended); it is host
+    logic and needs no GPU.  `SRContext.controller_step` measures the diff on the GPU and calls it."""
+
+    STATES = {SR_TRAINING: "training", SR_SUSPENDED: "suspended"}
+    EVENTS = {SR_EV_NONE: None, SR_EV_SUSPEND: "suspend", SR_EV_RESUME: "resume"}
+
+    def __init__(self, thresh_sat: float, count_sat: int, thresh_online: float, count_online: int):
+        self.lib = load()
+        self.c = _lib.sr_controller()
+        check(self.lib.sr_controller_init(C.byref(self.c), thresh_sat, count_sat, thresh_online, count_online),
+              None, "sr_controller_init")
+
+    @property
+    def state(self) -> str:
+        return self.STATES[self.c.state]
+
+    @property
+    def patience(self) -> int:
+        return self.c.patience
+
+    def update(self, diff: float):
+        ev = C.c_int(0)
+        check(self.lib.sr_controller_update(C.byref(self.c), float(diff), C.byref(ev)), None,
+              "sr_controller_update")
+        return self.EVENTS[ev.value]
 
 
 class SRContext:
@@ -158,6 +188,19 @@ class SRContext:
         check(self.lib.sr_psnr_gain(self.h, _model(a), _model(b), _ptr(lr), _ptr(hr), n, p, C.byref(q),
                                     _stream(stream)), self.h, "sr_psnr_gain")
         return q.psnr_a, q.psnr_b, q.gain
+
+    def controller_step(self, ctrl: Controller, lr, hr, stream=None) -> dict:
+        """Epoch-end / validation hook (sr_controller_step): PSNR of SERVE/PREV/INIT/bilinear on the recent
+        patches, Algorithm 1's diff and transition, and the Q_DNN feedback."""
+        r = _lib.sr_epoch_report()
+        n, p = lr.shape[0], lr.shape[1]
+        check(self.lib.sr_controller_step(self.h, C.byref(ctrl.c), _ptr(lr), _ptr(hr), n, p, C.byref(r),
+                                          _stream(stream)), self.h, "sr_controller_step")
+        out = {f: getattr(r, f) for f, _ in r._fields_}
+        out["state_before"] = Controller.STATES[r.state_before]
+        out["state_after"] = Controller.STATES[r.state_after]
+        out["event"] = Controller.EVENTS[r.event]
+        return out
 
     def set_fusion(self, fuse_blocks=True):
         check(self.lib.sr_set_fusion(self.h, int(fuse_blocks)), self.h, "sr_set_fusion")

@@ -24,6 +24,20 @@ class sr_quality(C.Structure):
     _fields_ = [("psnr_a", C.c_double), ("psnr_b", C.c_double), ("gain", C.c_double)]
 
 
+class sr_controller(C.Structure):
+    _fields_ = [("thresh_sat", C.c_double), ("count_sat", C.c_int), ("thresh_online", C.c_double),
+                ("count_online", C.c_int), ("state", C.c_int), ("patience", C.c_int)]
+
+
+class sr_epoch_report(C.Structure):
+    _fields_ = [("state_before", C.c_int), ("event", C.c_int), ("state_after", C.c_int), ("diff", C.c_double),
+                ("psnr_serve", C.c_double), ("psnr_prev", C.c_double), ("psnr_init", C.c_double),
+                ("psnr_bilinear", C.c_double), ("q_dnn", C.c_double), ("q_dnn_prev", C.c_double)]
+
+
+SR_TRAINING, SR_SUSPENDED = 0, 1
+SR_EV_NONE, SR_EV_SUSPEND, SR_EV_RESUME = 0, 1, 2
+
 _P = C.c_void_p
 _I = C.c_int
 _SIGS = {
@@ -47,6 +61,9 @@ _SIGS = {
     "sr_train_sampled": (_I, [_P, _I, _I, _I, _P, _P]),
     "sr_publish": (_I, [_P, _P]),
     "sr_psnr_gain": (_I, [_P, _I, _I, _P, _P, _I, _I, C.POINTER(sr_quality), _P]),
+    "sr_controller_init": (_I, [C.POINTER(sr_controller), C.c_double, _I, C.c_double, _I]),
+    "sr_controller_update": (_I, [C.POINTER(sr_controller), C.c_double, C.POINTER(_I)]),
+    "sr_controller_step": (_I, [_P, C.POINTER(sr_controller), _P, _P, _I, _I, C.POINTER(sr_epoch_report), _P]),
     "sr_sse_u8": (_I, [_P, _P, _I, C.c_int64, _P, _P]),
     "sr_launch_count": (C.c_uint64, [_P]),
     "sr_kernel_timing": (_I, [_P, _I]),

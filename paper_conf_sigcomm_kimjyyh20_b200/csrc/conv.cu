@@ -168,12 +168,17 @@ __device__ __forceinline__ void epi_act(const EpiParams& ep, const float* sbias,
 // Bilinear skip by output phase (half-pixel centres, edge replicate == PyTorch align_corners=False):
 //   x2: phase 0 -> 0.25 v[i-1] + 0.75 v[i];  phase 1 -> 0.75 v[i] + 0.25 v[i+1]
 //   x3: phase 0 -> v[i-1]/3 + 2 v[i]/3;  phase 1 -> v[i];  phase 2 -> 2 v[i]/3 + v[i+1]/3
+//   x4: source offsets (ph + 1/2)/4 - 1/2 = -3/8, -1/8, +1/8, +3/8 (exact binary fractions)
 template <int S>
 __device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp) {
   if (S == 2) {
     wm = ph == 0 ? 0.25f : 0.f;
     w0 = 0.75f;
     wp = ph == 1 ? 0.25f : 0.f;
+  } else if (S == 4) {
+    wm = ph == 0 ? 0.375f : (ph == 1 ? 0.125f : 0.f);
+    w0 = (ph == 0 || ph == 3) ? 0.625f : 0.875f;
+    wp = ph == 3 ? 0.375f : (ph == 2 ? 0.125f : 0.f);
   } else {
     const float t = 1.f / 3.f, tt = 2.f / 3.f;
     wm = ph == 0 ? t : 0.f;
@@ -376,7 +381,10 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
         } else if (EPI == EPI_ACT) {
           epi_act<COUTP>(ep, sbias, pix, v, pre);
         } else if (EPI == EPI_TAIL_U8) {
-          if (Y >= ep.hr_row0 && Y < ep.hr_row1)
+          if (ep.vsep > 0) {  // virtual batch of square images: image j at columns [j*vsep + 1, j*vsep + 1 + p)
+            const int j = X / ep.vsep, x = X - j * ep.vsep - 1;
+            if (x >= 0 && x < ep.vp) epi_tail<S, COUTP, false>(ep, sbias, j, Y, x, ep.vp, ep.vp, v, lsum, 0);
+          } else if (Y >= ep.hr_row0 && Y < ep.hr_row1)
             epi_tail<S, COUTP, false>(ep, sbias, n, Y, X, g.H, g.W, v, lsum, ((size_t)n * g.H + Y) * g.W + X);
         } else {
           const size_t vp = ((size_t)n * g.H + Y) * g.W + X;
@@ -440,10 +448,11 @@ cudaError_t launch_conv(int cinp, int coutp, int epi, const void* in, const bf16
   SR_CONV_CASE(16, 16) SR_CONV_CASE(16, 32) SR_CONV_CASE(16, 48) SR_CONV_CASE(16, 64)
   SR_CONV_CASE(32, 16) SR_CONV_CASE(32, 32) SR_CONV_CASE(32, 48) SR_CONV_CASE(32, 64)
   SR_CONV_CASE(48, 16) SR_CONV_CASE(48, 32) SR_CONV_CASE(48, 48)
-  SR_CONV_CASE(64, 16) SR_CONV_CASE(64, 32) SR_CONV_CASE(64, 64)
-  // up conv + tail (C -> 3 s^2 padded: 12 -> 16, 27 -> 32)
+  SR_CONV_CASE(64, 16) SR_CONV_CASE(64, 32) SR_CONV_CASE(64, 64) SR_CONV_CASE(48, 64)
+  // up conv + tail (C -> 3 s^2 padded: 12 -> 16, 27 -> 32, 48)
   SR_TAIL_CASE(16, 16, 2) SR_TAIL_CASE(32, 16, 2) SR_TAIL_CASE(48, 16, 2) SR_TAIL_CASE(64, 16, 2)
   SR_TAIL_CASE(16, 32, 3) SR_TAIL_CASE(32, 32, 3) SR_TAIL_CASE(48, 32, 3) SR_TAIL_CASE(64, 32, 3)
+  SR_TAIL_CASE(16, 48, 4) SR_TAIL_CASE(32, 48, 4) SR_TAIL_CASE(48, 48, 4) SR_TAIL_CASE(64, 48, 4)
   return cudaErrorNotSupported;
 }
 
@@ -666,7 +675,7 @@ cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, con
   SR_WG_CASE(16, 16) SR_WG_CASE(16, 32) SR_WG_CASE(16, 48) SR_WG_CASE(16, 64)
   SR_WG_CASE(32, 16) SR_WG_CASE(32, 32) SR_WG_CASE(32, 48) SR_WG_CASE(32, 64)
   SR_WG_CASE(48, 16) SR_WG_CASE(48, 32) SR_WG_CASE(48, 48)
-  SR_WG_CASE(64, 16) SR_WG_CASE(64, 32) SR_WG_CASE(64, 64)
+  SR_WG_CASE(64, 16) SR_WG_CASE(64, 32) SR_WG_CASE(64, 64) SR_WG_CASE(64, 48)
   return cudaErrorNotSupported;
 }
 
@@ -683,12 +692,13 @@ __global__ void k_bilinear_u8(const uint8_t* __restrict__ lr, int n, int h, int 
   EpiParams ep{};
   ep.lr = lr;
   ep.hr = hr;
-  float v[32];
+  constexpr int CO = S == 4 ? 48 : 32;
+  float v[CO];
 #pragma unroll
-  for (int k = 0; k < 32; ++k) v[k] = 0.f;
-  const float zb[32] = {0.f};
+  for (int k = 0; k < CO; ++k) v[k] = 0.f;
+  const float zb[CO] = {0.f};
   float ls = 0.f;
-  epi_tail<S, 32, false>(ep, zb, img, Y, X, h, w, v, ls, 0);
+  epi_tail<S, CO, false>(ep, zb, img, Y, X, h, w, v, ls, 0);
 }
 
 cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st) {
@@ -696,6 +706,7 @@ cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, ui
   unsigned blocks = (unsigned)((tot + 255) / 256);
   if (s == 2) return launch_k(k_bilinear_u8<2>, dim3(blocks), dim3(256), 0, st, lr, n, h, w, hr);
   if (s == 3) return launch_k(k_bilinear_u8<3>, dim3(blocks), dim3(256), 0, st, lr, n, h, w, hr);
+  if (s == 4) return launch_k(k_bilinear_u8<4>, dim3(blocks), dim3(256), 0, st, lr, n, h, w, hr);
   return cudaErrorNotSupported;
 }
 

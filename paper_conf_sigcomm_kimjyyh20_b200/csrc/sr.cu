@@ -56,7 +56,7 @@ struct sr_ctx {
   size_t batch_bytes_lr = 0, batch_bytes_hr = 0;
   long long sample_step = 0;
   // psnr
-  uint8_t *val_a = nullptr, *val_b = nullptr;
+  uint8_t* val_a = nullptr;  // one model's SR output of the validation patches
   size_t val_bytes = 0;
   unsigned long long* sse = nullptr;
   int sse_n = 0;
@@ -298,6 +298,58 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   return SR_OK;
 }
 
+// Batches of small square images (the validation patches of sr_psnr_gain / sr_controller_step): too narrow for
+// the wide kernels one by one, so they run as ONE virtual wide image, side by side with zero separator columns
+// (re-zeroed by every conv epilogue = each image's own zero padding), exactly like the training batch.  Same
+// math as forward_infer.
+static bool use_virtual_infer(const sr_ctx* ctx, int n, int h, int w) {
+  const int Wv = n * (w + 2);
+  return n > 1 && h == w && !roll_supported(16, ctx->Cp, w) && roll_supported(16, ctx->Cp, Wv) &&
+         roll_supported(ctx->Cp, ctx->Cp, Wv);
+}
+
+static sr_status forward_infer_virtual(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int p,
+                                       uint8_t* hr, cudaStream_t st) {
+  const int Hv = p, Wv = n * (p + 2), sep = p + 2;
+  TRY(ensure_infer_ws(ctx, (size_t)Hv * Wv));
+  const int Cp = ctx->Cp;
+  auto WO = [&](int ci) { return sn.wo + ctx->convs[ci].pk_off; };
+  auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
+  launch_pack_input_virtual(lr, n, p, ctx->x16, st);
+  ctx->launches++;
+  CKL();
+  TRY(roll_ex(ctx, "infer_v", 16, Cp, ctx->x16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ctx->f0, 1, Hv, Wv,
+              st));
+  bf16* cur = ctx->f0;
+  for (int b = 0; b < ctx->B; ++b) {
+    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+    if (ctx->fuse_blocks && resblock_supported(Cp, Wv)) {
+      cudaError_t e = launch_resblock(Cp, cur, WO(1 + 2 * b), WO(2 + 2 * b), Bv(1 + 2 * b), Bv(2 + 2 * b), nxt, 1, Hv,
+                                      Wv, st, nullptr, nullptr, sep);
+      ctx->launches++;
+      if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("resblock launch: ") + cudaGetErrorString(e));
+    } else {
+      TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1, sep, ctx->tt,
+                  1, Hv, Wv, st));
+      TRY(roll_ex(ctx, "infer_v", Cp, Cp, ctx->tt, WO(2 + 2 * b), Bv(2 + 2 * b), cur, nullptr, nullptr, 0, sep, nxt, 1,
+                  Hv, Wv, st));
+    }
+    cur = nxt;
+  }
+  const int cb = 1 + 2 * ctx->B, cu = cb + 1;
+  bf16* gbuf = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+  TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(cb), Bv(cb), ctx->f0, nullptr, nullptr, 0, sep, gbuf, 1, Hv, Wv, st));
+  EpiParams et{};
+  et.bias = Bv(cu);
+  et.scale = ctx->s;
+  et.lr = lr;
+  et.hr = hr;
+  et.vsep = sep;
+  et.vp = p;
+  TRY(conv(ctx, Cp, ctx->OUTP, EPI_TAIL_U8, gbuf, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, et, st));
+  return SR_OK;
+}
+
 static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
   if (pix <= ctx->tr_pix) return SR_OK;
   const int Cp = ctx->Cp;
@@ -512,8 +564,7 @@ extern "C" {
 sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, sr_ctx** out) {
   if (!out) return SR_E_INVAL;
   *out = nullptr;
-  if (scale == 4) return SR_E_UNSUPPORTED;
-  if ((scale != 2 && scale != 3) || blocks < 0 || channels < 1 || channels > 64) return SR_E_INVAL;
+  if ((scale < 2 || scale > 4) || blocks < 0 || channels < 1 || channels > 64) return SR_E_INVAL;
   sr_ctx* ctx = new sr_ctx();
   ctx->s = scale;
   ctx->B = blocks;
@@ -612,7 +663,7 @@ void sr_destroy(sr_ctx* ctx) {
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->counters,
                   ctx->adam_scal, ctx->pool_lr,
-                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->val_b, ctx->sse};
+                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].wo); cudaFree(ctx->snap[k].bias); }
@@ -738,6 +789,8 @@ sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, in
   }
   if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer: bad model");
   CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
+  if (use_virtual_infer(ctx, n, h, w) && ctx->virtual_train)
+    return forward_infer_virtual(ctx, ctx->snap[which], lr_dev, n, h, hr_dev, st);
   return forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st);
 }
 
@@ -966,36 +1019,119 @@ sr_status sr_sse_u8(const uint8_t* a_dev, const uint8_t* b_dev, int n, int64_t e
   return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
 }
 
-sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
-                       int p, sr_quality* out_host, sr_stream stream) {
-  GUARD();
-  if (!lr_dev || !hr_dev || !out_host || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_psnr_gain: bad args");
-  cudaStream_t st = (cudaStream_t)stream;
+// Mean per-patch PSNR of k models on the same validation patches (one sync).  Per patch: integer SSE (K9) ->
+// 10 log10(255^2 count / SSE), capped at 100 dB for SSE = 0.
+static sr_status mean_psnr(sr_ctx* ctx, const sr_model* models, int k, const uint8_t* lr_dev, const uint8_t* hr_dev,
+                           int n, int p, double* out, cudaStream_t st) {
   const int s = ctx->s;
   const size_t per = (size_t)s * p * s * p * 3, tot = per * n;
   if (tot > ctx->val_bytes) {
     CK(dalloc(&ctx->val_a, tot));
-    CK(dalloc(&ctx->val_b, tot));
     ctx->val_bytes = tot;
   }
-  if (n > ctx->sse_n) { CK(dalloc(&ctx->sse, 2 * (size_t)n)); ctx->sse_n = n; }
-  TRY(sr_infer(ctx, a, lr_dev, n, p, p, ctx->val_a, stream));
-  TRY(sr_infer(ctx, b, lr_dev, n, p, p, ctx->val_b, stream));
-  launch_sse_u8(ctx->val_a, hr_dev, n, (int64_t)per, ctx->sse, st);
-  launch_sse_u8(ctx->val_b, hr_dev, n, (int64_t)per, ctx->sse + n, st);
-  ctx->launches += 2;
-  CKL();
-  std::vector<unsigned long long> h(2 * (size_t)n);
+  if ((size_t)k * n > (size_t)ctx->sse_n) { CK(dalloc(&ctx->sse, (size_t)k * n)); ctx->sse_n = k * n; }
+  for (int m = 0; m < k; ++m) {
+    // sse of model m is launched on st right after its inference, so val_a can be reused (stream order)
+    TRY(sr_infer(ctx, models[m], lr_dev, n, p, p, ctx->val_a, (sr_stream)st));
+    launch_sse_u8(ctx->val_a, hr_dev, n, (int64_t)per, ctx->sse + (size_t)m * n, st);
+    ctx->launches++;
+    CKL();
+  }
+  std::vector<unsigned long long> h((size_t)k * n);
   CK(cudaMemcpyAsync(h.data(), ctx->sse, h.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  double sa = 0, sb = 0;
-  for (int i = 0; i < n; ++i) {
-    sa += h[i] == 0 ? 100.0 : 10.0 * std::log10(255.0 * 255.0 * (double)per / (double)h[i]);
-    sb += h[n + i] == 0 ? 100.0 : 10.0 * std::log10(255.0 * 255.0 * (double)per / (double)h[n + i]);
+  for (int m = 0; m < k; ++m) {
+    double acc = 0;
+    for (int i = 0; i < n; ++i) {
+      const unsigned long long e = h[(size_t)m * n + i];
+      acc += e == 0 ? 100.0 : 10.0 * std::log10(255.0 * 255.0 * (double)per / (double)e);
+    }
+    out[m] = acc / n;
   }
-  out_host->psnr_a = sa / n;
-  out_host->psnr_b = sb / n;
-  out_host->gain = out_host->psnr_a - out_host->psnr_b;
+  return SR_OK;
+}
+
+sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
+                       int p, sr_quality* out_host, sr_stream stream) {
+  GUARD();
+  if (!lr_dev || !hr_dev || !out_host || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_psnr_gain: bad args");
+  const sr_model ms[2] = {a, b};
+  double q[2];
+  TRY(mean_psnr(ctx, ms, 2, lr_dev, hr_dev, n, p, q, (cudaStream_t)stream));
+  out_host->psnr_a = q[0];
+  out_host->psnr_b = q[1];
+  out_host->gain = q[0] - q[1];
+  return SR_OK;
+}
+
+// ---- Algorithm 1 (App. A), written in the paper's line order
+sr_status sr_controller_init(sr_controller* c, double thresh_sat, int count_sat, double thresh_online,
+                             int count_online) {
+  if (!c || count_sat < 0 || count_online < 0) return SR_E_INVAL;
+  c->thresh_sat = thresh_sat;
+  c->count_sat = count_sat;
+  c->thresh_online = thresh_online;
+  c->count_online = count_online;
+  c->state = SR_TRAINING;  // line 1
+  c->patience = 0;
+  return SR_OK;
+}
+
+sr_status sr_controller_update(sr_controller* c, double diff, int* event_out) {
+  if (!c || (c->state != SR_TRAINING && c->state != SR_SUSPENDED)) return SR_E_INVAL;
+  int ev = SR_EV_NONE;
+  if (c->state == SR_TRAINING) {       // lines 4-14: one training epoch
+    if (diff < c->thresh_sat) {        // line 7
+      c->patience += 1;                // line 8
+      if (c->patience > c->count_sat) {  // line 9
+        ev = SR_EV_SUSPEND;            // line 10
+        c->state = SR_SUSPENDED;       // line 11
+        c->patience = 0;               // line 12
+      }
+    } else {
+      c->patience = 0;                 // line 14
+    }
+  } else {                             // lines 15-25: one validation period
+    if (diff < c->thresh_online) {     // line 18
+      c->patience += 1;                // line 19
+      if (c->patience > c->count_online) {  // line 20
+        ev = SR_EV_RESUME;             // line 21
+        c->state = SR_TRAINING;        // line 22
+        c->patience = 0;               // line 23
+      }
+    } else {
+      c->patience = 0;                 // line 25
+    }
+  }
+  if (event_out) *event_out = ev;
+  return SR_OK;
+}
+
+sr_status sr_controller_step(sr_ctx* ctx, sr_controller* c, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
+                             int p, sr_epoch_report* out_host, sr_stream stream) {
+  GUARD();
+  if (!c || !lr_dev || !hr_dev || !out_host || n < 1 || p < 1)
+    return fail(ctx, SR_E_INVAL, "sr_controller_step: bad args");
+  if (c->state != SR_TRAINING && c->state != SR_SUSPENDED)
+    return fail(ctx, SR_E_INVAL, "sr_controller_step: controller not initialised");
+  const sr_model ms[4] = {SR_SERVE, SR_PREV, SR_INIT, SR_BILINEAR};
+  double q[4];
+  TRY(mean_psnr(ctx, ms, 4, lr_dev, hr_dev, n, p, q, (cudaStream_t)stream));
+  sr_epoch_report r{};
+  r.psnr_serve = q[0];
+  r.psnr_prev = q[1];
+  r.psnr_init = q[2];
+  r.psnr_bilinear = q[3];
+  r.q_dnn = q[0] - q[3];
+  r.q_dnn_prev = q[1] - q[3];
+  r.state_before = c->state;
+  r.diff = c->state == SR_TRAINING ? q[0] - q[1] : q[0] - q[2];  // line 6 / line 17
+  int ev = SR_EV_NONE;
+  sr_status st = sr_controller_update(c, r.diff, &ev);
+  if (st != SR_OK) return fail(ctx, st, "sr_controller_step: update failed");
+  r.event = ev;
+  r.state_after = c->state;
+  *out_host = r;
   return SR_OK;
 }
 

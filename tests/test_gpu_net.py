@@ -39,7 +39,7 @@ def test_create_init_matches_synth_bitexact(cfg):
 
 
 # ---------------------------------------------------------------- inference
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_zero_weight_net_is_bilinear_bitexact(s):
     ctx = _ctx(s, 2, 8)
     ctx.set_params(np.zeros(ctx.num_params, np.float32))
@@ -52,7 +52,7 @@ def test_zero_weight_net_is_bilinear_bitexact(s):
     np.testing.assert_array_equal(got_b, ref)
 
 
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_pixel_shuffle_permutation_bitexact(s):
     B, C = 1, 8
     ctx = _ctx(s, B, C)
@@ -77,7 +77,7 @@ def test_tiny_config_inference_parity():
     _check_frames(got, ref, hr)
 
 
-@pytest.mark.parametrize("cfg", [(2, 8, 32), (3, 8, 48), (2, 8, 48)])
+@pytest.mark.parametrize("cfg", [(2, 8, 32), (3, 8, 48), (2, 8, 48), (4, 8, 48)])
 def test_real_net_inference_parity_small_frames(cfg):
     """The BASELINE nets on frames the oracle finishes in seconds (several tiles + ragged tails)."""
     s, B, C = cfg
@@ -106,7 +106,8 @@ def _oracle_pixel(p, lr_frame, s, B, C, y, x):
     return out[0, s * (y - y0):s * (y - y0) + s, s * (x - x0):s * (x - x0) + s]
 
 
-@pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (720, 1280), 2), ((2, 8, 32), (540, 960), 2)])
+@pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (720, 1280), 2), ((2, 8, 32), (540, 960), 2),
+                                      ((4, 8, 48), (270, 480), 2)])
 def test_full_size_frames_sampled_parity(cfg, hw, n):
     """BASELINE frame sizes (config 3: 720p x3 8x48; config 2: 540p x2 8x32) in the bench's launch
     configuration; sampled output pixels (incl. corners and tile seams) against the oracle."""
@@ -143,7 +144,8 @@ def test_strip_inference_bitexact():
 
 
 # ---------------------------------------------------------------- training
-@pytest.mark.parametrize("cfg,n,p", [((2, 2, 8), 4, 16), ((3, 2, 16), 3, 20), ((2, 8, 48), 2, 48)])
+@pytest.mark.parametrize("cfg,n,p", [((2, 2, 8), 4, 16), ((3, 2, 16), 3, 20), ((2, 8, 48), 2, 48),
+                                     ((4, 2, 16), 3, 16)])
 def test_train_gradient_and_adam_parity(cfg, n, p):
     s, B, C = cfg
     ctx = _ctx(s, B, C, seed=21)
@@ -208,6 +210,38 @@ def test_psnr_gain_matches_oracle():
     assert abs(pa - np.mean(O.psnr_u8(ref_sr, hrp))) < 0.05
 
 
+def test_controller_step_matches_oracle():
+    """sr_controller_step (Algorithm 1 epoch end / validation period): the four PSNRs equal the oracle's PSNR of
+    each model's SR output, and diff / transition / Q_DNN equal oracle.controller.epoch_report on them."""
+    from paper_conf_sigcomm_kimjyyh20_b200 import Controller
+    s, B, C = 2, 2, 8
+    ctx = _ctx(s, B, C, seed=21, lr=5e-3)
+    lrp, hrp, _ = synth_patch_pool(8, s, 40, seed=22, frame_hw=(120, 160))
+    lr_d, hr_d = torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda()
+    for _ in range(2):  # SERVE, PREV and INIT all different
+        for _ in range(3):
+            ctx.train_step(lr_d, hr_d)
+        ctx.publish()
+    params = dict(thresh_sat=100.0, count_sat=0, thresh_online=-100.0, count_online=1)
+    ctrl, ref = Controller(**params), O.Algorithm1(**params)
+    outs = {m: ctx.infer(lr_d, m).cpu().numpy() for m in ("serve", "prev", "init", "bilinear")}
+    q = {m: float(np.mean(O.psnr_u8(o, hrp))) for m, o in outs.items()}
+    for _ in range(3):  # Training -> suspend (diff < 100), then two validation periods with no resume
+        r = ctx.controller_step(ctrl, lr_d, hr_d)
+        rr = O.epoch_report(ref, q["serve"], q["prev"], q["init"], q["bilinear"])
+        for m in q:
+            assert abs(r["psnr_" + m] - q[m]) < 1e-9
+        for k in ("state_before", "event", "state_after"):
+            assert r[k] == rr[k], (k, r[k], rr[k])
+        for k in ("diff", "q_dnn", "q_dnn_prev"):
+            assert abs(r[k] - rr[k]) < 1e-9
+        assert ctrl.patience == ref.patience
+    assert ctrl.state == "suspended" and ctrl.patience == 0
+    # the SERVE PSNR is also the oracle network's within the PSNR bar
+    ref_sr = O.infer_u8(ctx.get_params("serve"), lrp, s, B, C)
+    assert abs(q["serve"] - float(np.mean(O.psnr_u8(ref_sr, hrp)))) < 0.05
+
+
 def test_publish_snapshots():
     s, B, C = 2, 1, 8
     ctx = _ctx(s, B, C, seed=3, lr=1e-2)
@@ -242,7 +276,7 @@ def test_fused_block_equals_unfused(cfg, hw):
     _check_frames(b.cpu().numpy(), ref)
 
 
-@pytest.mark.parametrize("cfg,n,p", [((3, 2, 32), 8, 24), ((2, 3, 48), 6, 48)])
+@pytest.mark.parametrize("cfg,n,p", [((3, 2, 32), 8, 24), ((2, 3, 48), 6, 48), ((4, 2, 32), 4, 24)])
 def test_virtual_batch_training_matches_oracle_and_narrow_path(cfg, n, p):
     """Training on the virtual wide batch (rolling kernels, zero separator columns) vs the per-patch tiled path
     and vs the oracle."""
@@ -263,6 +297,22 @@ def test_virtual_batch_training_matches_oracle_and_narrow_path(cfg, n, p):
         assert abs(lo - ref_loss) / ref_loss < 1e-2
         assert rel_l2(g, ref_g) < 1e-2, rel_l2(g, ref_g)
     assert rel_l2(grads[0][1], grads[1][1]) < 1e-2
+
+
+@pytest.mark.parametrize("cfg,n,p", [((3, 8, 48), 16, 48), ((2, 2, 8), 5, 20), ((4, 2, 32), 3, 40)])
+def test_small_image_batch_virtual_inference(cfg, n, p):
+    """A batch of small square images (validation patches) runs as one virtual wide image with zero separator
+    columns: equal to the oracle within the bar and to the image-by-image path (set_fusion bit 1) within 1 LSB."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=31)
+    lrp, hrp, _ = synth_patch_pool(n, s, s * p, seed=32, frame_hw=(s * p * 3, s * p * 4))
+    lr = torch.from_numpy(lrp).cuda()
+    got = ctx.infer(lr, "serve").cpu().numpy()
+    ctx.set_fusion(3)
+    narrow = ctx.infer(lr, "serve").cpu().numpy()
+    assert np.abs(got.astype(int) - narrow.astype(int)).max() <= 1
+    ref = O.infer_u8(ctx.get_params("serve"), lrp, s, B, C)
+    _check_frames(got, ref, hrp)
 
 
 def test_infer_host_pipeline_equals_device_path():

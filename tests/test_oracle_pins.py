@@ -87,7 +87,7 @@ def test_dgrad_wgrad_match_torch_autograd():
 
 
 # ---------------------------------------------------------------- pixel shuffle
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_pixel_shuffle_matches_torch_and_inverts(s):
     r = _rng(6)
     y = r.standard_normal((2, 4, 5, 3 * s * s))
@@ -98,7 +98,7 @@ def test_pixel_shuffle_matches_torch_and_inverts(s):
 
 
 # ---------------------------------------------------------------- bilinear skip
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_bilinear_matches_torch_interpolate(s):
     v = _rng(7).integers(0, 256, size=(2, 7, 9, 3)).astype(np.uint8)
     ref = torch.nn.functional.interpolate(torch.from_numpy(v.astype(np.float64)).permute(0, 3, 1, 2),
@@ -116,7 +116,7 @@ def test_bilinear_x2_values_are_sixteenths():
 
 
 # ---------------------------------------------------------------- whole net special cases
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_zero_weight_net_is_bilinear_bitexact(s):
     v = _rng(9).integers(0, 256, size=(2, 10, 12, 3)).astype(np.uint8)
     p = np.zeros(num_params(s, 2, 8), np.float32)
@@ -127,7 +127,7 @@ def test_zero_weight_net_is_bilinear_bitexact(s):
     np.testing.assert_array_equal(out, ref)
 
 
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_bias_only_up_conv_is_the_shuffle_permutation(s):
     """Zero input frame (skip = 0), zero weights, up-conv bias b[k] = k/255: HR pixel (s h+i, s w+j, c)
     must equal c s^2 + i s + j exactly (ESPCN/PyTorch channel order)."""
@@ -158,7 +158,7 @@ def test_translation_equivariance_interior():
 
 
 # ---------------------------------------------------------------- gradients: finite differences
-@pytest.mark.parametrize("s", [2, 3])
+@pytest.mark.parametrize("s", [2, 3, 4])
 def test_full_gradient_finite_difference(s):
     B, C = 2, 4
     r = _rng(13)
