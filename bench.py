@@ -281,7 +281,9 @@ def run_ours(args):
             "roofline": {"bound": "tensor", "kernel": dom, "achieved": round(achieved, 1),
                          "peak": sustained, "unit": "TFLOP/s", "frac": round(achieved / sustained, 4),
                          "peak_kind": "measured bf16_tflops_sustained (MEASURED_PEAKS.json)",
-                         "traffic": None, "launches": dv["launches"], "avg_ms": round(dv["ms"] / dv["launches"], 4)},
+                         "traffic": traffic_of(dom, frames), "traffic_unit": "bytes per launch (ncu dram read+write)",
+                         "algorithmic_bytes": round(dv["bytes"] / dv["launches"]),
+                         "launches": dv["launches"], "avg_ms": round(dv["ms"] / dv["launches"], 4)},
             "e2e": {"value": round(fps_e2e, 3), "unit": "frames/s",
                     "h2d_bytes_per_step": int(lr_host.numel()), "d2h_bytes_per_step": int(hr_host.numel() + 4)},
             "gpu_launches": int(launches),
@@ -341,6 +343,19 @@ def run_reference(args):
         "data": "synthetic", "config": {"workload": f"cfg3+cfg4 per step (oracle on a bounded sample)"},
         "cpu_baseline": cb, "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
+
+
+def traffic_of(kernel_class, frames):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu capture (profiles/r01_traffic.json),
+    when it was taken on the same launch shape; else None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
+            t = json.load(f).get(kernel_class)
+    except (OSError, ValueError):
+        return None
+    if not t or t.get("frames") != frames or (t.get("h"), t.get("w")) != (LR_H, LR_W):
+        return None
+    return int(t["dram_read"] + t["dram_write"])
 
 
 def main():
