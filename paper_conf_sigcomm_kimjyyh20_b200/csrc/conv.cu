@@ -21,8 +21,9 @@
 namespace sr {
 
 static constexpr int kConvThreads = 320;   // conv: TMA warp, MMA warp, 2 x 4 epilogue warps
-static constexpr int kWgradThreads = 192;  // wgrad: TMA warp, MMA warp, 4 epilogue warps
+static constexpr int kWgradThreads = 384;  // wgrad: TMA warp, MMA warp, 4 epilogue warps, 6 more for the reduction
 static constexpr int kStages = 2;
+static constexpr int kWgStages = 3;  // wgrad TMA ring depth
 static constexpr int kSmemLimit = 227 * 1024;
 
 int num_sms() {
@@ -457,19 +458,24 @@ cudaError_t launch_conv(int cinp, int coutp, int epi, const void* in, const bf16
 }
 
 // ------------------------------------------------------------------------------------------ weight grad
-// Stage: X tile (R+2) rows x P=TW+2 px, row-planar [row][chunk][px]; dY tile R rows x TW px row-planar.
-// A (MN-major) = X^T: 8-row groups g = dy*CCH + j at stride SBO = P*16 (rows are consecutive planes), K =
-// pixel at 16 B, K-groups LBO = 128.  B (MN-major) = dY: N-groups (co chunks) SBO = TW*16, LBO = 128.
-// D[dx][mt] (128 lanes = 16 groups of 8 (dy,ci) rows, COUTP columns), accumulated over all of this CTA's
-// K (split-K); written as a per-CTA partial, summed by k_wgrad_reduce in CTA order (deterministic).
+// Stage: X tile (R+2) rows x P = TW+2 px and dY tile R rows x TW px, both loaded by TMA in the MN-major
+// SWIZZLE_32B layout [row][16-ch block][px][16 ch] (32-B TMA inner unit: twice the TMA throughput of the
+// 16-B-chunk maps, which would otherwise bound this kernel; scripts/tma_rate.py).
+// A (MN-major) = X^T: M = (dy, ci) atoms of 16 channels a = dy*CB + cb at stride LBO = P*32 (rows are consecutive
+// planes, so the three dy of a tile row are consecutive atoms), K = pixels (8-row groups, SBO = 256; the dx tap
+// is a start-address shift of dx pixel rows).  B (MN-major) = dY: N = co atoms at LBO = TW*32.
+// D[dx][mt] (128 lanes = 8 atoms, COUTP columns), accumulated over all of this CTA's K (split-K) and written as
+// a per-CTA partial.  Then a grid barrier (cooperative launch: all CTAs are co-resident) and every CTA sums its
+// 1/grid slice of the outputs over all partials in CTA order (fixed order -> deterministic), scales and
+// scatters it into the canonical OIHW gradient.  No separate reduction kernel.
 static size_t wgrad_smem(int cinp, int coutp, int R, int TW) {
   const int P = TW + 2;
-  const int cch = cinp / 8, och = coutp / 8;
-  const int n_mt = (3 * cch + 15) / 16;
-  size_t xs = ((size_t)(R + 2) * cch * P * 16 + 1023) / 1024 * 1024;
-  size_t ys = ((size_t)R * och * TW * 16 + 1023) / 1024 * 1024;
-  long over = (long)(16 * n_mt - 3 * cch) * P * 16 + 64;  // rows read past the X tile by padded M-tiles
-  return 1024 + kStages * (xs + ys) + (over > 0 ? (size_t)over : 0) + 256;
+  const int cb = cinp / 16, ob = coutp / 16;
+  const int n_mt = (3 * cb + 7) / 8;
+  size_t xs = ((size_t)(R + 2) * cb * P * 32 + 1023) / 1024 * 1024;
+  size_t ys = ((size_t)R * ob * TW * 32 + 1023) / 1024 * 1024;
+  long over = (long)(8 * n_mt - 3 * cb) * P * 32 + 64;  // atoms read past the X tile by padded M-tiles
+  return 1024 + kWgStages * (xs + ys) + (over > 0 ? (size_t)over : 0) + 256;
 }
 
 WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes) {
@@ -490,9 +496,9 @@ WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem
 template <int CINP, int COUTP>
 __global__ void __launch_bounds__(kWgradThreads, 1)
 k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_dy, const WgradGeom g,
-        float* __restrict__ ws_w, float* __restrict__ ws_b) {
-  constexpr int CCH = CINP / 8, OCH = COUTP / 8;
-  constexpr int NMT = (3 * CCH + 15) / 16;
+        const WgradOut o) {
+  constexpr int CB = CINP / 16, OB = COUTP / 16, OCH = COUTP / 8;
+  constexpr int NMT = (3 * CB + 7) / 8;
   constexpr uint32_t TMEM_NEED = 3 * NMT * COUTP;
   constexpr uint32_t TMEM_COLS = TMEM_NEED <= 32 ? 32 : TMEM_NEED <= 64 ? 64 : TMEM_NEED <= 128 ? 128
                                  : TMEM_NEED <= 256 ? 256 : 512;
@@ -501,26 +507,30 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
 
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], done_bar;
+  constexpr int PER = 9 * CINP * COUTP, STRIDE = PER + COUTP;  // floats per partial
+  __shared__ __align__(8) uint64_t full_bar[kWgStages], empty_bar[kWgStages], done_bar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ float sdb[128 / OCH][COUTP];
 
   const int TW = g.TW, P = g.P, R = g.R;
-  const uint32_t xbox = (uint32_t)(R + 2) * CCH * P * 16, ybox = (uint32_t)R * OCH * TW * 16;  // TMA box bytes
-  const uint32_t xbytes = (xbox + 1023u) & ~1023u;      // dY tile offset inside a stage (128-B TMA alignment)
+  const uint32_t xbox = (uint32_t)(R + 2) * CB * P * 32, ybox = (uint32_t)R * OB * TW * 32;  // TMA box bytes
+  const uint32_t xbytes = (xbox + 1023u) & ~1023u;      // dY tile offset inside a stage (TMA alignment)
   const uint32_t ybytes = (ybox + 1023u) & ~1023u;
   const uint32_t stage_bytes = xbytes + ybytes;
   const int warp = warp_id();
   if (warp == 0 && lane_id() == 0) {
-    for (int s = 0; s < kStages; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 2); }
+    for (int s = 0; s < kWgStages; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 2); }
     mbar_init(&done_bar, 1);
     fence_barrier_init();
   }
+  long long* dbg = g.dbg ? g.dbg + (size_t)blockIdx.x * 8 : nullptr;
+  if (dbg && threadIdx.x == 0) dbg[0] = globaltimer();
   if (warp == 1) tmem_alloc<TMEM_COLS>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
-  pdl_enter();
+  pdl_wait();  // dependents are released only after the grid barrier below (no co-residency deadlock)
   tc_fence_after();
+  if (dbg && threadIdx.x == 0) dbg[1] = clock64();
   const uint32_t tmem = tmem_base_sh;
   const int tiles_xy = g.tiles_x * g.tiles_y;
 
@@ -534,11 +544,15 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
         const int n = u / tiles_xy, rem = u - n * tiles_xy;
         const int ty = rem / g.tiles_x, tx = rem - ty * g.tiles_x;
         mbar_wait(&empty_bar[s], ph ^ 1);
-        mbar_arrive_expect_tx(&full_bar[s], xbox + ybox);
-        uint8_t* base = smem + s * stage_bytes;
-        tma_load_5d(base, &tm_x, &full_bar[s], 0, tx * TW - 1, 0, ty * R - 1, n);
-        tma_load_5d(base + xbytes, &tm_dy, &full_bar[s], 0, tx * TW, 0, ty * R, n);
-        if (++s == kStages) { s = 0; ph ^= 1; }
+        if ((g.exp & 2) && u >= (int)blockIdx.x + kWgStages * (int)gridDim.x) {
+          mbar_arrive(&full_bar[s]);
+        } else {
+          mbar_arrive_expect_tx(&full_bar[s], xbox + ybox);
+          uint8_t* base = smem + s * stage_bytes;
+          tma_load_5d(base, &tm_x, &full_bar[s], 0, tx * TW - 1, 0, ty * R - 1, n);
+          tma_load_5d(base + xbytes, &tm_dy, &full_bar[s], 0, tx * TW, 0, ty * R, n);
+        }
+        if (++s == kWgStages) { s = 0; ph ^= 1; }
       }
     }
     __syncwarp();
@@ -547,36 +561,46 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
       int s = 0;
       uint32_t ph = 0;
       uint32_t acc = 0;
+      long long waited = 0;
       for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
+        const long long tw0 = dbg ? globaltimer() : 0;
         mbar_wait(&full_bar[s], ph);
+        if (dbg) {
+          const long long tw1 = globaltimer();
+          if (u == (int)blockIdx.x) dbg[2] = tw1;
+          else waited += tw1 - tw0;
+        }
         tc_fence_after();
         const uint32_t xb = smem_u32(smem + s * stage_bytes);
         const uint32_t yb = xb + xbytes;
-        const uint64_t a0 = make_desc(xb, 128, P * 16);
-        const uint64_t b0 = make_desc(yb, 128, TW * 16);
+        const uint64_t a0 = make_desc_sw(xb, P * 32, 256, 6);
+        const uint64_t b0 = make_desc_sw(yb, TW * 32, 256, 6);
         for (int r = 0; r < R; ++r) {
           for (int k16 = 0; k16 < TW / 16; ++k16) {
-            const uint32_t boff = (uint32_t)(r * OCH * TW + k16 * 16) * 16u;
+            const uint32_t boff = (uint32_t)(r * OB * TW + k16 * 16) * 32u;
 #pragma unroll
             for (int dx = 0; dx < 3; ++dx) {
 #pragma unroll
               for (int mt = 0; mt < NMT; ++mt) {
-                const uint32_t aoff = (uint32_t)((r * CCH + 16 * mt) * P + k16 * 16 + dx) * 16u;
-                mma_bf16_ss(tmem + (dx * NMT + mt) * COUTP, desc_add(a0, aoff), desc_add(b0, boff), IDESC, acc);
+                const uint32_t aoff = (uint32_t)((r * CB + 8 * mt) * P + k16 * 16 + dx) * 32u;
+                if (!(g.exp & 4))
+                  mma_bf16_ss(tmem + (dx * NMT + mt) * COUTP, desc_add(a0, aoff), desc_add(b0, boff), IDESC, acc);
               }
             }
             acc = 1;
           }
         }
         mma_commit(&empty_bar[s]);
-        if (++s == kStages) { s = 0; ph ^= 1; }
+        if (++s == kWgStages) { s = 0; ph ^= 1; }
       }
       mma_commit(&done_bar);
+      if (dbg) dbg[3] = globaltimer();
     }
     __syncwarp();
-  } else {
+  } else if (warp < 6) {
     // epilogue warps: bias gradient from the dY tiles while the MMAs run, then drain the accumulators.
-    // Thread et owns 8-channel chunk j = et % OCH and pixel subset grp = et / OCH (fixed order -> deterministic).
+    // Thread et owns 8-channel chunk j = et % OCH (block j/2, half j%2) and pixel subset grp = et / OCH (fixed
+    // order -> deterministic).  Half h of pixel p sits at 16 * (h ^ bit 2 of p) (SWIZZLE_32B).
     const int et = threadIdx.x - 64;  // 0..127
     constexpr int NG = 128 / OCH;
     const int j = et % OCH, grp = et / OCH;
@@ -587,11 +611,12 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
     uint32_t ph = 0;
     for (int u = blockIdx.x; u < g.units; u += gridDim.x) {
       mbar_wait(&full_bar[s], ph);
-      if (grp < NG) {
+      if (grp < NG && !(g.exp & 1)) {
         const uint8_t* yt = smem + s * stage_bytes + xbytes;
         for (int r = 0; r < R; ++r) {
           for (int p = grp; p < TW; p += NG) {
-            const uint4 q = *reinterpret_cast<const uint4*>(yt + ((size_t)(r * OCH + j) * TW + p) * 16);
+            const uint32_t off = ((uint32_t)(r * OB + (j >> 1)) * TW + p) * 32u + (((j & 1) ^ ((p >> 2) & 1)) << 4);
+            const uint4 q = *reinterpret_cast<const uint4*>(yt + off);
             const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q);
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
@@ -604,7 +629,7 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
       if (et == 0) mbar_arrive(&empty_bar[s]);
-      if (++s == kStages) { s = 0; ph ^= 1; }
+      if (++s == kWgStages) { s = 0; ph ^= 1; }
     }
     if (grp < NG) {
 #pragma unroll
@@ -614,44 +639,114 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
     if (et < COUTP) {
       float t = 0.f;
       for (int p2 = 0; p2 < NG; ++p2) t += sdb[p2][et];
-      ws_b[(size_t)blockIdx.x * COUTP + et] = t;
+      o.ws[(size_t)blockIdx.x * STRIDE + PER + et] = t;
     }
-    // drain: lane m of M-tile mt = row (16*mt + m/8 -> (dy, j)), ci = 8 j + m % 8
+    // drain: lane m of M-tile mt = atom a = 8 mt + m / 16 -> (dy, cb) = (a / CB, a % CB), ci = 16 cb + m % 16
     mbar_wait(&done_bar, 0);
+    if (dbg && et == 0) dbg[5] = globaltimer();
     tc_fence_after();
     const int quarter = warp & 3;
     const int m = quarter * 32 + lane_id();
-    float* outp = ws_w + (size_t)blockIdx.x * 9 * CINP * COUTP;
+    float* outp = o.ws + (size_t)blockIdx.x * STRIDE;
 #pragma unroll
     for (int dx = 0; dx < 3; ++dx) {
 #pragma unroll
       for (int mt = 0; mt < NMT; ++mt) {
-        const int grp = 16 * mt + m / 8;
-        const bool ok = grp < 3 * CCH;
-        const int dy = grp / CCH, j = grp % CCH;
-        const int ci = 8 * j + (m % 8);
+        const int a = 8 * mt + m / 16;
+        const bool ok = a < 3 * CB;
+        const int dy = a / CB, cb = a % CB;
+        const int ci = 16 * cb + (m % 16);
+        float v[COUTP];  // all columns of this accumulator row: one TMEM round trip
 #pragma unroll
-        for (int c0 = 0; c0 < COUTP; c0 += 16) {
-          float v[16];
-          tmem_ld16(tmem + ((uint32_t)(quarter * 32) << 16) + (dx * NMT + mt) * COUTP + c0, v);
-          tmem_ld_wait();
-          if (ok) {  // 16 consecutive floats: four 16-byte stores
-            float4* o = reinterpret_cast<float4*>(outp + ((size_t)(dy * 3 + dx) * CINP + ci) * COUTP + c0);
+        for (int c0 = 0; c0 < COUTP; c0 += 16)
+          tmem_ld16(tmem + ((uint32_t)(quarter * 32) << 16) + (dx * NMT + mt) * COUTP + c0, v + c0);
+        tmem_ld_wait();
+        if (ok) {  // COUTP consecutive floats: 16-byte stores
+          float4* dst = reinterpret_cast<float4*>(outp + ((size_t)(dy * 3 + dx) * CINP + ci) * COUTP);
 #pragma unroll
-            for (int q = 0; q < 4; ++q) o[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-          }
+          for (int q = 0; q < COUTP / 4; ++q) dst[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
         }
       }
     }
+    if (dbg && et == 0) { dbg[6] = globaltimer(); dbg[4] = clock64(); }
   }
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<TMEM_COLS>(tmem);
+  // ---- grid barrier: every partial written
+  if (threadIdx.x == 0) {
+    volatile unsigned* vgen = o.sync + 1;
+    const unsigned gen = *vgen;
+    __threadfence();
+    const unsigned arrived = atomicAdd(o.sync, 1u);
+    if (arrived == gridDim.x - 1) {
+      atomicExch(o.sync, 0u);
+      __threadfence();
+      atomicAdd(o.sync + 1, 1u);
+    } else {
+      while (*vgen == gen) {
+      }
+    }
+    __threadfence();
+  }
+  __syncthreads();
+  pdl_trigger();
+  if (dbg && threadIdx.x == 0) dbg[7] = globaltimer();
+  // ---- deterministic split-K reduction of this CTA's slice [lo, hi) of float4 outputs over all partials, in
+  // chunks of LC outputs: thread t sums partials q, q + NQ, ... (q = t / LC) of output t % LC, then the NQ group
+  // sums are added in order q = 0..NQ-1.
+  {
+    constexpr int TOT4 = STRIDE / 4;
+    const int G = gridDim.x;
+    const int lo = (int)((long long)blockIdx.x * TOT4 / G), hi = (int)((long long)(blockIdx.x + 1) * TOT4 / G);
+    float4* red = reinterpret_cast<float4*>(smem);  // stage buffers are free now
+    const int t = threadIdx.x;
+    for (int c0 = lo; c0 < hi; c0 += 48) {
+      const int LC = min(48, hi - c0);
+      const int NQ = min(32, kWgradThreads / LC);
+      const int oi = t % LC, q = t / LC;
+      if (q < NQ) {
+        const float4* src = reinterpret_cast<const float4*>(o.ws) + c0 + oi;
+        float4 acc4 = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int p = q; p < G; p += 16 * NQ) {  // 16 independent (predicated) loads in flight, added in order
+          float4 w4[16];
+#pragma unroll
+          for (int k = 0; k < 16; ++k)
+            w4[k] = p + k * NQ < G ? __ldcg(src + (size_t)(p + k * NQ) * TOT4) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+          for (int k = 0; k < 16; ++k) { acc4.x += w4[k].x; acc4.y += w4[k].y; acc4.z += w4[k].z; acc4.w += w4[k].w; }
+        }
+        red[q * LC + oi] = acc4;
+      }
+      __syncthreads();
+      if (t < LC) {
+        float4 s4 = red[t];
+        for (int qq = 1; qq < NQ; ++qq) {
+          const float4 w4 = red[qq * LC + t];
+          s4.x += w4.x; s4.y += w4.y; s4.z += w4.z; s4.w += w4.w;
+        }
+        const float sv[4] = {s4.x, s4.y, s4.z, s4.w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int i = 4 * (c0 + t) + e;
+          if (i < PER) {  // partial index [tap][ci][co]
+            const int co = i % COUTP, rest = i / COUTP;
+            const int ci = rest % CINP, tap = rest / CINP;
+            if (co < o.cout && ci < o.cin) o.gW[(co * o.cin + ci) * 9 + tap] = sv[e] * o.scale;
+          } else {
+            const int co = i - PER;
+            if (co < o.cout) o.gb[co] = sv[e] * o.scale;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
 }
 
 template <int CINP, int COUTP>
-static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, const WgradGeom& g, float* ws_w,
-                                  float* ws_b, size_t smem, int grid, cudaStream_t st) {
+static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, const WgradGeom& g,
+                                  const WgradOut& o, size_t smem, int grid, cudaStream_t st) {
   auto kern = k_wgrad<CINP, COUTP>;
   static size_t configured = 0;
   if (smem > configured) {
@@ -659,19 +754,17 @@ static cudaError_t launch_wgrad_t(const CUtensorMap& tx, const CUtensorMap& ty, 
     if (e != cudaSuccess) return e;
     configured = smem;
   }
-  return launch_k(kern, dim3(grid), dim3(kWgradThreads), smem, st, tx, ty, g, ws_w, ws_b);
+  return launch_coop(kern, dim3(grid), dim3(kWgradThreads), smem, st, tx, ty, g, o);
 }
 
 #define SR_WG_CASE(CI, CO) \
-  if (cinp == CI && coutp == CO) return launch_wgrad_t<CI, CO>(tx, ty, g, ws_w, ws_b, smem, grid, st);
+  if (cinp == CI && coutp == CO) return launch_wgrad_t<CI, CO>(tx, ty, g, o, smem, grid, st);
 
-cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, float* ws_w,
-                         float* ws_b, size_t smem, int grid, cudaStream_t st) {
+cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, const WgradOut& o,
+                         size_t smem, int grid, cudaStream_t st) {
   CUtensorMap tx, ty;
-  if (make_act_tmap(&tx, x, g.N, g.H, g.W, cinp, g.P, g.R + 2, cinp / 8, ROW_CHUNK_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
-  if (make_act_tmap(&ty, dy, g.N, g.H, g.W, coutp, g.TW, g.R, coutp / 8, ROW_CHUNK_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
+  if (make_act_tmap_sw32(&tx, x, g.N, g.H, g.W, cinp, g.P, g.R + 2) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (make_act_tmap_sw32(&ty, dy, g.N, g.H, g.W, coutp, g.TW, g.R) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   SR_WG_CASE(16, 16) SR_WG_CASE(16, 32) SR_WG_CASE(16, 48) SR_WG_CASE(16, 64)
   SR_WG_CASE(32, 16) SR_WG_CASE(32, 32) SR_WG_CASE(32, 48) SR_WG_CASE(32, 64)
   SR_WG_CASE(48, 16) SR_WG_CASE(48, 32) SR_WG_CASE(48, 48)

@@ -23,8 +23,9 @@
 // Per conv the out-row sequence of a piece has n_in + 2 entries (local q = -1 .. n_in); q in [1, n_in-2] are
 // the rows that are kept.
 //
-// Warps: 0 TMA producer, 1 TMEM alloc + MMA issuer (conv1 runs three rows ahead of conv2), 2..5 conv1
-// epilogue, 6..9 conv2 epilogue (residual from global/L2, rows -> smem -> TMA store).  The kernel is bound by the
+// Warps: 0 TMA producer, 1 TMEM alloc + conv1 MMA issuer, 10 conv2 MMA issuer (conv2 trails conv1 by three rows;
+// two issuers so that one waiting on a barrier does not starve the tensor pipe), 2..5 conv1 epilogue, 6..9 conv2
+// epilogue (residual from global/L2, rows -> smem -> TMA store).  The kernel is bound by the
 // 128 B/clk shared-memory port: per row-step the MMAs read ~155 KB of operands (A 4 KB + B 4.5 KB per MMA) and the
 // TMA/epilogue traffic adds ~49 KB (clock64 timeline, scripts/bench_block.py).
 #include <cuda.h>
@@ -36,7 +37,7 @@
 
 namespace sr {
 
-static constexpr int kBlkThreads = 320;
+static constexpr int kBlkThreads = 352;  // + warp 10: the conv2 MMA issuer
 static constexpr int kBlkTW = 126;  // output pixels per strip
 static constexpr int kBlkNF = 4;    // f-row ring
 static constexpr int kBlkNT = 3;    // t-row ring
@@ -60,7 +61,10 @@ __global__ void __launch_bounds__(kBlkThreads, 1)
 k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
            const float* __restrict__ b2, const bf16* __restrict__ fres, bf16* __restrict__ outp, const int N,
-           const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg) {
+           const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg,
+           const int exp) {
+  // exp (benchmarking experiments only, results wrong when set): 1 no residual load, 2 no output store, 4 no t
+  // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads
   // tsave (nullable): also write t = ReLU(conv1(f) + b1) to global (training saves it for the backward pass).
   // sep > 0: columns with col % sep in {0, sep-1} are separators of the virtual training batch -> t and out = 0.
   // dbg (benchmarking only, CTA 0): clock64 stamps [event][step], events: 0 f issued, 1 conv1 step issued,
@@ -68,7 +72,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 #define SR_DBG(ev, idx) \
   if (dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) dbg[(ev) * 256 + (idx)] = clock64();
   // more MMA-thread stamps: 7 step start, 8 conv1 blocks acquired, 9 f row landed, 10 conv2 part start,
-  // 11 conv2 blocks acquired, 12 t row ready
+  // 11 conv2 blocks acquired, 12 t row ready, 13 epi1 freed a block (by row), 14 epi2 freed a block (by row)
   using Cfg = BlkCfg<C>;
   constexpr int CCH = Cfg::CCH, RB = Cfg::RB;
   constexpr uint32_t PLANE = Cfg::PLANE, ROWB = Cfg::ROWB, OUTB = Cfg::OUTB;
@@ -149,55 +153,66 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     }
     __syncwarp();
   } else if (warp == 1) {
-    // ===================== MMA issuer: conv1 step st (f row st), then conv2 step st-3 (t row st-3) ===============
+    // ===================== conv1 MMA issuer: step st consumes f row st =====================
+    // (conv2 has its own issuer, warp 10: while one thread waits on a barrier the other keeps the tensor pipe fed)
     if (elect_one()) {
       mbar_wait(&w_bar, 0);
       const uint64_t bd1 = make_desc(smem_u32(sW1), Cfg::N * 16, 128);
-      const uint64_t bd2 = make_desc(smem_u32(sW2), Cfg::N * 16, 128);
-      int fs = 0, ts = 0;
-      uint32_t fph = 0, tph = 0;
-      long long G1 = 0, G2 = 0, acq1 = 0, acq2 = 0;  // out-row sequences (first row of the piece) / blocks acquired
+      int fs = 0;
+      uint32_t fph = 0;
+      long long G1 = 0, acq1 = 0;  // out-row sequence (first row of the piece) / blocks acquired
       SR_PIECE_BEGIN
-      for (int st = 0; st <= n_f + 2; ++st) {
+      for (int st = 0; st < n_f; ++st) {
         SR_DBG(7, st)
-        if (st < n_f) {
-          const long long g = G1 + st;
-          for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
-          SR_DBG(8, st)
-          mbar_wait(&f_full[fs], fph);
-          SR_DBG(9, st)
-          tc_fence_after();
+        const long long g = G1 + st;
+        for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
+        SR_DBG(8, st)
+        mbar_wait(&f_full[fs], fph);
+        SR_DBG(9, st)
+        tc_fence_after();
+        if (!(exp & 32))
           ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, PLANE);
-          mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
-          mma_commit(&f_empty[fs]);
-          if (st == n_f - 1) {                      // the last two rows of the piece receive nothing more
-            mma_commit(&r1_ready[ring_idx<RB>(g + 1)]);
-            mma_commit(&r1_ready[ring_idx<RB>(g + 2)]);
-          }
-          SR_DBG(1, st)
-          if (++fs == kBlkNF) { fs = 0; fph ^= 1; }
+        mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
+        mma_commit(&f_empty[fs]);
+        if (st == n_f - 1) {                      // the last two rows of the piece receive nothing more
+          mma_commit(&r1_ready[ring_idx<RB>(g + 1)]);
+          mma_commit(&r1_ready[ring_idx<RB>(g + 2)]);
         }
-        const int k = st - 3;
-        SR_DBG(10, st)
-        if (k >= 0 && k < n_t) {
-          const long long g = G2 + k;
-          for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
-          SR_DBG(11, st)
-          mbar_wait(&t_full[ts], tph);
-          SR_DBG(12, st)
-          tc_fence_after();
-          ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, PLANE);
-          mma_commit(&r2_ready[ring_idx<RB>(g)]);
-          mma_commit(&t_empty[ts]);
-          if (k == n_t - 1) {
-            mma_commit(&r2_ready[ring_idx<RB>(g + 1)]);
-            mma_commit(&r2_ready[ring_idx<RB>(g + 2)]);
-          }
-          SR_DBG(2, k)
-          if (++ts == kBlkNT) { ts = 0; tph ^= 1; }
-        }
+        SR_DBG(1, st)
+        if (++fs == kBlkNF) { fs = 0; fph ^= 1; }
       }
       G1 += n_f + 2;
+      SR_PIECE_END
+    }
+    __syncwarp();
+  } else if (warp == 10) {
+    // ===================== conv2 MMA issuer: step k consumes t row k =====================
+    if (elect_one()) {
+      mbar_wait(&w_bar, 0);
+      const uint64_t bd2 = make_desc(smem_u32(sW2), Cfg::N * 16, 128);
+      int ts = 0;
+      uint32_t tph = 0;
+      long long G2 = 0, acq2 = 0;
+      SR_PIECE_BEGIN
+      for (int k = 0; k < n_t; ++k) {
+        SR_DBG(10, k + 3)
+        const long long g = G2 + k;
+        for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
+        SR_DBG(11, k + 3)
+        mbar_wait(&t_full[ts], tph);
+        SR_DBG(12, k + 3)
+        tc_fence_after();
+        if (!(exp & 16))
+          ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, PLANE);
+        mma_commit(&r2_ready[ring_idx<RB>(g)]);
+        mma_commit(&t_empty[ts]);
+        if (k == n_t - 1) {
+          mma_commit(&r2_ready[ring_idx<RB>(g + 1)]);
+          mma_commit(&r2_ready[ring_idx<RB>(g + 2)]);
+        }
+        SR_DBG(2, k)
+        if (++ts == kBlkNT) { ts = 0; tph ^= 1; }
+      }
       G2 += n_t + 2;
       SR_PIECE_END
     }
@@ -234,11 +249,23 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       tc_fence_after();
       if (warp == 2 && lane_id() == 0) { SR_DBG(3, q + 1) }
       float v[C];
-      ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+      if (exp & 72) {
+        if (!(exp & 64)) {
+#pragma unroll
+          for (int c0 = 0; c0 < C; c0 += 8) tmem_ld8(ring1 + lane_off + b * C + c0, v + c0);
+          tmem_ld_wait();
+        } else {
+#pragma unroll
+          for (int c0 = 0; c0 < C; ++c0) v[c0] = (float)c0;
+        }
+      } else {
+        ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+      }
       tc_fence_before();
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&r1_free[b]);
-      if (emit) {
+      if (warp == 2 && lane_id() == 0) { SR_DBG(13, q + 1) }
+      if (emit && !(exp & 4)) {
         uint8_t* dst = sT + ts * ROWB + m * 16;
 #pragma unroll
         for (int j = 0; j < CCH; ++j) {
@@ -254,6 +281,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           if (save_col && q >= 2 && q <= n_f - 3)  // t rows y0 .. y1-1 belong to this piece
             reinterpret_cast<uint4*>(tsave + ((((size_t)n * H + trow) * W) + tcol) * C)[j] = u;
         }
+      }
+      if (emit) {
         fence_proxy_async_smem();
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&t_full[ts]);
@@ -263,7 +292,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     }
     G += n_f + 2;
     SR_PIECE_END
-  } else {
+  } else if (warp < 10) {
     // ===================== conv2 epilogue: drain finished rows -> + residual f -> smem -> TMA store ==========
     const int quarter = warp & 3;
     const int m = quarter * 32 + lane_id();
@@ -288,7 +317,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       const bool emit = q >= 1 && q <= n_t - 2;
       const int r = y0 - 1 + q;
       uint4 res[C / 8];
-      if (emit && lane_ok) {
+      if (emit && lane_ok && !(exp & 1)) {
         const uint4* rp = reinterpret_cast<const uint4*>(fres + ((((size_t)n * H + r) * W) + x0 + m) * C);
 #pragma unroll
         for (int j = 0; j < C / 8; ++j) res[j] = __ldg(rp + j);
@@ -297,13 +326,29 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
       tc_fence_after();
       if (warp == 6 && lane_id() == 0) { SR_DBG(5, q + 1) }
+      if (exp & 1) {
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) res[j] = make_uint4(0, 0, 0, 0);
+      }
       float v[C];
-      ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+      if (exp & 72) {
+        if (!(exp & 64)) {
+#pragma unroll
+          for (int c0 = 0; c0 < C; c0 += 8) tmem_ld8(ring2 + lane_off + b * C + c0, v + c0);
+          tmem_ld_wait();
+        } else {
+#pragma unroll
+          for (int c0 = 0; c0 < C; ++c0) v[c0] = (float)c0;
+        }
+      } else {
+        ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+      }
       tc_fence_before();
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&r2_free[b]);
+      if (warp == 6 && lane_id() == 0) { SR_DBG(14, q + 1) }
       if (emit) {
-        if (lane_ok) {
+        if (lane_ok && !(exp & 2)) {
           uint4* orow = reinterpret_cast<uint4*>(sO + os * OUTB + m * C * 2);
 #pragma unroll
           for (int j = 0; j < C / 8; ++j) {
@@ -325,7 +370,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         }
         fence_proxy_async_smem();
         named_bar_sync(2, 128);
-        if (leader) {
+        if (leader && !(exp & 2)) {
           tma_store_4d(&tm_out, sO + os * OUTB, 0, x0, r, n);
           bulk_commit();
           bulk_wait_read<kBlkNO - 2>();
@@ -349,7 +394,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 template <int C>
 static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, const bf16* w1, const bf16* w2,
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
-                                  int grid, bf16* tsave, int sep, long long* dbg, cudaStream_t st) {
+                                  int grid, bf16* tsave, int sep, long long* dbg, int exp, cudaStream_t st) {
   auto kern = k_resblock<C>;
   static bool configured = false;
   if (!configured) {
@@ -358,7 +403,7 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
     configured = true;
   }
   return launch_k(kern, dim3(grid), dim3(kBlkThreads), BlkCfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, out, N, H, W,
-                  tsave, sep, dbg);
+                  tsave, sep, dbg, exp);
 }
 
 bool resblock_supported(int cp, int W) {
@@ -371,16 +416,16 @@ bool resblock_supported(int cp, int W) {
 
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st, long long* dbg,
-                            bf16* tsave, int sep) {
+                            bf16* tsave, int sep, int exp) {
   CUtensorMap tf, to;
   if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (make_row_tmap(&to, out, N, H, W, cp, kBlkTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   const long long rows = (long long)N * ((W + kBlkTW - 1) / kBlkTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
-  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
-  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
-  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, st);
+  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
+  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
+  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
   return cudaErrorNotSupported;
 }
 

@@ -114,47 +114,6 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
   launch_k(k_pack_weights, grid, dim3(256), 0, st, params, convs_dev, nconv, wf, wd, wo, wdo, bias);
 }
 
-// --------------------------------------------------------------- wgrad split-K reduction (deterministic)
-// grad W[co][ci][ky][kx] = scale * sum_{cta in order} ws_w[cta][t][ci][co];  grad b[co] = scale * sum ws_b[cta][co]
-__global__ void k_wgrad_reduce(const float* __restrict__ ws_w, const float* __restrict__ ws_b, int nparts,
-                               int cinp, int coutp, int cin, int cout, float scale, float* __restrict__ gW,
-                               float* __restrict__ gb) {
-  pdl_enter();
-  // block = 32 outputs x 8 partial groups; group gi sums partials gi, gi+8, ... (fixed order), then the 8 group
-  // sums are added in order 0..7 -> deterministic.
-  __shared__ float part[8][33];
-  const int per = 9 * cinp * coutp;
-  const int i = blockIdx.x * 32 + threadIdx.x;
-  const int gi = threadIdx.y;
-  float s = 0.f;
-  if (i < per) {
-    for (int p = gi; p < nparts; p += 8) s += ws_w[(size_t)p * per + i];
-  } else if (i < per + coutp) {
-    for (int p = gi; p < nparts; p += 8) s += ws_b[(size_t)p * coutp + (i - per)];
-  }
-  part[gi][threadIdx.x] = s;
-  __syncthreads();
-  if (gi == 0) {
-    float t = 0.f;
-#pragma unroll
-    for (int q = 0; q < 8; ++q) t += part[q][threadIdx.x];
-    if (i < per) {
-      const int co = i % coutp, rest = i / coutp;
-      const int ci = rest % cinp, tap = rest / cinp;
-      if (co < cout && ci < cin) gW[(co * cin + ci) * 9 + tap] = t * scale;
-    } else if (i < per + coutp) {
-      const int co = i - per;
-      if (co < cout) gb[co] = t * scale;
-    }
-  }
-}
-
-void launch_wgrad_reduce(const float* ws_w, const float* ws_b, int nparts, int cinp, int coutp, int cin, int cout,
-                         float scale, float* gW, float* gb, cudaStream_t st) {
-  int tot = 9 * cinp * coutp + coutp;
-  launch_k(k_wgrad_reduce, dim3((tot + 31) / 32), dim3(32, 8), 0, st, ws_w, ws_b, nparts, cinp, coutp, cin, cout, scale, gW, gb);
-}
-
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
 // m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;  p -= (lr / bc1) * m / (sqrt(v) / sqrt(bc2) + eps),  g = s * grad
 // t and the bias corrections live on the device (k_adam_prep) so the step is replayable from a CUDA graph.

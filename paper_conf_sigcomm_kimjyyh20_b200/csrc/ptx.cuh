@@ -54,6 +54,12 @@ __device__ __forceinline__ bool mbar_try_wait(uint32_t addr, uint32_t phase) {
 }
 // Blocking wait on a phase parity.  A pipeline bug would otherwise hang the GPU: after ~2^35 cycles
 // (~17 s) the wait traps so the launch fails with an error instead.
+__device__ __forceinline__ long long globaltimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
   const uint32_t addr = smem_u32(bar);
   if (mbar_try_wait(addr, phase)) return;
@@ -142,6 +148,10 @@ __device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint
   d |= static_cast<uint64_t>(1) << 46;  // version = 1 (Blackwell)
   // base_offset = 0, lbo_mode = 0, layout_type (bits 61-63) = 0 = SWIZZLE_NONE
   return d;
+}
+// same with a layout type (bits 61-63): 0 SWIZZLE_NONE, 2 SWIZZLE_128B, 4 SWIZZLE_64B, 6 SWIZZLE_32B
+__device__ __forceinline__ uint64_t make_desc_sw(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout) {
+  return make_desc(saddr, lbo, sbo) | (static_cast<uint64_t>(layout & 7u) << 61);
 }
 // descriptors differ only in the start-address field: add (bytes >> 4)
 __device__ __forceinline__ uint64_t desc_add(uint64_t d, uint32_t bytes) { return d + (bytes >> 4); }

@@ -43,8 +43,9 @@ struct sr_ctx {
   bf16 *tx16 = nullptr, *tg = nullptr, *tdy = nullptr, *tdg = nullptr, *tdfa = nullptr, *tdfb = nullptr,
        *tdt = nullptr;
   std::vector<bf16*> tf, tts;
-  float *ws_w = nullptr, *ws_b = nullptr;
-  size_t ws_w_elems = 0, ws_b_elems = 0;
+  float* ws_w = nullptr;       // wgrad split-K partials [grid][9 cinp coutp + coutp]
+  size_t ws_w_elems = 0;
+  unsigned* wg_sync = nullptr; // wgrad grid barrier {count, generation}
   double* loss_sum = nullptr;
   long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t
   float* adam_scal = nullptr;     // device: lr/bc1, 1/sqrt(bc2)
@@ -199,23 +200,29 @@ static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N
   size_t smem = 0;
   WgradGeom g = make_wgrad_geom(N, H, W, d.cinp, d.coutp, &smem);
   int grid = std::min(g.units, num_sms());
-  size_t need_w = (size_t)grid * 9 * d.cinp * d.coutp, need_b = (size_t)grid * d.coutp;
+  size_t need_w = (size_t)grid * (9 * d.cinp * d.coutp + d.coutp);
   if (need_w > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, need_w)); ctx->ws_w_elems = need_w; }
-  if (need_b > ctx->ws_b_elems) { CK(dalloc(&ctx->ws_b, need_b)); ctx->ws_b_elems = need_b; }
+  if (!ctx->wg_sync) {
+    CK(dalloc(&ctx->wg_sync, 2));
+    CK(cudaMemsetAsync(ctx->wg_sync, 0, 2 * sizeof(unsigned), st));
+  }
   if (ctx->timing) {
     const double px = (double)N * H * W;
     tmark_begin(ctx, "wgrad_" + std::to_string(d.cinp) + "x" + std::to_string(d.coutp),
                 2.0 * 9 * d.cinp * d.coutp * px, px * 2.0 * (d.cinp + d.coutp), st);
   }
-  cudaError_t e = launch_wgrad(d.cinp, d.coutp, x, dy, g, ctx->ws_w, ctx->ws_b, smem, grid, st);
+  WgradOut o{};
+  o.ws = ctx->ws_w;
+  o.sync = ctx->wg_sync;
+  o.gW = ctx->grad + d.w_off;
+  o.gb = o.gW + (size_t)d.cout * d.cin * 9;
+  o.cin = d.cin;
+  o.cout = d.cout;
+  o.scale = scale;
+  cudaError_t e = launch_wgrad(d.cinp, d.coutp, x, dy, g, o, smem, grid, st);
   tmark_end(ctx, st);
   ctx->launches++;
   if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("wgrad launch: ") + cudaGetErrorString(e));
-  float* gW = ctx->grad + d.w_off;
-  float* gb = gW + (size_t)d.cout * d.cin * 9;
-  launch_wgrad_reduce(ctx->ws_w, ctx->ws_b, grid, d.cinp, d.coutp, d.cin, d.cout, scale, gW, gb, st);
-  ctx->launches++;
-  CKL();
   return SR_OK;
 }
 
@@ -661,7 +668,7 @@ void sr_destroy(sr_ctx* ctx) {
   cudaDeviceSynchronize();
   void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->x16, ctx->f0,
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
-                  ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->ws_b, ctx->loss_sum, ctx->counters,
+                  ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
                   ctx->adam_scal, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse};
   for (void* p : ptrs)
@@ -1196,19 +1203,21 @@ sr_status sr_test_wgrad(const void* x_dev, const void* dy_dev, int n, int h, int
   size_t smem = 0;
   WgradGeom g = make_wgrad_geom(n, h, w, cinp, coutp, &smem);
   int grid = std::min(g.units, num_sms());
-  float *ws_w = nullptr, *ws_b = nullptr, *gout = nullptr;
+  float *ws = nullptr, *gout = nullptr;
+  unsigned* sync = nullptr;
   const size_t np = (size_t)cout * cin * 9 + cout;
-  if (cudaMalloc(&ws_w, (size_t)grid * 9 * cinp * coutp * 4) || cudaMalloc(&ws_b, (size_t)grid * coutp * 4) ||
-      cudaMalloc(&gout, np * 4))
+  if (cudaMalloc(&ws, (size_t)grid * (9 * cinp * coutp + coutp) * 4) || cudaMalloc(&gout, np * 4) ||
+      cudaMalloc(&sync, 8))
     return SR_E_NOMEM;
-  cudaError_t e = launch_wgrad(cinp, coutp, (const bf16*)x_dev, (const bf16*)dy_dev, g, ws_w, ws_b, smem, grid, st);
-  launch_wgrad_reduce(ws_w, ws_b, grid, cinp, coutp, cin, cout, 1.0f, gout, gout + (size_t)cout * cin * 9, st);
+  cudaMemsetAsync(sync, 0, 8, st);
+  WgradOut o{ws, sync, gout, gout + (size_t)cout * cin * 9, cin, cout, 1.0f};
+  cudaError_t e = launch_wgrad(cinp, coutp, (const bf16*)x_dev, (const bf16*)dy_dev, g, o, smem, grid, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
   std::vector<float> h_(np);
   cudaMemcpy(h_.data(), gout, np * 4, cudaMemcpyDeviceToHost);
   memcpy(dw_host, h_.data(), (size_t)cout * cin * 9 * 4);
   memcpy(db_host, h_.data() + (size_t)cout * cin * 9, cout * 4);
-  cudaFree(ws_w); cudaFree(ws_b); cudaFree(gout);
+  cudaFree(ws); cudaFree(gout); cudaFree(sync);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
 

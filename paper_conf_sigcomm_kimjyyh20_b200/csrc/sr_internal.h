@@ -54,10 +54,24 @@ struct WgradGeom {
   int N, H, W;
   int TW, R, P;
   int tiles_x, tiles_y, units;
+  long long* dbg;  // optional per-CTA globaltimer stamps [grid][8] (benchmarking only)
+  int exp;         // benchmarking experiments (results wrong): bit 0 skip bias-grad reads, bit 1 no TMA after the
+                   // first ring fill, bit 2 skip the MMAs
+};
+// Where the weight gradient goes: per-CTA split-K partials ws [grid][9*cinp*coutp + coutp] (fp32), a grid
+// barrier {count, generation} (zero-initialised once, reusable), and the final
+// gW[co][ci][3][3] = scale * sum_cta partial, gb[co] likewise (canonical OIHW, unpadded cin x cout).
+struct WgradOut {
+  float* ws;
+  unsigned* sync;
+  float* gW;
+  float* gb;
+  int cin, cout;
+  float scale;
 };
 WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes);
-cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, float* ws_w,
-                         float* ws_b, size_t smem, int grid, cudaStream_t st);
+cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, const WgradOut& o,
+                         size_t smem, int grid, cudaStream_t st);
 
 int num_sms();
 

@@ -1,11 +1,20 @@
 // Test-only exports: validate the tcgen05 descriptor encodings and the 5-D TMA layouts the conv kernels
 // rely on, and micro-benchmark tcgen05.mma issue rate at the small N this network has.
+#include <cstdlib>
 #include "ptx.cuh"
 #include "tmap.h"
 #include "sr_internal.h"
 #include "kernels.h"
 
 namespace sr {
+
+// MN-major SWIZZLE_32B canonical offset of element (mn, k) of an [MN][K] operand: atom (mn / 16) at stride K*32,
+// K row k at 32 B (8-row groups of 256 B), the two 16-B halves of a row XOR-swapped by address bit 7 (Swizzle<1,4,3>).
+__device__ __forceinline__ uint32_t sw32_mn_off(int mn, int k, int K, int pad) {
+  const uint32_t base = (uint32_t)(mn / 16) * (uint32_t)(K * 32 + pad);
+  const uint32_t h = (uint32_t)((mn % 16) / 8) ^ (uint32_t)(((base + (uint32_t)k * 32u) >> 7) & 1);
+  return base + (uint32_t)k * 32u + h * 16u + (uint32_t)(mn % 8) * 2u;
+}
 
 // One CTA: D[128 x N] = A[128 x K] * B[N x K]^T.  A/B given row-major in global (K contiguous).
 // a_mn: stage A in the MN-major canonical layout instead of K-major (B likewise with b_mn).
@@ -18,7 +27,7 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
   __shared__ uint64_t bar;
   __shared__ uint32_t tmem_base;
   const int M = 128;
-  const int MA = M + 8;  // extra rows so shifted reads stay inside the buffer
+  const int MA = M + 16;  // extra rows so shifted reads stay inside the buffer
   uint8_t* sA = smem;
   uint8_t* sB = smem + MA * K * 2;
   // ---- stage A
@@ -27,14 +36,16 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
     __nv_bfloat16 v = m < M ? A[m * K + k] : __float2bfloat16(0.f);
     uint32_t off;
     if (!a_mn) off = (k / 8) * (MA * 16) + m * 16 + (k % 8) * 2;          // K-major: LBO = MA*16, SBO = 128
-    else off = (m / 8) * (K * 16) + k * 16 + (m % 8) * 2;                  // MN-major: SBO = K*16, LBO = 128
+    else if (a_mn == 1) off = (m / 8) * (K * 16) + k * 16 + (m % 8) * 2;  // MN-major: SBO = K*16, LBO = 128
+    else off = sw32_mn_off(m, k, K, shift >= 4 ? 64 : 0);                  // MN-major SWIZZLE_32B
     *reinterpret_cast<__nv_bfloat16*>(sA + off) = v;
   }
   for (int i = threadIdx.x; i < N * K; i += blockDim.x) {
     int n = i / K, k = i % K;
     uint32_t off;
     if (!b_mn) off = (k / 8) * (N * 16) + n * 16 + (k % 8) * 2;
-    else off = (n / 8) * (K * 16) + k * 16 + (n % 8) * 2;
+    else if (b_mn == 1) off = (n / 8) * (K * 16) + k * 16 + (n % 8) * 2;
+    else off = sw32_mn_off(n, k, K, 0);
     *reinterpret_cast<__nv_bfloat16*>(sB + off) = B[i];
   }
   fence_proxy_async_smem();
@@ -45,14 +56,21 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
   tc_fence_after();
   const uint32_t tmem = tmem_base;
   if (threadIdx.x == 0) {
-    const uint32_t idesc = make_idesc(128, N, a_mn, b_mn);
+    const uint32_t idesc = make_idesc(128, N, a_mn ? 1 : 0, b_mn ? 1 : 0);
     const uint32_t a0 = smem_u32(sA), b0 = smem_u32(sB);
-    uint64_t adesc = a_mn ? make_desc(a0, 128, K * 16) : make_desc(a0, MA * 16, 128);
-    uint64_t bdesc = b_mn ? make_desc(b0, 128, K * 16) : make_desc(b0, N * 16, 128);
+    // SWIZZLE_32B MN-major: atoms of 16 MN elements x 8 K rows (256 B); mode 2 puts the MN-atom stride (K*32) in
+    // LBO and the 8-row K-group stride (256) in SBO, mode 3 the other way round (to pin the encoding)
+    auto sw_desc = [&](uint32_t base, int mode, int pad) {
+      return mode == 2 ? make_desc_sw(base, K * 32 + pad, 256, 6) : make_desc_sw(base, 256, K * 32 + pad, 6);
+    };
+    uint64_t adesc = a_mn >= 2 ? sw_desc(a0, a_mn, shift >= 4 ? 64 : 0)
+                               : a_mn ? make_desc(a0, 128, K * 16) : make_desc(a0, MA * 16, 128);
+    uint64_t bdesc = b_mn >= 2 ? sw_desc(b0, b_mn, 0) : b_mn ? make_desc(b0, 128, K * 16) : make_desc(b0, N * 16, 128);
     const int ksteps = K / 16;
-    // one K step = 16 elements = 2 chunks: K-major advances by 2*LBO, MN-major by 2 LBO-groups (256 B)
-    const uint32_t a_step = a_mn ? 256 : 2 * MA * 16;
-    const uint32_t b_step = b_mn ? 256 : 2 * N * 16;
+    // one K step = 16 elements = 2 chunks: K-major advances by 2*LBO, MN-major by 2 LBO-groups (256 B),
+    // MN-major SWIZZLE_32B by 16 rows of 32 B (512 B)
+    const uint32_t a_step = a_mn >= 2 ? 512 : a_mn ? 256 : 2 * MA * 16;
+    const uint32_t b_step = b_mn >= 2 ? 512 : b_mn ? 256 : 2 * N * 16;
     long long t0 = clock64();
     if (reps > 0 && ksteps == 4) {
       // throughput mode: descriptors precomputed, 4 MMAs per iteration fully unrolled; shift=2 alternates
@@ -60,14 +78,26 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
       uint64_t ad[4], bd[4];
 #pragma unroll
       for (int ks = 0; ks < 4; ++ks) {
-        ad[ks] = desc_add(adesc, ks * a_step + (shift == 1 ? 16u * (ks % 3) : 0u));
+        ad[ks] = desc_add(adesc, ks * a_step + (shift == 1 ? 16u * (ks % 3) : (shift == 3 || shift == 5) ? 32u * (ks % 3) : 0u));
         bd[ks] = desc_add(bdesc, ks * b_step);
       }
-      const uint32_t d1 = shift == 2 ? tmem + 256 - N : tmem;
+      const uint32_t d1 = shift == 2 ? tmem + 256 - N : tmem;  // (shift 3: 32-B row shift; 4: atom pad; 5: both)
       mma_bf16_ss(tmem, ad[0], bd[0], idesc, 0u);
-      for (int r = 0; r < reps; ++r) {
+      if (shift == 6) {  // a ~40-cycle gap between MMAs: does the issuing thread overlap with MMA execution?
+        for (int r = 0; r < reps; ++r) {
 #pragma unroll
-        for (int ks = 0; ks < 4; ++ks) mma_bf16_ss((ks & 1) ? d1 : tmem, ad[ks], bd[ks], idesc, 1u);
+          for (int ks = 0; ks < 4; ++ks) {
+            const long long tg = clock64();
+            while (clock64() - tg < 40) {
+            }
+            mma_bf16_ss(tmem, ad[ks], bd[ks], idesc, 1u);
+          }
+        }
+      } else {
+        for (int r = 0; r < reps; ++r) {
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks) mma_bf16_ss((ks & 1) ? d1 : tmem, ad[ks], bd[ks], idesc, 1u);
+        }
       }
     } else {
       int total = reps > 0 ? reps : 1;
@@ -117,14 +147,78 @@ __global__ void k_test_tma(const __grid_constant__ CUtensorMap tm, uint8_t* out,
   for (uint32_t i = threadIdx.x; i < bytes; i += blockDim.x) out[i] = smem[i];
 }
 
+// TMA load throughput microbenchmark: every CTA streams boxes of a [1][H][W][Cp] activation (wgrad-like tiles:
+// 66 px x 6 rows x all channels) into a 4-stage ring, one thread issuing, `passes` sweeps over all tiles.
+// mode 0: 5-D ROW_CHUNK_PIX box (16-B innermost); mode 1: 5-D CHUNK_ROW_PIX; mode 2: 4-D plain box (Cp*2-B inner).
+__global__ void k_bench_tma(const __grid_constant__ CUtensorMap tm, int mode, int H, int W, int passes,
+                            uint32_t box_bytes) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t bar[4];
+  if (threadIdx.x != 0) return;
+  for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
+  fence_barrier_init();
+  const uint32_t stride = (box_bytes + 1023u) & ~1023u;
+  const int tx = (W + 63) / 64, ty = (H + 3) / 4, units = tx * ty;
+  int k = 0;
+  for (int pss = 0; pss < passes; ++pss) {
+    for (int u = blockIdx.x; u < units; u += gridDim.x, ++k) {
+      const int s = k & 3;
+      if (k >= 4) mbar_wait(&bar[s], ((k >> 2) - 1) & 1);
+      mbar_arrive_expect_tx(&bar[s], box_bytes);
+      const int x0 = (u % tx) * 64 - 1, y0 = (u / tx) * 4 - 1;
+      uint8_t* dst = smem + s * stride;
+      if (mode == 0) tma_load_5d(dst, &tm, &bar[s], 0, x0, 0, y0, 0);
+      else if (mode == 1) tma_load_5d(dst, &tm, &bar[s], 0, x0, y0, 0, 0);
+      else tma_load_4d(dst, &tm, &bar[s], 0, x0, y0, 0);
+    }
+  }
+  for (int j = (k > 4 ? k - 4 : 0); j < k; ++j) mbar_wait(&bar[j & 3], (j >> 2) & 1);
+}
+
 }  // namespace sr
 
 using namespace sr;
 
+extern "C" int sr_bench_tma(const void* act, int H, int W, int Cp, int mode, int grid, int passes, float* ms_out,
+                            void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  CUtensorMap tm;
+  uint32_t bytes = 66u * 6u * (uint32_t)Cp * 2u;
+  if (mode == 0 || mode == 1) {
+    if (make_act_tmap(&tm, act, 1, H, W, Cp, 66, 6, Cp / 8, mode == 0 ? ROW_CHUNK_PIX : CHUNK_ROW_PIX) != CUDA_SUCCESS)
+      return SR_E_CUDA;
+  } else {
+    auto fn = get_encode_fn();
+    cuuint64_t dims[4] = {(cuuint64_t)Cp, (cuuint64_t)W, (cuuint64_t)H, 1};
+    cuuint64_t strides[3] = {(cuuint64_t)Cp * 2, (cuuint64_t)W * Cp * 2, (cuuint64_t)H * W * Cp * 2};
+    cuuint32_t box[4] = {(cuuint32_t)Cp, 66, 6, 1};
+    cuuint32_t estr[4] = {1, 1, 1, 1};
+    if (fn(&tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(act), dims, strides, box, estr,
+           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return SR_E_CUDA;
+  }
+  size_t smem = 1024 + 4 * (size_t)((bytes + 1023u) & ~1023u);
+  cudaFuncSetAttribute(k_bench_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  k_bench_tma<<<grid, 32, smem, st>>>(tm, mode, H, W, 1, bytes);  // warm-up
+  cudaEventRecord(a, st);
+  k_bench_tma<<<grid, 32, smem, st>>>(tm, mode, H, W, passes, bytes);
+  cudaEventRecord(b, st);
+  cudaEventSynchronize(b);
+  cudaEventElapsedTime(ms_out, a, b);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
 extern "C" int sr_test_mma(const void* A, const void* B, float* D, int N, int K, int a_mn, int b_mn, int reps,
                            int shift, long long* cycles_dev, void* stream) {
   if (N % 16 || N < 16 || N > 256 || K % 16 || K < 16) return SR_E_INVAL;
-  size_t smem = (size_t)(128 + 8) * K * 2 + (size_t)N * K * 2 + 1024;
+  size_t smem = (size_t)(128 + 16) * K * 2 + (size_t)N * K * 2 + 1024 + 1024;
   if (smem > 200 * 1024) return SR_E_INVAL;
   cudaFuncSetAttribute(k_test_mma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k_test_mma<<<1, 128, smem, (cudaStream_t)stream>>>((const __nv_bfloat16*)A, (const __nv_bfloat16*)B, D, N, K,
@@ -212,9 +306,12 @@ extern "C" int sr_bench_resblock(int c, int n, int h, int w, int iters, float* m
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
-  cudaError_t e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, dbg_host ? dbg : nullptr);
+  const char* ex = std::getenv("SR_BLOCK_EXP");  // benchmarking experiments (see k_resblock)
+  const int exp = ex ? std::atoi(ex) : 0;
+  cudaError_t e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, dbg_host ? dbg : nullptr, nullptr, 0, exp);
   cudaEventRecord(a, st);
-  for (int i = 0; i < iters && e == cudaSuccess; ++i) e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st);
+  for (int i = 0; i < iters && e == cudaSuccess; ++i)
+    e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, nullptr, nullptr, 0, exp);
   cudaEventRecord(b, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
   float ms = 0.f;
@@ -255,4 +352,46 @@ extern "C" int sr_bench_roll_dbg(int cinp, int coutp, int n, int h, int w, int r
   cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
   cudaFree(x); cudaFree(y); cudaFree(r); cudaFree(wt); cudaFree(bias); cudaFree(dbg);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
+
+// Timing of one wgrad launch configuration (split-K + fused reduction) on device-resident data; dbg_host
+// (nullable) receives the per-CTA globaltimer stamps [grid][8] of one extra launch (benchmarking only).
+extern "C" int sr_bench_wgrad(const void* x, const void* dy, int n, int h, int w, int cinp, int coutp, int iters,
+                              float* ms_out, long long* dbg_host, int exp, void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  size_t smem = 0;
+  WgradGeom g = make_wgrad_geom(n, h, w, cinp, coutp, &smem);
+  g.exp = exp;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int grid = g.units < sms ? g.units : sms;
+  float *ws = nullptr, *gout = nullptr;
+  unsigned* sync = nullptr;
+  long long* dbg = nullptr;
+  if (cudaMalloc(&ws, (size_t)grid * (9 * cinp * coutp + coutp) * 4) ||
+      cudaMalloc(&gout, ((size_t)9 * cinp * coutp + coutp) * 4) || cudaMalloc(&dbg, (size_t)grid * 8 * 8) ||
+      cudaMalloc(&sync, 8))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(sync, 0, 8, st);
+  WgradOut o{ws, sync, gout, gout + (size_t)9 * cinp * coutp, cinp, coutp, 1.f};
+  cudaEvent_t a, b;
+  cudaEventCreate(&a); cudaEventCreate(&b);
+  launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, g, o, smem, grid, st);
+  cudaEventRecord(a, st);
+  for (int i = 0; i < iters; ++i) launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, g, o, smem, grid, st);
+  cudaEventRecord(b, st);
+  cudaEventSynchronize(b);
+  cudaEventElapsedTime(ms_out, a, b);
+  *ms_out /= iters;
+  if (dbg_host) {
+    WgradGeom gd = g;
+    gd.dbg = dbg;
+    launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, gd, o, smem, grid, st);
+    cudaMemcpyAsync(dbg_host, dbg, (size_t)grid * 8 * 8, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+  }
+  cudaEventDestroy(a); cudaEventDestroy(b);
+  cudaFree(ws); cudaFree(gout); cudaFree(dbg); cudaFree(sync);
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
 }

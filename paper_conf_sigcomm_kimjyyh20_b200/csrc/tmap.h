@@ -51,6 +51,24 @@ inline CUresult make_act_tmap(CUtensorMap* tm, const void* base, int N, int H, i
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+// NHWC bf16 [N][H][W][Cp] as a 5-D tensor {16, W, Cp/16, H, N} whose innermost unit is a 16-channel (32-byte)
+// block, SWIZZLE_32B: the box lands as smem [row][block][pixel][16 ch] with the two 16-B halves of each 32-B
+// pixel row swapped when address bit 7 is set -- the MN-major SWIZZLE_32B canonical layout (atoms of 16 channels
+// x 8 pixels).  Twice the TMA throughput of the 16-B-innermost maps above (scripts/tma_rate.py).
+inline CUresult make_act_tmap_sw32(CUtensorMap* tm, const void* base, int N, int H, int W, int Cp, int box_w,
+                                   int box_h) {
+  auto fn = get_encode_fn();
+  if (!fn) return CUDA_ERROR_NOT_SUPPORTED;
+  const uint64_t pix = (uint64_t)Cp * 2, row = (uint64_t)W * pix, img = (uint64_t)H * row;
+  cuuint64_t dims[5] = {16, (cuuint64_t)W, (cuuint64_t)(Cp / 16), (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[4] = {pix, 32, row, img};
+  cuuint32_t box[5] = {16, (cuuint32_t)box_w, (cuuint32_t)(Cp / 16), (cuuint32_t)box_h, 1};
+  cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+  return fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, const_cast<void*>(base), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+}
+
 // NHWC bf16 [N][H][W][Cp] as a 4-D tensor {Cp, W, H, N}; box {box_c, box_w, 1, 1} = (part of the channels of)
 // one row segment, smem layout [pixel][box_c] (residual rows; per-warp output slices for the TMA store).
 inline CUresult make_row_tmap(CUtensorMap* tm, const void* base, int N, int H, int W, int Cp, int box_w, int box_c) {

@@ -28,8 +28,15 @@ for c, n, h, w in ((48, 8, 720, 1280), (32, 30, 540, 960)):
     t0 = d[0, 0]
     names = ["f_iss", "E1_iss", "E2_iss", "e1_got", "e1_trow", "e2_got", "e2_store", "mma_st", "acq1", "f_ok",
              "c2_st", "acq2", "t_ok"]
-    for i in range(4, 14):
+    for i in range(4, 6):
         print("  step %3d " % i + " ".join(f"{nm}={(d[e, i] - t0) if d[e, i] else -1:7d}" for e, nm in enumerate(names)))
+    # block hand-off: MMA step st acquires ring-1 block of row st+2, last used by row st-3 (freed by epi1 at index
+    # st-3); ring-2 likewise with conv2 rows (conv2 step st handles t row k = st-3, acquires row k+2, freed k-3)
+    for st in range(8, 14):
+        k = st - 3
+        print(f"  step {st:3d}: acq1 wait {d[8, st] - d[7, st]:5d} (freed {d[13, st - 3] - d[7, st]:6d} rel. to step start)"
+              f"  acq2 wait {d[11, st] - d[10, st]:5d} (freed {d[14, k - 3] - d[10, st]:6d} rel. to conv2 part start)"
+              f"  f wait {d[9, st] - d[8, st]:5d}  t wait {d[12, st] - d[11, st]:5d}")
     for e, nm in enumerate(names[:7]):
         v = d[e, 20:200]
         v = v[v > 0]

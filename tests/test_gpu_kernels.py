@@ -31,7 +31,7 @@ def _s():
 # ------------------------------------------------------------------ tcgen05 descriptor / shape sanity
 @pytest.mark.parametrize("N", [16, 32, 48, 64, 144, 256])
 @pytest.mark.parametrize("K", [16, 64])
-@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (1, 1), (0, 1), (1, 0)])
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (1, 1), (0, 1), (1, 0), (2, 2), (2, 0)])  # 2: MN-major SWIZZLE_32B
 def test_mma_descriptors(lib, N, K, a_mn, b_mn):
     r = np.random.default_rng(N * 1000 + K + 10 * a_mn + b_mn)
     A = bf16_round(r.standard_normal((128, K)))
