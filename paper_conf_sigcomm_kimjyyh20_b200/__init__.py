@@ -128,6 +128,19 @@ class SRContext:
                                      _stream(stream)), self.h, "sr_infer_rows")
         return hr_frame
 
+    def infer_i420(self, y, u, v, which="serve", out=None, stream=None):
+        """I420 in (y [n,h,w], u/v [n,h/2,w/2] uint8 CUDA), I420 out at s x (sr_infer_i420)."""
+        import torch
+        n, h, w = y.shape
+        s = self.scale
+        if out is None:
+            out = (torch.empty((n, s * h, s * w), dtype=torch.uint8, device=y.device),
+                   torch.empty((n, s * h // 2, s * w // 2), dtype=torch.uint8, device=y.device),
+                   torch.empty((n, s * h // 2, s * w // 2), dtype=torch.uint8, device=y.device))
+        check(self.lib.sr_infer_i420(self.h, _model(which), _ptr(y), _ptr(u), _ptr(v), n, h, w, _ptr(out[0]),
+                                     _ptr(out[1]), _ptr(out[2]), _stream(stream)), self.h, "sr_infer_i420")
+        return out
+
     # ---------------------------------------------------------------- training
     def train_step(self, lr, hr, loss=None, stream=None):
         n, p = lr.shape[0], lr.shape[1]
@@ -157,6 +170,14 @@ class SRContext:
         n, pp = lr.shape[0], lr.shape[1]
         check(self.lib.sr_pool_push(self.h, _ptr(lr), _ptr(hr), n, pp, None, _stream(stream)), self.h,
               "sr_pool_push")
+
+    def pool_push_i420(self, y, u, v, hr, xy, stream=None):
+        """HR patches hr [n,s*pp,s*pp,3] with LR counterparts cropped from one decoded I420 frame (y [h,w], u/v
+        [h/2,w/2]) at LR corners xy [n,2] int32 (x, y)."""
+        h, w = y.shape[-2], y.shape[-1]
+        n, pp = hr.shape[0], hr.shape[1] // self.scale
+        check(self.lib.sr_pool_push_i420(self.h, _ptr(y), _ptr(u), _ptr(v), h, w, _ptr(hr), _ptr(xy), n, pp, None,
+                                         _stream(stream)), self.h, "sr_pool_push_i420")
 
     @property
     def pool_size(self) -> int:

@@ -50,6 +50,8 @@ _SIGS = {
     "sr_infer": (_I, [_P, _I, _P, _I, _I, _I, _P, _P]),
     "sr_infer_host": (_I, [_P, _I, _P, _I, _I, _I, _P, _P]),
     "sr_infer_rows": (_I, [_P, _I, _P, _I, _I, _I, _I, _P, _P]),
+    "sr_infer_i420": (_I, [_P, _I, _P, _P, _P, _I, _I, _I, _P, _P, _P, _P]),
+    "sr_pool_push_i420": (_I, [_P, _P, _P, _P, _I, _I, _P, _P, _I, _I, _P, _P]),
     "sr_train_step": (_I, [_P, _P, _P, _I, _I, _P, _P]),
     "sr_train_grad": (_I, [_P, _P, _P, _I, _I, _P, _P]),
     "sr_grad_buffer": (_P, [_P]),

@@ -64,7 +64,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
            const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg,
            const int exp) {
   // exp (benchmarking experiments only, results wrong when set): 1 no residual load, 2 no output store, 4 no t
-  // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads
+  // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads, 128 no f-row TMA
+  // after the first piece
   // tsave (nullable): also write t = ReLU(conv1(f) + b1) to global (training saves it for the backward pass).
   // sep > 0: columns with col % sep in {0, sep-1} are separators of the virtual training batch -> t and out = 0.
   // dbg (benchmarking only, CTA 0): clock64 stamps [event][step], events: 0 f issued, 1 conv1 step issued,
@@ -144,8 +145,12 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       SR_PIECE_BEGIN
       for (int i = 0; i < n_f; ++i) {
         mbar_wait(&f_empty[s], ph ^ 1);
-        mbar_arrive_expect_tx(&f_full[s], CCH * PLANE);
-        tma_load_5d(sF + s * ROWB, &tm_f, &f_full[s], 0, x0 - 2, y0 - 2 + i, 0, n);
+        if ((exp & 128) && pos > beg + 8) {
+          mbar_arrive(&f_full[s]);
+        } else {
+          mbar_arrive_expect_tx(&f_full[s], CCH * PLANE);
+          tma_load_5d(sF + s * ROWB, &tm_f, &f_full[s], 0, x0 - 2, y0 - 2 + i, 0, n);
+        }
         SR_DBG(0, i)
         if (++s == kBlkNF) { s = 0; ph ^= 1; }
       }

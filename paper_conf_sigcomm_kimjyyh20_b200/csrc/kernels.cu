@@ -28,6 +28,85 @@ void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st)
   launch_k(k_pack_input, dim3((unsigned)((npix + th - 1) / th)), dim3(th), 0, st, lr, npix, reinterpret_cast<uint4*>(x));
 }
 
+// ------------------------------------------------------------------ I420 <-> RGB (BT.601 studio swing, reading R21)
+// Integer conversion: C = Y - 16, D = U - 128, E = V - 128; R = (298 C + 409 E + 128) >> 8, G = (298 C - 100 D -
+// 208 E + 128) >> 8, B = (298 C + 516 D + 128) >> 8, clamped; chroma (y/2, x/2) is shared by its 2x2 block.
+__device__ __forceinline__ uint8_t clip8(int v) { return (uint8_t)min(max(v, 0), 255); }
+__device__ __forceinline__ void yuv_to_rgb(int Y, int U, int V, uint8_t* o) {
+  const int c = Y - 16, d = U - 128, e = V - 128;
+  o[0] = clip8((298 * c + 409 * e + 128) >> 8);
+  o[1] = clip8((298 * c - 100 * d - 208 * e + 128) >> 8);
+  o[2] = clip8((298 * c + 516 * d + 128) >> 8);
+}
+
+// one thread per pixel: planes y [n][h][w], u/v [n][h/2][w/2] -> rgb [n][h][w][3]
+__global__ void k_i420_to_rgb(const uint8_t* __restrict__ y, const uint8_t* __restrict__ u,
+                              const uint8_t* __restrict__ v, int n, int h, int w, uint8_t* __restrict__ rgb) {
+  pdl_enter();
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (long long)n * h * w) return;
+  const int x = (int)(i % w);
+  const long long r = i / w;
+  const int yy = (int)(r % h), f = (int)(r / h);
+  const size_t ci = ((size_t)f * (h / 2) + yy / 2) * (w / 2) + x / 2;
+  yuv_to_rgb(y[i], u[ci], v[ci], rgb + i * 3);
+}
+
+// one thread per 2x2 block: Y per pixel, U/V from the block's rounded mean colour
+__global__ void k_rgb_to_i420(const uint8_t* __restrict__ rgb, int n, int h, int w, uint8_t* __restrict__ y,
+                              uint8_t* __restrict__ u, uint8_t* __restrict__ v) {
+  pdl_enter();
+  const int hw = w / 2, hh = h / 2;
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (long long)n * hh * hw) return;
+  const int bx = (int)(i % hw);
+  const long long r = i / hw;
+  const int by = (int)(r % hh), f = (int)(r / hh);
+  int sr = 0, sg = 0, sb = 0;
+#pragma unroll
+  for (int dy = 0; dy < 2; ++dy)
+#pragma unroll
+    for (int dx = 0; dx < 2; ++dx) {
+      const size_t p = ((size_t)f * h + 2 * by + dy) * w + 2 * bx + dx;
+      const int R = rgb[p * 3], G = rgb[p * 3 + 1], B = rgb[p * 3 + 2];
+      y[p] = (uint8_t)(((66 * R + 129 * G + 25 * B + 128) >> 8) + 16);
+      sr += R; sg += G; sb += B;
+    }
+  const int R = (sr + 2) >> 2, G = (sg + 2) >> 2, B = (sb + 2) >> 2;
+  u[i] = (uint8_t)(((-38 * R - 74 * G + 112 * B + 128) >> 8) + 128);
+  v[i] = (uint8_t)(((112 * R - 94 * G - 18 * B + 128) >> 8) + 128);
+}
+
+// LR counterparts of arriving HR patches (§5.2): pp x pp RGB crops of decoded frame 0 at LR top-left
+// xy[j] = (x, y); grid (n, pp), one thread per pixel of a crop row.
+__global__ void k_i420_crop(const uint8_t* __restrict__ y, const uint8_t* __restrict__ u,
+                            const uint8_t* __restrict__ v, int h, int w, const int32_t* __restrict__ xy, int pp,
+                            uint8_t* __restrict__ out) {
+  pdl_enter();
+  const int j = blockIdx.x, r = blockIdx.y;
+  const int x0 = xy[2 * j], y0 = xy[2 * j + 1];
+  for (int c = threadIdx.x; c < pp; c += blockDim.x) {
+    const int X = x0 + c, Y = y0 + r;
+    const size_t ci = (size_t)(Y / 2) * (w / 2) + X / 2;
+    yuv_to_rgb(y[(size_t)Y * w + X], u[ci], v[ci], out + (((size_t)j * pp + r) * pp + c) * 3);
+  }
+}
+
+void launch_i420_to_rgb(const uint8_t* y, const uint8_t* u, const uint8_t* v, int n, int h, int w, uint8_t* rgb,
+                        cudaStream_t st) {
+  const long long tot = (long long)n * h * w;
+  launch_k(k_i420_to_rgb, dim3((unsigned)((tot + 255) / 256)), dim3(256), 0, st, y, u, v, n, h, w, rgb);
+}
+void launch_rgb_to_i420(const uint8_t* rgb, int n, int h, int w, uint8_t* y, uint8_t* u, uint8_t* v,
+                        cudaStream_t st) {
+  const long long tot = (long long)n * (h / 2) * (w / 2);
+  launch_k(k_rgb_to_i420, dim3((unsigned)((tot + 255) / 256)), dim3(256), 0, st, rgb, n, h, w, y, u, v);
+}
+void launch_i420_crop(const uint8_t* y, const uint8_t* u, const uint8_t* v, int h, int w, const int32_t* xy, int n,
+                      int pp, uint8_t* out, cudaStream_t st) {
+  launch_k(k_i420_crop, dim3(n, pp), dim3(64), 0, st, y, u, v, h, w, xy, pp, out);
+}
+
 // Virtual training batch: n patches p x p laid side by side in one p x (n (p+2)) image, patch j at columns
 // [j (p+2) + 1, j (p+2) + 1 + p); the separator columns j (p+2) and j (p+2) + p + 1 are zero and act as every
 // patch's own zero padding for all the 3x3 convs (which re-zero them in their epilogues).

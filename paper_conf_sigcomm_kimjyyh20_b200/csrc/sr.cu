@@ -58,6 +58,8 @@ struct sr_ctx {
   long long sample_step = 0;
   // psnr
   uint8_t* val_a = nullptr;  // one model's SR output of the validation patches
+  uint8_t *yuv_lr = nullptr, *yuv_hr = nullptr, *crop_buf = nullptr;  // I420 boundary staging (RGB)
+  size_t yuv_lr_bytes = 0, yuv_hr_bytes = 0, crop_bytes = 0;
   size_t val_bytes = 0;
   unsigned long long* sse = nullptr;
   int sse_n = 0;
@@ -670,7 +672,7 @@ void sr_destroy(sr_ctx* ctx) {
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
                   ctx->adam_scal, ctx->pool_lr,
-                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse};
+                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].wo); cudaFree(ctx->snap[k].bias); }
@@ -801,6 +803,27 @@ sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, in
   return forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st);
 }
 
+sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const uint8_t* u_dev,
+                        const uint8_t* v_dev, int n, int h, int w, uint8_t* hy_dev, uint8_t* hu_dev, uint8_t* hv_dev,
+                        sr_stream stream) {
+  GUARD();
+  if (!y_dev || !u_dev || !v_dev || !hy_dev || !hu_dev || !hv_dev || n < 1 || h < 2 || w < 2 || (h | w) & 1)
+    return fail(ctx, SR_E_INVAL, "sr_infer_i420: bad args (h, w must be even)");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int s = ctx->s;
+  const size_t lb = (size_t)n * h * w * 3, hb = lb * s * s;
+  if (lb > ctx->yuv_lr_bytes) { CK(dalloc(&ctx->yuv_lr, lb)); ctx->yuv_lr_bytes = lb; }
+  if (hb > ctx->yuv_hr_bytes) { CK(dalloc(&ctx->yuv_hr, hb)); ctx->yuv_hr_bytes = hb; }
+  launch_i420_to_rgb(y_dev, u_dev, v_dev, n, h, w, ctx->yuv_lr, st);
+  ctx->launches++;
+  CKL();
+  TRY(sr_infer(ctx, which, ctx->yuv_lr, n, h, w, ctx->yuv_hr, stream));
+  launch_rgb_to_i420(ctx->yuv_hr, n, s * h, s * w, hy_dev, hu_dev, hv_dev, st);
+  ctx->launches++;
+  CKL();
+  return SR_OK;
+}
+
 sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
                         uint8_t* hr_host, sr_stream stream) {
   GUARD();
@@ -902,13 +925,30 @@ sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev
     return fail(ctx, SR_E_INVAL, "sr_pool_push: patch size differs from the first push");
   }
   const size_t lb = (size_t)pp * pp * 3, hb = lb * s * s;
-  for (int i = 0; i < n; ++i) {
+  for (int i = 0; i < n;) {  // arrival order into the ring: at most two contiguous runs per call (wrap)
     const long long slot = (ctx->pool_total + i) % ctx->pool_cap;
-    CK(cudaMemcpyAsync(ctx->pool_lr + slot * lb, lr_dev + i * lb, lb, cudaMemcpyDeviceToDevice, st));
-    CK(cudaMemcpyAsync(ctx->pool_hr + slot * hb, hr_dev + i * hb, hb, cudaMemcpyDeviceToDevice, st));
+    const int run = (int)std::min<long long>(n - i, ctx->pool_cap - slot);
+    CK(cudaMemcpyAsync(ctx->pool_lr + slot * lb, lr_dev + i * lb, run * lb, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(ctx->pool_hr + slot * hb, hr_dev + i * hb, run * hb, cudaMemcpyDeviceToDevice, st));
+    i += run;
   }
   ctx->pool_total += n;
   return SR_OK;
+}
+
+sr_status sr_pool_push_i420(sr_ctx* ctx, const uint8_t* y_dev, const uint8_t* u_dev, const uint8_t* v_dev, int h,
+                            int w, const uint8_t* hr_dev, const int32_t* xy_dev, int n, int pp,
+                            const int64_t* arrival_ts, sr_stream stream) {
+  GUARD();
+  if (!y_dev || !u_dev || !v_dev || !hr_dev || !xy_dev || n < 1 || pp < 1 || h < 2 || w < 2 || (h | w) & 1)
+    return fail(ctx, SR_E_INVAL, "sr_pool_push_i420: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t need = (size_t)n * pp * pp * 3;
+  if (need > ctx->crop_bytes) { CK(dalloc(&ctx->crop_buf, need)); ctx->crop_bytes = need; }
+  launch_i420_crop(y_dev, u_dev, v_dev, h, w, xy_dev, n, pp, ctx->crop_buf, st);
+  ctx->launches++;
+  CKL();
+  return sr_pool_push(ctx, ctx->crop_buf, hr_dev, n, pp, arrival_ts, stream);
 }
 
 size_t sr_pool_size(const sr_ctx* ctx) {

@@ -325,3 +325,60 @@ def test_infer_host_pipeline_equals_device_path():
     out_h = torch.empty((7, 360, 600, 3), dtype=torch.uint8).pin_memory()
     ctx.infer_host(lr_h, out_h, "serve")
     assert torch.equal(out_h, dev)
+
+
+# ---------------------------------------------------------------- I420 boundary
+def _i420_frames(n, h, w, seed):
+    from oracle.color import rgb_to_i420
+    rgb = synth_frames(n, h, w, seed=seed)
+    return rgb_to_i420(rgb)
+
+
+@pytest.mark.parametrize("s", [2, 3, 4])
+def test_i420_bilinear_path_bitexact(s):
+    """Bilinear 'model': I420 -> RGB -> bilinear -> RGB -> I420 equals the oracle composition bit for bit."""
+    from oracle.color import i420_to_rgb, rgb_to_i420
+    ctx = _ctx(s, 1, 8)
+    y, u, v = _i420_frames(2, 36, 52, seed=41)
+    out = ctx.infer_i420(*(torch.from_numpy(a).cuda() for a in (y, u, v)), which="bilinear")
+    rgb = i420_to_rgb(y, u, v)
+    ref = rgb_to_i420(np.rint(np.clip(O.bilinear_up(rgb, s), 0, 255)).astype(np.uint8))
+    for g, r in zip(out, ref):
+        np.testing.assert_array_equal(g.cpu().numpy(), r)
+
+
+@pytest.mark.parametrize("cfg,hw", [((3, 8, 48), (90, 160)), ((2, 2, 16), (34, 60))])
+def test_i420_dnn_path(cfg, hw):
+    """DNN model: the conversions are exact around the product's RGB inference (bit-exact against the oracle
+    conversions applied to sr_infer's own output) and the whole path is within the bar of the oracle net."""
+    from oracle.color import i420_to_rgb, rgb_to_i420
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=5)
+    y, u, v = _i420_frames(2, hw[0], hw[1], seed=42)
+    out = ctx.infer_i420(*(torch.from_numpy(a).cuda() for a in (y, u, v)))
+    rgb = i420_to_rgb(y, u, v)
+    sr_rgb = ctx.infer(torch.from_numpy(rgb).cuda(), "serve").cpu().numpy()
+    for g, r in zip(out, rgb_to_i420(sr_rgb)):
+        np.testing.assert_array_equal(g.cpu().numpy(), r)
+    ref = rgb_to_i420(O.infer_u8(ctx.get_params("serve"), rgb, s, B, C))
+    assert np.abs(out[0].cpu().numpy().astype(int) - ref[0].astype(int)).max() <= 3
+
+
+def test_pool_push_i420_crops_the_decoded_frame():
+    from oracle.color import crop_rgb_from_i420
+    s, pp = 2, 16
+    ctx = _ctx(s, 1, 8)
+    y, u, v = _i420_frames(1, 64, 96, seed=43)
+    xy = np.array([[0, 0], [10, 6], [80, 48], [33, 21]], np.int32)
+    hr = np.random.default_rng(7).integers(0, 256, (4, s * pp, s * pp, 3)).astype(np.uint8)
+    ctx.pool_push_i420(*(torch.from_numpy(a[0]).cuda() for a in (y, u, v)), torch.from_numpy(hr).cuda(),
+                       torch.from_numpy(xy).cuda())
+    assert ctx.pool_size == 4
+    # sample every entry back (batch large enough to hit all four) and compare with the oracle crops
+    lr_b, hr_b, idx = ctx.sample_batch(0, 64, pp)
+    crops = crop_rgb_from_i420(y, u, v, xy, pp)
+    idx = idx.cpu().numpy()
+    for k in range(64):
+        j = int(idx[k])
+        np.testing.assert_array_equal(lr_b[k].cpu().numpy(), crops[j])
+        np.testing.assert_array_equal(hr_b[k].cpu().numpy(), hr[j])
