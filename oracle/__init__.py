@@ -10,7 +10,9 @@ Parity pins (tests/test_oracle_pins.py, `-m "not gpu"`): brute-force 7-loop conv
 kernels, pixel shuffle as a permutation, zero-weight net == bilinear skip (bit-exact u8, checked
 against torch.nn.functional.interpolate), finite-difference gradients of the whole net, PSNR closed
 form, Adam step-1 closed form (and torch.optim.Adam), sampler statistics, paper arithmetic facts,
-Algorithm 1 (oracle/controller.py) against traces worked out by hand from App. A (tests/golden/alg1_traces.json).
+Algorithm 1 (oracle/controller.py) against traces worked out by hand from App. A (tests/golden/alg1_traces.json),
+the I420 conversion (oracle/color.py) against the real-valued BT.601 matrices, and the client's patch selection
+(oracle/patch_select.py) against frames whose degraded cells are known by construction.
 "parity unpinned": none of the functions below; the learning-direction check (loss falls) is a
 sanity check only.
 """
@@ -20,3 +22,4 @@ from .srnet import (  # noqa: F401
     dp_aggregate, sample_indices, gather_patches, psnr_u8, psnr_gain, conv_shapes_oracle,
 )
 from .controller import Algorithm1, epoch_report  # noqa: F401
+from .patch_select import select_patches  # noqa: F401

@@ -223,6 +223,17 @@ class SRContext:
         out["event"] = Controller.EVENTS[r.event]
         return out
 
+    def patch_select(self, raw, dec, cell=120, max_sel=10, seed=0, step=0, stream=None):
+        """The ingest client's patch selection (sr_patch_select): [(x, y), ...] of the kept cells in order."""
+        import numpy as np
+        h, w = raw.shape[0], raw.shape[1]
+        xy = np.zeros(2 * max(max_sel, 1), np.int32)
+        n = C.c_int(0)
+        check(self.lib.sr_patch_select(self.h, _ptr(raw), _ptr(dec), h, w, cell, max_sel, seed, step,
+                                       xy.ctypes.data_as(C.c_void_p), C.byref(n), _stream(stream)), self.h,
+              "sr_patch_select")
+        return [(int(xy[2 * i]), int(xy[2 * i + 1])) for i in range(n.value)]
+
     def set_fusion(self, fuse_blocks=True):
         check(self.lib.sr_set_fusion(self.h, int(fuse_blocks)), self.h, "sr_set_fusion")
 

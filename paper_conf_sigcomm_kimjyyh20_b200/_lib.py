@@ -66,6 +66,7 @@ _SIGS = {
     "sr_controller_init": (_I, [C.POINTER(sr_controller), C.c_double, _I, C.c_double, _I]),
     "sr_controller_update": (_I, [C.POINTER(sr_controller), C.c_double, C.POINTER(_I)]),
     "sr_controller_step": (_I, [_P, C.POINTER(sr_controller), _P, _P, _I, _I, C.POINTER(sr_epoch_report), _P]),
+    "sr_patch_select": (_I, [_P, _P, _P, _I, _I, _I, _I, C.c_uint64, C.c_int64, _P, C.POINTER(_I), _P]),
     "sr_sse_u8": (_I, [_P, _P, _I, C.c_int64, _P, _P]),
     "sr_launch_count": (C.c_uint64, [_P]),
     "sr_kernel_timing": (_I, [_P, _I]),

@@ -107,6 +107,41 @@ void launch_i420_crop(const uint8_t* y, const uint8_t* u, const uint8_t* v, int 
   launch_k(k_i420_crop, dim3(n, pp), dim3(64), 0, st, y, u, v, h, w, xy, pp, out);
 }
 
+// ------------------------------------------------------------------ per-cell integer SSE (patch selection)
+// grid (ncx, ncy): block (cx, cy) sums (raw - dec)^2 over the (possibly partial) cell of a [h][w][3] frame.
+__global__ void k_cell_sse(const uint8_t* __restrict__ raw, const uint8_t* __restrict__ dec, int h, int w, int cell,
+                           unsigned long long* __restrict__ out) {
+  pdl_enter();
+  const int cx = blockIdx.x, cy = blockIdx.y;
+  const int x0 = cx * cell, y0 = cy * cell;
+  const int cw = min(cell, w - x0), ch = min(cell, h - y0);
+  const int rowb = cw * 3;
+  unsigned long long acc = 0;
+  for (int i = threadIdx.x; i < ch * rowb; i += blockDim.x) {
+    const int r = i / rowb, c = i - r * rowb;
+    const size_t o = ((size_t)(y0 + r) * w + x0) * 3 + c;
+    const int d = (int)raw[o] - (int)dec[o];
+    acc += (unsigned long long)(d * d);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  __shared__ unsigned long long part[32];
+  if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    unsigned long long t = threadIdx.x < (blockDim.x >> 5) ? part[threadIdx.x] : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    if (threadIdx.x == 0) out[(size_t)cy * gridDim.x + cx] = t;
+  }
+}
+
+void launch_cell_sse(const uint8_t* raw, const uint8_t* dec, int h, int w, int cell, unsigned long long* out,
+                     cudaStream_t st) {
+  const int nx = (w + cell - 1) / cell, ny = (h + cell - 1) / cell;
+  launch_k(k_cell_sse, dim3(nx, ny), dim3(256), 0, st, raw, dec, h, w, cell, out);
+}
+
 // Virtual training batch: n patches p x p laid side by side in one p x (n (p+2)) image, patch j at columns
 // [j (p+2) + 1, j (p+2) + 1 + p); the separator columns j (p+2) and j (p+2) + p + 1 are zero and act as every
 // patch's own zero padding for all the 3x3 convs (which re-zero them in their epilogues).

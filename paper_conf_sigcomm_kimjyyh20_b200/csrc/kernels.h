@@ -56,6 +56,8 @@ void launch_i420_to_rgb(const uint8_t* y, const uint8_t* u, const uint8_t* v, in
 void launch_rgb_to_i420(const uint8_t* rgb, int n, int h, int w, uint8_t* y, uint8_t* u, uint8_t* v, cudaStream_t st);
 void launch_i420_crop(const uint8_t* y, const uint8_t* u, const uint8_t* v, int h, int w, const int32_t* xy, int n,
                       int pp, uint8_t* out, cudaStream_t st);
+void launch_cell_sse(const uint8_t* raw, const uint8_t* dec, int h, int w, int cell, unsigned long long* out,
+                     cudaStream_t st);
 cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st);
 
 }  // namespace sr

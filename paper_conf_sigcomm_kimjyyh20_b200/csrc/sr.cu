@@ -60,6 +60,8 @@ struct sr_ctx {
   uint8_t* val_a = nullptr;  // one model's SR output of the validation patches
   uint8_t *yuv_lr = nullptr, *yuv_hr = nullptr, *crop_buf = nullptr;  // I420 boundary staging (RGB)
   size_t yuv_lr_bytes = 0, yuv_hr_bytes = 0, crop_bytes = 0;
+  unsigned long long* cell_sse = nullptr;  // patch selection
+  int cell_n = 0;
   size_t val_bytes = 0;
   unsigned long long* sse = nullptr;
   int sse_n = 0;
@@ -672,7 +674,7 @@ void sr_destroy(sr_ctx* ctx) {
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
                   ctx->adam_scal, ctx->pool_lr,
-                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf};
+                  ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf, ctx->cell_sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].wo); cudaFree(ctx->snap[k].bias); }
@@ -1108,6 +1110,47 @@ sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_de
   out_host->psnr_a = q[0];
   out_host->psnr_b = q[1];
   out_host->gain = q[0] - q[1];
+  return SR_OK;
+}
+
+// ---- client-side patch selection (§5.2; reading R22)
+sr_status sr_patch_select(sr_ctx* ctx, const uint8_t* raw_dev, const uint8_t* dec_dev, int h, int w, int cell,
+                          int max_sel, uint64_t seed, int64_t step, int32_t* xy_host, int* n_sel, sr_stream stream) {
+  GUARD();
+  if (!raw_dev || !dec_dev || !xy_host || !n_sel || h < 1 || w < 1 || cell < 1 || max_sel < 0)
+    return fail(ctx, SR_E_INVAL, "sr_patch_select: bad args");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int nx = (w + cell - 1) / cell, ny = (h + cell - 1) / cell;
+  if (nx * ny > ctx->cell_n) { CK(dalloc(&ctx->cell_sse, (size_t)nx * ny)); ctx->cell_n = nx * ny; }
+  launch_cell_sse(raw_dev, dec_dev, h, w, cell, ctx->cell_sse, st);
+  ctx->launches++;
+  CKL();
+  std::vector<unsigned long long> sse((size_t)nx * ny);
+  CK(cudaMemcpyAsync(sse.data(), ctx->cell_sse, sse.size() * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  unsigned long long s_frame = 0;
+  for (auto v : sse) s_frame += v;
+  const unsigned long long n_frame = (unsigned long long)h * w * 3;
+  const int gx = w / cell, gy = h / cell, n = gx * gy;  // whole cells are the candidates
+  std::vector<int> perm(n);
+  for (int k = 0; k < n; ++k) perm[k] = k;
+  for (int k = 0; k < n; ++k) {  // Fisher-Yates on the counter-based SplitMix64 stream
+    const uint64_t u = mix64h(seed + 0x9E3779B97F4A7C15ull * (((uint64_t)step << 32) + k + 1));
+    const int j = k + (int)(((unsigned __int128)u * (uint64_t)(n - k)) >> 64);
+    std::swap(perm[k], perm[j]);
+  }
+  int cnt = 0;
+  const unsigned long long n_cell = (unsigned long long)cell * cell * 3;
+  for (int i = 0; i < n && cnt < max_sel; ++i) {
+    const int cy = perm[i] / gx, cx = perm[i] % gx;
+    // PSNR(cell) < PSNR(frame)  <=>  SSE_cell * n_frame > SSE_frame * n_cell  (exact, 128-bit)
+    if ((unsigned __int128)sse[(size_t)cy * nx + cx] * n_frame > (unsigned __int128)s_frame * n_cell) {
+      xy_host[2 * cnt] = cx * cell;
+      xy_host[2 * cnt + 1] = cy * cell;
+      ++cnt;
+    }
+  }
+  *n_sel = cnt;
   return SR_OK;
 }
 

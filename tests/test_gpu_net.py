@@ -382,3 +382,22 @@ def test_pool_push_i420_crops_the_decoded_frame():
         j = int(idx[k])
         np.testing.assert_array_equal(lr_b[k].cpu().numpy(), crops[j])
         np.testing.assert_array_equal(hr_b[k].cpu().numpy(), hr[j])
+
+
+# ---------------------------------------------------------------- client patch selection
+@pytest.mark.parametrize("hw,cell,max_sel,seed,step", [((1080, 1920), 120, 10, 3, 0), ((250, 370), 60, 50, 1, 7),
+                                                        ((240, 360), 120, 10, 0, 1)])
+def test_patch_select_matches_oracle(hw, cell, max_sel, seed, step):
+    """sr_patch_select == oracle.select_patches exactly (integer decisions, same permutation) on a synthetic frame
+    and a degraded copy (area-downsampled and bilinearly upscaled: the 'decoded' low-bitrate proxy)."""
+    from oracle.patch_select import select_patches
+    from synth.gen import area_downsample
+    ctx = _ctx(2, 1, 8)
+    h, w = hw
+    raw = synth_frames(1, h, w, seed=51)[0]
+    dec = np.rint(np.clip(O.bilinear_up(area_downsample(raw[None, : h // 2 * 2, : w // 2 * 2], 2), 2), 0, 255))
+    dec_full = raw.copy()
+    dec_full[: h // 2 * 2, : w // 2 * 2] = dec[0].astype(np.uint8)
+    got = ctx.patch_select(torch.from_numpy(raw).cuda(), torch.from_numpy(dec_full).cuda(), cell, max_sel, seed, step)
+    assert got == select_patches(raw, dec_full, cell, max_sel, seed, step)
+    assert len(got) > 0
