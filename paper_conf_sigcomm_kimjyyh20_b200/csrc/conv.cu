@@ -190,7 +190,7 @@ __device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp)
 
 // Tail: y = acc + b (3 s^2 channels, index c*s^2 + i*s + j = pixel-shuffle phase (i,j) of colour c);
 // skip = bilinear_s(v) at HR (sY+i, sX+j).  Inference: u8 = RNE(clamp(255 y + skip, 0, 255)).
-// Training: o = y + skip/255, d = o - hr/255 -> loss += d^2, dy[c s^2 + i s + j] = 2 d.
+// Training: o = y + skip/255, d = o - hr/255 -> loss += d^2, dy[c s^2 + i s + j] = 2 d (L1: |d|, sign(d)).
 // (n, Y, X) addresses the LR image / HR target (n-th image of size H x W); dy_pix is the pixel index of this
 // output in the conv's own layout (equal to ((n H + Y) W + X) except for the virtual training batch).
 template <int S, int COUTP, bool TRAIN>
@@ -236,8 +236,13 @@ __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias
         if (TRAIN) {
           float o = y + skip * (1.f / 255.f);
           float d = o - (float)__ldg(trow + j * 3 + c) * (1.f / 255.f);
-          lsum += d * d;
-          dyv[k] = 2.f * d;
+          if (ep.l1) {  // L1 variant: |d|, d/d o = sign(d) (0 at 0)
+            lsum += fabsf(d);
+            dyv[k] = d > 0.f ? 1.f : (d < 0.f ? -1.f : 0.f);
+          } else {
+            lsum += d * d;
+            dyv[k] = 2.f * d;
+          }
         } else {
           float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
           hrow[j * 3 + c] = (uint8_t)__float2int_rn(o);

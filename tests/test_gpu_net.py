@@ -144,22 +144,24 @@ def test_strip_inference_bitexact():
 
 
 # ---------------------------------------------------------------- training
-@pytest.mark.parametrize("cfg,n,p", [((2, 2, 8), 4, 16), ((3, 2, 16), 3, 20), ((2, 8, 48), 2, 48),
-                                     ((4, 2, 16), 3, 16)])
-def test_train_gradient_and_adam_parity(cfg, n, p):
+@pytest.mark.parametrize("cfg,n,p,loss", [((2, 2, 8), 4, 16, "mse"), ((3, 2, 16), 3, 20, "mse"),
+                                          ((2, 8, 48), 2, 48, "mse"), ((4, 2, 16), 3, 16, "mse"),
+                                          ((2, 2, 8), 4, 16, "l1"), ((3, 3, 32), 6, 24, "l1")])
+def test_train_gradient_and_adam_parity(cfg, n, p, loss):
     s, B, C = cfg
-    ctx = _ctx(s, B, C, seed=21)
+    loss_kind = loss
+    ctx = _ctx(s, B, C, seed=21, loss=loss_kind)
     p0 = init_params(s, B, C, seed=21) * 2.0
     ctx.set_params(p0)
     lrp, hrp, _ = synth_patch_pool(n, s, s * p, seed=31, frame_hw=(s * p * 3, s * p * 4))
     lr = torch.from_numpy(lrp).cuda()
     hr = torch.from_numpy(hrp).cuda()
-    loss = torch.zeros(1, dtype=torch.float32, device="cuda")
-    ctx.train_grad(lr, hr, loss)
+    lo = torch.zeros(1, dtype=torch.float32, device="cuda")
+    ctx.train_grad(lr, hr, lo)
     g = ctx.grad_buffer().cpu().numpy().copy()
     pq = ctx.get_params("train")
-    ref_loss, ref_g = O.train_loss_and_grad(pq, lrp, hrp, s, B, C)
-    assert abs(loss.item() - ref_loss) / ref_loss < 1e-2
+    ref_loss, ref_g = O.train_loss_and_grad(pq, lrp, hrp, s, B, C, loss_kind=loss_kind)
+    assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
     assert rel_l2(g, ref_g) < 1e-2, rel_l2(g, ref_g)
     ctx.train_apply(1.0)
     p1 = ctx.get_params("train")

@@ -188,14 +188,16 @@ def test_full_gradient_finite_difference(s):
     assert abs(loss - L(p)) < 1e-15
 
 
-def test_gradient_matches_torch_autograd_net():
-    """Same net written with torch.nn.functional in float64 (library autograd)."""
+@pytest.mark.parametrize("loss_kind", ["mse", "l1"])
+def test_gradient_matches_torch_autograd_net(loss_kind):
+    """Same net written with torch.nn.functional in float64 (library autograd); MSE (R6) and the L1 variant
+    (torch's sign(0) = 0 convention)."""
     s, B, C = 3, 2, 4
     r = _rng(14)
     p = init_params(s, B, C, seed=5).astype(np.float64)
     lr = r.integers(0, 256, size=(2, 6, 5, 3)).astype(np.uint8)
     hr = r.integers(0, 256, size=(2, 18, 15, 3)).astype(np.uint8)
-    loss, g = O.train_loss_and_grad(p, lr, hr, s, B, C)
+    loss, g = O.train_loss_and_grad(p, lr, hr, s, B, C, loss_kind=loss_kind)
     pt = torch.from_numpy(p.copy()).requires_grad_(True)
     convs, off = [], 0
     for co, ci in O.conv_shapes_oracle(s, B, C):
@@ -214,7 +216,7 @@ def test_gradient_matches_torch_autograd_net():
     y = F.conv2d(gg, *convs[-1], padding=1)
     o = F.pixel_shuffle(y, s) + F.interpolate(v, scale_factor=s, mode="bilinear", align_corners=False) / 255.0
     t = torch.from_numpy(hr.astype(np.float64)).permute(0, 3, 1, 2) / 255.0
-    lt = ((o - t) ** 2).mean()
+    lt = ((o - t) ** 2).mean() if loss_kind == "mse" else (o - t).abs().mean()
     lt.backward()
     assert abs(lt.item() - loss) < 1e-14
     np.testing.assert_allclose(g, pt.grad.numpy(), rtol=1e-9, atol=1e-14)
