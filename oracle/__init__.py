@@ -18,7 +18,7 @@ sanity check only.
 """
 from .srnet import (  # noqa: F401
     conv3x3, conv3x3_bruteforce, conv3x3_dgrad, conv3x3_wgrad, pixel_shuffle, pixel_unshuffle,
-    bilinear_up, unpack_params, pack_params, forward, infer_u8, train_loss_and_grad, adam_step,
+    bilinear_up, bicubic_up, unpack_params, pack_params, forward, infer_u8, train_loss_and_grad, adam_step,
     dp_aggregate, sample_indices, gather_patches, psnr_u8, psnr_gain, conv_shapes_oracle,
 )
 from .controller import Algorithm1, epoch_report  # noqa: F401

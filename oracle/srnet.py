@@ -176,6 +176,51 @@ def bilinear_up(v_u8, s):
 
 
 # ----------------------------------------------------------------------------------------------------
+# bicubic up-scaling (the skip variant of SURVEY §8(f) NEXT 3; north star "bilinear/bicubic"; reading R23):
+# Keys cubic convolution with A = -0.75 (PyTorch bicubic, align_corners=False): src = (dst + 0.5)/s - 0.5 (no
+# clamp), i0 = floor(src), t = src - i0, out = sum_{k=-1..2} w(k - t) v[clamp(i0 + k, 0, n-1)],
+# w(x) = (A+2)|x|^3 - (A+3)|x|^2 + 1 for |x| <= 1, A|x|^3 - 5A|x|^2 + 8A|x| - 4A for 1 < |x| < 2.
+# ----------------------------------------------------------------------------------------------------
+
+def _cubic_w(x, A=-0.75):
+    x = abs(x)
+    if x <= 1.0:
+        return (A + 2.0) * x ** 3 - (A + 3.0) * x ** 2 + 1.0
+    if x < 2.0:
+        return A * x ** 3 - 5.0 * A * x ** 2 + 8.0 * A * x - 4.0 * A
+    return 0.0
+
+
+def _bicubic_axis(v, s, axis):
+    n = v.shape[axis]
+    out_shape = list(v.shape)
+    out_shape[axis] = n * s
+    out = np.zeros(out_shape, dtype=np.float64)
+    for dst in range(n * s):
+        src = (dst + 0.5) / s - 0.5
+        i0 = int(np.floor(src))
+        t = src - i0
+        acc = 0.0
+        for k in range(-1, 3):
+            idx = min(max(i0 + k, 0), n - 1)
+            acc = acc + _cubic_w(k - t) * np.take(v, idx, axis=axis)
+        sl = [slice(None)] * v.ndim
+        sl[axis] = dst
+        out[tuple(sl)] = acc
+    return out
+
+
+def bicubic_up(v_u8, s):
+    """u8 [N,H,W,3] -> fp64 [N,sH,sW,3] on the 0..255 scale (horizontal pass, then vertical)."""
+    v = np.asarray(v_u8, dtype=np.float64)
+    return _bicubic_axis(_bicubic_axis(v, s, 2), s, 1)
+
+
+def skip_up(v_u8, s, skip="bilinear"):
+    return bilinear_up(v_u8, s) if skip == "bilinear" else bicubic_up(v_u8, s)
+
+
+# ----------------------------------------------------------------------------------------------------
 # network forward (see module docstring)
 # ----------------------------------------------------------------------------------------------------
 
@@ -203,10 +248,10 @@ def forward(flat_params, lr_u8, scale, blocks, channels, keep=False):
     return y
 
 
-def infer_u8(flat_params, lr_u8, scale, blocks, channels, return_float=False):
-    """Inference output: u8 = rint(clip(255 PS(y) + bilinear(v), 0, 255)) (R5)."""
+def infer_u8(flat_params, lr_u8, scale, blocks, channels, return_float=False, skip="bilinear"):
+    """Inference output: u8 = rint(clip(255 PS(y) + bilinear(v), 0, 255)) (R5); skip="bicubic" for R23."""
     y = forward(flat_params, lr_u8, scale, blocks, channels)
-    o255 = 255.0 * pixel_shuffle(y, scale) + bilinear_up(lr_u8, scale)
+    o255 = 255.0 * pixel_shuffle(y, scale) + skip_up(lr_u8, scale, skip)
     u8 = np.rint(np.clip(o255, 0.0, 255.0)).astype(np.uint8)
     if return_float:
         return u8, o255
@@ -217,12 +262,12 @@ def infer_u8(flat_params, lr_u8, scale, blocks, channels, return_float=False):
 # training: MSE loss (R6) and the analytic backward pass (chain rule written out by hand)
 # ----------------------------------------------------------------------------------------------------
 
-def train_loss_and_grad(flat_params, lr_u8, hr_u8, scale, blocks, channels, loss_kind="mse"):
+def train_loss_and_grad(flat_params, lr_u8, hr_u8, scale, blocks, channels, loss_kind="mse", skip="bilinear"):
     """Returns (loss, flat gradient) of L = mean over all HR elements of (o - hr/255)^2,
     o = PS(y) + bilinear(v)/255 (no clamp).  Gradient w.r.t. the parameters only (no input grad)."""
     y, a = forward(flat_params, lr_u8, scale, blocks, channels, keep=True)
     convs = a["convs"]
-    o = pixel_shuffle(y, scale) + bilinear_up(lr_u8, scale) / 255.0
+    o = pixel_shuffle(y, scale) + skip_up(lr_u8, scale, skip) / 255.0
     t = np.asarray(hr_u8, dtype=np.float64) / 255.0
     n_el = o.size
     if loss_kind == "mse":

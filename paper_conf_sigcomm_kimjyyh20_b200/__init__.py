@@ -62,14 +62,15 @@ class SRContext:
 
     def __init__(self, scale: int, blocks: int, channels: int, seed: int = 0, lr: float = 0.0,
                  world: int = 1, rank: int = 0, dp_weight: float = 0.0, recent_k: int = 0, recent_w: int = 0,
-                 pool_capacity: int = 0, loss: str = "mse"):
+                 pool_capacity: int = 0, loss: str = "mse", skip: str = "bilinear"):
         import torch
         if not torch.cuda.is_available():
             raise SRError("SRContext needs a CUDA device (no CPU fallback)")
         self.lib = load()
         self.scale, self.blocks, self.channels = scale, blocks, channels
         opt = sr_options(seed=seed, lr=lr, world=world, rank=rank, dp_weight=dp_weight, recent_k=recent_k,
-                         recent_w=recent_w, pool_capacity=pool_capacity, loss={"mse": 0, "l1": 1}[loss])
+                         recent_w=recent_w, pool_capacity=pool_capacity, loss={"mse": 0, "l1": 1}[loss],
+                         skip={"bilinear": 0, "bicubic": 1}[skip])
         h = C.c_void_p()
         st = self.lib.sr_create(scale, blocks, channels, C.byref(opt), C.byref(h))
         if st != 0:

@@ -17,7 +17,8 @@ MODELS = {"train": SR_TRAIN, "serve": SR_SERVE, "prev": SR_PREV, "init": SR_INIT
 class sr_options(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("lr", C.c_float), ("beta1", C.c_float), ("beta2", C.c_float),
                 ("eps", C.c_float), ("recent_k", C.c_int), ("recent_w", C.c_int), ("world", C.c_int),
-                ("rank", C.c_int), ("dp_weight", C.c_float), ("pool_capacity", C.c_int), ("loss", C.c_int)]
+                ("rank", C.c_int), ("dp_weight", C.c_float), ("pool_capacity", C.c_int), ("loss", C.c_int),
+                ("skip", C.c_int)]
 
 
 class sr_quality(C.Structure):

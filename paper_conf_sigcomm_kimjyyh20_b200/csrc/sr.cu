@@ -301,6 +301,7 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   EpiParams et{};
   et.bias = Bv(cu);
   et.scale = ctx->s;
+  et.bicubic = ctx->opt.skip == 1;
   et.lr = lr;
   et.hr = hr;
   et.hr_row0 = row0;
@@ -353,6 +354,7 @@ static sr_status forward_infer_virtual(sr_ctx* ctx, const Snapshot& sn, const ui
   EpiParams et{};
   et.bias = Bv(cu);
   et.scale = ctx->s;
+  et.bicubic = ctx->opt.skip == 1;
   et.lr = lr;
   et.hr = hr;
   et.vsep = sep;
@@ -427,6 +429,7 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
     e.dy = ctx->tdy;
     e.loss_sum = ctx->loss_sum;
     e.l1 = ctx->opt.loss == 1;
+    e.bicubic = ctx->opt.skip == 1;
     e.vsep = sep;
     e.vp = p;
     TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, e, st));
@@ -512,6 +515,7 @@ static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, i
     e.dy = ctx->tdy;
     e.loss_sum = ctx->loss_sum;
     e.l1 = ctx->opt.loss == 1;
+    e.bicubic = ctx->opt.skip == 1;
     TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, W(cu), n, p, p, e, st));
   }
   const double n_el = (double)pix * ctx->s * ctx->s * 3;
@@ -596,7 +600,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   if (ctx->opt.dp_weight == 0.f) ctx->opt.dp_weight = 1.f;
   if (ctx->opt.pool_capacity <= 0) ctx->opt.pool_capacity = 8192;
   if (ctx->opt.rank < 0 || ctx->opt.rank >= ctx->opt.world) { delete ctx; return SR_E_INVAL; }
-  if (ctx->opt.loss < 0 || ctx->opt.loss > 1) { delete ctx; return SR_E_INVAL; }
+  if (ctx->opt.loss < 0 || ctx->opt.loss > 1 || ctx->opt.skip < 0 || ctx->opt.skip > 1) { delete ctx; return SR_E_INVAL; }
   // conv table in canonical order: head, (b.conv1, b.conv2) x B, body, up
   std::vector<std::pair<int, int>> shp;  // (cout, cin)
   shp.push_back({channels, 3});

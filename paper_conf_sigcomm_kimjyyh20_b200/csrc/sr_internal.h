@@ -45,6 +45,7 @@ struct EpiParams {
   int dbg;             // benchmarking only: 1 = drain TMEM and skip the epilogue, 2 = plain store (no bias/res)
   int vsep, vp;        // EPI_TAIL_TRAIN on the virtual training batch: column pitch p+2 and patch size p (0 = off)
   int l1;              // EPI_TAIL_TRAIN: L1 loss (loss += |d|, dy = sign(d)) instead of MSE
+  int bicubic;         // tails: bicubic skip (reading R23) instead of bilinear
 };
 
 ConvGeom make_geom(int N, int H, int W, int cinp, int coutp, size_t* smem_bytes);

@@ -403,3 +403,32 @@ def test_patch_select_matches_oracle(hw, cell, max_sel, seed, step):
     got = ctx.patch_select(torch.from_numpy(raw).cuda(), torch.from_numpy(dec_full).cuda(), cell, max_sel, seed, step)
     assert got == select_patches(raw, dec_full, cell, max_sel, seed, step)
     assert len(got) > 0
+
+
+# ---------------------------------------------------------------- bicubic skip variant
+@pytest.mark.parametrize("cfg,hw", [((2, 2, 16), (37, 130)), ((3, 8, 48), (45, 301)), ((4, 2, 16), (20, 110))])
+def test_bicubic_skip_inference_parity(cfg, hw):
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=9, skip="bicubic")
+    lr, hr = synth_frames(2, hw[0], hw[1], seed=19, scale=s)
+    got = ctx.infer(torch.from_numpy(lr).cuda(), "serve").cpu().numpy()
+    ref = O.infer_u8(ctx.get_params("serve"), lr, s, B, C, skip="bicubic")
+    _check_frames(got, ref, hr)
+    # zero weights: the output is the bicubic skip itself (fp32 weights vs fp64 -> within 1 LSB)
+    ctx.set_params(np.zeros(ctx.num_params, np.float32))
+    z = ctx.infer(torch.from_numpy(lr).cuda(), "serve").cpu().numpy()
+    zb = np.rint(np.clip(O.bicubic_up(lr, s), 0, 255))
+    assert np.abs(z.astype(int) - zb.astype(int)).max() <= 1
+
+
+@pytest.mark.parametrize("cfg,n,p", [((2, 2, 8), 4, 16), ((3, 2, 32), 6, 24)])
+def test_bicubic_skip_training_parity(cfg, n, p):
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=23, skip="bicubic")
+    lrp, hrp, _ = synth_patch_pool(n, s, s * p, seed=33, frame_hw=(s * p * 3, s * p * 4))
+    lo = torch.zeros(1, device="cuda")
+    ctx.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo)
+    g = ctx.grad_buffer().cpu().numpy().copy()
+    ref_loss, ref_g = O.train_loss_and_grad(ctx.get_params("train"), lrp, hrp, s, B, C, skip="bicubic")
+    assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
+    assert rel_l2(g, ref_g) < 1e-2

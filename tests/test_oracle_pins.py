@@ -107,6 +107,29 @@ def test_bilinear_matches_torch_interpolate(s):
     np.testing.assert_allclose(O.bilinear_up(v, s), ref, rtol=0, atol=1e-12)
 
 
+@pytest.mark.parametrize("s", [2, 3, 4])
+def test_bicubic_matches_torch_interpolate(s):
+    """The bicubic skip variant (R23) = PyTorch bicubic, align_corners=False, A = -0.75, clamped taps."""
+    v = _rng(17).integers(0, 256, size=(2, 7, 9, 3)).astype(np.uint8)
+    ref = torch.nn.functional.interpolate(torch.from_numpy(v.astype(np.float64)).permute(0, 3, 1, 2),
+                                          scale_factor=s, mode="bicubic", align_corners=False)
+    np.testing.assert_allclose(O.bicubic_up(v, s), ref.permute(0, 2, 3, 1).numpy(), rtol=0, atol=1e-10)
+
+
+def test_bicubic_hand_computed_weights():
+    """Constants are reproduced exactly (weights sum to 1), and on a ramp v[i] = 10 i the x2 outputs use the
+    A = -0.75 weights worked out by hand: t = 0.75 -> (-0.03515625, 0.26171875, 0.87890625, -0.10546875) on
+    taps i0-1..i0+2, t = 0.25 -> the mirror.  (A = -0.75 does not reproduce linear functions exactly.)"""
+    c = np.full((1, 6, 6, 3), 77, np.uint8)
+    np.testing.assert_allclose(O.bicubic_up(c, 3), 77.0, atol=1e-12)
+    ramp = np.tile(np.arange(0, 120, 10, dtype=np.uint8).reshape(1, 1, 12, 1), (1, 3, 1, 3))
+    up = O.bicubic_up(ramp, 2)[0, 1, :, 0]
+    w75 = [-0.03515625, 0.26171875, 0.87890625, -0.10546875]
+    assert abs(up[4] - 10 * sum(w * i for w, i in zip(w75, range(0, 4)))) < 1e-12        # src 1.75
+    assert abs(up[5] - 10 * sum(w * i for w, i in zip(w75[::-1], range(1, 5)))) < 1e-12  # src 2.25
+    assert abs(up[4] - 17.03125) < 1e-12 and abs(up[5] - 22.96875) < 1e-12
+
+
 def test_bilinear_x2_values_are_sixteenths():
     """At x2 the separable weights are 1/4, 3/4: every value is an exact multiple of 1/16 (ties real)."""
     v = _rng(8).integers(0, 256, size=(1, 16, 16, 3)).astype(np.uint8)
