@@ -25,6 +25,7 @@
 #include "sr_internal.h"
 #include "kernels.h"
 #include "launch.cuh"
+#include "tail.cuh"
 
 namespace sr {
 
@@ -56,6 +57,11 @@ struct RollArgs {
   int sep;  // > 0: output columns with col % sep in {0, sep-1} are forced to 0
   int N, H, W;
   long long* dbg;  // benchmarking only: CTA-0 clock64 stamps [event][step]
+  // tail mode (TS > 0, the up conv): pixel shuffle + skip + clamp + RNE u8 straight from the epilogue
+  const uint8_t* lr;  // [N,H,W,3] LR frames (skip input)
+  uint8_t* hr;        // [N,TS H,TS W,3]
+  int hr_row0, hr_row1;  // LR rows whose HR rows are written (strip mode)
+  int bicubic;
 };
 #define SR_RDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -67,7 +73,7 @@ __device__ __forceinline__ void ld_row(const bf16* base, uint4* dst) {
   for (int q = 0; q < CH / 8; ++q) dst[q] = __ldg(p + q);
 }
 
-template <int CINP, int COUTP>
+template <int CINP, int COUTP, int TS>
 __global__ void __launch_bounds__(kRollThreads, 1)
 k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
             const __grid_constant__ CUtensorMap tm_aux, const bf16* __restrict__ wfold, const RollArgs a) {
@@ -178,7 +184,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     __syncwarp();
   } else if (warp == 10) {
     // ===================== store warp: TMA-store finished rows in emission order =====================
-    if (elect_one()) {
+    if (TS == 0 && elect_one()) {
       tma_prefetch_desc(&tm_out);
       int os[2] = {0, 0};
       uint32_t oph[2] = {0, 0};
@@ -244,6 +250,18 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       if (lane_id() == 0) mbar_arrive(&r_free[b]);
       if (warp == 2 && lane_id() == 0) { SR_RDBG(6, q + 1) }
       if (!emit) continue;
+      if constexpr (TS > 0) {  // up conv: the tail straight from registers (the ring held the bias)
+        if (lane_ok && r >= a.hr_row0 && r < a.hr_row1) {
+          EpiParams ep{};
+          ep.scale = TS;
+          ep.lr = a.lr;
+          ep.hr = a.hr;
+          ep.bicubic = a.bicubic;
+          float ls = 0.f;
+          epi_tail<TS, COUTP, false>(ep, nullptr, n, r, xc, H, W, v, ls, 0);
+        }
+        continue;
+      }
       const uint4* aux = reinterpret_cast<const uint4*>(sA + (int)(xi % NAUX) * ROWB + m * COUTP * 2);
       if (has_aux) mbar_wait(&x_full[xi % NAUX], (uint32_t)(xi / NAUX) & 1u);
       mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);  // the store warp has read this staging row
@@ -311,10 +329,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-template <int CINP, int COUTP>
+template <int CINP, int COUTP, int TS = 0>
 static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, const CUtensorMap& tx,
                                  const bf16* wfold, const RollArgs& a, int grid, cudaStream_t st) {
-  auto kern = k_conv_roll<CINP, COUTP>;
+  auto kern = k_conv_roll<CINP, COUTP, TS>;
   constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
   static bool configured = false;
   if (!configured) {
@@ -346,7 +364,7 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
   const void* auxp = res1 ? (const void*)res1 : (mask ? (const void*)mask : (const void*)out);
   if (make_row_tmap(&tx, auxp, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (res1 && mask) return cudaErrorNotSupported;  // one TMA aux stream per launch
-  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg};
+  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
@@ -354,6 +372,25 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
   SR_ROLL_CASE(32, 16) SR_ROLL_CASE(32, 32) SR_ROLL_CASE(32, 48)
   SR_ROLL_CASE(48, 16) SR_ROLL_CASE(48, 32) SR_ROLL_CASE(48, 48)
   SR_ROLL_CASE(64, 16) SR_ROLL_CASE(64, 32) SR_ROLL_CASE(64, 48)
+  return cudaErrorNotSupported;
+}
+
+#define SR_ROLL_TAIL_CASE(CI, CO, S) \
+  if (cinp == CI && coutp == CO && s == S) return launch_roll_t<CI, CO, S>(ti, ti, ti, wfold, a, grid, st);
+
+cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
+                                  const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
+                                  int W, cudaStream_t st) {
+  CUtensorMap ti;
+  if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
+    return cudaErrorInvalidValue;
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, lr, hr, hr_row0, hr_row1, bicubic};
+  const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  SR_ROLL_TAIL_CASE(16, 16, 2) SR_ROLL_TAIL_CASE(32, 16, 2) SR_ROLL_TAIL_CASE(48, 16, 2) SR_ROLL_TAIL_CASE(64, 16, 2)
+  SR_ROLL_TAIL_CASE(16, 32, 3) SR_ROLL_TAIL_CASE(32, 32, 3) SR_ROLL_TAIL_CASE(48, 32, 3) SR_ROLL_TAIL_CASE(64, 32, 3)
+  SR_ROLL_TAIL_CASE(16, 48, 4) SR_ROLL_TAIL_CASE(32, 48, 4) SR_ROLL_TAIL_CASE(48, 48, 4) SR_ROLL_TAIL_CASE(64, 48, 4)
   return cudaErrorNotSupported;
 }
 

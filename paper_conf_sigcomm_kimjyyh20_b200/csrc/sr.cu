@@ -73,6 +73,7 @@ struct sr_ctx {
   // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
   bool timing = false;
   bool fuse_blocks = true;  // fused residual-block kernel for wide frames (sr_set_option)
+  bool roll_tail = true;    // rolling up conv with the tail epilogue for wide frames (sr_set_fusion bit 2 clears)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -298,6 +299,19 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   eb.res1 = ctx->f0;
   eb.out = gbuf;
   TRY(conv_fwd(ctx, Cp, Cp, cur, sn, cb, n, h, w, eb, st));
+  if (roll_supported(Cp, ctx->OUTP, w) && ctx->roll_tail) {  // rolling up conv with the tail in its epilogue
+    if (ctx->timing) {
+      const double px = (double)n * h * w;
+      tmark_begin(ctx, "conv_tail_roll_" + std::to_string(Cp) + "x" + std::to_string(ctx->OUTP),
+                  2.0 * 9 * Cp * ctx->OUTP * px, px * (2.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
+    }
+    cudaError_t e = launch_conv_roll_tail(Cp, ctx->OUTP, ctx->s, gbuf, sn.wo + ctx->convs[cu].pk_off, Bv(cu), lr, hr,
+                                          row0, row1, ctx->opt.skip == 1, n, h, w, st);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll tail launch: ") + cudaGetErrorString(e));
+    return SR_OK;
+  }
   EpiParams et{};
   et.bias = Bv(cu);
   et.scale = ctx->s;
@@ -700,6 +714,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   if (!ctx) return SR_E_INVAL;
   ctx->fuse_blocks = (fuse_blocks & 1) != 0;
   ctx->virtual_train = (fuse_blocks & 2) == 0;  // bit 1 set: per-patch (narrow tile) training path
+  ctx->roll_tail = (fuse_blocks & 4) == 0;      // bit 2 set: tiled up conv + tail instead of the rolling one
   return SR_OK;
 }
 

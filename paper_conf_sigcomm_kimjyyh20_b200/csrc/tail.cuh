@@ -1,0 +1,206 @@
+// Shared epilogue pieces of the up-conv tail (pixel shuffle + bilinear / bicubic skip + clamp + RNE u8, or the
+// training loss / dy), used by the tiled conv (conv.cu) and the rolling conv (conv_roll.cu).
+// sbias may be null when the accumulator already holds the bias (the rolling kernel's bias-armed TMEM ring).
+#pragma once
+#include "ptx.cuh"
+#include "sr_internal.h"
+
+namespace sr {
+
+template <int COUTP>
+__device__ __forceinline__ void store_bf16_row(bf16* p, const float* v) {
+  uint4* q = reinterpret_cast<uint4*>(p);
+#pragma unroll
+  for (int i = 0; i < COUTP / 8; ++i) {
+    uint4 u;
+    u.x = pack_bf16x2(v[i * 8 + 0], v[i * 8 + 1]);
+    u.y = pack_bf16x2(v[i * 8 + 2], v[i * 8 + 3]);
+    u.z = pack_bf16x2(v[i * 8 + 4], v[i * 8 + 5]);
+    u.w = pack_bf16x2(v[i * 8 + 6], v[i * 8 + 7]);
+    q[i] = u;
+  }
+}
+
+// Bilinear skip by output phase (half-pixel centres, edge replicate == PyTorch align_corners=False):
+//   x2: phase 0 -> 0.25 v[i-1] + 0.75 v[i];  phase 1 -> 0.75 v[i] + 0.25 v[i+1]
+//   x3: phase 0 -> v[i-1]/3 + 2 v[i]/3;  phase 1 -> v[i];  phase 2 -> 2 v[i]/3 + v[i+1]/3
+//   x4: source offsets (ph + 1/2)/4 - 1/2 = -3/8, -1/8, +1/8, +3/8 (exact binary fractions)
+template <int S>
+__device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp) {
+  if (S == 2) {
+    wm = ph == 0 ? 0.25f : 0.f;
+    w0 = 0.75f;
+    wp = ph == 1 ? 0.25f : 0.f;
+  } else if (S == 4) {
+    wm = ph == 0 ? 0.375f : (ph == 1 ? 0.125f : 0.f);
+    w0 = (ph == 0 || ph == 3) ? 0.625f : 0.875f;
+    wp = ph == 3 ? 0.375f : (ph == 2 ? 0.125f : 0.f);
+  } else {
+    const float t = 1.f / 3.f, tt = 2.f / 3.f;
+    wm = ph == 0 ? t : 0.f;
+    w0 = ph == 1 ? 1.f : tt;
+    wp = ph == 2 ? t : 0.f;
+  }
+}
+
+// Bicubic skip variant (reading R23: Keys, A = -0.75, half-pixel centres without clamping the source coordinate,
+// clamped taps = PyTorch bicubic align_corners=False).  Phase ph of S: source offset d = (ph + 1/2)/S - 1/2;
+// d < 0 -> taps rows -2..+1 with t = 1 + d, else rows -1..+2 with t = d.  w[0..4] are the weights of rows -2..+2.
+__device__ __forceinline__ float cubic_w(float x) {
+  const float A = -0.75f;
+  x = fabsf(x);
+  return x <= 1.f ? ((A + 2.f) * x - (A + 3.f)) * x * x + 1.f
+                  : (x < 2.f ? ((A * x - 5.f * A) * x + 8.f * A) * x - 4.f * A : 0.f);
+}
+template <int S>
+__device__ __forceinline__ void cubic_phase_w(int ph, float* w) {
+  const float d = ((float)ph + 0.5f) / (float)S - 0.5f;
+  const bool neg = d < 0.f;
+  const float t = neg ? 1.f + d : d;
+  const int base = neg ? 0 : 1;  // index of tap k = -1 in rows -2..+2
+#pragma unroll
+  for (int a = 0; a < 5; ++a) w[a] = 0.f;
+#pragma unroll
+  for (int k = -1; k <= 2; ++k) w[base + k + 1] = cubic_w((float)k - t);
+}
+
+// Tail with the bicubic skip: as epi_tail below, skip = bicubic_S(v) from the 5 x 5 LR neighbourhood.
+template <int S, int COUTP, bool TRAIN>
+__device__ __noinline__ void epi_tail_bicubic(const EpiParams& ep, const float* sbias, int n, int Y, int X, int H,
+                                              int W, float* v, float& lsum, size_t dy_pix) {
+  const uint8_t* lr = ep.lr + (size_t)n * H * W * 3;
+  float hrow[5][S][3];  // horizontal pass on the five LR rows Y-2..Y+2 (clamped), per output phase j
+#pragma unroll
+  for (int a = 0; a < 5; ++a) {
+    const int yy = min(max(Y + a - 2, 0), H - 1);
+    float px[5][3];
+#pragma unroll
+    for (int b = 0; b < 5; ++b) {
+      const int xx = min(max(X + b - 2, 0), W - 1);
+      const uint8_t* p = lr + ((size_t)yy * W + xx) * 3;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) px[b][c] = (float)__ldg(p + c);
+    }
+#pragma unroll
+    for (int j = 0; j < S; ++j) {
+      float wx[5];
+      cubic_phase_w<S>(j, wx);
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        float acc = 0.f;
+#pragma unroll
+        for (int b = 0; b < 5; ++b) acc = fmaf(wx[b], px[b][c], acc);
+        hrow[a][j][c] = acc;
+      }
+    }
+  }
+  const int sH = S * H, sW = S * W;
+  float dyv[COUTP];
+#pragma unroll
+  for (int k = 0; k < COUTP; ++k) dyv[k] = 0.f;
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    float wy[5];
+    cubic_phase_w<S>(i, wy);
+    uint8_t* orow = TRAIN ? nullptr : ep.hr + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3;
+    const uint8_t* trow =
+        TRAIN ? ep.hr_ref + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3 : nullptr;
+#pragma unroll
+    for (int j = 0; j < S; ++j) {
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        float skip = 0.f;
+#pragma unroll
+        for (int a = 0; a < 5; ++a) skip = fmaf(wy[a], hrow[a][j][c], skip);
+        const int k = c * S * S + i * S + j;
+        const float y = v[k] + (sbias ? sbias[k] : 0.f);
+        if (TRAIN) {
+          const float o = y + skip * (1.f / 255.f);
+          const float d = o - (float)__ldg(trow + j * 3 + c) * (1.f / 255.f);
+          if (ep.l1) {
+            lsum += fabsf(d);
+            dyv[k] = d > 0.f ? 1.f : (d < 0.f ? -1.f : 0.f);
+          } else {
+            lsum += d * d;
+            dyv[k] = 2.f * d;
+          }
+        } else {
+          const float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
+          orow[j * 3 + c] = (uint8_t)__float2int_rn(o);
+        }
+      }
+    }
+  }
+  if (TRAIN) store_bf16_row<COUTP>(ep.dy + dy_pix * COUTP, dyv);
+}
+
+// Tail: y = acc + b (3 s^2 channels, index c*s^2 + i*s + j = pixel-shuffle phase (i,j) of colour c);
+// skip = bilinear_s(v) at HR (sY+i, sX+j).  Inference: u8 = RNE(clamp(255 y + skip, 0, 255)).
+// Training: o = y + skip/255, d = o - hr/255 -> loss += d^2, dy[c s^2 + i s + j] = 2 d (L1: |d|, sign(d)).
+// (n, Y, X) addresses the LR image / HR target (n-th image of size H x W); dy_pix is the pixel index of this
+// output in the conv's own layout (equal to ((n H + Y) W + X) except for the virtual training batch).
+template <int S, int COUTP, bool TRAIN>
+__device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias, int n, int Y, int X, int H,
+                                         int W, float* v, float& lsum, size_t dy_pix) {
+  if (ep.bicubic) {
+    epi_tail_bicubic<S, COUTP, TRAIN>(ep, sbias, n, Y, X, H, W, v, lsum, dy_pix);
+    return;
+  }
+  const uint8_t* lr = ep.lr + (size_t)n * H * W * 3;
+  float nb[3][3][3];  // [dy][dx][c] neighbourhood of LR pixel (Y,X), clamped (edge replicate)
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    int yy = min(max(Y + a - 1, 0), H - 1);
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      int xx = min(max(X + b - 1, 0), W - 1);
+      const uint8_t* p = lr + ((size_t)yy * W + xx) * 3;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) nb[a][b][c] = (float)__ldg(p + c);
+    }
+  }
+  const int sH = S * H, sW = S * W;
+  float dyv[COUTP];
+#pragma unroll
+  for (int k = 0; k < COUTP; ++k) dyv[k] = 0.f;
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    float ym, y0, yp;
+    phase_w<S>(i, ym, y0, yp);
+    uint8_t* hrow = TRAIN ? nullptr : ep.hr + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3;
+    const uint8_t* trow =
+        TRAIN ? ep.hr_ref + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3 : nullptr;
+#pragma unroll
+    for (int j = 0; j < S; ++j) {
+      float xm, x0, xp;
+      phase_w<S>(j, xm, x0, xp);
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        // horizontal pass on the three LR rows, then vertical
+        float h0 = xm * nb[0][0][c] + x0 * nb[0][1][c] + xp * nb[0][2][c];
+        float h1 = xm * nb[1][0][c] + x0 * nb[1][1][c] + xp * nb[1][2][c];
+        float h2 = xm * nb[2][0][c] + x0 * nb[2][1][c] + xp * nb[2][2][c];
+        float skip = ym * h0 + y0 * h1 + yp * h2;
+        const int k = c * S * S + i * S + j;
+        float y = v[k] + (sbias ? sbias[k] : 0.f);
+        if (TRAIN) {
+          float o = y + skip * (1.f / 255.f);
+          float d = o - (float)__ldg(trow + j * 3 + c) * (1.f / 255.f);
+          if (ep.l1) {  // L1 variant: |d|, d/d o = sign(d) (0 at 0)
+            lsum += fabsf(d);
+            dyv[k] = d > 0.f ? 1.f : (d < 0.f ? -1.f : 0.f);
+          } else {
+            lsum += d * d;
+            dyv[k] = 2.f * d;
+          }
+        } else {
+          float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
+          hrow[j * 3 + c] = (uint8_t)__float2int_rn(o);
+        }
+      }
+    }
+  }
+  if (TRAIN) store_bf16_row<COUTP>(ep.dy + dy_pix * COUTP, dyv);
+}
+
+}  // namespace sr

@@ -432,3 +432,17 @@ def test_bicubic_skip_training_parity(cfg, n, p):
     ref_loss, ref_g = O.train_loss_and_grad(ctx.get_params("train"), lrp, hrp, s, B, C, skip="bicubic")
     assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
     assert rel_l2(g, ref_g) < 1e-2
+
+
+@pytest.mark.parametrize("cfg,hw", [((3, 8, 48), (50, 300)), ((2, 2, 16), (33, 130)), ((4, 2, 32), (20, 200))])
+def test_rolling_tail_equals_tiled_tail(cfg, hw):
+    """Up conv + tail on the rolling kernel (default for wide frames) vs the tiled one (set_fusion bit 2): same
+    math, different fp32 summation order -> within 1 LSB; strips (hr_row0/1) covered by test_strip_*."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=14)
+    lr = torch.from_numpy(synth_frames(2, hw[0], hw[1], seed=15)).cuda()
+    a = ctx.infer(lr, "serve").clone()
+    ctx.set_fusion(1 | 4)
+    b = ctx.infer(lr, "serve")
+    torch.cuda.synchronize()
+    assert (a.int() - b.int()).abs().max().item() <= 1
