@@ -176,7 +176,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_DBG(9, st)
         tc_fence_after();
         if (!(exp & 32))
-          ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, PLANE);
+          ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, 2 * PLANE);
         mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
         mma_commit(&f_empty[fs]);
         if (st == n_f - 1) {                      // the last two rows of the piece receive nothing more
@@ -208,7 +208,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_DBG(12, k + 3)
         tc_fence_after();
         if (!(exp & 16))
-          ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, PLANE);
+          ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, 2 * PLANE);
         mma_commit(&r2_ready[ring_idx<RB>(g)]);
         mma_commit(&t_empty[ts]);
         if (k == n_t - 1) {

@@ -168,7 +168,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         mbar_wait(&in_full[s], ph);
         SR_RDBG(3, i)
         tc_fence_after();
-        ring_mma_step<CINP, COUTP, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, PLANE);
+        ring_mma_step<CINP, COUTP, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, 2 * PLANE);
         mma_commit(&r_ready[ring_idx<RB>(g)]);
         mma_commit(&in_empty[s]);
         SR_RDBG(4, i)

@@ -11,9 +11,11 @@
 
 namespace sr {
 
-template <int CINP, int COUTP, int RB>
+// A operand = one input row: APX bytes per pixel row of a K-atom (16 for SWIZZLE_NONE 8-channel chunks, 32 for
+// SWIZZLE_32B 16-channel blocks); kstride = bytes from one K step (16 channels) to the next.
+template <int CINP, int COUTP, int RB, int APX = 16>
 __device__ __forceinline__ void ring_mma_step(uint32_t ring_base, long long g, uint64_t ad, uint64_t bd,
-                                              uint32_t plane) {
+                                              uint32_t kstride) {
   constexpr int CCH = CINP / 8, KS = CINP / 16, N = 3 * COUTP;
   const int i0 = ring_idx<RB>(g);
   int blkA, rowA, nA, blkB = 0, rowB = 0, nB = 0;
@@ -25,7 +27,7 @@ __device__ __forceinline__ void ring_mma_step(uint32_t ring_base, long long g, u
   for (int dx = 0; dx < 3; ++dx)
 #pragma unroll
     for (int ks = 0; ks < KS; ++ks)
-      mma_bf16_ss(ring_base + blkA * COUTP, desc_add(ad, dx * 16u + ks * 2u * plane),
+      mma_bf16_ss(ring_base + blkA * COUTP, desc_add(ad, dx * (uint32_t)APX + ks * kstride),
                   desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * N * 16u + rowA * 16u), idA, 1u);
   if (nB) {
     const uint32_t idB = make_idesc(128, nB, 0, 0);
@@ -33,7 +35,7 @@ __device__ __forceinline__ void ring_mma_step(uint32_t ring_base, long long g, u
     for (int dx = 0; dx < 3; ++dx)
 #pragma unroll
       for (int ks = 0; ks < KS; ++ks)
-        mma_bf16_ss(ring_base + blkB * COUTP, desc_add(ad, dx * 16u + ks * 2u * plane),
+        mma_bf16_ss(ring_base + blkB * COUTP, desc_add(ad, dx * (uint32_t)APX + ks * kstride),
                     desc_add(bd, (uint32_t)(dx * CCH + 2 * ks) * N * 16u + rowB * 16u), idB, 1u);
   }
 }

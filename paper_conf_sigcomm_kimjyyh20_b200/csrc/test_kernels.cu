@@ -37,7 +37,11 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
     uint32_t off;
     if (!a_mn) off = (k / 8) * (MA * 16) + m * 16 + (k % 8) * 2;          // K-major: LBO = MA*16, SBO = 128
     else if (a_mn == 1) off = (m / 8) * (K * 16) + k * 16 + (m % 8) * 2;  // MN-major: SBO = K*16, LBO = 128
-    else off = sw32_mn_off(m, k, K, shift >= 4 ? 64 : 0);                  // MN-major SWIZZLE_32B
+    else if (a_mn == 4) {                                                   // K-major SWIZZLE_32B
+      const uint32_t lin = (uint32_t)(k / 16) * (MA * 32) + (uint32_t)m * 32 + (uint32_t)((k % 16) / 8) * 16;
+      const uint32_t abs_ = smem_u32(sA) + lin;
+      off = (lin ^ ((abs_ & 0x80u) >> 3)) + (uint32_t)(k % 8) * 2;
+    } else off = sw32_mn_off(m, k, K, shift >= 4 ? 64 : 0);                // MN-major SWIZZLE_32B
     *reinterpret_cast<__nv_bfloat16*>(sA + off) = v;
   }
   for (int i = threadIdx.x; i < N * K; i += blockDim.x) {
@@ -56,20 +60,21 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
   tc_fence_after();
   const uint32_t tmem = tmem_base;
   if (threadIdx.x == 0) {
-    const uint32_t idesc = make_idesc(128, N, a_mn ? 1 : 0, b_mn ? 1 : 0);
+    const uint32_t idesc = make_idesc(128, N, (a_mn && a_mn != 4) ? 1 : 0, b_mn ? 1 : 0);
     const uint32_t a0 = smem_u32(sA), b0 = smem_u32(sB);
     // SWIZZLE_32B MN-major: atoms of 16 MN elements x 8 K rows (256 B); mode 2 puts the MN-atom stride (K*32) in
     // LBO and the 8-row K-group stride (256) in SBO, mode 3 the other way round (to pin the encoding)
     auto sw_desc = [&](uint32_t base, int mode, int pad) {
       return mode == 2 ? make_desc_sw(base, K * 32 + pad, 256, 6) : make_desc_sw(base, 256, K * 32 + pad, 6);
     };
-    uint64_t adesc = a_mn >= 2 ? sw_desc(a0, a_mn, shift >= 4 ? 64 : 0)
+    uint64_t adesc = a_mn == 4 ? make_desc_sw(a0, 16, 256, 6)
+                   : a_mn >= 2 ? sw_desc(a0, a_mn, shift >= 4 ? 64 : 0)
                                : a_mn ? make_desc(a0, 128, K * 16) : make_desc(a0, MA * 16, 128);
     uint64_t bdesc = b_mn >= 2 ? sw_desc(b0, b_mn, 0) : b_mn ? make_desc(b0, 128, K * 16) : make_desc(b0, N * 16, 128);
     const int ksteps = K / 16;
     // one K step = 16 elements = 2 chunks: K-major advances by 2*LBO, MN-major by 2 LBO-groups (256 B),
     // MN-major SWIZZLE_32B by 16 rows of 32 B (512 B)
-    const uint32_t a_step = a_mn >= 2 ? 512 : a_mn ? 256 : 2 * MA * 16;
+    const uint32_t a_step = a_mn == 4 ? MA * 32 : a_mn >= 2 ? 512 : a_mn ? 256 : 2 * MA * 16;
     const uint32_t b_step = b_mn >= 2 ? 512 : b_mn ? 256 : 2 * N * 16;
     long long t0 = clock64();
     if (reps > 0 && ksteps == 4) {
@@ -103,7 +108,7 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
       int total = reps > 0 ? reps : 1;
       for (int r = 0; r < total; ++r) {
         for (int ks = 0; ks < ksteps; ++ks) {
-          uint32_t sh = shift ? 16u * ((r * ksteps + ks) % 3) : 0u;
+          uint32_t sh = shift == 7 ? 32u : shift ? 16u * ((r * ksteps + ks) % 3) : 0u;
           mma_bf16_ss(tmem, desc_add(adesc, ks * a_step + sh), desc_add(bdesc, ks * b_step), idesc,
                       (r | ks) != 0);
         }
@@ -218,7 +223,7 @@ extern "C" int sr_bench_tma(const void* act, int H, int W, int Cp, int mode, int
 extern "C" int sr_test_mma(const void* A, const void* B, float* D, int N, int K, int a_mn, int b_mn, int reps,
                            int shift, long long* cycles_dev, void* stream) {
   if (N % 16 || N < 16 || N > 256 || K % 16 || K < 16) return SR_E_INVAL;
-  size_t smem = (size_t)(128 + 16) * K * 2 + (size_t)N * K * 2 + 1024 + 1024;
+  size_t smem = (size_t)(128 + 16) * K * 4 + (size_t)N * K * 2 + 1024 + 1024;
   if (smem > 200 * 1024) return SR_E_INVAL;
   cudaFuncSetAttribute(k_test_mma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k_test_mma<<<1, 128, smem, (cudaStream_t)stream>>>((const __nv_bfloat16*)A, (const __nv_bfloat16*)B, D, N, K,
