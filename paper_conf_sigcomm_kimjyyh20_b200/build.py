@@ -3,12 +3,14 @@ import os
 import shutil
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libsr.so")
-SOURCES = ["conv.cu", "conv_roll.cu", "conv_block.cu", "kernels.cu", "sr.cu", "test_kernels.cu"]
+SOURCES = ["conv.cu", "conv_roll.cu", "conv_block.cu", "conv_wgrad.cu", "kernels.cu", "sr.cu", "test_kernels.cu"]
+OBJDIR = os.path.join(ROOT, "build", "obj")
 
 
 def nvcc_path():
@@ -27,12 +29,29 @@ def needs_rebuild():
 
 
 def build(force=False, verbose=True):
+    """Compile every translation unit to an object in parallel (build/obj), then link libsr.so."""
     if not force and not needs_rebuild():
         return LIB
-    cmd = [nvcc_path(), "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
-           "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-v" if os.environ.get("SR_PTXAS_V") else "-O3",
-           "-I", os.path.join(ROOT, "include"), "-o", LIB + ".tmp"]
-    cmd += [os.path.join(CSRC, s) for s in SOURCES]
+    os.makedirs(OBJDIR, exist_ok=True)
+    flags = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-Xcompiler", "-fPIC",
+             "-Xptxas", "-v" if os.environ.get("SR_PTXAS_V") else "-O3", "-I", os.path.join(ROOT, "include")]
+    nvcc = nvcc_path()
+
+    def compile_one(src):
+        obj = os.path.join(OBJDIR, src.replace(".cu", ".o"))
+        cmd = [nvcc] + flags + ["-c", os.path.join(CSRC, src), "-o", obj]
+        if verbose:
+            print(" ".join(cmd), file=sys.stderr)
+        r = subprocess.run(cmd, cwd=CSRC, capture_output=True, text=True)
+        if r.stderr:
+            print(r.stderr, file=sys.stderr, end="")
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed on {src}")
+        return obj
+
+    with ThreadPoolExecutor(max_workers=min(len(SOURCES), os.cpu_count() or 4)) as ex:
+        objs = list(ex.map(compile_one, SOURCES))
+    cmd = [nvcc, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", LIB + ".tmp"] + objs
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.run(cmd, check=True, cwd=CSRC)

@@ -96,6 +96,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
 
   const int N = a.N, H = a.H, W = a.W;
   const int warp = warp_id();
+  if (threadIdx.x == 0) { SR_RDBG(8, 0) }  // kernel entry
   if (warp == 0 && lane_id() == 0) {
     for (int s = 0; s < kRollIn; ++s) { mbar_init(&in_full[s], 1); mbar_init(&in_empty[s], 1); }
     for (int s = 0; s < RB; ++s) { mbar_init(&r_ready[s], 1); mbar_init(&r_free[s], 4); }
@@ -108,6 +109,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   tc_fence_before();
   __syncthreads();
   pdl_enter();  // predecessor complete: global inputs are valid from here on
+  if (threadIdx.x == 0) { SR_RDBG(10, 0) }  // after setup + PDL wait
   if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
   __syncthreads();
   tc_fence_after();
@@ -326,6 +328,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
 #undef SR_PIECE_END
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) { SR_RDBG(9, 0) }  // all roles done
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 

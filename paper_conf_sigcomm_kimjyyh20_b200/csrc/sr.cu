@@ -43,6 +43,8 @@ struct sr_ctx {
   bf16 *tx16 = nullptr, *tg = nullptr, *tdy = nullptr, *tdg = nullptr, *tdfa = nullptr, *tdfb = nullptr,
        *tdt = nullptr;
   std::vector<bf16*> tf, tts;
+  std::vector<bf16*> tdf, tdtb;  // virtual training path: every block's df_b (B+1) and dt_b (B), kept for the
+                                 // batched wgrad at the end of the backward pass
   float* ws_w = nullptr;       // wgrad split-K partials [grid][9 cinp coutp + coutp]
   size_t ws_w_elems = 0;
   unsigned* wg_sync = nullptr; // wgrad grid barrier {count, generation}
@@ -104,6 +106,11 @@ static cudaError_t dalloc(T** p, size_t count) {
   return cudaMalloc(reinterpret_cast<void**>(p), count * sizeof(T));
 }
 static int rup16(int c) { return (c + 15) / 16 * 16; }
+#define TRY_(x)                  \
+  do {                           \
+    sr_status s_ = (x);          \
+    if (s_ != SR_OK) return s_;  \
+  } while (0)
 
 static uint64_t mix64h(uint64_t z) {
   z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
@@ -199,36 +206,71 @@ static sr_status roll_ex(sr_ctx* ctx, const char* cls, int cinp, int coutp, cons
   return SR_OK;
 }
 
-static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N, int H, int W, float scale,
-                       cudaStream_t st) {
+static WgradJob wjob(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy) {
   const ConvDesc& d = ctx->convs[ci];
-  size_t smem = 0;
-  WgradGeom g = make_wgrad_geom(N, H, W, d.cinp, d.coutp, &smem);
-  int grid = std::min(g.units, num_sms());
-  size_t need_w = (size_t)grid * (9 * d.cinp * d.coutp + d.coutp);
-  if (need_w > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, need_w)); ctx->ws_w_elems = need_w; }
+  float* gW = ctx->grad + d.w_off;
+  return WgradJob{x, dy, d.cinp, d.coutp, d.cin, d.cout, gW, gW + (size_t)d.cout * d.cin * 9};
+}
+
+static sr_status ensure_wg(sr_ctx* ctx, size_t elems, cudaStream_t st) {
+  if (elems > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, elems)); ctx->ws_w_elems = elems; }
   if (!ctx->wg_sync) {
     CK(dalloc(&ctx->wg_sync, 2));
     CK(cudaMemsetAsync(ctx->wg_sync, 0, 2 * sizeof(unsigned), st));
   }
-  if (ctx->timing) {
-    const double px = (double)N * H * W;
-    tmark_begin(ctx, "wgrad_" + std::to_string(d.cinp) + "x" + std::to_string(d.coutp),
-                2.0 * 9 * d.cinp * d.coutp * px, px * 2.0 * (d.cinp + d.coutp), st);
-  }
-  WgradOut o{};
-  o.ws = ctx->ws_w;
-  o.sync = ctx->wg_sync;
-  o.gW = ctx->grad + d.w_off;
-  o.gb = o.gW + (size_t)d.cout * d.cin * 9;
-  o.cin = d.cin;
-  o.cout = d.cout;
-  o.scale = scale;
-  cudaError_t e = launch_wgrad(d.cinp, d.coutp, x, dy, g, o, smem, grid, st);
-  tmark_end(ctx, st);
-  ctx->launches++;
-  if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("wgrad launch: ") + cudaGetErrorString(e));
   return SR_OK;
+}
+
+// Weight (+ bias) gradients of a list of convs whose inputs share one shape: grad <- scale * dL/dW.  Wide images: the
+// batched rolling kernel (one launch per kWgradMaxJobs convs); otherwise the tiled kernel, one launch per conv.
+static sr_status wgrad_jobs(sr_ctx* ctx, const WgradJob* jobs, int J, int N, int H, int W, float scale,
+                            cudaStream_t st) {
+  for (int k0 = 0; k0 < J; k0 += kWgradMaxJobs) {
+    const int nj = std::min(kWgradMaxJobs, J - k0);
+    const WgradJob* jb = jobs + k0;
+    if (!wgrad_multi_supported(jb, nj, W)) break;
+    const int grid = wgrad_multi_grid(nj, N, H, W);
+    TRY_(ensure_wg(ctx, wgrad_multi_ws_floats(jb, nj, grid), st));
+    if (ctx->timing) {
+      double fl = 0, by = 0;
+      const double px = (double)N * H * W;
+      for (int k = 0; k < nj; ++k) {
+        fl += 2.0 * 9 * jb[k].cinp * jb[k].coutp * px;
+        by += px * 2.0 * (jb[k].cinp + jb[k].coutp);
+      }
+      tmark_begin(ctx, nj > 1 ? "wgrad_batch" : "wgrad_" + std::to_string(jb[0].cinp) + "x" +
+                                                    std::to_string(jb[0].coutp), fl, by, st);
+    }
+    cudaError_t e = launch_wgrad_multi(jb, nj, N, H, W, scale, ctx->ws_w, ctx->wg_sync, grid, nullptr, st);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("wgrad launch: ") + cudaGetErrorString(e));
+    if (k0 + nj == J) return SR_OK;
+  }
+  for (int k = 0; k < J; ++k) {  // tiled kernel
+    const WgradJob& j = jobs[k];
+    size_t smem = 0;
+    WgradGeom g = make_wgrad_geom(N, H, W, j.cinp, j.coutp, &smem);
+    const int grid = std::min(g.units, num_sms());
+    TRY_(ensure_wg(ctx, (size_t)grid * (9 * j.cinp * j.coutp + j.coutp), st));
+    if (ctx->timing) {
+      const double px = (double)N * H * W;
+      tmark_begin(ctx, "wgrad_" + std::to_string(j.cinp) + "x" + std::to_string(j.coutp),
+                  2.0 * 9 * j.cinp * j.coutp * px, px * 2.0 * (j.cinp + j.coutp), st);
+    }
+    WgradOut o{ctx->ws_w, ctx->wg_sync, j.gW, j.gb, j.cin, j.cout, scale};
+    cudaError_t e = launch_wgrad(j.cinp, j.coutp, j.x, j.dy, g, o, smem, grid, st);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("wgrad launch: ") + cudaGetErrorString(e));
+  }
+  return SR_OK;
+}
+
+static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N, int H, int W, float scale,
+                       cudaStream_t st) {
+  const WgradJob j = wjob(ctx, ci, x, dy);
+  return wgrad_jobs(ctx, &j, 1, N, H, W, scale, st);
 }
 
 #define TRY(x)                   \
@@ -389,6 +431,8 @@ static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
   CK(dalloc(&ctx->tdfa, pix * Cp));
   CK(dalloc(&ctx->tdfb, pix * Cp));
   CK(dalloc(&ctx->tdt, pix * Cp));
+  for (auto& p : ctx->tdf) CK(dalloc(&p, pix * Cp));
+  for (auto& p : ctx->tdtb) CK(dalloc(&p, pix * Cp));
   ctx->tr_pix = pix;
   return SR_OK;
 }
@@ -454,26 +498,27 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
     ctx->launches++;
   }
   const float gscale = (float)((ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.0f) / n_el);
-  // ---- backward
-  TRY(wgrad(ctx, cu, ctx->tg, ctx->tdy, 1, Hv, Wv, gscale, st));
+  // ---- backward: the data-gradient chain (every df_b, dt_b kept), then all weight gradients in one batched launch
   TRY(roll_ex(ctx, "train_dgrad", OUTP, Cp, ctx->tdy, WDO(cu), nullptr, nullptr, nullptr, nullptr, 0, sep, ctx->tdg, 1,
               Hv, Wv, st));
-  TRY(wgrad(ctx, cb, ctx->tf[B], ctx->tdg, 1, Hv, Wv, gscale, st));
-  bf16* df = ctx->tdfa;
   TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdg, WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr,
-              0, sep, df, 1, Hv, Wv, st));
+              0, sep, ctx->tdf[B], 1, Hv, Wv, st));
   for (int b = B - 1; b >= 0; --b) {
-    TRY(wgrad(ctx, 2 + 2 * b, ctx->tts[b], df, 1, Hv, Wv, gscale, st));
-    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, df, WDO(2 + 2 * b), nullptr, nullptr, nullptr, ctx->tts[b], 0, sep,
-                ctx->tdt, 1, Hv, Wv, st));
-    TRY(wgrad(ctx, 1 + 2 * b, ctx->tf[b], ctx->tdt, 1, Hv, Wv, gscale, st));
-    bf16* dfn = (df == ctx->tdfa) ? ctx->tdfb : ctx->tdfa;
-    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdt, WDO(1 + 2 * b), nullptr, df, b == 0 ? ctx->tdg : nullptr,
-                nullptr, 0, sep, dfn, 1, Hv, Wv, st));
-    df = dfn;
+    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdf[b + 1], WDO(2 + 2 * b), nullptr, nullptr, nullptr, ctx->tts[b],
+                0, sep, ctx->tdtb[b], 1, Hv, Wv, st));
+    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdtb[b], WDO(1 + 2 * b), nullptr, ctx->tdf[b + 1],
+                b == 0 ? ctx->tdg : nullptr, nullptr, 0, sep, ctx->tdf[b], 1, Hv, Wv, st));
   }
-  TRY(wgrad(ctx, 0, ctx->tx16, df, 1, Hv, Wv, gscale, st));
-  return SR_OK;
+  // jobs in reverse production order of their dY (the most recent dY is the likeliest to still sit in L2)
+  std::vector<WgradJob> jobs;
+  jobs.push_back(wjob(ctx, 0, ctx->tx16, ctx->tdf[0]));
+  for (int b = 0; b < B; ++b) {
+    jobs.push_back(wjob(ctx, 1 + 2 * b, ctx->tf[b], ctx->tdtb[b]));
+    jobs.push_back(wjob(ctx, 2 + 2 * b, ctx->tts[b], ctx->tdf[b + 1]));
+  }
+  jobs.push_back(wjob(ctx, cb, ctx->tf[B], ctx->tdg));
+  jobs.push_back(wjob(ctx, cu, ctx->tg, ctx->tdy));
+  return wgrad_jobs(ctx, jobs.data(), (int)jobs.size(), 1, Hv, Wv, gscale, st);
 }
 
 // Forward with saved activations, MSE loss + gradient fused into the tail, backward (dgrad = the fwd conv
@@ -662,6 +707,8 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->adam_scal, 2);
   ctx->tf.assign(blocks + 1, nullptr);
   ctx->tts.assign(blocks, nullptr);
+  ctx->tdf.assign(blocks + 1, nullptr);
+  ctx->tdtb.assign(blocks, nullptr);
   if (st != SR_OK) { sr_destroy(ctx); return st; }
   if (cudaMemcpy(ctx->convs_dev, ctx->convs.data(), ctx->convs.size() * sizeof(ConvDesc),
                  cudaMemcpyHostToDevice) != cudaSuccess ||
@@ -701,6 +748,8 @@ void sr_destroy(sr_ctx* ctx) {
   for (int k = 0; k < 4; ++k) { cudaFree(ctx->snap[k].wf); cudaFree(ctx->snap[k].wo); cudaFree(ctx->snap[k].bias); }
   for (auto p : ctx->tf) if (p) cudaFree(p);
   for (auto p : ctx->tts) if (p) cudaFree(p);
+  for (auto p : ctx->tdf) if (p) cudaFree(p);
+  for (auto p : ctx->tdtb) if (p) cudaFree(p);
   if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
   if (ctx->train_graph) cudaGraphExecDestroy(ctx->train_graph);
   for (auto e : ctx->chunk_ev) if (e) cudaEventDestroy(e);
@@ -1300,30 +1349,37 @@ sr_status sr_test_conv(const void* x_dev, int n, int h, int w, int cin, int cout
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
 
+sr_status sr_test_wgrad_batch(int J, const void* const* x_devs, const void* const* dy_devs, int n, int h, int w,
+                              const int* cins, const int* couts, float* out_host, sr_stream stream) {
+  if (J < 1 || !x_devs || !dy_devs || !cins || !couts || !out_host) return SR_E_INVAL;
+  cudaStream_t st = (cudaStream_t)stream;
+  std::vector<size_t> off(J + 1, 0);
+  for (int k = 0; k < J; ++k) off[k + 1] = off[k] + (size_t)couts[k] * cins[k] * 9 + couts[k];
+  float* gout = nullptr;
+  if (cudaMalloc(&gout, off[J] * 4)) return SR_E_NOMEM;
+  std::vector<WgradJob> jobs(J);
+  for (int k = 0; k < J; ++k)
+    jobs[k] = WgradJob{(const bf16*)x_devs[k], (const bf16*)dy_devs[k], rup16(cins[k]), rup16(couts[k]), cins[k],
+                       couts[k], gout + off[k], gout + off[k] + (size_t)couts[k] * cins[k] * 9};
+  sr_ctx tmp;  // workspace holder only (the same batching/fallback logic as training)
+  sr_status rc = wgrad_jobs(&tmp, jobs.data(), J, n, h, w, 1.0f, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  if (rc == SR_OK && e2 == cudaSuccess) cudaMemcpy(out_host, gout, off[J] * 4, cudaMemcpyDeviceToHost);
+  cudaFree(gout);
+  if (tmp.ws_w) cudaFree(tmp.ws_w);
+  if (tmp.wg_sync) cudaFree(tmp.wg_sync);
+  return rc != SR_OK ? rc : (e2 == cudaSuccess ? SR_OK : SR_E_CUDA);
+}
+
 sr_status sr_test_wgrad(const void* x_dev, const void* dy_dev, int n, int h, int w, int cin, int cout,
                         float* dw_host, float* db_host, sr_stream stream) {
   if (!x_dev || !dy_dev || !dw_host || !db_host) return SR_E_INVAL;
-  cudaStream_t st = (cudaStream_t)stream;
-  const int cinp = rup16(cin), coutp = rup16(cout);
-  size_t smem = 0;
-  WgradGeom g = make_wgrad_geom(n, h, w, cinp, coutp, &smem);
-  int grid = std::min(g.units, num_sms());
-  float *ws = nullptr, *gout = nullptr;
-  unsigned* sync = nullptr;
-  const size_t np = (size_t)cout * cin * 9 + cout;
-  if (cudaMalloc(&ws, (size_t)grid * (9 * cinp * coutp + coutp) * 4) || cudaMalloc(&gout, np * 4) ||
-      cudaMalloc(&sync, 8))
-    return SR_E_NOMEM;
-  cudaMemsetAsync(sync, 0, 8, st);
-  WgradOut o{ws, sync, gout, gout + (size_t)cout * cin * 9, cin, cout, 1.0f};
-  cudaError_t e = launch_wgrad(cinp, coutp, (const bf16*)x_dev, (const bf16*)dy_dev, g, o, smem, grid, st);
-  cudaError_t e2 = cudaStreamSynchronize(st);
-  std::vector<float> h_(np);
-  cudaMemcpy(h_.data(), gout, np * 4, cudaMemcpyDeviceToHost);
+  std::vector<float> h_((size_t)cout * cin * 9 + cout);
+  sr_status rc = sr_test_wgrad_batch(1, &x_dev, &dy_dev, n, h, w, &cin, &cout, h_.data(), stream);
+  if (rc != SR_OK) return rc;
   memcpy(dw_host, h_.data(), (size_t)cout * cin * 9 * 4);
   memcpy(db_host, h_.data() + (size_t)cout * cin * 9, cout * 4);
-  cudaFree(ws); cudaFree(gout); cudaFree(sync);
-  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+  return SR_OK;
 }
 
 }  // extern "C"

@@ -75,6 +75,22 @@ WgradGeom make_wgrad_geom(int N, int H, int W, int cinp, int coutp, size_t* smem
 cudaError_t launch_wgrad(int cinp, int coutp, const bf16* x, const bf16* dy, const WgradGeom& g, const WgradOut& o,
                          size_t smem, int grid, cudaStream_t st);
 
+// Batched rolling wgrad for wide images (conv_wgrad.cu): up to kWgradMaxJobs convs over inputs of one shape in one
+// launch, partials ws[(grid + J)][max stride] (wgrad_multi_ws_floats), grid = wgrad_multi_grid, sync as WgradOut.
+static constexpr int kWgradMaxJobs = 20;
+struct WgradJob {
+  const bf16* x;   // conv input  [N,H,W,cinp]
+  const bf16* dy;  // conv output gradient [N,H,W,coutp]
+  int cinp, coutp, cin, cout;
+  float* gW;       // canonical OIHW [cout][cin][3][3]
+  float* gb;       // [cout]
+};
+bool wgrad_multi_supported(const WgradJob* jobs, int J, int W);
+int wgrad_multi_grid(int J, int N, int H, int W);
+size_t wgrad_multi_ws_floats(const WgradJob* jobs, int J, int grid);
+cudaError_t launch_wgrad_multi(const WgradJob* jobs, int J, int N, int H, int W, float scale, float* ws,
+                               unsigned* sync, int grid, long long* dbg, cudaStream_t st);
+
 int num_sms();
 
 }  // namespace sr

@@ -370,11 +370,13 @@ extern "C" int sr_bench_wgrad(const void* x, const void* dy, int n, int h, int w
   int dev = 0, sms = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const int grid = g.units < sms ? g.units : sms;
+  const bool roll = (exp & 8) != 0;  // exp bit 3: the rolling batched kernel with one job (W >= 128)
+  const int grid = roll ? wgrad_multi_grid(1, n, h, w) : (g.units < sms ? g.units : sms);
+  const WgradJob job{(const bf16*)x, (const bf16*)dy, cinp, coutp, cinp, coutp, nullptr, nullptr};
   float *ws = nullptr, *gout = nullptr;
   unsigned* sync = nullptr;
   long long* dbg = nullptr;
-  if (cudaMalloc(&ws, (size_t)grid * (9 * cinp * coutp + coutp) * 4) ||
+  if (cudaMalloc(&ws, (size_t)(grid + 1) * (9 * cinp * coutp + coutp) * 4) ||
       cudaMalloc(&gout, ((size_t)9 * cinp * coutp + coutp) * 4) || cudaMalloc(&dbg, (size_t)grid * 8 * 8) ||
       cudaMalloc(&sync, 8))
     return SR_E_NOMEM;
@@ -382,9 +384,16 @@ extern "C" int sr_bench_wgrad(const void* x, const void* dy, int n, int h, int w
   WgradOut o{ws, sync, gout, gout + (size_t)9 * cinp * coutp, cinp, coutp, 1.f};
   cudaEvent_t a, b;
   cudaEventCreate(&a); cudaEventCreate(&b);
-  launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, g, o, smem, grid, st);
+  auto run = [&](const WgradGeom& gg) {
+    WgradJob jb = job;
+    jb.gW = o.gW;
+    jb.gb = o.gb;
+    return roll ? launch_wgrad_multi(&jb, 1, n, h, w, 1.f, o.ws, o.sync, grid, gg.dbg, st)
+                : launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, gg, o, smem, grid, st);
+  };
+  if (run(g) != cudaSuccess) return SR_E_CUDA;
   cudaEventRecord(a, st);
-  for (int i = 0; i < iters; ++i) launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, g, o, smem, grid, st);
+  for (int i = 0; i < iters; ++i) run(g);
   cudaEventRecord(b, st);
   cudaEventSynchronize(b);
   cudaEventElapsedTime(ms_out, a, b);
@@ -392,7 +401,7 @@ extern "C" int sr_bench_wgrad(const void* x, const void* dy, int n, int h, int w
   if (dbg_host) {
     WgradGeom gd = g;
     gd.dbg = dbg;
-    launch_wgrad(cinp, coutp, (const bf16*)x, (const bf16*)dy, gd, o, smem, grid, st);
+    run(gd);
     cudaMemcpyAsync(dbg_host, dbg, (size_t)grid * 8 * 8, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
   }

@@ -25,9 +25,14 @@ for ci, co in ((48, 48), (16, 48), (48, 32)):
     print(f"wgrad {ci}x{co}: rc={rc} {ms.value * 1e3:.1f} us ({fl / ms.value / 1e9:.0f} TF/s) incl. the fused reduction")
     t0 = dbg[:, 0].min()
     d = (dbg - t0) / 1e3
-    names = ["entry", "pdl", "first_full", "mma_issued", "(waited)", "done_bar", "drained", "barrier"]
-    clk = (dbg[:, 4] - dbg[:, 1]) / (dbg[:, 6] - dbg[:, 0])
-    print(f"  SM clock during the launch: med {np.median(clk):.3f} GHz (min {clk.min():.3f}, max {clk.max():.3f})")
+    if EXP & 8:  # batched rolling kernel: slot 1 = reduction done, 2 = first MMA, 3 = MMAs issued
+        names = ["entry", "reduced", "first_mma", "mma_issued", "(clock)", "first_done", "drained", "barrier"]
+        skip = (4,)
+    else:
+        names = ["entry", "pdl", "first_full", "mma_issued", "(waited)", "done_bar", "drained", "barrier"]
+        skip = (1, 4)
+        clk = (dbg[:, 4] - dbg[:, 1]) / (dbg[:, 6] - dbg[:, 0])
+        print(f"  SM clock during the launch: med {np.median(clk):.3f} GHz (min {clk.min():.3f}, max {clk.max():.3f})")
     for k, nm in enumerate(names):
-        if k not in (1, 4):
+        if k not in skip:
             print(f"  {nm:11s} min {d[:, k].min():7.2f} med {np.median(d[:, k]):7.2f} max {d[:, k].max():7.2f} us")

@@ -147,7 +147,11 @@ def test_conv_dgrad_with_mask(lib, case):
 # ------------------------------------------------------------------ wgrad
 @pytest.mark.parametrize("case", [(2, 7, 20, 16, 48), (1, 9, 150, 48, 48), (4, 48, 48, 48, 48),
                                   (3, 11, 48, 32, 16), (2, 12, 48, 48, 32), (2, 13, 17, 8, 8),
-                                  (48, 48, 48, 48, 48), (2, 90, 300, 16, 48)])
+                                  (48, 48, 48, 48, 48), (2, 90, 300, 16, 48),
+                                  # rolling k_wgrad_roll (W >= 128): training virtual-batch shapes (head, body, up
+                                  # conv), ragged strips, 64 channels, a single row
+                                  (1, 48, 3200, 48, 48), (1, 48, 3200, 16, 48), (1, 48, 3200, 48, 27),
+                                  (3, 5, 260, 64, 64), (2, 7, 129, 32, 16), (1, 1, 128, 8, 8), (2, 3, 400, 48, 64)])
 def test_wgrad_matches_oracle(lib, case):
     n, h, w, cin, cout = case
     r = np.random.default_rng(4)
@@ -163,6 +167,45 @@ def test_wgrad_matches_oracle(lib, case):
     rW, rb = O.conv3x3_wgrad(x, dy)
     assert rel_l2(dw, rW) < 1e-5
     assert rel_l2(db, rb) < 1e-5
+
+
+@pytest.mark.parametrize("case", [
+    # n, h, w, [(cin, cout), ...]
+    (1, 48, 3200, [(16, 48)] + [(48, 48)] * 17 + [(48, 27)]),  # one training iteration of the 8x48 x3 net
+    (2, 5, 300, [(48, 48), (16, 48), (48, 32), (48, 48), (48, 16), (16, 16), (48, 48)]),  # CTAs span job ends
+    (1, 3, 256, [(32, 32), (16, 32), (32, 16)] * 6 + [(32, 32), (16, 16)]),  # 20 jobs, one row per CTA
+])
+def test_wgrad_batch_matches_oracle(lib, case):
+    """The batched wgrad launch (all convs of a training iteration at once, partials per (CTA, job) slot,
+    reduction over the CTAs touching each job) = the oracle per conv."""
+    n, h, w, shapes = case
+    r = np.random.default_rng(7)
+    xs, dys, xds, dyds = [], [], [], []
+    for cin, cout in shapes:
+        xs.append(bf16_round(r.standard_normal((n, h, w, cin))))
+        dys.append(bf16_round(r.standard_normal((n, h, w, cout))))
+        xds.append(to_dev_bf16(xs[-1], rup16(cin)))
+        dyds.append(to_dev_bf16(dys[-1], rup16(cout)))
+    J = len(shapes)
+    sizes = [co * ci * 9 + co for ci, co in shapes]
+    out = np.zeros(sum(sizes), np.float32)
+    P = C.c_void_p * J
+    cins = (C.c_int * J)(*[ci for ci, _ in shapes])
+    couts = (C.c_int * J)(*[co for _, co in shapes])
+    st = lib.sr_test_wgrad_batch(J, P(*[t.data_ptr() for t in xds]), P(*[t.data_ptr() for t in dyds]), n, h, w,
+                                 cins, couts, out.ctypes.data_as(C.c_void_p), _s())
+    assert st == 0
+    off = 0
+    for k, (cin, cout) in enumerate(shapes):
+        rW, rb = O.conv3x3_wgrad(xs[k], dys[k])
+        dw = out[off:off + cout * cin * 9].reshape(cout, cin, 3, 3)
+        db = out[off + cout * cin * 9:off + sizes[k]]
+        off += sizes[k]
+        # bf16 operands are exact in both; what differs is fp32 accumulation: each CTA's TMEM accumulator sums
+        # up to ~138 rows x 128 px = 17.7k products per output in the tensor core's fp32 adds (measured 2.2e-5
+        # at the training shape), vs 1e-5 for the per-conv kernels' shorter chains
+        assert rel_l2(dw, rW) < 1e-4, (k, rel_l2(dw, rW))
+        assert rel_l2(db, rb) < 1e-5, (k, rel_l2(db, rb))
 
 
 # ------------------------------------------------------------------ small kernels
