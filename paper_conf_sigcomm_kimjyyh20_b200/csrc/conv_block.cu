@@ -52,8 +52,9 @@ struct BlkCfg {
   static constexpr uint32_t ROWB = ((CCH * PLANE) + 1023u) & ~1023u;             // f / t ring slot
   static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
   static constexpr uint32_t OUTB = ((kBlkTW * C * 2) + 1023u) & ~1023u;          // staging row
+  static constexpr uint32_t ARMB = ((kArmOnesBytes + 2 * 2 * C * 16) + 1023u) & ~1023u;  // ones + 2 bias tiles
   static constexpr size_t SMEM = 1024 + 2 * WB_AL + (size_t)kBlkNF * ROWB + (size_t)kBlkNT * ROWB +
-                                 (size_t)kBlkNO * OUTB;
+                                 (size_t)kBlkNO * OUTB + ARMB;
 };
 
 template <int C>
@@ -85,6 +86,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   uint8_t* sF = sW2 + Cfg::WB_AL;
   uint8_t* sT = sF + kBlkNF * ROWB;
   uint8_t* sO = sT + kBlkNT * ROWB;
+  uint8_t* sOnes = sO + kBlkNO * OUTB;       // bias-arming MMA operands (ring.cuh)
+  uint8_t* sB1 = sOnes + kArmOnesBytes;
+  uint8_t* sB2 = sB1 + 2 * C * 16;
   __shared__ __align__(8) uint64_t f_full[kBlkNF], f_empty[kBlkNF], t_full[kBlkNT], t_empty[kBlkNT], r1_ready[RB],
       r1_free[RB], r2_ready[RB], r2_free[RB], w_bar;
   __shared__ uint32_t tmem_base_sh;
@@ -115,6 +119,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     reinterpret_cast<float*>(sb1v)[threadIdx.x] = b1[threadIdx.x];
     reinterpret_cast<float*>(sb2v)[threadIdx.x] = b2[threadIdx.x];
   }
+  arm_tiles_fill(sOnes, sB1, b1, C, threadIdx.x, blockDim.x);
+  arm_tiles_fill(sOnes, sB2, b2, C, threadIdx.x, blockDim.x);
+  fence_proxy_async_smem();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
@@ -175,6 +182,11 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         mbar_wait(&f_full[fs], fph);
         SR_DBG(9, st)
         tc_fence_after();
+        if (st == 0) {  // the piece's first two rows receive no earlier contribution
+          ring_arm<C, RB>(ring1, g, smem_u32(sOnes), smem_u32(sB1));
+          ring_arm<C, RB>(ring1, g + 1, smem_u32(sOnes), smem_u32(sB1));
+        }
+        ring_arm<C, RB>(ring1, g + 2, smem_u32(sOnes), smem_u32(sB1));  // its first contribution comes now
         if (!(exp & 32))
           ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, 2 * PLANE);
         mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
@@ -207,6 +219,11 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         mbar_wait(&t_full[ts], tph);
         SR_DBG(12, k + 3)
         tc_fence_after();
+        if (k == 0) {
+          ring_arm<C, RB>(ring2, g, smem_u32(sOnes), smem_u32(sB2));
+          ring_arm<C, RB>(ring2, g + 1, smem_u32(sOnes), smem_u32(sB2));
+        }
+        ring_arm<C, RB>(ring2, g + 2, smem_u32(sOnes), smem_u32(sB2));
         if (!(exp & 16))
           ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, 2 * PLANE);
         mma_commit(&r2_ready[ring_idx<RB>(g)]);
@@ -227,15 +244,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     const int quarter = warp & 3;
     const int m = quarter * 32 + lane_id();
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
-    {  // arm every ring block with b1
-      float v[C];
-      for (int b = 0; b < RB; ++b) {
-        ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
-        tc_fence_before();
-        __syncwarp();
-        if (lane_id() == 0) mbar_arrive(&r1_free[b]);
-      }
-    }
+    for (int b = 0; b < RB; ++b)  // every ring block starts free (the MMA issuer arms blocks itself)
+      if (lane_id() == 0) mbar_arrive(&r1_free[b]);
     int ts = 0;
     uint32_t tph = 0;
     long long G = 0;
@@ -264,7 +274,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           for (int c0 = 0; c0 < C; ++c0) v[c0] = (float)c0;
         }
       } else {
-        ring_drain<C>(ring1 + lane_off + b * C, v, sb1v);
+#pragma unroll
+        for (int c0 = 0; c0 < C; c0 += 8) tmem_ld8(ring1 + lane_off + b * C + c0, v + c0);
+        tmem_ld_wait();
       }
       tc_fence_before();
       __syncwarp();
@@ -303,15 +315,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     const int m = quarter * 32 + lane_id();
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
     const bool leader = (warp == 6 && lane_id() == 0);
-    {
-      float v[C];
-      for (int b = 0; b < RB; ++b) {
-        ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
-        tc_fence_before();
-        __syncwarp();
-        if (lane_id() == 0) mbar_arrive(&r2_free[b]);
-      }
-    }
+    for (int b = 0; b < RB; ++b)
+      if (lane_id() == 0) mbar_arrive(&r2_free[b]);
     int os = 0;
     long long G = 0;
     SR_PIECE_BEGIN
@@ -346,7 +351,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           for (int c0 = 0; c0 < C; ++c0) v[c0] = (float)c0;
         }
       } else {
-        ring_drain<C>(ring2 + lane_off + b * C, v, sb2v);
+#pragma unroll
+        for (int c0 = 0; c0 < C; c0 += 8) tmem_ld8(ring2 + lane_off + b * C + c0, v + c0);
+        tmem_ld_wait();
       }
       tc_fence_before();
       __syncwarp();

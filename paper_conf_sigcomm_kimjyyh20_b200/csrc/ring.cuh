@@ -59,4 +59,37 @@ __device__ __forceinline__ void ring_drain(uint32_t taddr, float* v, const float
   tmem_st_wait();
 }
 
+// ---- arming a ring block with the bias inside the tensor pipe (instead of tcgen05.st from the epilogue): one
+// non-accumulating MMA, M = 128, N = COUTP, K = 16, A = "ones" tile (A[m][k] = 1 for k < 3), B[n][k] = the bias split
+// into three bf16 terms (hi, mid, lo: hi + mid + lo = the fp32 bias to ~2^-24 relative), so D[m][n] = bias[n].
+// Both tiles are K-major SWIZZLE_NONE: element (row, k) at (row%8)*16 + (row/8)*128 + (k/8)*LBO + (k%8)*2 with
+// LBO = rows*16.  The MMA issuer arms the block of an output row right before that row's first contribution, so
+// the epilogue only drains (tcgen05.ld) and frees the block.
+static constexpr uint32_t kArmOnesBytes = 128 * 16 * 2;  // A tile: 128 rows x 16 K
+
+__device__ __forceinline__ void arm_tiles_fill(uint8_t* ones, uint8_t* btile, const float* bias, int coutp,
+                                               int tid, int nthreads) {
+  for (int i = tid; i < 128 * 16; i += nthreads) {
+    const int r = i / 16, k = i % 16;
+    *reinterpret_cast<__nv_bfloat16*>(ones + (r % 8) * 16 + (r / 8) * 128 + (k / 8) * 2048 + (k % 8) * 2) =
+        __float2bfloat16(k < 3 ? 1.f : 0.f);
+  }
+  for (int i = tid; i < coutp * 16; i += nthreads) {
+    const int n = i / 16, k = i % 16;
+    const float b = bias[n];
+    const __nv_bfloat16 hi = __float2bfloat16(b);
+    const __nv_bfloat16 mid = __float2bfloat16(b - __bfloat162float(hi));
+    const __nv_bfloat16 lo = __float2bfloat16(b - __bfloat162float(hi) - __bfloat162float(mid));
+    const __nv_bfloat16 v = k == 0 ? hi : k == 1 ? mid : k == 2 ? lo : __float2bfloat16(0.f);
+    *reinterpret_cast<__nv_bfloat16*>(btile + (n % 8) * 16 + (n / 8) * 128 + (k / 8) * (coutp * 16) + (k % 8) * 2) = v;
+  }
+}
+
+template <int COUTP, int RB>
+__device__ __forceinline__ void ring_arm(uint32_t ring_base, long long g, uint32_t ones_saddr, uint32_t btile_saddr) {
+  constexpr uint32_t id = make_idesc(128, COUTP, 0, 0);
+  mma_bf16_ss(ring_base + ring_idx<RB>(g) * COUTP, make_desc(ones_saddr, 2048, 128),
+              make_desc(btile_saddr, COUTP * 16, 128), id, 0u);
+}
+
 }  // namespace sr
