@@ -49,7 +49,7 @@ struct BlkCfg {
   static constexpr int RB = (256 / C) < 8 ? (256 / C) : 8;  // TMEM ring blocks per conv (256 columns each)
   static constexpr uint32_t WBYTES = 9u * C * C * 2u;
   static constexpr uint32_t PLANE = 130 * 16;
-  static constexpr uint32_t ROWB = ((CCH * PLANE) + 1023u) & ~1023u;             // f / t ring slot
+  static constexpr uint32_t ROWB = ((CCH * PLANE) + 127u) & ~127u;  // f / t ring slot (TMA: 128-B aligned)
   static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
   static constexpr uint32_t OUTB = ((kBlkTW * C * 2) + 1023u) & ~1023u;          // staging row
   static constexpr uint32_t ARMB = ((kArmOnesBytes + 2 * 2 * C * 16) + 1023u) & ~1023u;  // ones + 2 bias tiles
@@ -322,16 +322,24 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     SR_PIECE_BEGIN
     const bool lane_ok = m < kBlkTW && x0 + m < W;
     const bool sep0 = sep > 0 && (((x0 + m) % sep) == 0 || ((x0 + m) % sep) == sep - 1);
+    // the residual row is loaded one row ahead (res_nx), so its L2 latency overlaps a whole row-step
+    uint4 res_nx[C / 8];
+    auto ld_res = [&](int q) {
+      if (q >= 1 && q <= n_t - 2 && lane_ok && !(exp & 1)) {
+        const uint4* rp = reinterpret_cast<const uint4*>(fres + ((((size_t)n * H + y0 - 1 + q) * W) + x0 + m) * C);
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) res_nx[j] = __ldg(rp + j);
+      }
+    };
+    ld_res(-1);
     for (int q = -1; q <= n_t; ++q) {         // out rows of conv2 = output rows y0-1+q
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
       const int r = y0 - 1 + q;
       uint4 res[C / 8];
-      if (emit && lane_ok && !(exp & 1)) {
-        const uint4* rp = reinterpret_cast<const uint4*>(fres + ((((size_t)n * H + r) * W) + x0 + m) * C);
 #pragma unroll
-        for (int j = 0; j < C / 8; ++j) res[j] = __ldg(rp + j);
-      }
+      for (int j = 0; j < C / 8; ++j) res[j] = res_nx[j];
+      ld_res(q + 1);
       const int b = ring_idx<RB>(g);
       mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
       tc_fence_after();
