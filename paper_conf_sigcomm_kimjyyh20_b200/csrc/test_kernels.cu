@@ -134,6 +134,81 @@ k_test_mma(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict_
   if (warp_id() == 0) tmem_dealloc<256>(tmem);
 }
 
+// A operand from TMEM: lane m of A column c holds (A[m][2c], A[m][2c+1]) as bf16x2 (pack = 0: even k in the low
+// half; 1: high half), written with tcgen05.st; B K-major SWIZZLE_NONE in smem.  D[128 x N] = A * B^T.
+// reps > 0: also time `reps` x (K/16) MMAs (cycles[0]).
+__global__ void __launch_bounds__(128, 1)
+k_test_mma_ts(const __nv_bfloat16* __restrict__ A, const __nv_bfloat16* __restrict__ B, float* __restrict__ D, int N,
+              int K, int pack, int reps, long long* cycles) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tmem_base;
+  uint8_t* sB = smem;
+  for (int i = threadIdx.x; i < N * K; i += blockDim.x) {
+    const int n = i / K, k = i % K;
+    *reinterpret_cast<__nv_bfloat16*>(sB + (k / 8) * (N * 16) + n * 16 + (k % 8) * 2) = B[i];
+  }
+  fence_proxy_async_smem();
+  if (warp_id() == 0) tmem_alloc<512>(&tmem_base);
+  if (threadIdx.x == 0) { mbar_init(&bar, 1); fence_barrier_init(); }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base, ta = tmem + 384;
+  const int row = warp_id() * 32 + lane_id();
+  const uint32_t lane_off = (warp_id() * 32u) << 16;
+  for (int c0 = 0; c0 < K / 2; c0 += 8) {
+    float v[8];
+    for (int c = 0; c < 8; ++c) {
+      __nv_bfloat16 lo = A[row * K + 2 * (c0 + c)], hi = A[row * K + 2 * (c0 + c) + 1];
+      if (pack == 2) { lo = __float2bfloat16((float)(row + 1)); hi = __float2bfloat16(-(float)(row + 1)); }
+      if (pack == 3) { lo = __float2bfloat16((float)(c0 + c + 1)); hi = __float2bfloat16(-(float)(c0 + c + 1)); }
+      __nv_bfloat162 h = pack == 1 ? __halves2bfloat162(hi, lo) : __halves2bfloat162(lo, hi);
+      v[c] = __uint_as_float(*reinterpret_cast<uint32_t*>(&h));
+    }
+    tmem_st8(ta + lane_off + c0, v);
+  }
+  tmem_st_wait();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (threadIdx.x == 0) {
+    const uint32_t idesc = make_idesc(128, N, 0, 0);
+    const uint64_t bdesc = make_desc(smem_u32(sB), N * 16, 128);
+    const long long t0 = clock64();
+    const int total = reps > 0 ? reps : 1;
+    if (reps > 0 && K == 64) {  // throughput: descriptors precomputed, 4 MMAs per iteration, two D chains
+      uint64_t bd[4];
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) bd[ks] = desc_add(bdesc, ks * 2 * N * 16);
+      mma_bf16_ts(tmem, ta, bd[0], idesc, 0u);
+      mma_bf16_ts(tmem + 176, ta, bd[0], idesc, 0u);
+      for (int r = 0; r < reps; ++r) {
+#pragma unroll
+        for (int ks = 0; ks < 4; ++ks) mma_bf16_ts(tmem + ((ks & 1) ? 176u : 0u), ta + ks * 8, bd[ks], idesc, 1u);
+      }
+    } else
+    for (int r = 0; r < total; ++r)  // reps > 0: odd reps accumulate into a second D (independent chains)
+      for (int ks = 0; ks < K / 16; ++ks)
+        mma_bf16_ts(tmem + ((reps > 0 && (r & 1)) ? 176u : 0u), ta + ks * 8, desc_add(bdesc, ks * 2 * N * 16), idesc,
+                    (r > 1 || ks) != 0);
+    mma_commit(&bar);
+    mbar_wait(&bar, 0);
+    if (cycles) cycles[0] = clock64() - t0;
+  }
+  __syncthreads();
+  tc_fence_after();
+  for (int c0 = 0; c0 < N; c0 += 16) {
+    float v[16];
+    tmem_ld16(tmem + lane_off + c0, v);
+    tmem_ld_wait();
+    for (int j = 0; j < 16; ++j) D[row * N + c0 + j] = v[j];
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp_id() == 0) tmem_dealloc<512>(tmem);
+}
+
 // Dump what a 5-D TMA box lands in shared memory (to check the chunk-planar layouts and OOB zero fill).
 __global__ void k_test_tma(const __grid_constant__ CUtensorMap tm, uint8_t* out, uint32_t bytes, int c1, int c2,
                            int c3, int c4) {
@@ -357,6 +432,16 @@ extern "C" int sr_bench_roll_dbg(int cinp, int coutp, int n, int h, int w, int r
   cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
   cudaFree(x); cudaFree(y); cudaFree(r); cudaFree(wt); cudaFree(bias); cudaFree(dbg);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
+
+extern "C" int sr_test_mma_ts(const void* A, const void* B, float* D, int N, int K, int pack, int reps,
+                              long long* cycles_dev, void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t smem = (size_t)N * K * 2;
+  cudaFuncSetAttribute(k_test_mma_ts, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_test_mma_ts<<<1, 128, smem, st>>>((const __nv_bfloat16*)A, (const __nv_bfloat16*)B, D, N, K, pack, reps,
+                                      cycles_dev);
+  return cudaStreamSynchronize(st) == cudaSuccess ? 0 : -3;
 }
 
 // Timing of one wgrad launch configuration (split-K + fused reduction) on device-resident data; dbg_host
