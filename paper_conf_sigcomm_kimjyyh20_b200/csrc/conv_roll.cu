@@ -40,10 +40,11 @@ struct RollCfg {
   static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
   static constexpr uint32_t PLANE = (kRollTW + 2) * 16;
   static constexpr uint32_t IN_BOX = (CINP / 8) * PLANE;
-  static constexpr uint32_t IN_STRIDE = (IN_BOX + 1023u) & ~1023u;
+  static constexpr uint32_t IN_STRIDE = (IN_BOX + 127u) & ~127u;  // TMA destination: 128-B aligned
   static constexpr uint32_t ROWB = ((kRollTW * COUTP * 2) + 1023u) & ~1023u;
   static constexpr int NAUX = 4;  // residual / mask rows (TMA)
-  static constexpr size_t BASE = 1024 + WB_AL + (size_t)2 * kRollNO * ROWB + (size_t)NAUX * ROWB;
+  static constexpr uint32_t ARMB = ((kArmOnesBytes + COUTP * 32) + 127u) & ~127u;  // bias-arming MMA operands
+  static constexpr size_t BASE = 1024 + WB_AL + (size_t)2 * kRollNO * ROWB + (size_t)NAUX * ROWB + ARMB;
   static constexpr int NIN = (BASE + 4 * IN_STRIDE <= 227 * 1024) ? 4 : 3;  // input-row ring slots
   static constexpr size_t SMEM = BASE + (size_t)NIN * IN_STRIDE;
 };
@@ -87,6 +88,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   uint8_t* sIn = sW + Cfg::WB_AL;
   uint8_t* sO = sIn + kRollIn * IN_STRIDE;
   uint8_t* sA = sO + 2 * kRollNO * ROWB;
+  uint8_t* sOnes = sA + NAUX * ROWB;  // ring.cuh: ones x bias MMA arms a ring block
+  uint8_t* sBt = sOnes + kArmOnesBytes;
   __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
       x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar;
   // the aux row (res1 or mask) travels by TMA; res2 (used once per backward pass) by plain loads
@@ -111,6 +114,9 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   pdl_enter();  // predecessor complete: global inputs are valid from here on
   if (threadIdx.x == 0) { SR_RDBG(10, 0) }  // after setup + PDL wait
   if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
+  __syncthreads();
+  arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, threadIdx.x, blockDim.x);
+  fence_proxy_async_smem();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
@@ -170,6 +176,11 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         mbar_wait(&in_full[s], ph);
         SR_RDBG(3, i)
         tc_fence_after();
+        if (i == 0) {  // the piece's first two rows receive no earlier contribution
+          ring_arm<COUTP, RB>(tmem, g, smem_u32(sOnes), smem_u32(sBt));
+          ring_arm<COUTP, RB>(tmem, g + 1, smem_u32(sOnes), smem_u32(sBt));
+        }
+        ring_arm<COUTP, RB>(tmem, g + 2, smem_u32(sOnes), smem_u32(sBt));  // its first contribution comes now
         ring_mma_step<CINP, COUTP, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, 2 * PLANE);
         mma_commit(&r_ready[ring_idx<RB>(g)]);
         mma_commit(&in_empty[s]);
@@ -218,13 +229,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
     uint8_t* stage = sO + grp * kRollNO * ROWB;
     uint32_t ophase = 0;
-    for (int b = grp; b < RB; b += 2) {  // arm this group's ring blocks with the bias (RB is even)
-      float v[COUTP];
-      ring_drain<COUTP>(tmem + lane_off + b * COUTP, v, sbv);
-      tc_fence_before();
-      __syncwarp();
+    for (int b = grp; b < RB; b += 2)  // this group's ring blocks start free (RB is even; the MMA issuer arms)
       if (lane_id() == 0) mbar_arrive(&r_free[b]);
-    }
     int os = 0;
     long long G = 0, emitted = 0;  // emitted: output rows of both groups so far (aux ring order)
     SR_PIECE_BEGIN
@@ -246,7 +252,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       tc_fence_after();
       if (warp == 2 && lane_id() == 0) { SR_RDBG(5, q + 1) }
       float v[COUTP];
-      ring_drain<COUTP>(tmem + lane_off + b * COUTP, v, sbv);
+      ring_load<COUTP>(tmem + lane_off + b * COUTP, v);
       tc_fence_before();
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&r_free[b]);

@@ -59,6 +59,17 @@ __device__ __forceinline__ void ring_drain(uint32_t taddr, float* v, const float
   tmem_st_wait();
 }
 
+// Load COLS accumulator columns of a ring block (this thread's lane) without re-arming (blocks armed by ring_arm).
+template <int COLS>
+__device__ __forceinline__ void ring_load(uint32_t taddr, float* v) {
+  static_assert(COLS % 8 == 0, "ring_load: columns must be a multiple of 8");
+  constexpr int C16 = COLS / 16 * 16;
+#pragma unroll
+  for (int c0 = 0; c0 < C16; c0 += 16) tmem_ld16(taddr + c0, v + c0);
+  if (COLS % 16) tmem_ld8(taddr + C16, v + C16);
+  tmem_ld_wait();
+}
+
 // ---- arming a ring block with the bias inside the tensor pipe (instead of tcgen05.st from the epilogue): one
 // non-accumulating MMA, M = 128, N = COUTP, K = 16, A = "ones" tile (A[m][k] = 1 for k < 3), B[n][k] = the bias split
 // into three bf16 terms (hi, mid, lo: hi + mid + lo = the fp32 bias to ~2^-24 relative), so D[m][n] = bias[n].
