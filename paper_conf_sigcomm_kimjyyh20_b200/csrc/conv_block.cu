@@ -57,17 +57,19 @@ struct BlkCfg {
                                  (size_t)kBlkNO * OUTB + ARMB;
 };
 
-template <int C>
+template <int C, bool BWD>
 __global__ void __launch_bounds__(kBlkThreads, 1)
 k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
            const float* __restrict__ b2, const bf16* __restrict__ fres, bf16* __restrict__ outp, const int N,
            const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg,
-           const int exp) {
+           const int exp, const bf16* __restrict__ mask, const bf16* __restrict__ res2) {
   // exp (benchmarking experiments only, results wrong when set): 1 no residual load, 2 no output store, 4 no t
   // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads, 128 no f-row TMA
   // after the first piece
   // tsave (nullable): also write t = ReLU(conv1(f) + b1) to global (training saves it for the backward pass).
+  // mask (nullable): the data-gradient block of the backward pass -- t = conv1(f) * 1[mask > 0] (ReLU' through the
+  // saved forward t) instead of ReLU; res2 (nullable): conv2's output also adds res2 (the global-skip gradient).
   // sep > 0: columns with col % sep in {0, sep-1} are separators of the virtual training batch -> t and out = 0.
   // dbg (benchmarking only, CTA 0): clock64 stamps [event][step], events: 0 f issued, 1 conv1 step issued,
   // 2 conv2 step issued, 3 epi1 got a block, 4 epi1 t row done, 5 epi2 got a block, 6 epi2 row stored
@@ -253,11 +255,28 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     const int tcol = x0 - 1 + m;
     const bool col_ok = tcol >= 0 && tcol < W && !(sep > 0 && ((tcol % sep) == 0 || (tcol % sep) == sep - 1));
     const bool save_col = tsave != nullptr && m >= 1 && m <= kBlkTW && tcol < W;  // this strip's own columns
+    // backward mode: the ReLU' mask row (saved forward t) is loaded one row ahead, like the residual below
+    uint4 mk_nx[BWD ? C / 8 : 1];
+    auto ld_mask = [&](int q) {
+      const int trow = y0 - 2 + q;
+      if (BWD && q >= 1 && q <= n_f - 2 && col_ok && trow >= 0 && trow < H) {
+        const uint4* mp = reinterpret_cast<const uint4*>(mask + ((((size_t)n * H + trow) * W) + tcol) * C);
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) mk_nx[j] = __ldg(mp + j);
+      }
+    };
+    ld_mask(-1);
     for (int q = -1; q <= n_f; ++q) {         // out rows of conv1 = t rows y0-2+q
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_f - 2;
       const int trow = y0 - 2 + q;
       const bool ok = col_ok && trow >= 0 && trow < H;
+      uint4 mk[BWD ? C / 8 : 1];
+      if constexpr (BWD) {
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) mk[j] = mk_nx[j];
+        ld_mask(q + 1);
+      }
       if (emit) mbar_wait(&t_empty[ts], tph ^ 1);
       const int b = ring_idx<RB>(g);
       mbar_wait(&r1_ready[b], (uint32_t)(g / RB) & 1u);
@@ -287,8 +306,18 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 #pragma unroll
         for (int j = 0; j < CCH; ++j) {
           float a[8];
+          if constexpr (BWD) {  // ReLU' = 1[t > 0] of the forward t
+            const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&mk[j]);
 #pragma unroll
-          for (int e = 0; e < 8; ++e) a[e] = ok ? fmaxf(v[8 * j + e], 0.f) : 0.f;
+            for (int e = 0; e < 4; ++e) {
+              const float2 f2 = __bfloat1622float2(h2[e]);
+              a[2 * e] = ok && f2.x > 0.f ? v[8 * j + 2 * e] : 0.f;
+              a[2 * e + 1] = ok && f2.y > 0.f ? v[8 * j + 2 * e + 1] : 0.f;
+            }
+          } else {
+#pragma unroll
+            for (int e = 0; e < 8; ++e) a[e] = ok ? fmaxf(v[8 * j + e], 0.f) : 0.f;
+          }
           uint4 u;
           u.x = pack_bf16x2(a[0], a[1]);
           u.y = pack_bf16x2(a[2], a[3]);
@@ -324,11 +353,18 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     const bool sep0 = sep > 0 && (((x0 + m) % sep) == 0 || ((x0 + m) % sep) == sep - 1);
     // the residual row is loaded one row ahead (res_nx), so its L2 latency overlaps a whole row-step
     uint4 res_nx[C / 8];
+    uint4 r2_nx[BWD ? C / 8 : 1];
     auto ld_res = [&](int q) {
       if (q >= 1 && q <= n_t - 2 && lane_ok && !(exp & 1)) {
-        const uint4* rp = reinterpret_cast<const uint4*>(fres + ((((size_t)n * H + y0 - 1 + q) * W) + x0 + m) * C);
+        const size_t pix = (((size_t)n * H + y0 - 1 + q) * W) + x0 + m;
+        const uint4* rp = reinterpret_cast<const uint4*>(fres + pix * C);
 #pragma unroll
         for (int j = 0; j < C / 8; ++j) res_nx[j] = __ldg(rp + j);
+        if (BWD && res2) {
+          const uint4* rp2 = reinterpret_cast<const uint4*>(res2 + pix * C);
+#pragma unroll
+          for (int j = 0; j < C / 8; ++j) r2_nx[j] = __ldg(rp2 + j);
+        }
       }
     };
     ld_res(-1);
@@ -336,9 +372,13 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
       const int r = y0 - 1 + q;
-      uint4 res[C / 8];
+      uint4 res[C / 8], rs2[BWD ? C / 8 : 1];
 #pragma unroll
       for (int j = 0; j < C / 8; ++j) res[j] = res_nx[j];
+      if (BWD && res2) {
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) rs2[j] = r2_nx[j];
+      }
       ld_res(q + 1);
       const int b = ring_idx<RB>(g);
       mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
@@ -377,8 +417,21 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
               const float2 f2 = __bfloat1622float2(h2[e]);
-              a[2 * e] = sep0 ? 0.f : v[8 * j + 2 * e] + f2.x;
-              a[2 * e + 1] = sep0 ? 0.f : v[8 * j + 2 * e + 1] + f2.y;
+              a[2 * e] = v[8 * j + 2 * e] + f2.x;
+              a[2 * e + 1] = v[8 * j + 2 * e + 1] + f2.y;
+            }
+            if (BWD && res2) {
+              const __nv_bfloat162* g2 = reinterpret_cast<const __nv_bfloat162*>(&rs2[j]);
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const float2 f2 = __bfloat1622float2(g2[e]);
+                a[2 * e] += f2.x;
+                a[2 * e + 1] += f2.y;
+              }
+            }
+            if (sep0) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) a[e] = 0.f;
             }
             uint4 u;
             u.x = pack_bf16x2(a[0], a[1]);
@@ -414,16 +467,17 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
 template <int C>
 static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, const bf16* w1, const bf16* w2,
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
-                                  int grid, bf16* tsave, int sep, long long* dbg, int exp, cudaStream_t st) {
-  auto kern = k_resblock<C>;
-  static bool configured = false;
-  if (!configured) {
+                                  int grid, bf16* tsave, int sep, long long* dbg, int exp, const bf16* mask,
+                                  const bf16* res2, cudaStream_t st) {
+  auto kern = mask ? k_resblock<C, true> : k_resblock<C, false>;
+  static bool configured[2] = {false, false};
+  if (!configured[mask != nullptr]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BlkCfg<C>::SMEM);
     if (e != cudaSuccess) return e;
-    configured = true;
+    configured[mask != nullptr] = true;
   }
   return launch_k(kern, dim3(grid), dim3(kBlkThreads), BlkCfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, out, N, H, W,
-                  tsave, sep, dbg, exp);
+                  tsave, sep, dbg, exp, mask, res2);
 }
 
 bool resblock_supported(int cp, int W) {
@@ -436,16 +490,19 @@ bool resblock_supported(int cp, int W) {
 
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st, long long* dbg,
-                            bf16* tsave, int sep, int exp) {
+                            bf16* tsave, int sep, int exp, const bf16* mask, const bf16* res2) {
   CUtensorMap tf, to;
   if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (make_row_tmap(&to, out, N, H, W, cp, kBlkTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   const long long rows = (long long)N * ((W + kBlkTW - 1) / kBlkTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
-  if (cp == 16) return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
-  if (cp == 32) return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
-  if (cp == 48) return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, st);
+  if (cp == 16)
+    return launch_block_t<16>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, mask, res2, st);
+  if (cp == 32)
+    return launch_block_t<32>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, mask, res2, st);
+  if (cp == 48)
+    return launch_block_t<48>(tf, to, w1fold, w2fold, b1, b2, f, out, N, H, W, grid, tsave, sep, dbg, exp, mask, res2, st);
   return cudaErrorNotSupported;
 }
 

@@ -44,7 +44,8 @@ cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, co
 bool resblock_supported(int cp, int W);
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,
-                            long long* dbg = nullptr, bf16* tsave = nullptr, int sep = 0, int exp = 0);
+                            long long* dbg = nullptr, bf16* tsave = nullptr, int sep = 0, int exp = 0,
+                            const bf16* mask = nullptr, const bf16* res2 = nullptr);
 // Device-side step counters (so a training iteration can be captured once in a CUDA graph and replayed):
 // counters[0] = sampler step, counters[1] = Adam step t; scal[0] = lr / (1 - b1^t), scal[1] = 1/sqrt(1 - b2^t).
 void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st);

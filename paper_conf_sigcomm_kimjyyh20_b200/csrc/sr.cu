@@ -51,6 +51,7 @@ struct sr_ctx {
   double* loss_sum = nullptr;
   long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t
   float* adam_scal = nullptr;     // device: lr/bc1, 1/sqrt(bc2)
+  float* zero_bias = nullptr;     // device: 64 zeros (the bias of the data-gradient convs)
   // patch pool (device ring)
   uint8_t *pool_lr = nullptr, *pool_hr = nullptr;
   long long pool_total = 0, pool_cap = 0;
@@ -76,6 +77,7 @@ struct sr_ctx {
   bool timing = false;
   bool fuse_blocks = true;  // fused residual-block kernel for wide frames (sr_set_option)
   bool roll_tail = true;    // rolling up conv with the tail epilogue for wide frames (sr_set_fusion bit 2 clears)
+  bool fuse_bwd = false;    // fused data-gradient residual blocks (sr_set_fusion bit 3; slower at the training shape)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -504,6 +506,21 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
   TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdg, WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr,
               0, sep, ctx->tdf[B], 1, Hv, Wv, st));
   for (int b = B - 1; b >= 0; --b) {
+    if (ctx->fuse_blocks && ctx->fuse_bwd && resblock_supported(Cp, Wv)) {
+      // the block's data gradient in one fused kernel (k_resblock in mask mode): dt = dgrad_conv2(df) * 1[t > 0]
+      // stays in shared memory (and is saved for the wgrad), df' = df + dgrad_conv1(dt) (+ dg into f0 at b = 0)
+      if (ctx->timing) {
+        const double px = (double)Hv * Wv;
+        tmark_begin(ctx, "train_dgrad_block_" + std::to_string(Cp), 2 * 2.0 * 9 * Cp * Cp * px, px * 2.0 * 4 * Cp, st);
+      }
+      cudaError_t e = launch_resblock(Cp, ctx->tdf[b + 1], WDO(2 + 2 * b), WDO(1 + 2 * b), ctx->zero_bias,
+                                      ctx->zero_bias, ctx->tdf[b], 1, Hv, Wv, st, nullptr, ctx->tdtb[b], sep, 0,
+                                      ctx->tts[b], b == 0 ? ctx->tdg : nullptr);
+      tmark_end(ctx, st);
+      ctx->launches++;
+      if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("dgrad block launch: ") + cudaGetErrorString(e));
+      continue;
+    }
     TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdf[b + 1], WDO(2 + 2 * b), nullptr, nullptr, nullptr, ctx->tts[b],
                 0, sep, ctx->tdtb[b], 1, Hv, Wv, st));
     TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdtb[b], WDO(1 + 2 * b), nullptr, ctx->tdf[b + 1],
@@ -705,6 +722,8 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->loss_sum, 1);
   al(&ctx->counters, 2);
   al(&ctx->adam_scal, 2);
+  al(&ctx->zero_bias, 64);
+  if (st == SR_OK && cudaMemset(ctx->zero_bias, 0, 64 * sizeof(float)) != cudaSuccess) st = SR_E_CUDA;
   ctx->tf.assign(blocks + 1, nullptr);
   ctx->tts.assign(blocks, nullptr);
   ctx->tdf.assign(blocks + 1, nullptr);
@@ -741,7 +760,7 @@ void sr_destroy(sr_ctx* ctx) {
   void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->x16, ctx->f0,
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
-                  ctx->adam_scal, ctx->pool_lr,
+                  ctx->adam_scal, ctx->zero_bias, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf, ctx->cell_sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -764,6 +783,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->fuse_blocks = (fuse_blocks & 1) != 0;
   ctx->virtual_train = (fuse_blocks & 2) == 0;  // bit 1 set: per-patch (narrow tile) training path
   ctx->roll_tail = (fuse_blocks & 4) == 0;      // bit 2 set: tiled up conv + tail instead of the rolling one
+  ctx->fuse_bwd = (fuse_blocks & 8) != 0;       // bit 3 set: fused data-gradient blocks in training
   return SR_OK;
 }
 

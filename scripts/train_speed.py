@@ -10,6 +10,8 @@ from synth import synth_patch_pool  # noqa: E402
 
 s, B, C = 3, 8, 48
 ctx = SRContext(s, B, C, seed=0)
+if len(sys.argv) > 1:
+    ctx.set_fusion(int(sys.argv[1]))  # e.g. 9: fused data-gradient blocks
 plr, phr, _ = synth_patch_pool(256, s, 180, seed=1, frame_hw=(540, 900))
 ctx.pool_push(torch.from_numpy(plr).cuda(), torch.from_numpy(phr).cuda())
 st = torch.cuda.Stream()

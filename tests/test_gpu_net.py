@@ -286,7 +286,7 @@ def test_virtual_batch_training_matches_oracle_and_narrow_path(cfg, n, p):
     lrp, hrp, _ = synth_patch_pool(n, s, s * p, seed=41, frame_hw=(s * p * 3, s * p * 4))
     lr, hr = torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda()
     grads = []
-    for mode in (1, 0, 3):  # bit 0: fused blocks, bit 1: per-patch path
+    for mode in (1, 0, 3, 9):  # bit 0: fused blocks, bit 1: per-patch path, bit 3: fused data-gradient blocks
         ctx = _ctx(s, B, C, seed=22)
         ctx.set_params(init_params(s, B, C, seed=22) * 1.5)  # bf16 storage: rel L2 ~4e-3 at x1, ~8.5e-3 at x2
         ctx.set_fusion(mode)
