@@ -33,6 +33,11 @@ static constexpr int kRollThreads = 352;  // + warp 10: TMA-store warp
 static constexpr int kRollNO = 3;    // output staging rows per epilogue group
 static constexpr int kRollTW = 128;  // output pixels per strip (= MMA M)
 
+static constexpr int kTailLrChunks = 26;  // 416 B: LR pixels x0-5 .. x0+133 of a 128-pixel strip
+static constexpr uint32_t kTailLrSlot = (16 * kTailLrChunks * 5 + 127) & ~127u;  // 5 LR rows per slot
+// LR-row ring depth of the staged tail (in the aux area, unused by the tail): deep enough that the producer, which
+// runs up to NIN + RB rows ahead of the epilogue, never waits on it (a shallow ring stalls the input rows)
+
 template <int CINP, int COUTP>
 struct RollCfg {
   static constexpr int RB = (512 / COUTP) < 8 ? (512 / COUTP) : 8;
@@ -43,9 +48,13 @@ struct RollCfg {
   static constexpr uint32_t IN_STRIDE = (IN_BOX + 127u) & ~127u;  // TMA destination: 128-B aligned
   static constexpr uint32_t ROWB = ((kRollTW * COUTP * 2) + 1023u) & ~1023u;
   static constexpr int NAUX = 4;  // residual / mask rows (TMA)
+  static constexpr int NLR = (int)((NAUX * ROWB) / kTailLrSlot) < 16 ? (int)((NAUX * ROWB) / kTailLrSlot) : 16;
   static constexpr uint32_t ARMB = ((kArmOnesBytes + COUTP * 32) + 127u) & ~127u;  // bias-arming MMA operands
   static constexpr size_t BASE = 1024 + WB_AL + (size_t)2 * kRollNO * ROWB + (size_t)NAUX * ROWB + ARMB;
-  static constexpr int NIN = (BASE + 4 * IN_STRIDE <= 227 * 1024) ? 4 : 3;  // input-row ring slots
+  // input-row ring slots: as many as fit (up to 8) -- the TMA loads in flight per SM are what keeps HBM busy
+  static constexpr int NIN_FIT = (int)((227 * 1024 - BASE) / IN_STRIDE);
+  static constexpr int NIN = NIN_FIT > 8 ? 8 : NIN_FIT;
+  static constexpr bool FITS = NIN >= 3;  // else not offered (roll_supported)
   static constexpr size_t SMEM = BASE + (size_t)NIN * IN_STRIDE;
 };
 
@@ -63,6 +72,10 @@ struct RollArgs {
   uint8_t* hr;        // [N,TS H,TS W,3]
   int hr_row0, hr_row1;  // LR rows whose HR rows are written (strip mode)
   int bicubic;
+  // tail_tma: LR neighbourhood rows arrive by TMA (tm_aux, make_u8_rows_tmap, box kTailLrChunks x 5 rows) and the
+  // S HR rows of every LR row are staged in smem and leave by one TMA store (tm_out); needs W % 16 == 0.
+  // Otherwise every lane reads its 3x3 (5x5) LR neighbourhood and writes its S x S x 3 bytes from/to global.
+  int tail_tma;
 };
 #define SR_RDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -91,7 +104,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   uint8_t* sOnes = sA + NAUX * ROWB;  // ring.cuh: ones x bias MMA arms a ring block
   uint8_t* sBt = sOnes + kArmOnesBytes;
   __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
-      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar;
+      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar, l_full[TS > 0 ? Cfg::NLR : 1],
+      l_empty[TS > 0 ? Cfg::NLR : 1];
   // the aux row (res1 or mask) travels by TMA; res2 (used once per backward pass) by plain loads
   const bool has_aux = a.res1 != nullptr || a.mask != nullptr;
   __shared__ uint32_t tmem_base_sh;
@@ -104,6 +118,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     for (int s = 0; s < kRollIn; ++s) { mbar_init(&in_full[s], 1); mbar_init(&in_empty[s], 1); }
     for (int s = 0; s < RB; ++s) { mbar_init(&r_ready[s], 1); mbar_init(&r_free[s], 4); }
     for (int s = 0; s < NAUX; ++s) { mbar_init(&x_full[s], 1); mbar_init(&x_empty[s], 4); }
+    if (TS > 0)
+      for (int s = 0; s < Cfg::NLR; ++s) { mbar_init(&l_full[s], 1); mbar_init(&l_empty[s], 4); }
     for (int s = 0; s < 2 * kRollNO; ++s) { mbar_init(&o_full[s], 4); mbar_init(&o_free[s], 1); }
     mbar_init(&w_bar, 1);
     fence_barrier_init();
@@ -140,8 +156,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       tma_prefetch_desc(&tm_in);
       mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
       bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
-      int s = 0, xs = 0;
-      uint32_t ph = 0, xph = 0;
+      int s = 0, xs = 0, ls = 0;
+      uint32_t ph = 0, xph = 0, lph = 0;
       SR_PIECE_BEGIN
       for (int i = 0; i < n_in; ++i) {
         mbar_wait(&in_empty[s], ph ^ 1);
@@ -149,6 +165,12 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         tma_load_5d(sIn + s * IN_STRIDE, &tm_in, &in_full[s], 0, x0 - 1, y0 - 1 + i, 0, n);
         SR_RDBG(0, i)
         if (++s == kRollIn) { s = 0; ph ^= 1; }
+        if (TS > 0 && a.tail_tma && i >= 1 && i - 1 < y1 - y0) {  // LR rows r-2..r+2 of output row r = y0+i-1
+          mbar_wait(&l_empty[ls], lph ^ 1);
+          mbar_arrive_expect_tx(&l_full[ls], 16 * kTailLrChunks * 5);
+          tma_load_4d(sA + ls * kTailLrSlot, &tm_aux, &l_full[ls], 0, 3 * x0 / 16 - 1, y0 + i - 3, n);
+          if (++ls == Cfg::NLR) { ls = 0; lph ^= 1; }
+        }
         if (has_aux && i >= 1 && i - 1 < y1 - y0) {  // aux row of output row y0+i-1 (needed after input row y0+i)
           mbar_wait(&x_empty[xs], xph ^ 1);
           mbar_arrive_expect_tx(&x_full[xs], kRollTW * COUTP * 2);
@@ -197,7 +219,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     __syncwarp();
   } else if (warp == 10) {
     // ===================== store warp: TMA-store finished rows in emission order =====================
-    if (TS == 0 && elect_one()) {
+    if ((TS == 0 || a.tail_tma) && elect_one()) {
       tma_prefetch_desc(&tm_out);
       int os[2] = {0, 0};
       uint32_t oph[2] = {0, 0};
@@ -209,11 +231,22 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         const int grp = (int)(g & 1);
         const int b = grp * kRollNO + os[grp];
         mbar_wait(&o_full[b], oph[grp]);
-        tma_store_4d(&tm_out, sO + b * ROWB, 0, x0, y0 - 1 + q, n);
-        bulk_commit();
-        bulk_wait_read<1>();        // the previous store has read its staging row
-        if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
-        pend_b = b;
+        const int r = y0 - 1 + q;
+        if (TS == 0 || (r >= a.hr_row0 && r < a.hr_row1)) {
+          if (TS > 0)  // the S HR rows of LR row r
+            tma_store_4d(&tm_out, sO + b * ROWB, 0, x0 * TS * 3 / 16, TS * r, n);
+          else
+            tma_store_4d(&tm_out, sO + b * ROWB, 0, x0, r, n);
+          bulk_commit();
+          bulk_wait_read<1>();        // the previous store has read its staging row
+          if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
+          pend_b = b;
+        } else {  // strip mode: row outside [hr_row0, hr_row1), nothing to store
+          bulk_wait_read<0>();
+          if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
+          pend_b = -1;
+          mbar_arrive(&o_free[b]);
+        }
         if (++os[grp] == kRollNO) { os[grp] = 0; oph[grp] ^= 1; }
       }
       G += n_in + 2;
@@ -259,14 +292,31 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       if (warp == 2 && lane_id() == 0) { SR_RDBG(6, q + 1) }
       if (!emit) continue;
       if constexpr (TS > 0) {  // up conv: the tail straight from registers (the ring held the bias)
+        if (a.tail_tma) {  // LR rows from the TMA ring, HR rows staged for the store warp
+          constexpr int NLR = TS > 0 ? Cfg::NLR : 1;
+          mbar_wait(&l_full[xi % NLR], (uint32_t)(xi / NLR) & 1u);
+          mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);
+          if (lane_ok)
+            tail_u8_smem<TS>(smem_u32(sA) + (uint32_t)(xi % NLR) * kTailLrSlot, 16 * kTailLrChunks, 3 * x0 - 16,
+                             smem_u32(stage + os * ROWB), kRollTW * TS * 3, 3 * TS * m, r, xc, H, W, v, a.bicubic);
+          __syncwarp();
+          if (lane_id() == 0) mbar_arrive(&l_empty[xi % NLR]);
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane_id() == 0) mbar_arrive(&o_full[grp * kRollNO + os]);
+          if (++os == kRollNO) { os = 0; ophase ^= 1; }
+          continue;
+        }
         if (lane_ok && r >= a.hr_row0 && r < a.hr_row1) {
           EpiParams ep{};
           ep.scale = TS;
           ep.lr = a.lr;
           ep.hr = a.hr;
           ep.bicubic = a.bicubic;
-          float ls = 0.f;
-          epi_tail<TS, COUTP, false>(ep, nullptr, n, r, xc, H, W, v, ls, 0);
+          float ls = 0.f, vv[COUTP];  // a copy: epi_tail may pass it to a non-inlined call (keeps v in registers)
+#pragma unroll
+          for (int k = 0; k < COUTP; ++k) vv[k] = v[k];
+          epi_tail<TS, COUTP, false>(ep, nullptr, n, r, xc, H, W, vv, ls, 0);
         }
         continue;
       }
@@ -341,22 +391,32 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
 template <int CINP, int COUTP, int TS = 0>
 static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, const CUtensorMap& tx,
                                  const bf16* wfold, const RollArgs& a, int grid, cudaStream_t st) {
-  auto kern = k_conv_roll<CINP, COUTP, TS>;
-  constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
-  static bool configured = false;
-  if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    configured = true;
+  if constexpr (!RollCfg<CINP, COUTP>::FITS) {
+    return cudaErrorNotSupported;
+  } else {
+    auto kern = k_conv_roll<CINP, COUTP, TS>;
+    constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
+    static bool configured = false;
+    if (!configured) {
+      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e != cudaSuccess) return e;
+      configured = true;
+    }
+    return launch_k(kern, dim3(grid), dim3(kRollThreads), smem, st, ti, to, tx, wfold, a);
   }
-  return launch_k(kern, dim3(grid), dim3(kRollThreads), smem, st, ti, to, tx, wfold, a);
-  return cudaGetLastError();
 }
 
 static bool ch_ok(int c) { return c == 16 || c == 32 || c == 48 || c == 64; }
 
+template <int CI>
+static bool roll_fits(int coutp) {
+  return coutp == 16 ? RollCfg<CI, 16>::FITS : coutp == 32 ? RollCfg<CI, 32>::FITS : RollCfg<CI, 48>::FITS;
+}
+
 bool roll_supported(int cinp, int coutp, int W) {
-  return W >= 96 && ch_ok(cinp) && (coutp == 16 || coutp == 32 || coutp == 48);
+  if (W < 96 || !ch_ok(cinp) || !(coutp == 16 || coutp == 32 || coutp == 48)) return false;
+  return cinp == 16 ? roll_fits<16>(coutp) : cinp == 32 ? roll_fits<32>(coutp)
+       : cinp == 48 ? roll_fits<48>(coutp) : roll_fits<64>(coutp);
 }
 
 #define SR_ROLL_CASE(CI, CO) \
@@ -373,7 +433,7 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
   const void* auxp = res1 ? (const void*)res1 : (mask ? (const void*)mask : (const void*)out);
   if (make_row_tmap(&tx, auxp, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (res1 && mask) return cudaErrorNotSupported;  // one TMA aux stream per launch
-  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0};
+  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0, 0};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
@@ -385,15 +445,21 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
 }
 
 #define SR_ROLL_TAIL_CASE(CI, CO, S) \
-  if (cinp == CI && coutp == CO && s == S) return launch_roll_t<CI, CO, S>(ti, ti, ti, wfold, a, grid, st);
+  if (cinp == CI && coutp == CO && s == S) return launch_roll_t<CI, CO, S>(ti, th, tl, wfold, a, grid, st);
 
 cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
                                   const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
-                                  int W, cudaStream_t st) {
+                                  int W, cudaStream_t st, int tail_tma_ok) {
   CUtensorMap ti;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
-  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, lr, hr, hr_row0, hr_row1, bicubic};
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, lr, hr, hr_row0, hr_row1, bicubic, 0};
+  // TMA-staged tail when both u8 images are 16-B row-aligned (W % 16 == 0) and 16-B based
+  CUtensorMap tl = ti, th = ti;
+  if (tail_tma_ok && W % 16 == 0 &&
+      make_u8_rows_tmap(&tl, lr, N, H, 3LL * W, kTailLrChunks, 5) == CUDA_SUCCESS &&
+      make_u8_rows_tmap(&th, hr, N, s * H, 3LL * s * W, kRollTW * s * 3 / 16, s) == CUDA_SUCCESS)
+    a.tail_tma = 1;
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;

@@ -78,6 +78,7 @@ struct sr_ctx {
   bool fuse_blocks = true;  // fused residual-block kernel for wide frames (sr_set_option)
   bool roll_tail = true;    // rolling up conv with the tail epilogue for wide frames (sr_set_fusion bit 2 clears)
   bool fuse_bwd = false;    // fused data-gradient residual blocks (sr_set_fusion bit 3; slower at the training shape)
+  bool tail_tma = true;     // TMA-staged LR/HR rows in the rolling tail (sr_set_fusion bit 4 clears)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -350,7 +351,7 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
                   2.0 * 9 * Cp * ctx->OUTP * px, px * (2.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
     }
     cudaError_t e = launch_conv_roll_tail(Cp, ctx->OUTP, ctx->s, gbuf, sn.wo + ctx->convs[cu].pk_off, Bv(cu), lr, hr,
-                                          row0, row1, ctx->opt.skip == 1, n, h, w, st);
+                                          row0, row1, ctx->opt.skip == 1, n, h, w, st, ctx->tail_tma);
     tmark_end(ctx, st);
     ctx->launches++;
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll tail launch: ") + cudaGetErrorString(e));
@@ -784,6 +785,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->virtual_train = (fuse_blocks & 2) == 0;  // bit 1 set: per-patch (narrow tile) training path
   ctx->roll_tail = (fuse_blocks & 4) == 0;      // bit 2 set: tiled up conv + tail instead of the rolling one
   ctx->fuse_bwd = (fuse_blocks & 8) != 0;       // bit 3 set: fused data-gradient blocks in training
+  ctx->tail_tma = (fuse_blocks & 16) == 0;      // bit 4 set: rolling tail reads/writes u8 pixels per lane
   return SR_OK;
 }
 

@@ -43,6 +43,25 @@ __device__ __forceinline__ void phase_w(int ph, float& wm, float& w0, float& wp)
   }
 }
 
+// One separable bilinear pass at output phase ph: weights of (v[i-1], v[i], v[i+1]); zero taps are skipped at
+// compile time (each phase has at most two), which is exact: the dropped terms are +0 on non-negative values.
+template <int S>
+__device__ __forceinline__ float bil3(int ph, float a, float b, float c) {
+  float wm, w0, wp;
+  phase_w<S>(ph, wm, w0, wp);
+  float acc = w0 * b;
+  if (wm != 0.f) acc = fmaf(wm, a, acc);
+  if (wp != 0.f) acc = fmaf(wp, c, acc);
+  return acc;
+}
+
+// clamp(x, 0, 255) rounded half-to-even to u8 in one instruction (NaN -> 0)
+__device__ __forceinline__ uint8_t f2u8_rn_sat(float x) {
+  uint32_t r;
+  asm("cvt.rni.sat.u8.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return (uint8_t)r;
+}
+
 // Bicubic skip variant (reading R23: Keys, A = -0.75, half-pixel centres without clamping the source coordinate,
 // clamped taps = PyTorch bicubic align_corners=False).  Phase ph of S: source offset d = (ph + 1/2)/S - 1/2;
 // d < 0 -> taps rows -2..+1 with t = 1 + d, else rows -1..+2 with t = d.  w[0..4] are the weights of rows -2..+2.
@@ -125,8 +144,7 @@ __device__ __noinline__ void epi_tail_bicubic(const EpiParams& ep, const float* 
             dyv[k] = 2.f * d;
           }
         } else {
-          const float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
-          orow[j * 3 + c] = (uint8_t)__float2int_rn(o);
+          orow[j * 3 + c] = f2u8_rn_sat(fmaf(255.f, y, skip));
         }
       }
     }
@@ -159,28 +177,28 @@ __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias
       for (int c = 0; c < 3; ++c) nb[a][b][c] = (float)__ldg(p + c);
     }
   }
+  float hx[3][S][3];  // horizontal pass per LR row and output column phase
+#pragma unroll
+  for (int a = 0; a < 3; ++a)
+#pragma unroll
+    for (int j = 0; j < S; ++j)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) hx[a][j][c] = bil3<S>(j, nb[a][0][c], nb[a][1][c], nb[a][2][c]);
   const int sH = S * H, sW = S * W;
   float dyv[COUTP];
 #pragma unroll
   for (int k = 0; k < COUTP; ++k) dyv[k] = 0.f;
 #pragma unroll
   for (int i = 0; i < S; ++i) {
-    float ym, y0, yp;
-    phase_w<S>(i, ym, y0, yp);
     uint8_t* hrow = TRAIN ? nullptr : ep.hr + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3;
     const uint8_t* trow =
         TRAIN ? ep.hr_ref + (((size_t)n * sH + (size_t)S * Y + i) * sW + (size_t)S * X) * 3 : nullptr;
 #pragma unroll
     for (int j = 0; j < S; ++j) {
-      float xm, x0, xp;
-      phase_w<S>(j, xm, x0, xp);
 #pragma unroll
       for (int c = 0; c < 3; ++c) {
-        // horizontal pass on the three LR rows, then vertical
-        float h0 = xm * nb[0][0][c] + x0 * nb[0][1][c] + xp * nb[0][2][c];
-        float h1 = xm * nb[1][0][c] + x0 * nb[1][1][c] + xp * nb[1][2][c];
-        float h2 = xm * nb[2][0][c] + x0 * nb[2][1][c] + xp * nb[2][2][c];
-        float skip = ym * h0 + y0 * h1 + yp * h2;
+        // horizontal pass on the three LR rows (hx), then vertical
+        const float skip = bil3<S>(i, hx[0][j][c], hx[1][j][c], hx[2][j][c]);
         const int k = c * S * S + i * S + j;
         float y = v[k] + (sbias ? sbias[k] : 0.f);
         if (TRAIN) {
@@ -194,13 +212,102 @@ __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias
             dyv[k] = 2.f * d;
           }
         } else {
-          float o = fminf(fmaxf(fmaf(255.f, y, skip), 0.f), 255.f);
-          hrow[j * 3 + c] = (uint8_t)__float2int_rn(o);
+          hrow[j * 3 + c] = f2u8_rn_sat(fmaf(255.f, y, skip));
         }
       }
     }
   }
   if (TRAIN) store_bf16_row<COUTP>(ep.dy + dy_pix * COUTP, dyv);
+}
+
+__device__ __forceinline__ float lds_u8f(uint32_t a) {
+  uint32_t r;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(r) : "r"(a));
+  return (float)r;
+}
+__device__ __forceinline__ void sts_u8(uint32_t a, uint8_t v) {
+  asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "h"((unsigned short)v) : "memory");
+}
+
+// Inference tail with both u8 images in shared memory (the rolling kernel's TMA-staged path):
+//   L: LR rows Y-2 .. Y+2 of the strip (rows outside the image are zero-filled; the clamp below never reads
+//      them), lpitch bytes per row, LR pixel p of a row at byte 3 p - lbase;
+//   O: the S HR rows of LR row Y, opitch bytes each, HR pixel (S Y + i, S X + j) at byte i opitch + ox + 3 j.
+// Arithmetic and its order are those of epi_tail / epi_tail_bicubic (no bias term: the ring held it), so the
+// u8 result is bit-identical to the global-memory path.
+template <int S>
+__device__ __forceinline__ void tail_u8_smem(uint32_t L, int lpitch, int lbase, uint32_t O, int opitch,
+                                             int ox, int Y, int X, int H, int W, const float* v, int bicubic) {
+  // L, O: shared-memory (state space) addresses
+  if (bicubic) {
+    float hrow[5][S][3];
+#pragma unroll
+    for (int a = 0; a < 5; ++a) {
+      const uint32_t lrow = L + (min(max(Y + a - 2, 0), H - 1) - Y + 2) * lpitch - lbase;
+      float px[5][3];
+#pragma unroll
+      for (int b = 0; b < 5; ++b) {
+        const uint32_t p = lrow + 3 * min(max(X + b - 2, 0), W - 1);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) px[b][c] = lds_u8f(p + c);
+      }
+#pragma unroll
+      for (int j = 0; j < S; ++j) {
+        float wx[5];
+        cubic_phase_w<S>(j, wx);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          float acc = 0.f;
+#pragma unroll
+          for (int b = 0; b < 5; ++b) acc = fmaf(wx[b], px[b][c], acc);
+          hrow[a][j][c] = acc;
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      float wy[5];
+      cubic_phase_w<S>(i, wy);
+#pragma unroll
+      for (int j = 0; j < S; ++j) {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          float skip = 0.f;
+#pragma unroll
+          for (int a = 0; a < 5; ++a) skip = fmaf(wy[a], hrow[a][j][c], skip);
+          sts_u8(O + i * opitch + ox + 3 * j + c, f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip)));
+        }
+      }
+    }
+    return;
+  }
+  float nb[3][3][3];
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    const uint32_t lrow = L + (min(max(Y + a - 1, 0), H - 1) - Y + 2) * lpitch - lbase;
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      const uint32_t p = lrow + 3 * min(max(X + b - 1, 0), W - 1);
+#pragma unroll
+      for (int c = 0; c < 3; ++c) nb[a][b][c] = lds_u8f(p + c);
+    }
+  }
+  float hx[3][S][3];
+#pragma unroll
+  for (int a = 0; a < 3; ++a)
+#pragma unroll
+    for (int j = 0; j < S; ++j)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) hx[a][j][c] = bil3<S>(j, nb[a][0][c], nb[a][1][c], nb[a][2][c]);
+#pragma unroll
+  for (int i = 0; i < S; ++i)
+#pragma unroll
+    for (int j = 0; j < S; ++j)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        const float skip = bil3<S>(i, hx[0][j][c], hx[1][j][c], hx[2][j][c]);
+        sts_u8(O + i * opitch + ox + 3 * j + c, f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip)));
+      }
 }
 
 }  // namespace sr

@@ -83,4 +83,23 @@ inline CUresult make_row_tmap(CUtensorMap* tm, const void* base, int N, int H, i
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
+// u8 image rows [N][H][row_bytes] (NHWC RGB frames: row_bytes = 3 W) as a 4-D tensor {16, row_bytes/16, H, N}
+// whose innermost unit is a 16-byte chunk; box {16, box_chunks, box_rows, 1} lands as smem [row][chunk][16], i.e.
+// box_rows dense rows of 16 * box_chunks bytes.  Needs row_bytes % 16 == 0 and a 16-B aligned base.  Used by the
+// up-conv tail: LR neighbourhood rows in, staged HR rows out (one TMA per LR row instead of 27 byte accesses per
+// lane).  Out-of-bounds box bytes are zero-filled (loads) / clipped (stores).
+inline CUresult make_u8_rows_tmap(CUtensorMap* tm, const void* base, int N, int H, long long row_bytes,
+                                  int box_chunks, int box_rows) {
+  auto fn = get_encode_fn();
+  if (!fn) return CUDA_ERROR_NOT_SUPPORTED;
+  if (row_bytes % 16 != 0 || (reinterpret_cast<uintptr_t>(base) & 15) != 0) return CUDA_ERROR_INVALID_VALUE;
+  cuuint64_t dims[4] = {16, (cuuint64_t)(row_bytes / 16), (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[3] = {16, (cuuint64_t)row_bytes, (cuuint64_t)row_bytes * H};
+  cuuint32_t box[4] = {16, (cuuint32_t)box_chunks, (cuuint32_t)box_rows, 1};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  return fn(tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void*>(base), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+}
+
 }  // namespace sr

@@ -6,9 +6,10 @@ lib = load()
 lib.sr_bench_roll_dbg.restype = C.c_int
 lib.sr_bench_roll_dbg.argtypes = [C.c_int] * 6 + [C.c_void_p, C.c_void_p, C.c_void_p]
 st = C.c_void_p(torch.cuda.current_stream().cuda_stream)
+CI, CO = (int(sys.argv[1]), int(sys.argv[2])) if len(sys.argv) > 2 else (48, 48)
 for res in (0, 1):
     dbg = np.zeros(16 * 256, np.int64); ms = C.c_float()
-    rc = lib.sr_bench_roll_dbg(48, 48, 8, 720, 1280, res, dbg.ctypes.data_as(C.c_void_p), C.byref(ms), st)
+    rc = lib.sr_bench_roll_dbg(CI, CO, 8, 720, 1280, res, dbg.ctypes.data_as(C.c_void_p), C.byref(ms), st)
     d = dbg.reshape(16, 256); t0 = d[0, 0]
     print(f"res={res} rc={rc} {ms.value*1e3:.1f} us")
     names = ["in_iss", "mma_st", "acq", "in_ok", "mma_iss", "ep_got", "ep_drained", "ep_stored"]

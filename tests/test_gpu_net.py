@@ -446,3 +446,35 @@ def test_rolling_tail_equals_tiled_tail(cfg, hw):
     b = ctx.infer(lr, "serve")
     torch.cuda.synchronize()
     assert (a.int() - b.int()).abs().max().item() <= 1
+
+
+@pytest.mark.parametrize("cfg,hw,skip", [((3, 8, 48), (37, 272), "bilinear"), ((2, 2, 16), (21, 400), "bilinear"),
+                                         ((4, 2, 48), (19, 144), "bilinear"), ((3, 2, 16), (23, 272), "bicubic"),
+                                         ((2, 2, 16), (17, 528), "bicubic"), ((4, 2, 16), (13, 256), "bicubic")])
+def test_staged_tail_bitexact_and_oracle(cfg, hw, skip):
+    """Rolling tail with TMA-staged LR rows / HR rows (W % 16 == 0; ragged last strip) == the per-lane global path
+    (set_fusion bit 4) bit for bit, and == the oracle within the north-star bar."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=31, skip=skip)
+    lr, hr = synth_frames(2, hw[0], hw[1], seed=32, scale=s)
+    lrd = torch.from_numpy(lr).cuda()
+    a = ctx.infer(lrd, "serve").clone()
+    ctx.set_fusion(1 | 16)
+    b = ctx.infer(lrd, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
+    ref = O.infer_u8(ctx.get_params("serve"), lr, s, B, C, skip=skip)
+    _check_frames(a.cpu().numpy(), ref, hr)
+
+
+def test_staged_tail_strips_bitexact():
+    """Strip mode on the staged tail: rows outside [row0, row1) are neither computed into nor stored."""
+    s, B, C = 3, 2, 16
+    ctx = _ctx(s, B, C, seed=41)
+    lr = torch.from_numpy(synth_frames(1, 77, 272, seed=42)).cuda()
+    full = ctx.infer(lr, "serve")
+    hr = torch.full_like(full[0], 7)
+    for r0, r1 in ((0, 13), (13, 50), (50, 51), (51, 77)):
+        ctx.infer_rows(lr[0], r0, r1, hr, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(hr, full[0])
