@@ -304,6 +304,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
           fence_proxy_async_smem();
           __syncwarp();
           if (lane_id() == 0) mbar_arrive(&o_full[grp * kRollNO + os]);
+          if (warp == 2 && lane_id() == 0) { SR_RDBG(7, q + 1) }
           if (++os == kRollNO) { os = 0; ophase ^= 1; }
           continue;
         }
@@ -449,11 +450,11 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
 
 cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
                                   const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
-                                  int W, cudaStream_t st, int tail_tma_ok) {
+                                  int W, cudaStream_t st, int tail_tma_ok, long long* dbg) {
   CUtensorMap ti;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
-  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, lr, hr, hr_row0, hr_row1, bicubic, 0};
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, dbg, lr, hr, hr_row0, hr_row1, bicubic, 0};
   // TMA-staged tail when both u8 images are 16-B row-aligned (W % 16 == 0) and 16-B based
   CUtensorMap tl = ti, th = ti;
   if (tail_tma_ok && W % 16 == 0 &&

@@ -40,7 +40,13 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
 // rolling up conv + tail (pixel shuffle + skip + clamp + RNE u8 into hr rows of LR rows [hr_row0, hr_row1))
 cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
                                   const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
-                                  int W, cudaStream_t st, int tail_tma_ok = 1);
+                                  int W, cudaStream_t st, int tail_tma_ok = 1, long long* dbg = nullptr);
+// fused body conv (+ f0) + up conv + tail (g kept in shared memory); needs W % 16 == 0 and a 16-B aligned LR frame
+bool bodytail_supported(int cp, int s, int W, const void* lr, const void* hr);
+cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const bf16* w1fold, const bf16* w2fold,
+                            const float* b1, const float* b2, const uint8_t* lr, uint8_t* hr, int hr_row0,
+                            int hr_row1, int bicubic, int N, int H, int W, cudaStream_t st,
+                            long long* dbg = nullptr);
 bool resblock_supported(int cp, int W);
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,

@@ -79,6 +79,7 @@ struct sr_ctx {
   bool roll_tail = true;    // rolling up conv with the tail epilogue for wide frames (sr_set_fusion bit 2 clears)
   bool fuse_bwd = false;    // fused data-gradient residual blocks (sr_set_fusion bit 3; slower at the training shape)
   bool tail_tma = true;     // TMA-staged LR/HR rows in the rolling tail (sr_set_fusion bit 4 clears)
+  bool fuse_bodytail = true;  // body conv + up conv + tail as one kernel, g in smem (sr_set_fusion bit 5 clears)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -338,6 +339,21 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
     cur = nxt;
   }
   const int cb = 1 + 2 * ctx->B, cu = cb + 1;
+  if (ctx->fuse_bodytail && ctx->roll_tail && ctx->OUTP == (ctx->s == 2 ? 16 : ctx->s == 3 ? 32 : 48) &&
+      bodytail_supported(Cp, ctx->s, w, lr, hr)) {  // g = f0 + body(f) stays in shared memory
+    if (ctx->timing) {
+      const double px = (double)n * h * w;
+      tmark_begin(ctx, "bodytail_" + std::to_string(Cp) + "x" + std::to_string(ctx->OUTP),
+                  2.0 * 9 * Cp * (Cp + ctx->OUTP) * px, px * (4.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
+    }
+    cudaError_t e = launch_bodytail(Cp, ctx->s, cur, ctx->f0, sn.wo + ctx->convs[cb].pk_off,
+                                    sn.wo + ctx->convs[cu].pk_off, Bv(cb), Bv(cu), lr, hr, row0, row1,
+                                    ctx->opt.skip == 1, n, h, w, st);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("bodytail launch: ") + cudaGetErrorString(e));
+    return SR_OK;
+  }
   bf16* gbuf = (cur == ctx->fa) ? ctx->fb : ctx->fa;
   EpiParams eb{};
   eb.bias = Bv(cb);
@@ -786,6 +802,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->roll_tail = (fuse_blocks & 4) == 0;      // bit 2 set: tiled up conv + tail instead of the rolling one
   ctx->fuse_bwd = (fuse_blocks & 8) != 0;       // bit 3 set: fused data-gradient blocks in training
   ctx->tail_tma = (fuse_blocks & 16) == 0;      // bit 4 set: rolling tail reads/writes u8 pixels per lane
+  ctx->fuse_bodytail = (fuse_blocks & 32) == 0; // bit 5 set: body conv and up conv + tail as two kernels
   return SR_OK;
 }
 

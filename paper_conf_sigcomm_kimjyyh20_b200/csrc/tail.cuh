@@ -229,16 +229,15 @@ __device__ __forceinline__ void sts_u8(uint32_t a, uint8_t v) {
   asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "h"((unsigned short)v) : "memory");
 }
 
-// Inference tail with both u8 images in shared memory (the rolling kernel's TMA-staged path):
+// Inference tail from an LR neighbourhood in shared memory, result in registers:
 //   L: LR rows Y-2 .. Y+2 of the strip (rows outside the image are zero-filled; the clamp below never reads
-//      them), lpitch bytes per row, LR pixel p of a row at byte 3 p - lbase;
-//   O: the S HR rows of LR row Y, opitch bytes each, HR pixel (S Y + i, S X + j) at byte i opitch + ox + 3 j.
+//      them), lpitch bytes per row, LR pixel p of a row at byte 3 p - lbase (shared-memory state-space address);
+//   o[(i S + j) 3 + c] = u8 of HR pixel (S Y + i, S X + j), colour c.
 // Arithmetic and its order are those of epi_tail / epi_tail_bicubic (no bias term: the ring held it), so the
 // u8 result is bit-identical to the global-memory path.
 template <int S>
-__device__ __forceinline__ void tail_u8_smem(uint32_t L, int lpitch, int lbase, uint32_t O, int opitch,
-                                             int ox, int Y, int X, int H, int W, const float* v, int bicubic) {
-  // L, O: shared-memory (state space) addresses
+__device__ __forceinline__ void tail_u8_px(uint32_t L, int lpitch, int lbase, int Y, int X, int H, int W,
+                                           const float* v, int bicubic, uint8_t* o) {
   if (bicubic) {
     float hrow[5][S][3];
 #pragma unroll
@@ -275,7 +274,7 @@ __device__ __forceinline__ void tail_u8_smem(uint32_t L, int lpitch, int lbase, 
           float skip = 0.f;
 #pragma unroll
           for (int a = 0; a < 5; ++a) skip = fmaf(wy[a], hrow[a][j][c], skip);
-          sts_u8(O + i * opitch + ox + 3 * j + c, f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip)));
+          o[(i * S + j) * 3 + c] = f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip));
         }
       }
     }
@@ -306,8 +305,20 @@ __device__ __forceinline__ void tail_u8_smem(uint32_t L, int lpitch, int lbase, 
 #pragma unroll
       for (int c = 0; c < 3; ++c) {
         const float skip = bil3<S>(i, hx[0][j][c], hx[1][j][c], hx[2][j][c]);
-        sts_u8(O + i * opitch + ox + 3 * j + c, f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip)));
+        o[(i * S + j) * 3 + c] = f2u8_rn_sat(fmaf(255.f, v[c * S * S + i * S + j] + 0.f, skip));
       }
+}
+
+// The same with the S HR rows written to shared memory: HR pixel (S Y + i, S X + j) at O + i opitch + ox + 3 j.
+template <int S>
+__device__ __forceinline__ void tail_u8_smem(uint32_t L, int lpitch, int lbase, uint32_t O, int opitch,
+                                             int ox, int Y, int X, int H, int W, const float* v, int bicubic) {
+  uint8_t o[S * S * 3];
+  tail_u8_px<S>(L, lpitch, lbase, Y, X, H, W, v, bicubic, o);
+#pragma unroll
+  for (int i = 0; i < S; ++i)
+#pragma unroll
+    for (int k = 0; k < 3 * S; ++k) sts_u8(O + i * opitch + ox + k, o[i * 3 * S + k]);
 }
 
 }  // namespace sr

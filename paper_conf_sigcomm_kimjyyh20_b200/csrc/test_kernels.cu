@@ -423,6 +423,7 @@ extern "C" int sr_bench_roll_dbg(int cinp, int coutp, int n, int h, int w, int r
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
+  launch_conv_roll_ex(cinp, coutp, x, wt, bias, res ? r : nullptr, nullptr, nullptr, !res, 0, y, n, h, w, st);  // warm
   cudaEventRecord(a, st);
   cudaError_t e = launch_conv_roll_ex(cinp, coutp, x, wt, bias, res ? r : nullptr, nullptr, nullptr, !res, 0, y, n, h,
                                       w, st, dbg);
@@ -493,4 +494,72 @@ extern "C" int sr_bench_wgrad(const void* x, const void* dy, int n, int h, int w
   cudaEventDestroy(a); cudaEventDestroy(b);
   cudaFree(ws); cudaFree(gout); cudaFree(dbg); cudaFree(sync);
   return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
+}
+
+// Timeline of one rolling up-conv + tail launch (x s, Cin = cinp -> 3 s^2 (padded) outputs) on device-resident
+// synthetic data (benchmarking only): CTA-0 clock64 stamps as sr_bench_roll_dbg.
+extern "C" int sr_bench_roll_tail_dbg(int cinp, int s, int n, int h, int w, long long* dbg_host, float* ms_out,
+                                      void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const int coutp = s == 2 ? 16 : (s == 3 ? 32 : 48);
+  const size_t pix = (size_t)n * h * w;
+  bf16 *x = nullptr, *wt = nullptr;
+  uint8_t *lr = nullptr, *hr = nullptr;
+  float* bias = nullptr;
+  long long* dbg = nullptr;
+  if (cudaMalloc(&x, pix * cinp * 2) || cudaMalloc(&lr, pix * 3) || cudaMalloc(&hr, pix * 3 * s * s) ||
+      cudaMalloc(&wt, 9 * cinp * coutp * 2) || cudaMalloc(&bias, coutp * 4) || cudaMalloc(&dbg, 16 * 256 * 8))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(x, 0x3c, pix * cinp * 2, st);
+  cudaMemsetAsync(lr, 0x50, pix * 3, st);
+  cudaMemsetAsync(wt, 0x1c, 9 * cinp * coutp * 2, st);
+  cudaMemsetAsync(bias, 0, coutp * 4, st);
+  cudaMemsetAsync(dbg, 0, 16 * 256 * 8, st);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  launch_conv_roll_tail(cinp, coutp, s, x, wt, bias, lr, hr, 0, h, 0, n, h, w, st);  // warm
+  cudaEventRecord(a, st);
+  cudaError_t e = launch_conv_roll_tail(cinp, coutp, s, x, wt, bias, lr, hr, 0, h, 0, n, h, w, st, 1, dbg);
+  cudaEventRecord(b, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  cudaEventElapsedTime(ms_out, a, b);
+  cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
+  cudaFree(x); cudaFree(lr); cudaFree(hr); cudaFree(wt); cudaFree(bias); cudaFree(dbg);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
+}
+
+// Timeline of one fused body + up conv + tail launch (Cin = cp, x s) on synthetic device data (benchmarking only).
+extern "C" int sr_bench_bodytail_dbg(int cp, int s, int n, int h, int w, long long* dbg_host, float* ms_out,
+                                     void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  const int co2 = s == 2 ? 16 : (s == 3 ? 32 : 48);
+  const size_t pix = (size_t)n * h * w;
+  bf16 *x = nullptr, *f0 = nullptr, *w1 = nullptr, *w2 = nullptr;
+  uint8_t *lr = nullptr, *hr = nullptr;
+  float* bias = nullptr;
+  long long* dbg = nullptr;
+  if (cudaMalloc(&x, pix * cp * 2) || cudaMalloc(&f0, pix * cp * 2) || cudaMalloc(&lr, pix * 3) ||
+      cudaMalloc(&hr, pix * 3 * s * s) || cudaMalloc(&w1, 9 * cp * cp * 2) || cudaMalloc(&w2, 9 * cp * co2 * 2) ||
+      cudaMalloc(&bias, 64 * 4) || cudaMalloc(&dbg, 16 * 256 * 8))
+    return SR_E_NOMEM;
+  cudaMemsetAsync(x, 0x3c, pix * cp * 2, st);
+  cudaMemsetAsync(f0, 0x3c, pix * cp * 2, st);
+  cudaMemsetAsync(lr, 0x50, pix * 3, st);
+  cudaMemsetAsync(w1, 0x1c, 9 * cp * cp * 2, st);
+  cudaMemsetAsync(w2, 0x1c, 9 * cp * co2 * 2, st);
+  cudaMemsetAsync(bias, 0, 64 * 4, st);
+  cudaMemsetAsync(dbg, 0, 16 * 256 * 8, st);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  launch_bodytail(cp, s, x, f0, w1, w2, bias, bias, lr, hr, 0, h, 0, n, h, w, st);  // warm
+  cudaEventRecord(a, st);
+  cudaError_t e = launch_bodytail(cp, s, x, f0, w1, w2, bias, bias, lr, hr, 0, h, 0, n, h, w, st, dbg);
+  cudaEventRecord(b, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  cudaEventElapsedTime(ms_out, a, b);
+  cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
+  cudaFree(x); cudaFree(f0); cudaFree(lr); cudaFree(hr); cudaFree(w1); cudaFree(w2); cudaFree(bias); cudaFree(dbg);
+  return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }

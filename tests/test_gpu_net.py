@@ -478,3 +478,43 @@ def test_staged_tail_strips_bitexact():
         ctx.infer_rows(lr[0], r0, r1, hr, "serve")
     torch.cuda.synchronize()
     assert torch.equal(hr, full[0])
+
+
+@pytest.mark.parametrize("cfg,hw,skip", [((3, 8, 48), (41, 272), "bilinear"), ((2, 3, 32), (29, 400), "bilinear"),
+                                         ((4, 2, 48), (19, 144), "bicubic"), ((3, 2, 16), (33, 528), "bicubic"),
+                                         ((2, 2, 16), (8, 256), "bilinear")])
+def test_fused_bodytail_equals_two_kernels(cfg, hw, skip):
+    """Body conv + up conv + tail as one kernel (g kept in shared memory; default when W % 16 == 0) == the two
+    rolling kernels (set_fusion bit 5): same per-row MMA order and the same bf16 rounding of g -> bit-identical;
+    and the oracle within the north-star bar."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=51, skip=skip)
+    lr, hr = synth_frames(2, hw[0], hw[1], seed=52, scale=s)
+    lrd = torch.from_numpy(lr).cuda()
+    a = ctx.infer(lrd, "serve").clone()
+    ctx.set_fusion(1 | 32)
+    b = ctx.infer(lrd, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
+    ref = O.infer_u8(ctx.get_params("serve"), lr, s, B, C, skip=skip)
+    _check_frames(a.cpu().numpy(), ref, hr)
+
+
+def test_fused_bodytail_strips_and_unaligned_output():
+    """Strip pieces through the fused kernel == whole frame; an HR buffer at an odd byte offset (16-B copy-out with
+    ragged head/tail bytes) gives the same bytes."""
+    s, B, C = 3, 2, 16
+    ctx = _ctx(s, B, C, seed=61)
+    lr = torch.from_numpy(synth_frames(1, 61, 400, seed=62)).cuda()
+    full = ctx.infer(lr, "serve")
+    hr = torch.full_like(full[0], 3)
+    for r0, r1 in ((0, 20), (20, 21), (21, 61)):
+        ctx.infer_rows(lr[0], r0, r1, hr, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(hr, full[0])
+    flat = torch.zeros(full[0].numel() + 7, dtype=torch.uint8, device="cuda")
+    view = flat[5:5 + full[0].numel()].view(full[0].shape)
+    ctx.infer_rows(lr[0], 0, 61, view, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(view, full[0])
+    assert int(flat[:5].sum()) == 0 and int(flat[5 + full[0].numel():].sum()) == 0
