@@ -167,7 +167,7 @@ k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const bf16* __restrict__ wp
   constexpr uint32_t IDESC = make_idesc(128, COUTP, 0, 0);
 
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // stays in the shared window (LDS/STS, not generic)
   __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], tfull_bar[NSLOT], tempty_bar[NSLOT];
   __shared__ __align__(8) uint64_t w_bar;
   __shared__ uint32_t tmem_base_sh;
@@ -411,7 +411,7 @@ k_wgrad(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtens
   constexpr uint32_t IDESC = make_idesc(128, COUTP, 1, 1);
 
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // stays in the shared window (LDS/STS, not generic)
   constexpr int PER = 9 * CINP * COUTP, STRIDE = PER + COUTP;  // floats per partial
   __shared__ __align__(8) uint64_t full_bar[kWgStages], empty_bar[kWgStages], done_bar;
   __shared__ uint32_t tmem_base_sh;

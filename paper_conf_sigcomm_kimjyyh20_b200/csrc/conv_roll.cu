@@ -87,6 +87,56 @@ __device__ __forceinline__ void ld_row(const bf16* base, uint4* dst) {
   for (int q = 0; q < CH / 8; ++q) dst[q] = __ldg(p + q);
 }
 
+// One output row of one lane into the staging row: v (bias included) + res1 (aux row) + res2 -> ReLU -> x 1[mask > 0]
+// (aux row) -> 0 in separator columns -> bf16.  M: variant bits (1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU);
+// M = 32: generic body, the variant is read from em at run time.
+template <int COUTP, int M>
+__device__ __forceinline__ void roll_stage(uint4* orow, const float* v, const uint4* aux, const uint4* r2, bool sep0,
+                                           int em) {
+  const int mm = (M & 32) ? em : M;
+#pragma unroll
+  for (int j = 0; j < COUTP / 8; ++j) {
+    float o[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) o[e] = v[8 * j + e];
+    if (mm & 1) {
+      const uint4 t = aux[j];
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
+    }
+    if (mm & 2) {
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&r2[j]);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
+    }
+    if (mm & 16) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
+    }
+    if (mm & 4) {
+      const uint4 t = aux[j];
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __bfloat1622float2(h[e]);
+        o[2 * e] = f.x > 0.f ? o[2 * e] : 0.f;
+        o[2 * e + 1] = f.y > 0.f ? o[2 * e + 1] : 0.f;
+      }
+    }
+    if ((mm & 8) && sep0) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) o[e] = 0.f;
+    }
+    uint4 u;
+    u.x = pack_bf16x2(o[0], o[1]);
+    u.y = pack_bf16x2(o[2], o[3]);
+    u.z = pack_bf16x2(o[4], o[5]);
+    u.w = pack_bf16x2(o[6], o[7]);
+    orow[j] = u;
+  }
+}
+
 template <int CINP, int COUTP, int TS>
 __global__ void __launch_bounds__(kRollThreads, 1)
 k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
@@ -96,7 +146,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   constexpr uint32_t PLANE = Cfg::PLANE, IN_STRIDE = Cfg::IN_STRIDE, ROWB = Cfg::ROWB;
 
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // stays in the shared window (LDS/STS, not generic)
   uint8_t* sW = smem;
   uint8_t* sIn = sW + Cfg::WB_AL;
   uint8_t* sO = sIn + kRollIn * IN_STRIDE;
@@ -270,6 +320,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     const int xc = x0 + m;
     const bool lane_ok = xc < W;
     const bool sep0 = a.sep > 0 && ((xc % a.sep) == 0 || (xc % a.sep) == a.sep - 1);
+    // epilogue variant bits: 1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU
+    const int emode = (a.res1 ? 1 : 0) | (a.res2 ? 2 : 0) | (a.mask ? 4 : 0) | (a.sep > 0 ? 8 : 0) | (a.relu ? 16 : 0);
     for (int q = -1; q <= n_in; ++q) {
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_in - 2;
@@ -324,55 +376,30 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       const uint4* aux = reinterpret_cast<const uint4*>(sA + (int)(xi % NAUX) * ROWB + m * COUTP * 2);
       if (has_aux) mbar_wait(&x_full[xi % NAUX], (uint32_t)(xi / NAUX) & 1u);
       mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);  // the store warp has read this staging row
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(11, q + 1) }
       if (lane_ok) {
         uint4* orow = reinterpret_cast<uint4*>(stage + os * ROWB + m * COUTP * 2);
-#pragma unroll
-        for (int j = 0; j < COUTP / 8; ++j) {
-          float o[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) o[e] = v[8 * j + e];
-          if (a.res1) {
-            const uint4 t = aux[j];
-            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
-#pragma unroll
-            for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
-          }
-          if (a.res2) {
-            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&r2[j]);
-#pragma unroll
-            for (int e = 0; e < 4; ++e) { const float2 f = __bfloat1622float2(h[e]); o[2 * e] += f.x; o[2 * e + 1] += f.y; }
-          }
-          if (a.relu) {
-#pragma unroll
-            for (int e = 0; e < 8; ++e) o[e] = fmaxf(o[e], 0.f);
-          }
-          if (a.mask) {
-            const uint4 t = aux[j];
-            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
-#pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const float2 f = __bfloat1622float2(h[e]);
-              o[2 * e] = f.x > 0.f ? o[2 * e] : 0.f;
-              o[2 * e + 1] = f.y > 0.f ? o[2 * e + 1] : 0.f;
-            }
-          }
-          if (sep0) {
-#pragma unroll
-            for (int e = 0; e < 8; ++e) o[e] = 0.f;
-          }
-          uint4 u;
-          u.x = pack_bf16x2(o[0], o[1]);
-          u.y = pack_bf16x2(o[2], o[3]);
-          u.z = pack_bf16x2(o[4], o[5]);
-          u.w = pack_bf16x2(o[6], o[7]);
-          orow[j] = u;
+        // the epilogue variant is uniform across the launch: dispatch once per row to straight-line code
+        // (a generic body predicates every variant's instructions -- ~600 per row -- and the per-row chain of
+        // the epilogue group is what bounds the launch)
+        switch (emode) {  // the variants the library launches; anything else takes the generic body
+          case 0: roll_stage<COUTP, 0>(orow, v, aux, r2, sep0, emode); break;
+          case 1: roll_stage<COUTP, 1>(orow, v, aux, r2, sep0, emode); break;
+          case 8: roll_stage<COUTP, 8>(orow, v, aux, r2, sep0, emode); break;
+          case 1 | 8: roll_stage<COUTP, 1 | 8>(orow, v, aux, r2, sep0, emode); break;
+          case 1 | 2 | 8: roll_stage<COUTP, 1 | 2 | 8>(orow, v, aux, r2, sep0, emode); break;
+          case 4 | 8: roll_stage<COUTP, 4 | 8>(orow, v, aux, r2, sep0, emode); break;
+          case 16 | 8: roll_stage<COUTP, 16 | 8>(orow, v, aux, r2, sep0, emode); break;
+          default: roll_stage<COUTP, 32>(orow, v, aux, r2, sep0, emode); break;
         }
       }
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(12, q + 1) }
       if (has_aux) {
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&x_empty[xi % NAUX]);
       }
       fence_proxy_async_smem();
+      if (warp == 2 && lane_id() == 0) { SR_RDBG(13, q + 1) }
       __syncwarp();
       if (lane_id() == 0) mbar_arrive(&o_full[grp * kRollNO + os]);
       if (warp == 2 && lane_id() == 0) { SR_RDBG(7, q + 1) }

@@ -87,7 +87,7 @@ __global__ void __launch_bounds__(kWrThreads, 1) k_wgrad_multi(const __grid_cons
   constexpr uint32_t ATOM = Cfg::ATOM, S = Cfg::S, DYS = Cfg::DYS;
 
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // stays in the shared window (LDS/STS, not generic)
   uint8_t* sX = smem;
   uint8_t* sDY = smem + Cfg::XRING;
   __shared__ __align__(8) uint64_t x_full[NX], x_empty[NX], d_full[NS], d_empty[NS], done_bar, t_empty;

@@ -233,7 +233,7 @@ __global__ void k_test_tma(const __grid_constant__ CUtensorMap tm, uint8_t* out,
 __global__ void k_bench_tma(const __grid_constant__ CUtensorMap tm, int mode, int H, int W, int passes,
                             uint32_t box_bytes) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // stays in the shared window (LDS/STS, not generic)
   __shared__ __align__(8) uint64_t bar[4];
   if (threadIdx.x != 0) return;
   for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);

@@ -15,6 +15,9 @@ for res in (0, 1):
     names = ["in_iss", "mma_st", "acq", "in_ok", "mma_iss", "ep_got", "ep_drained", "ep_stored"]
     for i in range(6, 14):
         print("  %3d " % i + " ".join(f"{nm}={(d[e, i] - t0) if d[e, i] else -1:7d}" for e, nm in enumerate(names)))
+    a_, b_ = d[11, 10:40], d[6, 10:40]; m_ = (a_ > 0) & (b_ > 0)
+    if m_.any(): print(f"  o_free wait mean {np.mean(a_[m_] - b_[m_]):7.1f}  pack+sts {np.mean(d[12,10:40][m_] - a_[m_]):7.1f}"
+                       f"  fence {np.mean(d[13,10:40][m_] - d[12,10:40][m_]):7.1f}  arrive {np.mean(d[7,10:40][m_] - d[13,10:40][m_]):7.1f}")
     for e, nm in enumerate(names):
         v = d[e, 10:40]; v = v[v > 0]
         if len(v) > 2: print(f"  {nm:10s} interval {np.mean(np.diff(v)):7.1f}")
