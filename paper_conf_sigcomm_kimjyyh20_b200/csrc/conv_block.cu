@@ -57,13 +57,19 @@ struct BlkCfg {
                                  (size_t)kBlkNO * OUTB + ARMB;
 };
 
-template <int C, bool BWD>
+// GEN = false: the inference instantiation -- no experiments, no t save, no separators, no timeline (those runtime
+// checks otherwise put predicated instructions on the epilogues' per-row chains).
+template <int C, bool BWD, bool GEN>
 __global__ void __launch_bounds__(kBlkThreads, 1)
 k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
            const float* __restrict__ b2, const bf16* __restrict__ fres, bf16* __restrict__ outp, const int N,
-           const int H, const int W, bf16* __restrict__ tsave, const int sep, long long* __restrict__ dbg,
-           const int exp, const bf16* __restrict__ mask, const bf16* __restrict__ res2) {
+           const int H, const int W, bf16* __restrict__ tsave_in, const int sep_in, long long* __restrict__ dbg_in,
+           const int exp_in, const bf16* __restrict__ mask, const bf16* __restrict__ res2) {
+  bf16* const tsave = GEN ? tsave_in : nullptr;
+  const int sep = GEN ? sep_in : 0;
+  long long* const dbg = GEN ? dbg_in : nullptr;
+  const int exp = GEN ? exp_in : 0;
   // exp (benchmarking experiments only, results wrong when set): 1 no residual load, 2 no output store, 4 no t
   // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads, 128 no f-row TMA
   // after the first piece
@@ -253,7 +259,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     long long G = 0;
     SR_PIECE_BEGIN
     const int tcol = x0 - 1 + m;
-    const bool col_ok = tcol >= 0 && tcol < W && !(sep > 0 && ((tcol % sep) == 0 || (tcol % sep) == sep - 1));
+    const bool col_ok = tcol >= 0 && tcol < W && !(sep > 0 && ((tcol % max(sep, 1)) == 0 || (tcol % max(sep, 1)) == sep - 1));
     const bool save_col = tsave != nullptr && m >= 1 && m <= kBlkTW && tcol < W;  // this strip's own columns
     // backward mode: the ReLU' mask row (saved forward t) is loaded one row ahead, like the residual below
     uint4 mk_nx[BWD ? C / 8 : 1];
@@ -350,7 +356,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     long long G = 0;
     SR_PIECE_BEGIN
     const bool lane_ok = m < kBlkTW && x0 + m < W;
-    const bool sep0 = sep > 0 && (((x0 + m) % sep) == 0 || ((x0 + m) % sep) == sep - 1);
+    const bool sep0 = sep > 0 && (((x0 + m) % max(sep, 1)) == 0 || ((x0 + m) % max(sep, 1)) == sep - 1);
     // the residual row is loaded one row ahead (res_nx), so its L2 latency overlaps a whole row-step
     uint4 res_nx[C / 8];
     uint4 r2_nx[BWD ? C / 8 : 1];
@@ -469,12 +475,14 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
                                   int grid, bf16* tsave, int sep, long long* dbg, int exp, const bf16* mask,
                                   const bf16* res2, cudaStream_t st) {
-  auto kern = mask ? k_resblock<C, true> : k_resblock<C, false>;
-  static bool configured[2] = {false, false};
-  if (!configured[mask != nullptr]) {
+  const bool gen = tsave || sep > 0 || dbg || exp;
+  auto kern = mask ? k_resblock<C, true, true> : (gen ? k_resblock<C, false, true> : k_resblock<C, false, false>);
+  const int ki = mask ? 2 : (gen ? 1 : 0);
+  static bool configured[3] = {false, false, false};
+  if (!configured[ki]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BlkCfg<C>::SMEM);
     if (e != cudaSuccess) return e;
-    configured[mask != nullptr] = true;
+    configured[ki] = true;
   }
   return launch_k(kern, dim3(grid), dim3(kBlkThreads), BlkCfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, out, N, H, W,
                   tsave, sep, dbg, exp, mask, res2);
