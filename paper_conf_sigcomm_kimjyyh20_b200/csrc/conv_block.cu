@@ -57,9 +57,10 @@ struct BlkCfg {
                                  (size_t)kBlkNO * OUTB + ARMB;
 };
 
-// GEN = false: the inference instantiation -- no experiments, no t save, no separators, no timeline (those runtime
-// checks otherwise put predicated instructions on the epilogues' per-row chains).
-template <int C, bool BWD, bool GEN>
+// GEN = 0: the inference instantiation -- no experiments, no t save, no separators, no timeline (those runtime
+// checks otherwise put predicated instructions on the epilogues' per-row chains); 1: training forward (t save and
+// separators, no experiments / timeline); 2: everything read at run time.
+template <int C, bool BWD, int GEN>
 __global__ void __launch_bounds__(kBlkThreads, 1)
 k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
@@ -68,8 +69,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
            const int exp_in, const bf16* __restrict__ mask, const bf16* __restrict__ res2) {
   bf16* const tsave = GEN ? tsave_in : nullptr;
   const int sep = GEN ? sep_in : 0;
-  long long* const dbg = GEN ? dbg_in : nullptr;
-  const int exp = GEN ? exp_in : 0;
+  long long* const dbg = GEN == 2 ? dbg_in : nullptr;
+  const int exp = GEN == 2 ? exp_in : 0;
   // exp (benchmarking experiments only, results wrong when set): 1 no residual load, 2 no output store, 4 no t
   // smem write, 8 no bias re-arm, 16 no conv2 MMAs, 32 no conv1 MMAs, 64 no accumulator loads, 128 no f-row TMA
   // after the first piece
@@ -475,10 +476,10 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
                                   int grid, bf16* tsave, int sep, long long* dbg, int exp, const bf16* mask,
                                   const bf16* res2, cudaStream_t st) {
-  const bool gen = tsave || sep > 0 || dbg || exp;
-  auto kern = mask ? k_resblock<C, true, true> : (gen ? k_resblock<C, false, true> : k_resblock<C, false, false>);
-  const int ki = mask ? 2 : (gen ? 1 : 0);
-  static bool configured[3] = {false, false, false};
+  const int ki = mask ? 3 : ((dbg || exp) ? 2 : ((tsave || sep > 0) ? 1 : 0));
+  auto kern = ki == 3 ? k_resblock<C, true, 2>
+                      : (ki == 2 ? k_resblock<C, false, 2> : (ki == 1 ? k_resblock<C, false, 1> : k_resblock<C, false, 0>));
+  static bool configured[4] = {false, false, false, false};
   if (!configured[ki]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BlkCfg<C>::SMEM);
     if (e != cudaSuccess) return e;
