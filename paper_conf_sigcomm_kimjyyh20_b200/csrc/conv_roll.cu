@@ -76,6 +76,7 @@ struct RollArgs {
   // S HR rows of every LR row are staged in smem and leave by one TMA store (tm_out); needs W % 16 == 0.
   // Otherwise every lane reads its 3x3 (5x5) LR neighbourhood and writes its S x S x 3 bytes from/to global.
   int tail_tma;
+  int w_early;  // weights / bias may be fetched before the PDL wait (see the kernel prologue)
 };
 #define SR_RDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -177,13 +178,25 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
+  // Weights and bias were written at least two kernels upstream when the caller sets w_early (every launch inside the
+  // library's forward / backward chains: the kernel that packed them has completed before our predecessor passed its
+  // own griddepcontrol.wait, i.e. before we were scheduled), so they are fetched before the PDL wait and the fetch
+  // overlaps the predecessor's tail.  Everything the predecessor writes (activations) is read only after the wait.
+  auto load_params = [&]() {
+    if (threadIdx.x == 0) {
+      mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
+      bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
+    }
+    if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
+    __syncthreads();
+    arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, threadIdx.x, blockDim.x);
+    fence_proxy_async_smem();
+    __syncthreads();
+  };
+  if (a.w_early) load_params();
   pdl_enter();  // predecessor complete: global inputs are valid from here on
   if (threadIdx.x == 0) { SR_RDBG(10, 0) }  // after setup + PDL wait
-  if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
-  __syncthreads();
-  arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, threadIdx.x, blockDim.x);
-  fence_proxy_async_smem();
-  __syncthreads();
+  if (!a.w_early) load_params();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
 
@@ -204,8 +217,6 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     // ===================== TMA producer: weights, then input rows y0-1 .. y1 of each piece =====================
     if (elect_one()) {
       tma_prefetch_desc(&tm_in);
-      mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
-      bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
       int s = 0, xs = 0, ls = 0;
       uint32_t ph = 0, xph = 0, lph = 0;
       SR_PIECE_BEGIN
@@ -452,7 +463,7 @@ bool roll_supported(int cinp, int coutp, int W) {
 
 cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
                                 const bf16* res1, const bf16* res2, const bf16* mask, int relu, int sep, bf16* out,
-                                int N, int H, int W, cudaStream_t st, long long* dbg) {
+                                int N, int H, int W, cudaStream_t st, long long* dbg, int w_early) {
   CUtensorMap ti, to;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
@@ -461,7 +472,7 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
   const void* auxp = res1 ? (const void*)res1 : (mask ? (const void*)mask : (const void*)out);
   if (make_row_tmap(&tx, auxp, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (res1 && mask) return cudaErrorNotSupported;  // one TMA aux stream per launch
-  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0, 0};
+  RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0, 0, w_early};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
@@ -477,11 +488,11 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
 
 cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
                                   const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
-                                  int W, cudaStream_t st, int tail_tma_ok, long long* dbg) {
+                                  int W, cudaStream_t st, int tail_tma_ok, long long* dbg, int w_early) {
   CUtensorMap ti;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
-  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, dbg, lr, hr, hr_row0, hr_row1, bicubic, 0};
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, dbg, lr, hr, hr_row0, hr_row1, bicubic, 0, w_early};
   // TMA-staged tail when both u8 images are 16-B row-aligned (W % 16 == 0) and 16-B based
   CUtensorMap tl = ti, th = ti;
   if (tail_tma_ok && W % 16 == 0 &&
@@ -498,8 +509,9 @@ cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, co
 }
 
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
-                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st) {
-  return launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res, nullptr, nullptr, relu, 0, out, N, H, W, st);
+                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st, int w_early) {
+  return launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res, nullptr, nullptr, relu, 0, out, N, H, W, st, nullptr,
+                             w_early);
 }
 
 }  // namespace sr

@@ -32,15 +32,16 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStream_t st);
 bool roll_supported(int cinp, int coutp, int W);
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
-                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st);
+                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st), int w_early = 0;
 // general rolling conv: + res1 + res2, ReLU, x 1[mask > 0], zero-forced separator columns (sep > 0)
 cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
                                 const bf16* res1, const bf16* res2, const bf16* mask, int relu, int sep, bf16* out,
-                                int N, int H, int W, cudaStream_t st, long long* dbg = nullptr);
+                                int N, int H, int W, cudaStream_t st, long long* dbg = nullptr, int w_early = 0);
 // rolling up conv + tail (pixel shuffle + skip + clamp + RNE u8 into hr rows of LR rows [hr_row0, hr_row1))
 cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, const bf16* wfold, const float* bias,
                                   const uint8_t* lr, uint8_t* hr, int hr_row0, int hr_row1, int bicubic, int N, int H,
-                                  int W, cudaStream_t st, int tail_tma_ok = 1, long long* dbg = nullptr);
+                                  int W, cudaStream_t st, int tail_tma_ok = 1, long long* dbg = nullptr,
+                                  int w_early = 0);
 // fused body conv (+ f0) + up conv + tail (g kept in shared memory); needs W % 16 == 0 and a 16-B aligned LR frame
 bool bodytail_supported(int cp, int s, int W, const void* lr, const void* hr);
 cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const bf16* w1fold, const bf16* w2fold,

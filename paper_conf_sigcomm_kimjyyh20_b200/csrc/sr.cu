@@ -185,7 +185,7 @@ static sr_status conv_fwd(sr_ctx* ctx, int cinp, int coutp, const void* in, cons
                   2.0 * 9 * cinp * coutp * px, px * 2.0 * (cinp + coutp), st);
     }
     cudaError_t e = launch_conv_roll(cinp, coutp, in, sn.wo + ctx->convs[ci].pk_off, ep.bias, ep.res1, ep.relu,
-                                     ep.out, N, H, W, st);
+                                     ep.out, N, H, W, st, 1);  // inside a chain that starts with k_pack_input
     tmark_end(ctx, st);
     ctx->launches++;
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("conv_roll launch: ") + cudaGetErrorString(e));
@@ -203,7 +203,10 @@ static sr_status roll_ex(sr_ctx* ctx, const char* cls, int cinp, int coutp, cons
     tmark_begin(ctx, std::string(cls) + "_" + std::to_string(cinp) + "x" + std::to_string(coutp),
                 2.0 * 9 * cinp * coutp * px, px * 2.0 * (cinp + coutp), st);
   }
-  cudaError_t e = launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res1, res2, mask, relu, sep, out, N, H, W, st);
+  // w_early: every roll_ex launch sits inside a forward / backward chain that starts with a packing kernel, so its
+  // weights were written >= 2 kernels upstream (see k_conv_roll's prologue)
+  cudaError_t e = launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res1, res2, mask, relu, sep, out, N, H, W, st,
+                                      nullptr, 1);
   tmark_end(ctx, st);
   ctx->launches++;
   if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll launch: ") + cudaGetErrorString(e));
@@ -367,7 +370,7 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
                   2.0 * 9 * Cp * ctx->OUTP * px, px * (2.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
     }
     cudaError_t e = launch_conv_roll_tail(Cp, ctx->OUTP, ctx->s, gbuf, sn.wo + ctx->convs[cu].pk_off, Bv(cu), lr, hr,
-                                          row0, row1, ctx->opt.skip == 1, n, h, w, st, ctx->tail_tma);
+                                          row0, row1, ctx->opt.skip == 1, n, h, w, st, ctx->tail_tma, nullptr, 1);
     tmark_end(ctx, st);
     ctx->launches++;
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll tail launch: ") + cudaGetErrorString(e));
