@@ -32,7 +32,7 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStream_t st);
 bool roll_supported(int cinp, int coutp, int W);
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
-                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st), int w_early = 0;
+                             const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st, int w_early = 0);
 // general rolling conv: + res1 + res2, ReLU, x 1[mask > 0], zero-forced separator columns (sep > 0)
 cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
                                 const bf16* res1, const bf16* res2, const bf16* mask, int relu, int sep, bf16* out,
