@@ -476,10 +476,10 @@ static cudaError_t launch_block_t(const CUtensorMap& tf, const CUtensorMap& to, 
                                   const float* b1, const float* b2, const bf16* f, bf16* out, int N, int H, int W,
                                   int grid, bf16* tsave, int sep, long long* dbg, int exp, const bf16* mask,
                                   const bf16* res2, cudaStream_t st) {
-  const int ki = mask ? 3 : ((dbg || exp) ? 2 : ((tsave || sep > 0) ? 1 : 0));
-  auto kern = ki == 3 ? k_resblock<C, true, 2>
+  const int ki = mask ? ((dbg || exp) ? 4 : 3) : ((dbg || exp) ? 2 : ((tsave || sep > 0) ? 1 : 0));
+  auto kern = ki == 4 ? k_resblock<C, true, 2> : ki == 3 ? k_resblock<C, true, 1>
                       : (ki == 2 ? k_resblock<C, false, 2> : (ki == 1 ? k_resblock<C, false, 1> : k_resblock<C, false, 0>));
-  static bool configured[4] = {false, false, false, false};
+  static bool configured[5] = {false, false, false, false, false};
   if (!configured[ki]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BlkCfg<C>::SMEM);
     if (e != cudaSuccess) return e;
