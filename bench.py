@@ -143,9 +143,15 @@ def run_ours(args):
     if not args.no_graph:
         graph = torch.cuda.CUDAGraph()
         lc = ctx.launches
-        with torch.cuda.graph(graph):
-            train_iter()
-        launches_per_iter = ctx.launches - lc   # our kernels inside one captured iteration
+        try:
+            with torch.cuda.graph(graph):
+                train_iter()
+            launches_per_iter = ctx.launches - lc   # our kernels inside one captured iteration
+        except Exception as exc:  # e.g. a collective that cannot be captured: launch the iterations eagerly
+            print(f"[bench] rank {rank}: training-iteration graph capture failed ({exc}); eager iterations",
+                  file=sys.stderr, flush=True)
+            graph = None
+            torch.cuda.synchronize()
 
     ctrl = Controller(thresh_sat=0.05, count_sat=2, thresh_online=0.5, count_online=2)
     state["iters"] = 0  # training iterations since the last epoch end
