@@ -955,8 +955,23 @@ sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int
   // Chunked pipeline: all H2D copies go first on their own stream (per-chunk events), chunk k is super-resolved
   // on `stream` as soon as its frames landed, and its D2H runs on a third stream while chunk k+1 computes.
   // PCIe (55 GB/s measured) then hides behind the tensor work; only the last chunk's D2H is exposed.
+  // Chunk sizes: ~96 MB of HR output per chunk, except a one-frame first chunk (compute starts after one frame's
+  // H2D) and a one-frame last chunk (only one frame's D2H is left exposed after the last kernel).
   const int F = std::max(1, std::min(n, (int)std::max<size_t>(1, (size_t)(96u << 20) / std::max<size_t>(fh, 1))));
-  const int nch = (n + F - 1) / F;
+  std::vector<int> c0s;  // first frame of each chunk (+ n at the end)
+  {
+    int f = 0;
+    c0s.push_back(0);
+    if (n >= 3 && F > 1) { f = 1; c0s.push_back(f); }
+    while (f < n) {
+      const int left = n - f;
+      int take = std::min(F, left);
+      if (F > 1 && left > 1 && take == left) take = left - 1;  // keep the final frame as its own chunk
+      f += take;
+      c0s.push_back(f);
+    }
+  }
+  const int nch = (int)c0s.size() - 1;
   while ((int)ctx->chunk_ev.size() < 2 * nch + 1) {
     cudaEvent_t e;
     CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
@@ -967,12 +982,12 @@ sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int
   CK(cudaStreamWaitEvent(ctx->h2d_st, ev[0], 0));  // copies follow earlier work on `stream`
   CK(cudaStreamWaitEvent(ctx->copy_st, ev[0], 0));
   for (int c = 0; c < nch; ++c) {
-    const int f0 = c * F, fn = std::min(F, n - f0);
+    const int f0 = c0s[c], fn = c0s[c + 1] - c0s[c];
     CK(cudaMemcpyAsync(ctx->stage_lr + f0 * fl, lr_host + f0 * fl, fn * fl, cudaMemcpyHostToDevice, ctx->h2d_st));
     CK(cudaEventRecord(ev[1 + c], ctx->h2d_st));
   }
   for (int c = 0; c < nch; ++c) {
-    const int f0 = c * F, fn = std::min(F, n - f0);
+    const int f0 = c0s[c], fn = c0s[c + 1] - c0s[c];
     CK(cudaStreamWaitEvent(st, ev[1 + c], 0));
     TRY(sr_infer(ctx, which, ctx->stage_lr + f0 * fl, fn, h, w, ctx->stage_hr + f0 * fh, stream));
     CK(cudaEventRecord(ev[1 + nch + c], st));
