@@ -226,9 +226,13 @@ def run_ours(args):
     loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
 
     def step_e2e():
-        ctx.infer_host(lr_host, hr_host, "serve")
+        # a serving loop: frames in and out through the host API; the training iterations are enqueued behind the
+        # inference and run while the last HR chunks drain over PCIe; the step ends when its HR frames are in host
+        # memory (sr_infer_host_wait) and its loss has been read back
+        ctx.infer_host_async(lr_host, hr_host, "serve")
         train_iters()
         loss_host.copy_(loss, non_blocking=True)
+        ctx.infer_host_wait()
 
     step_e2e()
     barrier()

@@ -123,6 +123,16 @@ class SRContext:
                                      _stream(stream)), self.h, "sr_infer_host")
         return out_host
 
+    def infer_host_async(self, lr_host, out_host, which="serve", stream=None):
+        """sr_infer_host_async: enqueue H2D / compute / D2H and return; out_host is valid after infer_host_wait()."""
+        n, h, w, _ = lr_host.shape
+        check(self.lib.sr_infer_host_async(self.h, _model(which), _ptr(lr_host), n, h, w, _ptr(out_host),
+                                           _stream(stream)), self.h, "sr_infer_host_async")
+        return out_host
+
+    def infer_host_wait(self):
+        check(self.lib.sr_infer_host_wait(self.h), self.h, "sr_infer_host_wait")
+
     def infer_rows(self, lr_frame, row0, row1, hr_frame, which="serve", stream=None):
         h, w, _ = lr_frame.shape
         check(self.lib.sr_infer_rows(self.h, _model(which), _ptr(lr_frame), h, w, row0, row1, _ptr(hr_frame),

@@ -50,6 +50,8 @@ _SIGS = {
     "sr_set_params": (_I, [_P, _P, C.c_size_t]),
     "sr_infer": (_I, [_P, _I, _P, _I, _I, _I, _P, _P]),
     "sr_infer_host": (_I, [_P, _I, _P, _I, _I, _I, _P, _P]),
+    "sr_infer_host_async": (_I, [_P, _I, _P, _I, _I, _I, _P, _P]),
+    "sr_infer_host_wait": (_I, [_P]),
     "sr_infer_rows": (_I, [_P, _I, _P, _I, _I, _I, _I, _P, _P]),
     "sr_infer_i420": (_I, [_P, _I, _P, _P, _P, _I, _I, _I, _P, _P, _P, _P]),
     "sr_pool_push_i420": (_I, [_P, _P, _P, _P, _I, _I, _P, _P, _I, _I, _P, _P]),

@@ -37,6 +37,7 @@ struct sr_ctx {
   uint8_t *stage_lr = nullptr, *stage_hr = nullptr;
   cudaStream_t copy_st = nullptr, h2d_st = nullptr;  // sr_infer_host: PCIe copies overlapped with the tensor work
   std::vector<cudaEvent_t> chunk_ev;
+  bool host_pending = false;  // an sr_infer_host_async call whose D2H copies may still be in flight
   size_t stage_lr_bytes = 0, stage_hr_bytes = 0;
   // training workspace
   size_t tr_pix = 0;
@@ -939,10 +940,13 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
   return SR_OK;
 }
 
-sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
-                        uint8_t* hr_host, sr_stream stream) {
-  GUARD();
+static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
+                                 uint8_t* hr_host, sr_stream stream, bool sync) {
   if (!lr_host || !hr_host || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer_host: bad args");
+  if (ctx->host_pending) {  // the staging buffers and chunk events are reused: finish the previous async call
+    CK(cudaStreamSynchronize(ctx->copy_st));
+    ctx->host_pending = false;
+  }
   cudaStream_t st = (cudaStream_t)stream;
   const size_t fl = (size_t)h * w * 3, fh = fl * ctx->s * ctx->s;
   const size_t lb = (size_t)n * fl, hb = (size_t)n * fh;
@@ -994,7 +998,32 @@ sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int
     CK(cudaStreamWaitEvent(ctx->copy_st, ev[1 + nch + c], 0));
     CK(cudaMemcpyAsync(hr_host + f0 * fh, ctx->stage_hr + f0 * fh, fn * fh, cudaMemcpyDeviceToHost, ctx->copy_st));
   }
-  CK(cudaStreamSynchronize(ctx->copy_st));
+  if (sync) {
+    CK(cudaStreamSynchronize(ctx->copy_st));
+  } else {
+    ctx->host_pending = true;
+  }
+  return SR_OK;
+}
+
+sr_status sr_infer_host(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
+                        uint8_t* hr_host, sr_stream stream) {
+  GUARD();
+  return infer_host_impl(ctx, which, lr_host, n, h, w, hr_host, stream, true);
+}
+
+sr_status sr_infer_host_async(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
+                              uint8_t* hr_host, sr_stream stream) {
+  GUARD();
+  return infer_host_impl(ctx, which, lr_host, n, h, w, hr_host, stream, false);
+}
+
+sr_status sr_infer_host_wait(sr_ctx* ctx) {
+  GUARD();
+  if (ctx->host_pending) {
+    CK(cudaStreamSynchronize(ctx->copy_st));
+    ctx->host_pending = false;
+  }
   return SR_OK;
 }
 

@@ -327,6 +327,14 @@ def test_infer_host_pipeline_equals_device_path():
     out_h = torch.empty((7, 360, 600, 3), dtype=torch.uint8).pin_memory()
     ctx.infer_host(lr_h, out_h, "serve")
     assert torch.equal(out_h, dev)
+    # asynchronous form: enqueue, queue more work behind it, then wait; a second call waits for the first
+    out_a = torch.zeros_like(out_h).pin_memory()
+    out_b = torch.zeros_like(out_h).pin_memory()
+    ctx.infer_host_async(lr_h, out_a, "serve")
+    ctx.infer(torch.from_numpy(lr).cuda(), "serve")
+    ctx.infer_host_async(lr_h, out_b, "serve")
+    ctx.infer_host_wait()
+    assert torch.equal(out_a, dev) and torch.equal(out_b, dev)
 
 
 # ---------------------------------------------------------------- I420 boundary
