@@ -128,11 +128,13 @@ def run_ours(args):
     state = {"q": None}
 
     wdev = torch.ones(1, dtype=torch.float32, device=dev)  # this rank's gradient weight w_r
+    inv_w = wdev.reciprocal()  # single GPU: the Adam scale 1 / w_0 (no exchange step)
 
     def train_iter():
         ctx.sample_batch(-1, BATCH, PATCH, out=(blr, bhr, bidx))   # device-side step counter
         ctx.train_grad(blr, bhr, loss)                            # grad <- w_r g_r
-        scale = dp_allreduce_grad_dev(grad, wdev)                 # NCCL over NVLink (N > 1); 1 / sum_r w_r
+        # NCCL sum-allreduce over NVLink (N > 1) -> Adam scale 1 / sum_r w_r
+        scale = dp_allreduce_grad_dev(grad, wdev) if world > 1 else inv_w
         ctx.train_apply_dev(scale)
 
     # one training iteration captured as a CUDA graph (after an eager warm-up that sizes the workspaces)

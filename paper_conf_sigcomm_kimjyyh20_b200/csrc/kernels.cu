@@ -174,8 +174,11 @@ void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStr
 // dfold: Wdo[kx'][co/8][ky' cinp + ci][co%8] = W[co][ci][2-ky'][2-kx']  (dy-fold weights of the data-grad conv)
 __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc* __restrict__ convs, int nconv,
                                bf16* __restrict__ wf, bf16* __restrict__ wd, bf16* __restrict__ wo,
-                               bf16* __restrict__ wdo, float* __restrict__ bias) {
+                               bf16* __restrict__ wdo, float* __restrict__ bias, long long* __restrict__ bump) {
   pdl_enter();
+  // bump (training only): the Adam step counter, advanced here -- after k_adam of this step has read it -- instead
+  // of by a separate launch before k_adam
+  if (bump && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) ++*bump;
   const int c = blockIdx.y;
   if (c >= nconv) return;
   const ConvDesc d = convs[c];
@@ -223,9 +226,9 @@ __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc*
 }
 
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st) {
+                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st, long long* bump) {
   dim3 grid((max_elems + 255) / 256, nconv);
-  launch_k(k_pack_weights, grid, dim3(256), 0, st, params, convs_dev, nconv, wf, wd, wo, wdo, bias);
+  launch_k(k_pack_weights, grid, dim3(256), 0, st, params, convs_dev, nconv, wf, wd, wo, wdo, bias, bump);
 }
 
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
@@ -242,12 +245,21 @@ void launch_adam_prep(long long* counters, float* scal, double lr, double b1, do
   launch_k(k_adam_prep, dim3(1), dim3(1), 0, st, counters, scal, lr, b1, b2);
 }
 
+// k_adam computes the bias corrections itself from the device step counter: t = counters[1] + 1 (the counter is
+// advanced by the TRAIN repack that follows, k_pack_weights' bump) -- one launch less per training iteration.
 __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
                        const float* __restrict__ grad, size_t n, const float* __restrict__ gscale_dev, float gscale,
-                       const float* __restrict__ scal, float b1, float b2, float eps) {
+                       const long long* __restrict__ counters, double lr, float b1, float b2, float eps) {
   pdl_enter();
+  __shared__ float s_bc[2];
+  if (threadIdx.x == 0) {
+    const double t = (double)(counters[1] + 1);
+    s_bc[0] = (float)(lr / (1.0 - pow((double)b1, t)));
+    s_bc[1] = (float)(1.0 / sqrt(1.0 - pow((double)b2, t)));
+  }
+  __syncthreads();
   const float gs = gscale * (gscale_dev ? *gscale_dev : 1.f);
-  const float lr_bc1 = scal[0], inv_sqrt_bc2 = scal[1];
+  const float lr_bc1 = s_bc[0], inv_sqrt_bc2 = s_bc[1];
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   const size_t stride = (size_t)gridDim.x * blockDim.x;
   for (; i < n; i += stride) {
@@ -261,11 +273,11 @@ __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __re
 }
 
 void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
-                 const float* scal, float b1, float b2, float eps, cudaStream_t st) {
+                 const long long* counters, double lr, float b1, float b2, float eps, cudaStream_t st) {
   int th = 256;
   int blocks = (int)((n + th - 1) / th);
   if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
-  launch_k(k_adam, dim3(blocks), dim3(th), 0, st, p, m, v, g, n, gscale_dev, gscale, scal, b1, b2, eps);
+  launch_k(k_adam, dim3(blocks), dim3(th), 0, st, p, m, v, g, n, gscale_dev, gscale, counters, lr, b1, b2, eps);
 }
 
 __global__ void k_counter_add(long long* c, long long d) {

@@ -28,7 +28,8 @@ struct SampleArgs {
 
 void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st);
 void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nconv, int max_elems, bf16* wf,
-                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st);
+                         bf16* wd, bf16* wo, bf16* wdo, float* bias, cudaStream_t st,
+                         long long* bump = nullptr);
 void launch_pack_input_virtual(const uint8_t* lr, int n, int p, bf16* x, cudaStream_t st);
 bool roll_supported(int cinp, int coutp, int W);
 cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wfold, const float* bias,
@@ -57,7 +58,7 @@ cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf1
 // counters[0] = sampler step, counters[1] = Adam step t; scal[0] = lr / (1 - b1^t), scal[1] = 1/sqrt(1 - b2^t).
 void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st);
 void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
-                 const float* scal, float b1, float b2, float eps, cudaStream_t st);
+                 const long long* counters, double lr, float b1, float b2, float eps, cudaStream_t st);
 void launch_counter_add(long long* counter, long long delta, cudaStream_t st);
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st);
 void launch_sse_u8(const uint8_t* a, const uint8_t* b, int n, int64_t elems, unsigned long long* out,

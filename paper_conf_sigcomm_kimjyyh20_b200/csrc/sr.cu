@@ -123,10 +123,10 @@ static uint64_t mix64h(uint64_t z) {
   return z ^ (z >> 31);
 }
 
-static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st) {
+static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st, long long* bump = nullptr) {
   launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, ctx->snap[which].wf,
                       with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].wo,
-                      with_dgrad ? ctx->wdo_train : nullptr, ctx->snap[which].bias, st);
+                      with_dgrad ? ctx->wdo_train : nullptr, ctx->snap[which].bias, st, bump);
   ctx->launches++;
   CKL();
   return SR_OK;
@@ -662,12 +662,11 @@ static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, i
 
 static sr_status train_apply(sr_ctx* ctx, float grad_scale, const float* grad_scale_dev, cudaStream_t st) {
   ctx->t += 1;  // host mirror only; the kernels use the device counter (graph-replayable)
-  launch_adam_prep(ctx->counters, ctx->adam_scal, ctx->opt.lr, ctx->opt.beta1, ctx->opt.beta2, st);
-  launch_adam(ctx->params, ctx->m, ctx->v, ctx->grad, ctx->nparams, grad_scale_dev, grad_scale, ctx->adam_scal,
-              ctx->opt.beta1, ctx->opt.beta2, ctx->opt.eps, st);
-  ctx->launches += 2;
+  launch_adam(ctx->params, ctx->m, ctx->v, ctx->grad, ctx->nparams, grad_scale_dev, grad_scale, ctx->counters,
+              ctx->opt.lr, ctx->opt.beta1, ctx->opt.beta2, ctx->opt.eps, st);
+  ctx->launches += 1;
   CKL();
-  return repack(ctx, SR_TRAIN, true, st);
+  return repack(ctx, SR_TRAIN, true, st, ctx->counters + 1);  // the repack advances the Adam step counter
 }
 
 static bool valid_model(sr_model m) { return m >= SR_TRAIN && m <= SR_INIT; }
