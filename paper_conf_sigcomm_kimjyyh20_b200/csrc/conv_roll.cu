@@ -138,8 +138,14 @@ __device__ __forceinline__ void roll_stage(uint4* orow, const float* v, const ui
   }
 }
 
-template <int CINP, int COUTP, int TS>
-__global__ void __launch_bounds__(kRollThreads, 1)
+// U8 (head conv only, CINP = 16): the input is the u8 RGB frame itself.  The producer TMA-loads u8 rows (16-B
+// chunk map, W % 16 == 0) into a small ring in the aux area and warp 11 expands each row into the bf16 A slot
+// (x = v/255 in channels 0..2, exactly k_pack_input's arithmetic; channel chunk 1 is a zero plane written once),
+// so k_pack_input's 32 B/px write and the head's 32 B/px read become a 3 B/px read.
+static constexpr int kU8Slots = 8;
+static constexpr uint32_t kU8Slot = 512;  // 26 chunks = 416 B per u8 row
+template <int CINP, int COUTP, int TS, bool U8 = false>
+__global__ void __launch_bounds__(kRollThreads + (U8 ? 32 : 0), 1)
 k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
             const __grid_constant__ CUtensorMap tm_aux, const bf16* __restrict__ wfold, const RollArgs a) {
   using Cfg = RollCfg<CINP, COUTP>;
@@ -156,7 +162,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   uint8_t* sBt = sOnes + kArmOnesBytes;
   __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
       x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar, l_full[TS > 0 ? Cfg::NLR : 1],
-      l_empty[TS > 0 ? Cfg::NLR : 1];
+      l_empty[TS > 0 ? Cfg::NLR : 1], u_full[U8 ? kU8Slots : 1], u_empty[U8 ? kU8Slots : 1];
   // the aux row (res1 or mask) travels by TMA; res2 (used once per backward pass) by plain loads
   const bool has_aux = a.res1 != nullptr || a.mask != nullptr;
   __shared__ uint32_t tmem_base_sh;
@@ -172,10 +178,19 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     if (TS > 0)
       for (int s = 0; s < Cfg::NLR; ++s) { mbar_init(&l_full[s], 1); mbar_init(&l_empty[s], 4); }
     for (int s = 0; s < 2 * kRollNO; ++s) { mbar_init(&o_full[s], 4); mbar_init(&o_free[s], 1); }
+    if (U8)
+      for (int s = 0; s < kU8Slots; ++s) { mbar_init(&u_full[s], 1); mbar_init(&u_empty[s], 1); }
     mbar_init(&w_bar, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
+  if constexpr (U8) {  // channel chunk 1 (channels 8..15) of every input slot stays zero
+    static_assert(CINP == 16, "u8 input: head conv only");
+    for (int i = threadIdx.x; i < kRollIn * (int)(PLANE / 16); i += blockDim.x)
+      *reinterpret_cast<uint4*>(sIn + (i / (PLANE / 16)) * IN_STRIDE + PLANE + (i % (PLANE / 16)) * 16) =
+          make_uint4(0u, 0u, 0u, 0u);
+    fence_proxy_async_smem();
+  }
   tc_fence_before();
   __syncthreads();
   // Weights and bias were written at least two kernels upstream when the caller sets w_early (every launch inside the
@@ -217,15 +232,22 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     // ===================== TMA producer: weights, then input rows y0-1 .. y1 of each piece =====================
     if (elect_one()) {
       tma_prefetch_desc(&tm_in);
-      int s = 0, xs = 0, ls = 0;
-      uint32_t ph = 0, xph = 0, lph = 0;
+      int s = 0, xs = 0, ls = 0, us = 0;
+      uint32_t ph = 0, xph = 0, lph = 0, uph = 0;
       SR_PIECE_BEGIN
       for (int i = 0; i < n_in; ++i) {
-        mbar_wait(&in_empty[s], ph ^ 1);
-        mbar_arrive_expect_tx(&in_full[s], Cfg::IN_BOX);
-        tma_load_5d(sIn + s * IN_STRIDE, &tm_in, &in_full[s], 0, x0 - 1, y0 - 1 + i, 0, n);
+        if constexpr (U8) {  // u8 row y0-1+i, pixels x0-1 .. x0+128 (+ chunk alignment), for warp 11 to expand
+          mbar_wait(&u_empty[us], uph ^ 1);
+          mbar_arrive_expect_tx(&u_full[us], 16 * 26);
+          tma_load_4d(sA + us * kU8Slot, &tm_in, &u_full[us], 0, (3 * x0 - 3) >> 4, y0 - 1 + i, n);
+          if (++us == kU8Slots) { us = 0; uph ^= 1; }
+        } else {
+          mbar_wait(&in_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&in_full[s], Cfg::IN_BOX);
+          tma_load_5d(sIn + s * IN_STRIDE, &tm_in, &in_full[s], 0, x0 - 1, y0 - 1 + i, 0, n);
+          if (++s == kRollIn) { s = 0; ph ^= 1; }
+        }
         SR_RDBG(0, i)
-        if (++s == kRollIn) { s = 0; ph ^= 1; }
         if (TS > 0 && a.tail_tma && i >= 1 && i - 1 < y1 - y0) {  // LR rows r-2..r+2 of output row r = y0+i-1
           mbar_wait(&l_empty[ls], lph ^ 1);
           mbar_arrive_expect_tx(&l_full[ls], 16 * kTailLrChunks * 5);
@@ -278,6 +300,49 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       SR_PIECE_END
     }
     __syncwarp();
+  } else if (U8 && warp == 11) {
+    // ===================== u8 -> bf16 A-operand expansion (head conv) =====================
+    int s = 0, us = 0;
+    uint32_t ph = 0, uph = 0;
+    SR_PIECE_BEGIN
+    const int lbase = 16 * ((3 * x0 - 3) >> 4);
+    for (int i = 0; i < n_in; ++i) {
+      mbar_wait(&u_full[us], uph);
+      mbar_wait(&in_empty[s], ph ^ 1);
+      const uint32_t src = smem_u32(sA + us * kU8Slot) + (uint32_t)(3 * (x0 - 1) - lbase);
+      uint8_t* dst = sIn + s * IN_STRIDE;
+      constexpr int kIt = (kRollTW + 2 + 31) / 32;
+      float px[kIt][3];
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {  // all loads first, so their latencies overlap
+        const int p = lane_id() + 32 * k;
+        const uint32_t q = src + 3 * min(p, kRollTW + 1);
+        px[k][0] = lds_u8f(q);
+        px[k][1] = lds_u8f(q + 1);
+        px[k][2] = lds_u8f(q + 2);
+      }
+#pragma unroll
+      for (int k = 0; k < kIt; ++k) {
+        const int p = lane_id() + 32 * k;
+        if (p < kRollTW + 2) {
+          uint4 v;
+          v.x = pack_bf16x2(px[k][0] * (1.f / 255.f), px[k][1] * (1.f / 255.f));
+          v.y = pack_bf16x2(px[k][2] * (1.f / 255.f), 0.f);
+          v.z = 0u;
+          v.w = 0u;
+          *reinterpret_cast<uint4*>(dst + p * 16) = v;
+        }
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane_id() == 0) {
+        mbar_arrive(&u_empty[us]);
+        mbar_arrive(&in_full[s]);
+      }
+      if (++us == kU8Slots) { us = 0; uph ^= 1; }
+      if (++s == kRollIn) { s = 0; ph ^= 1; }
+    }
+    SR_PIECE_END
   } else if (warp == 10) {
     // ===================== store warp: TMA-store finished rows in emission order =====================
     if ((TS == 0 || a.tail_tma) && elect_one()) {
@@ -427,13 +492,13 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-template <int CINP, int COUTP, int TS = 0>
+template <int CINP, int COUTP, int TS = 0, bool U8 = false>
 static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, const CUtensorMap& tx,
                                  const bf16* wfold, const RollArgs& a, int grid, cudaStream_t st) {
   if constexpr (!RollCfg<CINP, COUTP>::FITS) {
     return cudaErrorNotSupported;
   } else {
-    auto kern = k_conv_roll<CINP, COUTP, TS>;
+    auto kern = k_conv_roll<CINP, COUTP, TS, U8>;
     constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
     static bool configured = false;
     if (!configured) {
@@ -441,8 +506,28 @@ static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, c
       if (e != cudaSuccess) return e;
       configured = true;
     }
-    return launch_k(kern, dim3(grid), dim3(kRollThreads), smem, st, ti, to, tx, wfold, a);
+    return launch_k(kern, dim3(grid), dim3(kRollThreads + (U8 ? 32 : 0)), smem, st, ti, to, tx, wfold, a);
   }
+}
+
+bool roll_head_u8_supported(int coutp, int W, const void* lr) {
+  return W >= 96 && W % 16 == 0 && (reinterpret_cast<uintptr_t>(lr) & 15) == 0 &&
+         (coutp == 16 || coutp == 32 || coutp == 48);
+}
+
+cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* wfold, const float* bias, bf16* out,
+                                     int N, int H, int W, cudaStream_t st, int w_early) {
+  if (!roll_head_u8_supported(coutp, W, lr)) return cudaErrorNotSupported;
+  CUtensorMap ti, to;
+  if (make_u8_rows_tmap(&ti, lr, N, H, 3LL * W, 26, 1) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, nullptr, nullptr, 0, 0, 0, 0, w_early};
+  const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  if (coutp == 16) return launch_roll_t<16, 16, 0, true>(ti, to, to, wfold, a, grid, st);
+  if (coutp == 32) return launch_roll_t<16, 32, 0, true>(ti, to, to, wfold, a, grid, st);
+  return launch_roll_t<16, 48, 0, true>(ti, to, to, wfold, a, grid, st);
 }
 
 static bool ch_ok(int c) { return c == 16 || c == 32 || c == 48 || c == 64; }

@@ -81,6 +81,7 @@ struct sr_ctx {
   bool fuse_bwd = false;    // fused data-gradient residual blocks (sr_set_fusion bit 3; slower at the training shape)
   bool tail_tma = true;     // TMA-staged LR/HR rows in the rolling tail (sr_set_fusion bit 4 clears)
   bool fuse_bodytail = true;  // body conv + up conv + tail as one kernel, g in smem (sr_set_fusion bit 5 clears)
+  bool fuse_head = true;      // head conv reads the u8 frame directly (sr_set_fusion bit 6 clears)
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -305,15 +306,27 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
   const size_t pix = (size_t)n * h * w;
   TRY(ensure_infer_ws(ctx, pix));
   const int Cp = ctx->Cp;
-  launch_pack_input(lr, pix, ctx->x16, st);
-  ctx->launches++;
-  CKL();
   auto W = [&](int ci) { return sn.wf + ctx->convs[ci].pk_off; };
   auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
-  EpiParams ep{};
-  ep.bias = Bv(0);
-  ep.out = ctx->f0;
-  TRY(conv_fwd(ctx, 16, Cp, ctx->x16, sn, 0, n, h, w, ep, st));
+  if (ctx->fuse_head && roll_supported(16, Cp, w) && roll_head_u8_supported(Cp, w, lr)) {
+    // head conv straight from the u8 frame (x = v/255 expanded in shared memory; no k_pack_input pass)
+    if (ctx->timing) {
+      const double px = (double)n * h * w;
+      tmark_begin(ctx, "conv_roll_16x" + std::to_string(Cp), 2.0 * 9 * 16 * Cp * px, px * (3.0 + 2.0 * Cp), st);
+    }
+    cudaError_t e = launch_conv_roll_head_u8(Cp, lr, sn.wo + ctx->convs[0].pk_off, Bv(0), ctx->f0, n, h, w, st, 1);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("u8 head launch: ") + cudaGetErrorString(e));
+  } else {
+    launch_pack_input(lr, pix, ctx->x16, st);
+    ctx->launches++;
+    CKL();
+    EpiParams ep{};
+    ep.bias = Bv(0);
+    ep.out = ctx->f0;
+    TRY(conv_fwd(ctx, 16, Cp, ctx->x16, sn, 0, n, h, w, ep, st));
+  }
   bf16* cur = ctx->f0;
   for (int b = 0; b < ctx->B; ++b) {
     bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
@@ -806,6 +819,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->fuse_bwd = (fuse_blocks & 8) != 0;       // bit 3 set: fused data-gradient blocks in training
   ctx->tail_tma = (fuse_blocks & 16) == 0;      // bit 4 set: rolling tail reads/writes u8 pixels per lane
   ctx->fuse_bodytail = (fuse_blocks & 32) == 0; // bit 5 set: body conv and up conv + tail as two kernels
+  ctx->fuse_head = (fuse_blocks & 64) == 0;     // bit 6 set: k_pack_input + head conv on the bf16 copy
   return SR_OK;
 }
 

@@ -526,3 +526,22 @@ def test_fused_bodytail_strips_and_unaligned_output():
     torch.cuda.synchronize()
     assert torch.equal(view, full[0])
     assert int(flat[:5].sum()) == 0 and int(flat[5 + full[0].numel():].sum()) == 0
+
+
+@pytest.mark.parametrize("cfg,hw", [((3, 8, 48), (37, 272)), ((2, 3, 32), (29, 400)), ((4, 2, 16), (19, 144)),
+                                    ((3, 2, 48), (5, 1296))])
+def test_u8_head_equals_packed_head(cfg, hw):
+    """Head conv reading the u8 frame directly (x = v/255 expanded in shared memory; default when W % 16 == 0) ==
+    k_pack_input + head conv (set_fusion bit 6), bit for bit -- same bf16 operands, same MMA order."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=71)
+    lr, hr = synth_frames(2, hw[0], hw[1], seed=72, scale=s)
+    lrd = torch.from_numpy(lr).cuda()
+    a = ctx.infer(lrd, "serve").clone()
+    ctx.set_fusion(1 | 64)
+    b = ctx.infer(lrd, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
+    if hw[1] <= 400:
+        ref = O.infer_u8(ctx.get_params("serve"), lr, s, B, C)
+        _check_frames(a.cpu().numpy(), ref, hr)
