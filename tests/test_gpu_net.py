@@ -545,3 +545,49 @@ def test_u8_head_equals_packed_head(cfg, hw):
     if hw[1] <= 400:
         ref = O.infer_u8(ctx.get_params("serve"), lr, s, B, C)
         _check_frames(a.cpu().numpy(), ref, hr)
+
+
+def test_sampler_rank_views_bitexact():
+    """world = 2: each rank samples from its arrival-order chunk of the pool (SURVEY §8(c)
+    step 10) -- indices within the view, crop offsets and gathered bytes equal the oracle's."""
+    s, B, C = 2, 1, 8
+    lrp, hrp, _ = synth_patch_pool(301, s, 120, seed=5, frame_hw=(240, 600))
+    for rank in (0, 1):
+        ctx = _ctx(s, B, C, seed=78, world=2, rank=rank)
+        ctx.pool_push(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda())
+        lo, hi = 301 * rank // 2, 301 * (rank + 1) // 2
+        for step in (0, 3):
+            lr, hr, idx = ctx.sample_batch(step, 32, 48)
+            ridx, oy, ox = O.sample_indices(78, step, hi - lo, 32, 60, 48, rank=rank, world=2)
+            np.testing.assert_array_equal(idx.cpu().numpy(), ridx)
+            rl, rh = O.gather_patches(lrp[lo:hi], hrp[lo:hi], ridx, oy, ox, 48, s)
+            np.testing.assert_array_equal(lr.cpu().numpy(), rl)
+            np.testing.assert_array_equal(hr.cpu().numpy(), rh)
+
+
+def test_two_rank_dp_step_matches_oracle():
+    """The DP training step of two ranks, both on this GPU with the allreduce done by hand (what NCCL sums):
+    grad = w_0 g_0 + w_1 g_1 from each rank's sr_train_grad (dp_weight pre-scales), Adam with 1 / (w_0 + w_1)
+    -> the oracle's dp_aggregate + adam_step; both ranks end with identical parameters."""
+    s, B, C = 2, 2, 16
+    lrp, hrp, _ = synth_patch_pool(6, s, 2 * 20, seed=81, frame_hw=(2 * 20 * 3, 2 * 20 * 4))
+    w = (1.0, 3.0)
+    ctxs = [_ctx(s, B, C, seed=82, world=2, rank=r, dp_weight=w[r]) for r in (0, 1)]
+    p0 = ctxs[0].get_params("train")
+    halves = [(slice(0, 3)), (slice(3, 6))]
+    grads, ref_g = [], []
+    for r, ctx in enumerate(ctxs):
+        lo = torch.zeros(1, device="cuda")
+        ctx.train_grad(torch.from_numpy(lrp[halves[r]]).cuda(), torch.from_numpy(hrp[halves[r]]).cuda(), lo)
+        grads.append(ctx.grad_buffer().clone())
+        ref_g.append(O.train_loss_and_grad(p0, lrp[halves[r]], hrp[halves[r]], s, B, C)[1])
+    total = grads[0] + grads[1]  # the sum-allreduce
+    for ctx in ctxs:
+        ctx.grad_buffer().copy_(total)
+        ctx.train_apply(1.0 / sum(w))
+    pa, pb = ctxs[0].get_params("train"), ctxs[1].get_params("train")
+    np.testing.assert_array_equal(pa, pb)
+    g = O.dp_aggregate(ref_g, list(w))
+    rp, _, _ = O.adam_step(p0, np.zeros_like(p0), np.zeros_like(p0), g, 1)
+    assert rel_l2(pa, rp) < 1e-3
+    assert rel_l2(total.cpu().numpy() / sum(w), g) < 1e-2
