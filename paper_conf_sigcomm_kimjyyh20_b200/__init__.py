@@ -248,6 +248,10 @@ class SRContext:
     def set_fusion(self, fuse_blocks=True):
         check(self.lib.sr_set_fusion(self.h, int(fuse_blocks)), self.h, "sr_set_fusion")
 
+    def set_sm_split(self, train_sms):
+        """sr_set_sm_split: training-side calls use train_sms SMs, inference-side calls the rest (0 = all)."""
+        check(self.lib.sr_set_sm_split(self.h, int(train_sms)), self.h, "sr_set_sm_split")
+
     def kernel_timing(self, enable=True):
         check(self.lib.sr_kernel_timing(self.h, int(enable)), self.h, "sr_kernel_timing")
 

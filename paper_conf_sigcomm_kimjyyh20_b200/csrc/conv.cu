@@ -27,6 +27,11 @@ static constexpr int kStages = 2;
 static constexpr int kWgStages = 3;  // wgrad TMA ring depth
 static constexpr int kSmemLimit = 227 * 1024;
 
+// Grid sizing.  Every persistent kernel takes one CTA per SM; set_grid_cap limits that to the SM share of the
+// calling API entry (sr_set_sm_split: inference and training running concurrently on disjoint SM sets).
+static thread_local int g_grid_cap = 0;
+void set_grid_cap(int cap) { g_grid_cap = cap; }
+int grid_cap() { return g_grid_cap; }
 int num_sms() {
   static int n = 0;
   if (!n) {
@@ -35,7 +40,7 @@ int num_sms() {
     cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
     if (n <= 0) n = 148;
   }
-  return n;
+  return (g_grid_cap > 0 && g_grid_cap < n) ? g_grid_cap : n;
 }
 
 // ------------------------------------------------------------------------------------------ geometry

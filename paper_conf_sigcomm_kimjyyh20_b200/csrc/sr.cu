@@ -82,6 +82,8 @@ struct sr_ctx {
   bool tail_tma = true;     // TMA-staged LR/HR rows in the rolling tail (sr_set_fusion bit 4 clears)
   bool fuse_bodytail = true;  // body conv + up conv + tail as one kernel, g in smem (sr_set_fusion bit 5 clears)
   bool fuse_head = true;      // head conv reads the u8 frame directly (sr_set_fusion bit 6 clears)
+  int sm_train = 0;           // sr_set_sm_split: SMs given to the training kernels (0 = all SMs to every call)
+  int sm_total = 0;
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
   size_t tnext = 0;
@@ -823,6 +825,16 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   return SR_OK;
 }
 
+sr_status sr_set_sm_split(sr_ctx* ctx, int train_sms) {
+  if (!ctx) return SR_E_INVAL;
+  set_grid_cap(0);
+  const int n = num_sms();
+  if (train_sms < 0 || train_sms >= n) return fail(ctx, SR_E_INVAL, "sr_set_sm_split: need 0 <= train_sms < #SMs");
+  ctx->sm_total = n;
+  ctx->sm_train = train_sms;
+  return SR_OK;
+}
+
 sr_status sr_kernel_timing(sr_ctx* ctx, int enable) {
   if (!ctx) return SR_E_INVAL;
   ctx->timing = enable != 0;
@@ -869,6 +881,18 @@ float* sr_grad_buffer(sr_ctx* ctx) { return ctx ? ctx->grad : nullptr; }
     if (!ctx) return SR_E_INVAL;                                                 \
     if (ctx->poisoned) return fail(ctx, SR_E_STATE, "ctx poisoned: " + ctx->err); \
   } while (0)
+
+// SM share of an API entry (restored on return): inference-side calls get sm_total - sm_train SMs, training-side
+// calls sm_train, when a split is set.
+struct GridCapScope {
+  int prev;
+  GridCapScope(const sr_ctx* ctx, bool train) : prev(grid_cap()) {
+    if (ctx && ctx->sm_train > 0) set_grid_cap(train ? ctx->sm_train : ctx->sm_total - ctx->sm_train);
+  }
+  ~GridCapScope() { set_grid_cap(prev); }
+};
+#define CAP_INFER() GridCapScope cap_scope_(ctx, false)
+#define CAP_TRAIN() GridCapScope cap_scope_(ctx, true)
 
 sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
   GUARD();
@@ -917,6 +941,7 @@ sr_status sr_get_params(sr_ctx* ctx, sr_model which, float* host_out, size_t n) 
 sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, int h, int w, uint8_t* hr_dev,
                    sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!lr_dev || !hr_dev || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer: bad args");
   cudaStream_t st = (cudaStream_t)stream;
   if (which == SR_BILINEAR) {
@@ -936,6 +961,7 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
                         const uint8_t* v_dev, int n, int h, int w, uint8_t* hy_dev, uint8_t* hu_dev, uint8_t* hv_dev,
                         sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!y_dev || !u_dev || !v_dev || !hy_dev || !hu_dev || !hv_dev || n < 1 || h < 2 || w < 2 || (h | w) & 1)
     return fail(ctx, SR_E_INVAL, "sr_infer_i420: bad args (h, w must be even)");
   cudaStream_t st = (cudaStream_t)stream;
@@ -955,6 +981,7 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
 
 static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_host, int n, int h, int w,
                                  uint8_t* hr_host, sr_stream stream, bool sync) {
+  CAP_INFER();
   if (!lr_host || !hr_host || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer_host: bad args");
   if (ctx->host_pending) {  // the staging buffers and chunk events are reused: finish the previous async call
     CK(cudaStreamSynchronize(ctx->copy_st));
@@ -1043,6 +1070,7 @@ sr_status sr_infer_host_wait(sr_ctx* ctx) {
 sr_status sr_infer_rows(sr_ctx* ctx, sr_model which, const uint8_t* lr_full_dev, int h, int w, int row0, int row1,
                         uint8_t* hr_full_dev, sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!lr_full_dev || !hr_full_dev || h < 1 || w < 1 || row0 < 0 || row1 > h || row0 >= row1)
     return fail(ctx, SR_E_INVAL, "sr_infer_rows: bad args");
   if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer_rows: bad model");
@@ -1058,17 +1086,20 @@ sr_status sr_infer_rows(sr_ctx* ctx, sr_model which, const uint8_t* lr_full_dev,
 sr_status sr_train_grad(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
                         sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   if (!lr_dev || !hr_dev || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_grad: bad args");
   return train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, (cudaStream_t)stream);
 }
 
 sr_status sr_train_apply(sr_ctx* ctx, float grad_scale, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   return train_apply(ctx, grad_scale, nullptr, (cudaStream_t)stream);
 }
 
 sr_status sr_train_apply_dev(sr_ctx* ctx, const float* grad_scale_dev, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   if (!grad_scale_dev) return fail(ctx, SR_E_INVAL, "sr_train_apply_dev: null scale");
   return train_apply(ctx, 1.0f, grad_scale_dev, (cudaStream_t)stream);
 }
@@ -1076,6 +1107,7 @@ sr_status sr_train_apply_dev(sr_ctx* ctx, const float* grad_scale_dev, sr_stream
 sr_status sr_train_step(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
                         sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   TRY(sr_train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, stream));
   const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
   return train_apply(ctx, 1.0f / w, nullptr, (cudaStream_t)stream);
@@ -1085,6 +1117,7 @@ sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev
                        const int64_t* arrival_ts, sr_stream stream) {
   (void)arrival_ts;
   GUARD();
+  CAP_TRAIN();
   if (!lr_dev || !hr_dev || n < 1 || pp < 1) return fail(ctx, SR_E_INVAL, "sr_pool_push: bad args");
   cudaStream_t st = (cudaStream_t)stream;
   const int s = ctx->s;
@@ -1112,6 +1145,7 @@ sr_status sr_pool_push_i420(sr_ctx* ctx, const uint8_t* y_dev, const uint8_t* u_
                             int w, const uint8_t* hr_dev, const int32_t* xy_dev, int n, int pp,
                             const int64_t* arrival_ts, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   if (!y_dev || !u_dev || !v_dev || !hr_dev || !xy_dev || n < 1 || pp < 1 || h < 2 || w < 2 || (h | w) & 1)
     return fail(ctx, SR_E_INVAL, "sr_pool_push_i420: bad args");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1131,6 +1165,7 @@ size_t sr_pool_size(const sr_ctx* ctx) {
 sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* lr_out_dev, uint8_t* hr_out_dev,
                           int32_t* idx_out_dev, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   if (!lr_out_dev || !hr_out_dev || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_sample_batch: bad args");
   if (ctx->pool_total == 0) return fail(ctx, SR_E_STATE, "sr_sample_batch: empty pool");
   if (p > ctx->pool_pp) return fail(ctx, SR_E_INVAL, "sr_sample_batch: p larger than pool patch");
@@ -1169,6 +1204,7 @@ sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* 
 
 sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss_dev, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   if (iters < 1 || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_sampled: bad args");
   if (ctx->opt.world != 1) return fail(ctx, SR_E_STATE, "sr_train_sampled: world > 1 needs the split API");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1214,6 +1250,7 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
 
 sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
   GUARD();
+  CAP_TRAIN();
   cudaStream_t st = (cudaStream_t)stream;
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wf, ctx->snap[SR_SERVE].wf, ctx->pk_total * sizeof(bf16),
                      cudaMemcpyDeviceToDevice, st));
@@ -1273,6 +1310,7 @@ static sr_status mean_psnr(sr_ctx* ctx, const sr_model* models, int k, const uin
 sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
                        int p, sr_quality* out_host, sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!lr_dev || !hr_dev || !out_host || n < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_psnr_gain: bad args");
   const sr_model ms[2] = {a, b};
   double q[2];
@@ -1287,6 +1325,7 @@ sr_status sr_psnr_gain(sr_ctx* ctx, sr_model a, sr_model b, const uint8_t* lr_de
 sr_status sr_patch_select(sr_ctx* ctx, const uint8_t* raw_dev, const uint8_t* dec_dev, int h, int w, int cell,
                           int max_sel, uint64_t seed, int64_t step, int32_t* xy_host, int* n_sel, sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!raw_dev || !dec_dev || !xy_host || !n_sel || h < 1 || w < 1 || cell < 1 || max_sel < 0)
     return fail(ctx, SR_E_INVAL, "sr_patch_select: bad args");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1370,6 +1409,7 @@ sr_status sr_controller_update(sr_controller* c, double diff, int* event_out) {
 sr_status sr_controller_step(sr_ctx* ctx, sr_controller* c, const uint8_t* lr_dev, const uint8_t* hr_dev, int n,
                              int p, sr_epoch_report* out_host, sr_stream stream) {
   GUARD();
+  CAP_INFER();
   if (!c || !lr_dev || !hr_dev || !out_host || n < 1 || p < 1)
     return fail(ctx, SR_E_INVAL, "sr_controller_step: bad args");
   if (c->state != SR_TRAINING && c->state != SR_SUSPENDED)

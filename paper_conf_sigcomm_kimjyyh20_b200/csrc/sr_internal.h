@@ -92,5 +92,7 @@ cudaError_t launch_wgrad_multi(const WgradJob* jobs, int J, int N, int H, int W,
                                unsigned* sync, int grid, long long* dbg, cudaStream_t st);
 
 int num_sms();
+void set_grid_cap(int cap);
+int grid_cap();
 
 }  // namespace sr

@@ -591,3 +591,26 @@ def test_two_rank_dp_step_matches_oracle():
     rp, _, _ = O.adam_step(p0, np.zeros_like(p0), np.zeros_like(p0), g, 1)
     assert rel_l2(pa, rp) < 1e-3
     assert rel_l2(total.cpu().numpy() / sum(w), g) < 1e-2
+
+
+def test_sm_split_grids():
+    """sr_set_sm_split sizes the persistent grids of inference-side and training-side calls for disjoint SM
+    shares: inference is bit-identical at any grid (every output row's MMA order is fixed by the row, not the CTA);
+    training at a 20-SM grid still matches the oracle (split-K grouping of the weight gradient changes)."""
+    s, B, C = 3, 2, 16
+    ctx = _ctx(s, B, C, seed=91)
+    lr, _ = synth_frames(2, 33, 272, seed=92, scale=s)
+    lrd = torch.from_numpy(lr).cuda()
+    a = ctx.infer(lrd, "serve").clone()
+    for k in (20, 100):
+        ctx.set_sm_split(k)
+        assert torch.equal(ctx.infer(lrd, "serve"), a)
+    ctx.set_sm_split(20)
+    lrp, hrp, _ = synth_patch_pool(6, s, s * 24, seed=93, frame_hw=(s * 24 * 3, s * 24 * 4))
+    lo = torch.zeros(1, device="cuda")
+    ctx.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo)
+    g = ctx.grad_buffer().cpu().numpy().copy()
+    ref_loss, ref_g = O.train_loss_and_grad(ctx.get_params("train"), lrp, hrp, s, B, C)
+    assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
+    assert rel_l2(g, ref_g) < 1e-2
+    ctx.set_sm_split(0)
