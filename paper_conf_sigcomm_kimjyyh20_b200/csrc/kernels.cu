@@ -233,17 +233,7 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 
 // --------------------------------------------------------------- fused Adam (PyTorch semantics)
 // m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;  p -= (lr / bc1) * m / (sqrt(v) / sqrt(bc2) + eps),  g = s * grad
-// t and the bias corrections live on the device (k_adam_prep) so the step is replayable from a CUDA graph.
-__global__ void k_adam_prep(long long* counters, float* scal, double lr, double b1, double b2) {
-  pdl_enter();
-  const long long t = ++counters[1];
-  scal[0] = (float)(lr / (1.0 - pow(b1, (double)t)));
-  scal[1] = (float)(1.0 / sqrt(1.0 - pow(b2, (double)t)));
-}
-
-void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st) {
-  launch_k(k_adam_prep, dim3(1), dim3(1), 0, st, counters, scal, lr, b1, b2);
-}
+// t lives on the device (counters[1]) so the step is replayable from a CUDA graph.
 
 // k_adam computes the bias corrections itself from the device step counter: t = counters[1] + 1 (the counter is
 // advanced by the TRAIN repack that follows, k_pack_weights' bump) -- one launch less per training iteration.

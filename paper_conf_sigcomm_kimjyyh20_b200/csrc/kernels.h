@@ -60,7 +60,6 @@ cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf1
                             const bf16* mask = nullptr, const bf16* res2 = nullptr);
 // Device-side step counters (so a training iteration can be captured once in a CUDA graph and replayed):
 // counters[0] = sampler step, counters[1] = Adam step t; scal[0] = lr / (1 - b1^t), scal[1] = 1/sqrt(1 - b2^t).
-void launch_adam_prep(long long* counters, float* scal, double lr, double b1, double b2, cudaStream_t st);
 void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
                  const long long* counters, double lr, float b1, float b2, float eps, cudaStream_t st);
 void launch_counter_add(long long* counter, long long delta, cudaStream_t st);

@@ -51,7 +51,6 @@ struct sr_ctx {
   unsigned* wg_sync = nullptr; // wgrad grid barrier {count, generation}
   double* loss_sum = nullptr;
   long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t
-  float* adam_scal = nullptr;     // device: lr/bc1, 1/sqrt(bc2)
   float* zero_bias = nullptr;     // device: 64 zeros (the bias of the data-gradient convs)
   // patch pool (device ring)
   uint8_t *pool_lr = nullptr, *pool_hr = nullptr;
@@ -756,7 +755,6 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->wdo_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
   al(&ctx->counters, 2);
-  al(&ctx->adam_scal, 2);
   al(&ctx->zero_bias, 64);
   if (st == SR_OK && cudaMemset(ctx->zero_bias, 0, 64 * sizeof(float)) != cudaSuccess) st = SR_E_CUDA;
   ctx->tf.assign(blocks + 1, nullptr);
@@ -795,7 +793,7 @@ void sr_destroy(sr_ctx* ctx) {
   void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->x16, ctx->f0,
                   ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
-                  ctx->adam_scal, ctx->zero_bias, ctx->pool_lr,
+                  ctx->zero_bias, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf, ctx->cell_sse};
   for (void* p : ptrs)
     if (p) cudaFree(p);
