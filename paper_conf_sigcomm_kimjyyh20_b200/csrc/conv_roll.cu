@@ -77,6 +77,14 @@ struct RollArgs {
   // Otherwise every lane reads its 3x3 (5x5) LR neighbourhood and writes its S x S x 3 bytes from/to global.
   int tail_tma;
   int w_early;  // weights / bias may be fetched before the PDL wait (see the kernel prologue)
+  // training tail (TS > 0, train = 1): o = PS(y) + skip/255 against hr_ref, loss += (o - t)^2 (L1: |o - t|) into
+  // *loss_sum, dy = 2 (o - t) (L1: sign) as a bf16 row per pixel; vsep > 0: virtual batch of vp x vp patches at
+  // columns [j vsep + 1, j vsep + 1 + vp), separator columns get dy = 0 and no loss
+  int train;
+  const uint8_t* hr_ref;
+  bf16* dy;
+  double* loss_sum;
+  int vsep, vp, l1;
 };
 #define SR_RDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -391,6 +399,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     for (int b = grp; b < RB; b += 2)  // this group's ring blocks start free (RB is even; the MMA issuer arms)
       if (lane_id() == 0) mbar_arrive(&r_free[b]);
     int os = 0;
+    float tr_lsum = 0.f;  // training tail: this thread's loss partial
     long long G = 0, emitted = 0;  // emitted: output rows of both groups so far (aux ring order)
     SR_PIECE_BEGIN
     const int xc = x0 + m;
@@ -420,6 +429,35 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       if (warp == 2 && lane_id() == 0) { SR_RDBG(6, q + 1) }
       if (!emit) continue;
       if constexpr (TS > 0) {  // up conv: the tail straight from registers (the ring held the bias)
+        if (a.train) {  // training tail: loss partial + dy row (same arithmetic as the tiled EPI_TAIL_TRAIN)
+          if (lane_ok) {
+            EpiParams ep{};
+            ep.scale = TS;
+            ep.lr = a.lr;
+            ep.hr_ref = a.hr_ref;
+            ep.dy = a.dy;
+            ep.l1 = a.l1;
+            ep.bicubic = a.bicubic;
+            float vv[COUTP];  // a copy: epi_tail may pass it to a non-inlined call (keeps v in registers)
+#pragma unroll
+            for (int k = 0; k < COUTP; ++k) vv[k] = v[k];
+            const size_t vpix = ((size_t)n * H + r) * W + xc;
+            if (a.vsep > 0) {
+              const int j = xc / a.vsep, x = xc - j * a.vsep - 1;
+              if (x < 0 || x >= a.vp) {
+                float z[COUTP];
+#pragma unroll
+                for (int k = 0; k < COUTP; ++k) z[k] = 0.f;
+                store_bf16_row<COUTP>(a.dy + vpix * COUTP, z);
+              } else {
+                epi_tail<TS, COUTP, true>(ep, nullptr, j, r, x, a.vp, a.vp, vv, tr_lsum, vpix);
+              }
+            } else {
+              epi_tail<TS, COUTP, true>(ep, nullptr, n, r, xc, H, W, vv, tr_lsum, vpix);
+            }
+          }
+          continue;
+        }
         if (a.tail_tma) {  // LR rows from the TMA ring, HR rows staged for the store warp
           constexpr int NLR = TS > 0 ? Cfg::NLR : 1;
           mbar_wait(&l_full[xi % NLR], (uint32_t)(xi / NLR) & 1u);
@@ -483,6 +521,11 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     }
     G += n_in + 2;
     SR_PIECE_END
+    if (TS > 0 && a.train) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) tr_lsum += __shfl_xor_sync(0xffffffffu, tr_lsum, o);
+      if (lane_id() == 0) atomicAdd(a.loss_sum, (double)tr_lsum);
+    }
   }
 #undef SR_PIECE_BEGIN
 #undef SR_PIECE_END
@@ -587,6 +630,31 @@ cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, co
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
+  SR_ROLL_TAIL_CASE(16, 16, 2) SR_ROLL_TAIL_CASE(32, 16, 2) SR_ROLL_TAIL_CASE(48, 16, 2) SR_ROLL_TAIL_CASE(64, 16, 2)
+  SR_ROLL_TAIL_CASE(16, 32, 3) SR_ROLL_TAIL_CASE(32, 32, 3) SR_ROLL_TAIL_CASE(48, 32, 3) SR_ROLL_TAIL_CASE(64, 32, 3)
+  SR_ROLL_TAIL_CASE(16, 48, 4) SR_ROLL_TAIL_CASE(32, 48, 4) SR_ROLL_TAIL_CASE(48, 48, 4) SR_ROLL_TAIL_CASE(64, 48, 4)
+  return cudaErrorNotSupported;
+}
+
+cudaError_t launch_conv_roll_tail_train(int cinp, int coutp, int s, const void* in, const bf16* wfold,
+                                        const float* bias, const uint8_t* lr, const uint8_t* hr_ref, bf16* dy,
+                                        double* loss_sum, int vsep, int vp, int l1, int bicubic, int N, int H, int W,
+                                        cudaStream_t st, int w_early) {
+  CUtensorMap ti;
+  if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
+    return cudaErrorInvalidValue;
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, lr, nullptr, 0, H, bicubic, 0, w_early};
+  a.train = 1;
+  a.hr_ref = hr_ref;
+  a.dy = dy;
+  a.loss_sum = loss_sum;
+  a.vsep = vsep;
+  a.vp = vp;
+  a.l1 = l1;
+  const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  CUtensorMap tl = ti, th = ti;
   SR_ROLL_TAIL_CASE(16, 16, 2) SR_ROLL_TAIL_CASE(32, 16, 2) SR_ROLL_TAIL_CASE(48, 16, 2) SR_ROLL_TAIL_CASE(64, 16, 2)
   SR_ROLL_TAIL_CASE(16, 32, 3) SR_ROLL_TAIL_CASE(32, 32, 3) SR_ROLL_TAIL_CASE(48, 32, 3) SR_ROLL_TAIL_CASE(64, 32, 3)
   SR_ROLL_TAIL_CASE(16, 48, 4) SR_ROLL_TAIL_CASE(32, 48, 4) SR_ROLL_TAIL_CASE(48, 48, 4) SR_ROLL_TAIL_CASE(64, 48, 4)

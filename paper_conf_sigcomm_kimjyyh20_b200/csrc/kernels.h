@@ -53,6 +53,11 @@ cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const 
 bool roll_head_u8_supported(int coutp, int W, const void* lr);
 cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* wfold, const float* bias, bf16* out,
                                      int N, int H, int W, cudaStream_t st, int w_early);
+// rolling up conv + training tail (loss partial into *loss_sum, dy rows; vsep > 0: virtual patch batch)
+cudaError_t launch_conv_roll_tail_train(int cinp, int coutp, int s, const void* in, const bf16* wfold,
+                                        const float* bias, const uint8_t* lr, const uint8_t* hr_ref, bf16* dy,
+                                        double* loss_sum, int vsep, int vp, int l1, int bicubic, int N, int H, int W,
+                                        cudaStream_t st, int w_early);
 bool resblock_supported(int cp, int W);
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                             const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,

@@ -527,7 +527,20 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
     e.bicubic = ctx->opt.skip == 1;
     e.vsep = sep;
     e.vp = p;
-    TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, e, st));
+    if (ctx->roll_tail && roll_supported(Cp, OUTP, Wv)) {  // rolling up conv with the training tail epilogue
+      if (ctx->timing) {
+        const double px = (double)Hv * Wv;
+        tmark_begin(ctx, "conv_tail_train_roll_" + std::to_string(Cp) + "x" + std::to_string(OUTP),
+                    2.0 * 9 * Cp * OUTP * px, px * (2.0 * Cp + 2.0 * OUTP), st);
+      }
+      cudaError_t er = launch_conv_roll_tail_train(Cp, OUTP, ctx->s, ctx->tg, WO(cu), Bv(cu), lr, hr, ctx->tdy,
+                                                   ctx->loss_sum, sep, p, e.l1, e.bicubic, 1, Hv, Wv, st, 1);
+      tmark_end(ctx, st);
+      ctx->launches++;
+      if (er != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll train tail: ") + cudaGetErrorString(er));
+    } else {
+      TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, e, st));
+    }
   }
   const double n_el = (double)n * p * p * ctx->s * ctx->s * 3;
   if (loss_dev) {

@@ -614,3 +614,20 @@ def test_sm_split_grids():
     assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
     assert rel_l2(g, ref_g) < 1e-2
     ctx.set_sm_split(0)
+
+
+@pytest.mark.parametrize("cfg,loss", [((3, 2, 48), "mse"), ((2, 2, 16), "l1"), ((4, 1, 16), "mse")])
+def test_rolling_training_tail_equals_tiled(cfg, loss):
+    """Training tail on the rolling kernel (default for the virtual batch) vs the tiled EPI_TAIL_TRAIN kernel
+    (set_fusion bit 2): same math, different fp32 order of the up-conv sums -> loss and gradients agree closely."""
+    s, B, C = cfg
+    lrp, hrp, _ = synth_patch_pool(5, s, s * 24, seed=95, frame_hw=(s * 24 * 3, s * 24 * 4))
+    out = []
+    for fusion in (1, 1 | 4):
+        ctx = _ctx(s, B, C, seed=96, loss=loss)
+        ctx.set_fusion(fusion)
+        lo = torch.zeros(1, device="cuda")
+        ctx.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo)
+        out.append((lo.item(), ctx.grad_buffer().cpu().numpy().copy()))
+    assert abs(out[0][0] - out[1][0]) <= 1e-4 * abs(out[1][0])
+    assert rel_l2(out[0][1], out[1][1]) < 2e-3
