@@ -315,18 +315,34 @@ __global__ void k_sample_gather(SampleArgs a) {
   __syncthreads();
   const int slot = s_slot, oy = s_oy, ox = s_ox;
   const int p = a.p, pp = a.pp, s = a.scale;
-  const int rb = 3 * p;  // bytes per LR crop row
-  const uint8_t* src = a.lr_pool + (size_t)slot * pp * pp * 3;
-  uint8_t* dst = a.lr_out + (size_t)j * p * p * 3;
-  for (int r = blockIdx.y; r < p; r += gridDim.y)
-    for (int c = threadIdx.x; c < rb; c += blockDim.x)
-      dst[r * rb + c] = src[((size_t)(oy + r) * pp + ox) * 3 + c];
-  const int sp = s * p, spp = s * pp, hb = 3 * sp;
-  const uint8_t* hsrc = a.hr_pool + (size_t)slot * spp * spp * 3;
-  uint8_t* hdst = a.hr_out + (size_t)j * sp * sp * 3;
-  for (int r = blockIdx.y; r < sp; r += gridDim.y)
-    for (int c = threadIdx.x; c < hb; c += blockDim.x)
-      hdst[r * hb + c] = hsrc[((size_t)(s * oy + r) * spp + s * ox) * 3 + c];
+  // Crop copies: one warp per crop row (rows r = part, part + gridDim.y, ... of this block, warps round-robin);
+  // the lanes issue all of a row's byte loads (coalesced, up to 16 per lane) before its stores, so the load
+  // latencies overlap instead of one load-store round trip per byte.
+  auto copy_rows = [&](const uint8_t* __restrict__ src, uint8_t* __restrict__ dst, int rows, int rowb, int src_pitch,
+                       int src_x0b, int src_y0) {
+    const int lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    for (int r = (int)blockIdx.y + (int)(threadIdx.x >> 5) * (int)gridDim.y; r < rows; r += nw * (int)gridDim.y) {
+      const uint8_t* __restrict__ sr = src + (size_t)(src_y0 + r) * src_pitch + src_x0b;
+      uint8_t* __restrict__ dr = dst + (size_t)r * rowb;
+      for (int c0 = 0; c0 < rowb; c0 += 32 * 16) {
+        uint8_t v[16];
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+          const int c = c0 + 32 * k + lane;
+          if (c < rowb) v[k] = __ldg(sr + c);
+        }
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+          const int c = c0 + 32 * k + lane;
+          if (c < rowb) dr[c] = v[k];
+        }
+      }
+    }
+  };
+  copy_rows(a.lr_pool + (size_t)slot * pp * pp * 3, a.lr_out + (size_t)j * p * p * 3, p, 3 * p, 3 * pp, 3 * ox, oy);
+  const int sp = s * p, spp = s * pp;
+  copy_rows(a.hr_pool + (size_t)slot * spp * spp * 3, a.hr_out + (size_t)j * sp * sp * 3, sp, 3 * sp, 3 * spp,
+            3 * s * ox, s * oy);
 }
 
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st) {
