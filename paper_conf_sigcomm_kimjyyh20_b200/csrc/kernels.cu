@@ -185,7 +185,7 @@ __global__ void k_pack_weights(const float* __restrict__ params, const ConvDesc*
   const float* W = params + d.w_off;
   const int tot = 9 * d.cinp * d.coutp;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < tot; i += gridDim.x * blockDim.x) {
-    {  // fwd element i = ((t * cinp/8 + j) * coutp + co) * 8 + e
+    if (wf) {  // fwd element i = ((t * cinp/8 + j) * coutp + co) * 8 + e
       int e = i & 7, r = i >> 3;
       int co = r % d.coutp; r /= d.coutp;
       int j = r % (d.cinp / 8), t = r / (d.cinp / 8);

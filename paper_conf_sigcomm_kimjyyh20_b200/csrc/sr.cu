@@ -82,6 +82,7 @@ struct sr_ctx {
   bool fuse_bodytail = true;  // body conv + up conv + tail as one kernel, g in smem (sr_set_fusion bit 5 clears)
   bool fuse_head = true;      // head conv reads the u8 frame directly (sr_set_fusion bit 6 clears)
   int sm_train = 0;           // sr_set_sm_split: SMs given to the training kernels (0 = all SMs to every call)
+  bool train_fold_only = false;  // TRAIN's tiled layouts (wf, wd) may be stale: rebuild before reading them
   int sm_total = 0;
   struct TRec { std::string cls; cudaEvent_t a, b; double flops, bytes; };
   std::vector<TRec> trec;
@@ -125,12 +126,18 @@ static uint64_t mix64h(uint64_t z) {
   return z ^ (z >> 31);
 }
 
-static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st, long long* bump = nullptr) {
-  launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, ctx->snap[which].wf,
-                      with_dgrad ? ctx->wd_train : nullptr, ctx->snap[which].wo,
+static sr_status repack(sr_ctx* ctx, int which, bool with_dgrad, cudaStream_t st, long long* bump = nullptr,
+                        bool fold_only = false) {
+  launch_pack_weights(ctx->params, ctx->convs_dev, ctx->nconv, ctx->max_pk, fold_only ? nullptr : ctx->snap[which].wf,
+                      (with_dgrad && !fold_only) ? ctx->wd_train : nullptr, ctx->snap[which].wo,
                       with_dgrad ? ctx->wdo_train : nullptr, ctx->snap[which].bias, st, bump);
   ctx->launches++;
   CKL();
+  return SR_OK;
+}
+
+static sr_status ensure_full_train_pack(sr_ctx* ctx, cudaStream_t st) {
+  if (ctx->train_fold_only) return repack(ctx, SR_TRAIN, true, st);
   return SR_OK;
 }
 
@@ -304,6 +311,7 @@ static sr_status ensure_infer_ws(sr_ctx* ctx, size_t pix) {
 // g = f0 + body(f); tail(up(g)) -> u8 with pixel shuffle + bilinear skip + clamp + RNE.
 static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
                                uint8_t* hr, int row0, int row1, cudaStream_t st) {
+  if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const size_t pix = (size_t)n * h * w;
   TRY(ensure_infer_ws(ctx, pix));
   const int Cp = ctx->Cp;
@@ -415,6 +423,7 @@ static bool use_virtual_infer(const sr_ctx* ctx, int n, int h, int w) {
 
 static sr_status forward_infer_virtual(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int p,
                                        uint8_t* hr, cudaStream_t st) {
+  if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const int Hv = p, Wv = n * (p + 2), sep = p + 2;
   TRY(ensure_infer_ws(ctx, (size_t)Hv * Wv));
   const int Cp = ctx->Cp;
@@ -539,6 +548,7 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
       ctx->launches++;
       if (er != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll train tail: ") + cudaGetErrorString(er));
     } else {
+      TRY(ensure_full_train_pack(ctx, st));  // the tiled tail reads TRAIN's tiled layout
       TRY(conv(ctx, Cp, OUTP, EPI_TAIL_TRAIN, ctx->tg, sn.wf + ctx->convs[cu].pk_off, 1, Hv, Wv, e, st));
     }
   }
@@ -593,6 +603,7 @@ static sr_status train_grad(sr_ctx* ctx, const uint8_t* lr, const uint8_t* hr, i
                             cudaStream_t st) {
   if (ctx->virtual_train && roll_supported(ctx->OUTP, ctx->Cp, n * (p + 2)) && roll_supported(16, ctx->Cp, n * (p + 2)))
     return train_grad_virtual(ctx, lr, hr, n, p, loss_dev, st);
+  TRY(ensure_full_train_pack(ctx, st));
   const size_t pix = (size_t)n * p * p;
   TRY(ensure_train_ws(ctx, pix));
   const int Cp = ctx->Cp, B = ctx->B, OUTP = ctx->OUTP;
@@ -693,7 +704,11 @@ static sr_status train_apply(sr_ctx* ctx, float grad_scale, const float* grad_sc
               ctx->opt.lr, ctx->opt.beta1, ctx->opt.beta2, ctx->opt.eps, st);
   ctx->launches += 1;
   CKL();
-  return repack(ctx, SR_TRAIN, true, st, ctx->counters + 1);  // the repack advances the Adam step counter
+  // The per-step repack writes only the dy-fold layouts the wide (virtual-batch) path reads; the tiled layouts of
+  // TRAIN are rebuilt on demand (ensure_full_train_pack) by the calls that read them.  The flag is sticky: graph
+  // replays of this step do not pass through the host.
+  if (ctx->virtual_train) ctx->train_fold_only = true;
+  return repack(ctx, SR_TRAIN, true, st, ctx->counters + 1, ctx->virtual_train);  // + Adam step counter
 }
 
 static bool valid_model(sr_model m) { return m >= SR_TRAIN && m <= SR_INIT; }
@@ -1263,6 +1278,7 @@ sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
   GUARD();
   CAP_TRAIN();
   cudaStream_t st = (cudaStream_t)stream;
+  TRY(ensure_full_train_pack(ctx, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wf, ctx->snap[SR_SERVE].wf, ctx->pk_total * sizeof(bf16),
                      cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].bias, ctx->snap[SR_SERVE].bias, ctx->b_total * sizeof(float),

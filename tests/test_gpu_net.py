@@ -631,3 +631,28 @@ def test_rolling_training_tail_equals_tiled(cfg, loss):
         out.append((lo.item(), ctx.grad_buffer().cpu().numpy().copy()))
     assert abs(out[0][0] - out[1][0]) <= 1e-4 * abs(out[1][0])
     assert rel_l2(out[0][1], out[1][1]) < 2e-3
+
+
+def test_tiled_layouts_follow_fold_only_training_steps():
+    """Virtual-batch training steps repack only the dy-fold weight layouts; publish, TRAIN-snapshot inference and the
+    narrow training path rebuild the tiled layouts first -- their results equal a fresh context holding the same
+    fp32 parameters (narrow frames use the tiled kernels)."""
+    s, B, C = 2, 2, 16
+    ctx = _ctx(s, B, C, seed=101)
+    lrp, hrp, _ = synth_patch_pool(6, s, s * 24, seed=102, frame_hw=(s * 24 * 3, s * 24 * 4))
+    for _ in range(2):
+        ctx.train_step(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda())
+    p = ctx.get_params("train")
+    fresh = _ctx(s, B, C, seed=5)
+    fresh.set_params(p)
+    small = torch.from_numpy(synth_frames(1, 24, 40, seed=103)).cuda()  # W < 96: tiled kernels
+    assert torch.equal(ctx.infer(small, "train"), fresh.infer(small, "serve"))
+    ctx.publish()
+    assert torch.equal(ctx.infer(small, "serve"), fresh.infer(small, "serve"))
+    for c in (ctx, fresh):
+        c.set_fusion(1 | 2)  # narrow (per-patch) training path: tiled forward and data-gradient layouts
+    lo1, lo2 = torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    ctx.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo1)
+    g1 = ctx.grad_buffer().clone()
+    fresh.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo2)
+    assert torch.equal(g1, fresh.grad_buffer()) and lo1.item() == lo2.item()
