@@ -343,6 +343,18 @@ __global__ void k_sample_gather(SampleArgs a) {
   const int sp = s * p, spp = s * pp;
   copy_rows(a.hr_pool + (size_t)slot * spp * spp * 3, a.hr_out + (size_t)j * sp * sp * 3, sp, 3 * sp, 3 * spp,
             3 * s * ox, s * oy);
+  if (a.step_bump) {  // every block read the step before arriving: the last arrival advances it for the next draw
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      const unsigned nb = gridDim.x * gridDim.y;
+      if (atomicAdd(a.done, 1u) == nb - 1) {
+        *a.step_bump += 1;
+        *a.done = 0u;
+        __threadfence();
+      }
+    }
+  }
 }
 
 void launch_sample_gather(const SampleArgs& a, int batch, cudaStream_t st) {

@@ -24,6 +24,9 @@ struct SampleArgs {
   uint8_t* lr_out;
   uint8_t* hr_out;
   int32_t* idx_out;
+  // device step mode: the last block to finish advances *step_dev (done = its block counter, reset by that block)
+  long long* step_bump;
+  unsigned* done;
 };
 
 void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st);

@@ -782,7 +782,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->wd_train, ctx->pk_total);
   al(&ctx->wdo_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
-  al(&ctx->counters, 2);
+  al(&ctx->counters, 3);  // [0] sampler step, [1] Adam t, [2] gather block counter
   al(&ctx->zero_bias, 64);
   if (st == SR_OK && cudaMemset(ctx->zero_bias, 0, 64 * sizeof(float)) != cudaSuccess) st = SR_E_CUDA;
   ctx->tf.assign(blocks + 1, nullptr);
@@ -927,7 +927,7 @@ sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
   CK(cudaMemset(ctx->m, 0, n * sizeof(float)));
   CK(cudaMemset(ctx->v, 0, n * sizeof(float)));
   CK(cudaMemset(ctx->grad, 0, n * sizeof(float)));
-  CK(cudaMemset(ctx->counters, 0, 2 * sizeof(long long)));
+  CK(cudaMemset(ctx->counters, 0, 3 * sizeof(long long)));
   ctx->t = 0;
   TRY(repack(ctx, SR_TRAIN, true, 0));
   for (int k = 1; k < 4; ++k) {
@@ -1218,12 +1218,12 @@ sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* 
   a.lr_out = lr_out_dev;
   a.hr_out = hr_out_dev;
   a.idx_out = idx_out_dev;
+  if (step < 0) {  // graph mode: the gather's last block advances the device-side sampler step
+    a.step_bump = ctx->counters;
+    a.done = reinterpret_cast<unsigned*>(ctx->counters + 2);
+  }
   launch_sample_gather(a, batch, (cudaStream_t)stream);
   ctx->launches++;
-  if (step < 0) {  // graph mode: advance the device-side sampler step
-    launch_counter_add(ctx->counters, 1, (cudaStream_t)stream);
-    ctx->launches++;
-  }
   CKL();
   return SR_OK;
 }

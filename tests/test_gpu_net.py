@@ -197,6 +197,11 @@ def test_sampler_gather_bitexact():
         rl, rh = O.gather_patches(lrp, hrp, ridx, oy, ox, 48, s)
         np.testing.assert_array_equal(lr.cpu().numpy(), rl)
         np.testing.assert_array_equal(hr.cpu().numpy(), rh)
+    # device step counter (graph mode): consecutive step = -1 calls draw steps 0, 1, 2 (the gather's last block
+    # advances the counter)
+    for step in range(3):
+        _, _, idx = ctx.sample_batch(-1, 64, 48)
+        np.testing.assert_array_equal(idx.cpu().numpy(), O.sample_indices(77, step, 300, 64, 60, 48)[0])
 
 
 def test_psnr_gain_matches_oracle():
