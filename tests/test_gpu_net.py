@@ -107,7 +107,7 @@ def _oracle_pixel(p, lr_frame, s, B, C, y, x):
 
 
 @pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (720, 1280), 2), ((2, 8, 32), (540, 960), 2),
-                                      ((4, 8, 48), (270, 480), 2)])
+                                      ((4, 8, 48), (270, 480), 2), ((2, 8, 48), (1080, 1920), 1)])
 def test_full_size_frames_sampled_parity(cfg, hw, n):
     """BASELINE frame sizes (config 3: 720p x3 8x48; config 2: 540p x2 8x32) in the bench's launch
     configuration; sampled output pixels (incl. corners and tile seams) against the oracle."""
