@@ -438,9 +438,6 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
             ep.dy = a.dy;
             ep.l1 = a.l1;
             ep.bicubic = a.bicubic;
-            float vv[COUTP];  // a copy: epi_tail may pass it to a non-inlined call (keeps v in registers)
-#pragma unroll
-            for (int k = 0; k < COUTP; ++k) vv[k] = v[k];
             const size_t vpix = ((size_t)n * H + r) * W + xc;
             if (a.vsep > 0) {
               const int j = xc / a.vsep, x = xc - j * a.vsep - 1;
@@ -450,10 +447,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
                 for (int k = 0; k < COUTP; ++k) z[k] = 0.f;
                 store_bf16_row<COUTP>(a.dy + vpix * COUTP, z);
               } else {
-                epi_tail<TS, COUTP, true>(ep, nullptr, j, r, x, a.vp, a.vp, vv, tr_lsum, vpix);
+                epi_tail<TS, COUTP, true>(ep, nullptr, j, r, x, a.vp, a.vp, v, tr_lsum, vpix);
               }
             } else {
-              epi_tail<TS, COUTP, true>(ep, nullptr, n, r, xc, H, W, vv, tr_lsum, vpix);
+              epi_tail<TS, COUTP, true>(ep, nullptr, n, r, xc, H, W, v, tr_lsum, vpix);
             }
           }
           continue;
@@ -480,10 +477,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
           ep.lr = a.lr;
           ep.hr = a.hr;
           ep.bicubic = a.bicubic;
-          float ls = 0.f, vv[COUTP];  // a copy: epi_tail may pass it to a non-inlined call (keeps v in registers)
-#pragma unroll
-          for (int k = 0; k < COUTP; ++k) vv[k] = v[k];
-          epi_tail<TS, COUTP, false>(ep, nullptr, n, r, xc, H, W, vv, ls, 0);
+          float ls = 0.f;
+          epi_tail<TS, COUTP, false>(ep, nullptr, n, r, xc, H, W, v, ls, 0);
         }
         continue;
       }

@@ -160,8 +160,11 @@ __device__ __noinline__ void epi_tail_bicubic(const EpiParams& ep, const float* 
 template <int S, int COUTP, bool TRAIN>
 __device__ __forceinline__ void epi_tail(const EpiParams& ep, const float* sbias, int n, int Y, int X, int H,
                                          int W, float* v, float& lsum, size_t dy_pix) {
-  if (ep.bicubic) {
-    epi_tail_bicubic<S, COUTP, TRAIN>(ep, sbias, n, Y, X, H, W, v, lsum, dy_pix);
+  if (ep.bicubic) {  // a copy goes to the non-inlined variant, so v itself never escapes (stays in registers)
+    float vb[COUTP];
+#pragma unroll
+    for (int k = 0; k < COUTP; ++k) vb[k] = v[k];
+    epi_tail_bicubic<S, COUTP, TRAIN>(ep, sbias, n, Y, X, H, W, vb, lsum, dy_pix);
     return;
   }
   const uint8_t* lr = ep.lr + (size_t)n * H * W * 3;
