@@ -153,7 +153,7 @@ __device__ __forceinline__ void roll_stage(uint4* orow, const float* v, const ui
 static constexpr int kU8Slots = 8;
 static constexpr uint32_t kU8Slot = 512;  // 26 chunks = 416 B per u8 row
 template <int CINP, int COUTP, int TS, bool U8 = false>
-__global__ void __launch_bounds__(kRollThreads + (U8 ? 32 : 0), 1)
+__global__ void __launch_bounds__(kRollThreads + (U8 ? 64 : 0), 1)
 k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
             const __grid_constant__ CUtensorMap tm_aux, const bf16* __restrict__ wfold, const RollArgs a) {
   using Cfg = RollCfg<CINP, COUTP>;
@@ -308,13 +308,19 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       SR_PIECE_END
     }
     __syncwarp();
-  } else if (U8 && warp == 11) {
-    // ===================== u8 -> bf16 A-operand expansion (head conv) =====================
+  } else if (U8 && warp >= 11) {
+    // ===================== u8 -> bf16 A-operand expansion (head conv): warps 11, 12 take alternate rows ==========
     int s = 0, us = 0;
     uint32_t ph = 0, uph = 0;
+    long long rowc = 0;  // rows seen so far (both warps count every row; each converts its parity)
     SR_PIECE_BEGIN
     const int lbase = 16 * ((3 * x0 - 3) >> 4);
-    for (int i = 0; i < n_in; ++i) {
+    for (int i = 0; i < n_in; ++i, ++rowc) {
+      if ((int)(rowc & 1) != warp - 11) {
+        if (++us == kU8Slots) { us = 0; uph ^= 1; }
+        if (++s == kRollIn) { s = 0; ph ^= 1; }
+        continue;
+      }
       mbar_wait(&u_full[us], uph);
       mbar_wait(&in_empty[s], ph ^ 1);
       const uint32_t src = smem_u32(sA + us * kU8Slot) + (uint32_t)(3 * (x0 - 1) - lbase);
@@ -544,7 +550,7 @@ static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, c
       if (e != cudaSuccess) return e;
       configured = true;
     }
-    return launch_k(kern, dim3(grid), dim3(kRollThreads + (U8 ? 32 : 0)), smem, st, ti, to, tx, wfold, a);
+    return launch_k(kern, dim3(grid), dim3(kRollThreads + (U8 ? 64 : 0)), smem, st, ti, to, tx, wfold, a);
   }
 }
 
