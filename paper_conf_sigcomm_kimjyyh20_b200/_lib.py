@@ -18,7 +18,7 @@ class sr_options(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("lr", C.c_float), ("beta1", C.c_float), ("beta2", C.c_float),
                 ("eps", C.c_float), ("recent_k", C.c_int), ("recent_w", C.c_int), ("world", C.c_int),
                 ("rank", C.c_int), ("dp_weight", C.c_float), ("pool_capacity", C.c_int), ("loss", C.c_int),
-                ("skip", C.c_int)]
+                ("skip", C.c_int), ("device", C.c_int), ("nccl_id", C.c_void_p)]
 
 
 class sr_quality(C.Structure):
@@ -60,6 +60,11 @@ _SIGS = {
     "sr_grad_buffer": (_P, [_P]),
     "sr_train_apply": (_I, [_P, C.c_float, _P]),
     "sr_train_apply_dev": (_I, [_P, _P, _P]),
+    "sr_train_allreduce": (_I, [_P, _P]),
+    "sr_dp_weight_sum": (C.c_double, [_P]),
+    "sr_nccl_unique_id": (_I, [_P, C.c_size_t]),
+    "sr_get_adam_state": (_I, [_P, _P, _P, C.c_size_t, C.POINTER(C.c_int64)]),
+    "sr_pool_stats": (_I, [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
     "sr_pool_push": (_I, [_P, _P, _P, _I, _I, _P, _P]),
     "sr_pool_size": (C.c_size_t, [_P]),
     "sr_sample_batch": (_I, [_P, C.c_int64, _I, _I, _P, _P, _P, _P]),

@@ -78,13 +78,17 @@ __global__ void k_rgb_to_i420(const uint8_t* __restrict__ rgb, int n, int h, int
 }
 
 // LR counterparts of arriving HR patches (§5.2): pp x pp RGB crops of decoded frame 0 at LR top-left
-// xy[j] = (x, y); grid (n, pp), one thread per pixel of a crop row.
+// xy[j] = (x, y); grid (n, pp), one thread per pixel of a crop row.  The corners come from the ingest client, i.e.
+// they are external input: a crop that does not lie inside the frame is clamped into it (pp <= h, w is checked by
+// the host) and counted once in *rejected, so a bad corner can never read outside the planes.
 __global__ void k_i420_crop(const uint8_t* __restrict__ y, const uint8_t* __restrict__ u,
                             const uint8_t* __restrict__ v, int h, int w, const int32_t* __restrict__ xy, int pp,
-                            uint8_t* __restrict__ out) {
+                            uint8_t* __restrict__ out, unsigned long long* __restrict__ rejected) {
   pdl_enter();
   const int j = blockIdx.x, r = blockIdx.y;
-  const int x0 = xy[2 * j], y0 = xy[2 * j + 1];
+  const int xr = xy[2 * j], yr = xy[2 * j + 1];
+  const int x0 = min(max(xr, 0), w - pp), y0 = min(max(yr, 0), h - pp);
+  if ((x0 != xr || y0 != yr) && r == 0 && threadIdx.x == 0 && rejected) atomicAdd(rejected, 1ull);
   for (int c = threadIdx.x; c < pp; c += blockDim.x) {
     const int X = x0 + c, Y = y0 + r;
     const size_t ci = (size_t)(Y / 2) * (w / 2) + X / 2;
@@ -103,8 +107,8 @@ void launch_rgb_to_i420(const uint8_t* rgb, int n, int h, int w, uint8_t* y, uin
   launch_k(k_rgb_to_i420, dim3((unsigned)((tot + 255) / 256)), dim3(256), 0, st, rgb, n, h, w, y, u, v);
 }
 void launch_i420_crop(const uint8_t* y, const uint8_t* u, const uint8_t* v, int h, int w, const int32_t* xy, int n,
-                      int pp, uint8_t* out, cudaStream_t st) {
-  launch_k(k_i420_crop, dim3(n, pp), dim3(64), 0, st, y, u, v, h, w, xy, pp, out);
+                      int pp, uint8_t* out, unsigned long long* rejected, cudaStream_t st) {
+  launch_k(k_i420_crop, dim3(n, pp), dim3(64), 0, st, y, u, v, h, w, xy, pp, out, rejected);
 }
 
 // ------------------------------------------------------------------ per-cell integer SSE (patch selection)
@@ -300,7 +304,15 @@ __global__ void k_sample_gather(SampleArgs a) {
     const uint64_t u0 = mix64(a.seed + GAMMA * (base + 1));
     const uint64_t u1 = mix64(a.seed + GAMMA * (base + 2));
     const uint64_t u2 = mix64(a.seed + GAMMA * (base + 3));
-    const uint64_t n = (uint64_t)a.n_view;
+    long long n_view = a.n_view, view_base = a.view_base;
+    if (a.pool_total_dev) {  // the rank's arrival-order chunk of the pool as it is now (stream-ordered with pushes)
+      const long long tot = *a.pool_total_dev;
+      const long long avail = tot < a.capacity ? tot : a.capacity;
+      const long long lo = avail * a.rank / a.world, hi = avail * (a.rank + 1) / a.world;
+      n_view = hi - lo;
+      view_base = tot - avail + lo;
+    }
+    const uint64_t n = n_view > 0 ? (uint64_t)n_view : 1ull;
     const uint64_t kp = n < (uint64_t)a.recent_k ? n : (uint64_t)a.recent_k;
     const uint64_t Wt = (uint64_t)a.recent_w * kp + (n - kp);
     const uint64_t q = __umul64hi(u0, Wt);
@@ -308,9 +320,9 @@ __global__ void k_sample_gather(SampleArgs a) {
     const uint64_t span = (uint64_t)(a.pp - a.p + 1);
     s_oy = (int)__umul64hi(u1, span);
     s_ox = (int)__umul64hi(u2, span);
-    const int64_t arrival = a.view_base + (int64_t)idx;
-    s_slot = (int)(arrival % a.capacity);
-    if (a.idx_out && blockIdx.y == 0) a.idx_out[j] = (int32_t)idx;
+    const int64_t arrival = view_base + (int64_t)idx;
+    s_slot = n_view > 0 ? (int)(arrival % a.capacity) : -1;  // empty view: zero patches, index -1
+    if (a.idx_out && blockIdx.y == 0) a.idx_out[j] = n_view > 0 ? (int32_t)idx : -1;
   }
   __syncthreads();
   const int slot = s_slot, oy = s_oy, ox = s_ox;
@@ -339,10 +351,17 @@ __global__ void k_sample_gather(SampleArgs a) {
       }
     }
   };
-  copy_rows(a.lr_pool + (size_t)slot * pp * pp * 3, a.lr_out + (size_t)j * p * p * 3, p, 3 * p, 3 * pp, 3 * ox, oy);
   const int sp = s * p, spp = s * pp;
-  copy_rows(a.hr_pool + (size_t)slot * spp * spp * 3, a.hr_out + (size_t)j * sp * sp * 3, sp, 3 * sp, 3 * spp,
-            3 * s * ox, s * oy);
+  if (slot >= 0) {
+    copy_rows(a.lr_pool + (size_t)slot * pp * pp * 3, a.lr_out + (size_t)j * p * p * 3, p, 3 * p, 3 * pp, 3 * ox, oy);
+    copy_rows(a.hr_pool + (size_t)slot * spp * spp * 3, a.hr_out + (size_t)j * sp * sp * 3, sp, 3 * sp, 3 * spp,
+              3 * s * ox, s * oy);
+  } else {
+    for (int i = threadIdx.x + blockIdx.y * blockDim.x; i < 3 * p * p; i += blockDim.x * gridDim.y)
+      a.lr_out[(size_t)j * p * p * 3 + i] = 0;
+    for (int i = threadIdx.x + blockIdx.y * blockDim.x; i < 3 * sp * sp; i += blockDim.x * gridDim.y)
+      a.hr_out[(size_t)j * sp * sp * 3 + i] = 0;
+  }
   if (a.step_bump) {  // every block read the step before arriving: the last arrival advances it for the next draw
     __syncthreads();
     if (threadIdx.x == 0) {

@@ -17,6 +17,10 @@ struct SampleArgs {
   const long long* step_dev;
   int world, rank;
   long long n_view, view_base, capacity;
+  // non-null: the pool size is read on the device (arrivals counted by sr_pool_push's k_counter_add), and the rank's
+  // view [lo, hi) of the min(total, capacity) pooled patches is derived from it -- a captured graph then keeps seeing
+  // new arrivals; n_view / view_base are ignored
+  const long long* pool_total_dev;
   int recent_k, recent_w;
   int p, pp, scale;
   const uint8_t* lr_pool;
@@ -78,8 +82,9 @@ void launch_loss_finalize(const double* sum, double inv_n, float* out, cudaStrea
 void launch_i420_to_rgb(const uint8_t* y, const uint8_t* u, const uint8_t* v, int n, int h, int w, uint8_t* rgb,
                         cudaStream_t st);
 void launch_rgb_to_i420(const uint8_t* rgb, int n, int h, int w, uint8_t* y, uint8_t* u, uint8_t* v, cudaStream_t st);
+// out-of-frame corners are clamped into the frame (no out-of-bounds reads) and counted in *rejected
 void launch_i420_crop(const uint8_t* y, const uint8_t* u, const uint8_t* v, int h, int w, const int32_t* xy, int n,
-                      int pp, uint8_t* out, cudaStream_t st);
+                      int pp, uint8_t* out, unsigned long long* rejected, cudaStream_t st);
 void launch_cell_sse(const uint8_t* raw, const uint8_t* dec, int h, int w, int cell, unsigned long long* out,
                      cudaStream_t st);
 cudaError_t launch_bilinear_u8(const uint8_t* lr, int n, int h, int w, int s, uint8_t* hr, cudaStream_t st);

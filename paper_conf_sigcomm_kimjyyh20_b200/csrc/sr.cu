@@ -7,10 +7,44 @@
 #include <string>
 #include <vector>
 #include <algorithm>
+#include <dlfcn.h>
+#include <nccl.h>  // types only: libnccl is dlopen'ed at sr_create when world > 1 (libsr.so loads without it)
 #include "sr_internal.h"
 #include "kernels.h"
 
 using namespace sr;
+
+// ---------------------------------------------------------------------------------- NCCL (T5)
+// The data-parallel gradient exchange is one sum-allreduce of the flat fp32 gradient over NVLink/NVSwitch.  libnccl
+// is resolved at run time (SR_NCCL_LIB, else the soname "libnccl.so.2": the copy torch already loaded if any, else the
+// system one), so the library itself carries no link-time NCCL dependency.
+namespace {
+struct NcclApi {
+  bool tried = false, ok = false;
+  std::string why;
+  decltype(&ncclGetUniqueId) get_id = nullptr;
+  decltype(&ncclCommInitRank) init_rank = nullptr;
+  decltype(&ncclAllReduce) all_reduce = nullptr;
+  decltype(&ncclCommDestroy) destroy = nullptr;
+  decltype(&ncclGetErrorString) err = nullptr;
+};
+NcclApi& nccl() {
+  static NcclApi a;
+  if (a.tried) return a;
+  a.tried = true;
+  const char* path = std::getenv("SR_NCCL_LIB");
+  void* h = dlopen(path && path[0] ? path : "libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) { a.why = std::string("dlopen libnccl: ") + dlerror(); return a; }
+  a.get_id = (decltype(a.get_id))dlsym(h, "ncclGetUniqueId");
+  a.init_rank = (decltype(a.init_rank))dlsym(h, "ncclCommInitRank");
+  a.all_reduce = (decltype(a.all_reduce))dlsym(h, "ncclAllReduce");
+  a.destroy = (decltype(a.destroy))dlsym(h, "ncclCommDestroy");
+  a.err = (decltype(a.err))dlsym(h, "ncclGetErrorString");
+  a.ok = a.get_id && a.init_rank && a.all_reduce && a.destroy && a.err;
+  if (!a.ok) a.why = "libnccl lacks ncclGetUniqueId/ncclCommInitRank/ncclAllReduce/ncclCommDestroy";
+  return a;
+}
+}  // namespace
 
 struct Snapshot {
   bf16* wf = nullptr;    // packed fwd weights (all convs)
@@ -50,7 +84,8 @@ struct sr_ctx {
   size_t ws_w_elems = 0;
   unsigned* wg_sync = nullptr; // wgrad grid barrier {count, generation}
   double* loss_sum = nullptr;
-  long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t
+  long long* counters = nullptr;  // device: [0] sampler step (graph mode), [1] Adam t, [2] gather block counter,
+                                  // [3] pooled patches (arrivals), [4] i420 crops clamped into the frame
   float* zero_bias = nullptr;     // device: 64 zeros (the bias of the data-gradient convs)
   // patch pool (device ring)
   uint8_t *pool_lr = nullptr, *pool_hr = nullptr;
@@ -69,9 +104,20 @@ struct sr_ctx {
   unsigned long long* sse = nullptr;
   int sse_n = 0;
   cudaEvent_t publish_ev = nullptr;
-  // CUDA graph of one sampled training iteration (sample -> fwd/bwd -> Adam), per (batch, p)
+  // CUDA graph of one sampled training iteration (sample -> fwd/bwd -> [allreduce] -> Adam), per (batch, p); re-captured
+  // when the loss pointer or any workspace it references changes (ws_gen counts training-workspace reallocations)
   cudaGraphExec_t train_graph = nullptr;
   int graph_batch = 0, graph_p = 0;
+  float* graph_loss = nullptr;
+  unsigned long long graph_kernels = 0;  // our kernels in one captured iteration
+  unsigned long long ws_gen = 0, graph_gen = 0;
+  // data parallelism (T5): NCCL communicator owned by the ctx (created from sr_options.nccl_id), sum of the ranks'
+  // gradient weights (allreduced once at sr_create)
+  ncclComm_t comm = nullptr;
+  double sum_w = 1.0;
+  int device = 0;
+  // inference calls in flight per stream (sr_publish makes its snapshot copies wait for them)
+  std::vector<std::pair<cudaStream_t, cudaEvent_t>> infer_evs;
   unsigned long long launches = 0;
   // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
   bool timing = false;
@@ -230,7 +276,7 @@ static WgradJob wjob(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy) {
 }
 
 static sr_status ensure_wg(sr_ctx* ctx, size_t elems, cudaStream_t st) {
-  if (elems > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, elems)); ctx->ws_w_elems = elems; }
+  if (elems > ctx->ws_w_elems) { CK(dalloc(&ctx->ws_w, elems)); ctx->ws_w_elems = elems; ctx->ws_gen++; }
   if (!ctx->wg_sync) {
     CK(dalloc(&ctx->wg_sync, 2));
     CK(cudaMemsetAsync(ctx->wg_sync, 0, 2 * sizeof(unsigned), st));
@@ -467,6 +513,7 @@ static sr_status forward_infer_virtual(sr_ctx* ctx, const Snapshot& sn, const ui
 
 static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
   if (pix <= ctx->tr_pix) return SR_OK;
+  ctx->ws_gen++;
   const int Cp = ctx->Cp;
   CK(dalloc(&ctx->tx16, pix * 16));
   for (auto& p : ctx->tf) CK(dalloc(&p, pix * Cp));
@@ -713,6 +760,61 @@ static sr_status train_apply(sr_ctx* ctx, float grad_scale, const float* grad_sc
 
 static bool valid_model(sr_model m) { return m >= SR_TRAIN && m <= SR_INIT; }
 
+#define NCK(call)                                                                                           \
+  do {                                                                                                      \
+    ncclResult_t r_ = (call);                                                                               \
+    if (r_ != ncclSuccess) return fail(ctx, SR_E_NCCL, std::string(#call) + ": " + nccl().err(r_));        \
+  } while (0)
+
+// Communicator of the DP group from the caller's ncclUniqueId (collective over the ranks: every rank calls sr_create
+// with the same id), then sum_r w_r of the ranks' gradient weights, once (the weights are fixed per ctx).
+static sr_status comm_init(sr_ctx* ctx) {
+  NcclApi& a = nccl();
+  if (!a.ok) return fail(ctx, SR_E_NCCL, a.why);
+  ncclUniqueId id;
+  memcpy(&id, ctx->opt.nccl_id, sizeof(id));
+  NCK(a.init_rank(&ctx->comm, ctx->opt.world, id, ctx->opt.rank));
+  float* w = nullptr;
+  CK(cudaMalloc(&w, sizeof(float)));
+  const float mine = ctx->opt.dp_weight;
+  CK(cudaMemcpy(w, &mine, sizeof(float), cudaMemcpyHostToDevice));
+  ncclResult_t r = a.all_reduce(w, w, 1, ncclFloat32, ncclSum, ctx->comm, 0);
+  float tot = 0.f;
+  cudaError_t e = cudaMemcpy(&tot, w, sizeof(float), cudaMemcpyDeviceToHost);
+  cudaFree(w);
+  if (r != ncclSuccess) return fail(ctx, SR_E_NCCL, std::string("ncclAllReduce(weights): ") + a.err(r));
+  CK(e);
+  if (!(tot > 0.f)) return fail(ctx, SR_E_INVAL, "sum of dp_weight over ranks must be > 0");
+  ctx->sum_w = tot;
+  return SR_OK;
+}
+
+// T5 exchange: grad <- sum_r (w_r g_r) over the DP group, in place, stream-ordered (graph-capturable).
+static sr_status grad_exchange(sr_ctx* ctx, cudaStream_t st) {
+  if (!ctx->comm) {
+    if (ctx->opt.world > 1)
+      return fail(ctx, SR_E_STATE, "world > 1 without sr_options.nccl_id: exchange the gradient yourself "
+                                   "(sr_grad_buffer) and call sr_train_apply");
+    return SR_OK;
+  }
+  NCK(nccl().all_reduce(ctx->grad, ctx->grad, ctx->nparams, ncclFloat32, ncclSum, ctx->comm, st));
+  return SR_OK;  // (NCCL's kernel, not counted in sr_launch_count)
+}
+
+// the stream's last inference call (sr_publish orders its snapshot copies after it)
+static sr_status note_infer(sr_ctx* ctx, cudaStream_t st) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  CK(cudaStreamIsCapturing(st, &cs));
+  if (cs != cudaStreamCaptureStatusNone) return SR_OK;  // inside a caller's graph capture: the caller orders it
+  for (auto& pe : ctx->infer_evs)
+    if (pe.first == st) { CK(cudaEventRecord(pe.second, st)); return SR_OK; }
+  cudaEvent_t e;
+  CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  ctx->infer_evs.push_back({st, e});
+  CK(cudaEventRecord(e, st));
+  return SR_OK;
+}
+
 // ------------------------------------------------------------------------------------------ C ABI
 extern "C" {
 
@@ -738,6 +840,10 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   if (ctx->opt.dp_weight == 0.f) ctx->opt.dp_weight = 1.f;
   if (ctx->opt.pool_capacity <= 0) ctx->opt.pool_capacity = 8192;
   if (ctx->opt.rank < 0 || ctx->opt.rank >= ctx->opt.world) { delete ctx; return SR_E_INVAL; }
+  if (opt && opt->device >= 0) {
+    if (cudaSetDevice(opt->device) != cudaSuccess) { delete ctx; return SR_E_INVAL; }
+  }
+  if (cudaGetDevice(&ctx->device) != cudaSuccess) { delete ctx; return SR_E_CUDA; }
   if (ctx->opt.loss < 0 || ctx->opt.loss > 1 || ctx->opt.skip < 0 || ctx->opt.skip > 1) { delete ctx; return SR_E_INVAL; }
   // conv table in canonical order: head, (b.conv1, b.conv2) x B, body, up
   std::vector<std::pair<int, int>> shp;  // (cout, cin)
@@ -782,9 +888,10 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   al(&ctx->wd_train, ctx->pk_total);
   al(&ctx->wdo_train, ctx->pk_total);
   al(&ctx->loss_sum, 1);
-  al(&ctx->counters, 3);  // [0] sampler step, [1] Adam t, [2] gather block counter
+  al(&ctx->counters, 5);  // [0] sampler step, [1] Adam t, [2] gather block counter, [3] pool arrivals, [4] clamped crops
   al(&ctx->zero_bias, 64);
   if (st == SR_OK && cudaMemset(ctx->zero_bias, 0, 64 * sizeof(float)) != cudaSuccess) st = SR_E_CUDA;
+  if (st == SR_OK && cudaMemset(ctx->counters, 0, 5 * sizeof(long long)) != cudaSuccess) st = SR_E_CUDA;
   ctx->tf.assign(blocks + 1, nullptr);
   ctx->tts.assign(blocks, nullptr);
   ctx->tdf.assign(blocks + 1, nullptr);
@@ -811,6 +918,19 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   }
   st = sr_set_params(ctx, h.data(), h.size());
   if (st != SR_OK) { sr_destroy(ctx); return st; }
+  if (ctx->opt.nccl_id) {  // T5: the ctx owns the NCCL communicator of the data-parallel group
+    st = comm_init(ctx);
+    if (st != SR_OK) {
+      std::string msg = ctx->err;
+      sr_destroy(ctx);
+      fprintf(stderr, "sr_create: %s\n", msg.c_str());
+      return st;
+    }
+  } else {
+    // world 1: the rank's own weight; world > 1 without a communicator: external exchange (the caller allreduces
+    // sr_grad_buffer and passes 1 / sum_r w_r to sr_train_apply), sum unknown here
+    ctx->sum_w = ctx->opt.world > 1 ? 0.0 : ctx->opt.dp_weight;
+  }
   *out = ctx;
   return SR_OK;
 }
@@ -831,6 +951,8 @@ void sr_destroy(sr_ctx* ctx) {
   for (auto p : ctx->tdf) if (p) cudaFree(p);
   for (auto p : ctx->tdtb) if (p) cudaFree(p);
   if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
+  for (auto& pe : ctx->infer_evs) cudaEventDestroy(pe.second);
+  if (ctx->comm) nccl().destroy(ctx->comm);
   if (ctx->train_graph) cudaGraphExecDestroy(ctx->train_graph);
   for (auto e : ctx->chunk_ev) if (e) cudaEventDestroy(e);
   if (ctx->copy_st) cudaStreamDestroy(ctx->copy_st);
@@ -902,11 +1024,19 @@ size_t sr_num_params(const sr_ctx* ctx) { return ctx ? ctx->nparams : 0; }
 uint64_t sr_launch_count(const sr_ctx* ctx) { return ctx ? ctx->launches : 0; }
 float* sr_grad_buffer(sr_ctx* ctx) { return ctx ? ctx->grad : nullptr; }
 
+// Every call runs on the ctx's device (restored on return), so one process may drive ctxs on several GPUs.
+struct DeviceScope {
+  int prev = -1;
+  explicit DeviceScope(const sr_ctx* ctx) {
+    if (ctx && cudaGetDevice(&prev) == cudaSuccess && prev != ctx->device) cudaSetDevice(ctx->device);
+    else prev = -1;
+  }
+  ~DeviceScope() { if (prev >= 0) cudaSetDevice(prev); }
+};
 #define GUARD()                                                                  \
-  do {                                                                           \
-    if (!ctx) return SR_E_INVAL;                                                 \
-    if (ctx->poisoned) return fail(ctx, SR_E_STATE, "ctx poisoned: " + ctx->err); \
-  } while (0)
+  if (!ctx) return SR_E_INVAL;                                                   \
+  DeviceScope dev_scope_(ctx);                                                   \
+  if (ctx->poisoned) return fail(ctx, SR_E_STATE, "ctx poisoned: " + ctx->err)
 
 // SM share of an API entry (restored on return): inference-side calls get sm_total - sm_train SMs, training-side
 // calls sm_train, when a split is set.
@@ -979,8 +1109,10 @@ sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, in
   if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer: bad model");
   CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
   if (use_virtual_infer(ctx, n, h, w) && ctx->virtual_train)
-    return forward_infer_virtual(ctx, ctx->snap[which], lr_dev, n, h, hr_dev, st);
-  return forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st);
+    TRY(forward_infer_virtual(ctx, ctx->snap[which], lr_dev, n, h, hr_dev, st));
+  else
+    TRY(forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st));
+  return note_infer(ctx, st);
 }
 
 sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const uint8_t* u_dev,
@@ -1105,8 +1237,9 @@ sr_status sr_infer_rows(sr_ctx* ctx, sr_model which, const uint8_t* lr_full_dev,
   const int lo = std::max(0, row0 - halo), hi = std::min(h, row1 + halo);
   const int s = ctx->s;
   CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
-  return forward_infer(ctx, ctx->snap[which], lr_full_dev + (size_t)lo * w * 3, 1, hi - lo, w,
-                       hr_full_dev + (size_t)lo * s * (size_t)s * w * 3, row0 - lo, row1 - lo, st);
+  TRY(forward_infer(ctx, ctx->snap[which], lr_full_dev + (size_t)lo * w * 3, 1, hi - lo, w,
+                    hr_full_dev + (size_t)lo * s * (size_t)s * w * 3, row0 - lo, row1 - lo, st));
+  return note_infer(ctx, st);
 }
 
 sr_status sr_train_grad(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int p, float* loss_dev,
@@ -1134,10 +1267,20 @@ sr_status sr_train_step(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_de
                         sr_stream stream) {
   GUARD();
   CAP_TRAIN();
+  if (ctx->opt.world > 1 && !ctx->comm)
+    return fail(ctx, SR_E_STATE, "sr_train_step: world > 1 needs sr_options.nccl_id (or sr_train_grad + your "
+                                 "allreduce + sr_train_apply)");
   TRY(sr_train_grad(ctx, lr_dev, hr_dev, n, p, loss_dev, stream));
-  const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
-  return train_apply(ctx, 1.0f / w, nullptr, (cudaStream_t)stream);
+  TRY(grad_exchange(ctx, (cudaStream_t)stream));  // T5: sum_r w_r g_r over the DP group (no-op at world 1)
+  return train_apply(ctx, (float)(1.0 / ctx->sum_w), nullptr, (cudaStream_t)stream);
 }
+
+sr_status sr_train_allreduce(sr_ctx* ctx, sr_stream stream) {
+  GUARD();
+  return grad_exchange(ctx, (cudaStream_t)stream);
+}
+
+double sr_dp_weight_sum(const sr_ctx* ctx) { return ctx ? ctx->sum_w : 0.0; }
 
 sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev, int n, int pp,
                        const int64_t* arrival_ts, sr_stream stream) {
@@ -1164,6 +1307,9 @@ sr_status sr_pool_push(sr_ctx* ctx, const uint8_t* lr_dev, const uint8_t* hr_dev
     i += run;
   }
   ctx->pool_total += n;
+  launch_counter_add(ctx->counters + 3, n, st);  // the device-side arrival count the sampler reads (graph replays)
+  ctx->launches++;
+  CKL();
   return SR_OK;
 }
 
@@ -1172,12 +1318,14 @@ sr_status sr_pool_push_i420(sr_ctx* ctx, const uint8_t* y_dev, const uint8_t* u_
                             const int64_t* arrival_ts, sr_stream stream) {
   GUARD();
   CAP_TRAIN();
-  if (!y_dev || !u_dev || !v_dev || !hr_dev || !xy_dev || n < 1 || pp < 1 || h < 2 || w < 2 || (h | w) & 1)
-    return fail(ctx, SR_E_INVAL, "sr_pool_push_i420: bad args");
+  if (!y_dev || !u_dev || !v_dev || !hr_dev || !xy_dev || n < 1 || pp < 1 || h < 2 || w < 2 || (h | w) & 1 ||
+      pp > h || pp > w)
+    return fail(ctx, SR_E_INVAL, "sr_pool_push_i420: bad args (even h, w >= pp)");
   cudaStream_t st = (cudaStream_t)stream;
   const size_t need = (size_t)n * pp * pp * 3;
   if (need > ctx->crop_bytes) { CK(dalloc(&ctx->crop_buf, need)); ctx->crop_bytes = need; }
-  launch_i420_crop(y_dev, u_dev, v_dev, h, w, xy_dev, n, pp, ctx->crop_buf, st);
+  launch_i420_crop(y_dev, u_dev, v_dev, h, w, xy_dev, n, pp, ctx->crop_buf,
+                   reinterpret_cast<unsigned long long*>(ctx->counters + 4), st);
   ctx->launches++;
   CKL();
   return sr_pool_push(ctx, ctx->crop_buf, hr_dev, n, pp, arrival_ts, stream);
@@ -1186,6 +1334,16 @@ sr_status sr_pool_push_i420(sr_ctx* ctx, const uint8_t* y_dev, const uint8_t* u_
 size_t sr_pool_size(const sr_ctx* ctx) {
   if (!ctx) return 0;
   return (size_t)std::min(ctx->pool_total, ctx->pool_cap);
+}
+
+sr_status sr_pool_stats(sr_ctx* ctx, int64_t* arrivals, int64_t* clamped) {
+  GUARD();
+  long long h[2] = {0, 0};
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(h, ctx->counters + 3, sizeof h, cudaMemcpyDeviceToHost));
+  if (arrivals) *arrivals = h[0];
+  if (clamped) *clamped = h[1];
+  return SR_OK;
 }
 
 sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* lr_out_dev, uint8_t* hr_out_dev,
@@ -1207,6 +1365,7 @@ sr_status sr_sample_batch(sr_ctx* ctx, int64_t step, int batch, int p, uint8_t* 
   a.rank = r;
   a.n_view = hi - lo;
   a.view_base = ctx->pool_total - avail + lo;
+  a.pool_total_dev = ctx->counters + 3;  // the same view, derived on the device (stays current in graph replays)
   a.capacity = ctx->pool_cap;
   a.recent_k = ctx->opt.recent_k;
   a.recent_w = ctx->opt.recent_w;
@@ -1232,18 +1391,24 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
   GUARD();
   CAP_TRAIN();
   if (iters < 1 || batch < 1 || p < 1) return fail(ctx, SR_E_INVAL, "sr_train_sampled: bad args");
-  if (ctx->opt.world != 1) return fail(ctx, SR_E_STATE, "sr_train_sampled: world > 1 needs the split API");
+  if (ctx->opt.world > 1 && !ctx->comm)
+    return fail(ctx, SR_E_STATE, "sr_train_sampled: world > 1 needs sr_options.nccl_id (the ctx's communicator)");
   cudaStream_t st = (cudaStream_t)stream;
   const size_t lb = (size_t)batch * p * p * 3, hb = lb * ctx->s * ctx->s;
+  // one iteration: sample + gather from the device-side pool view and step counter (T1), forward / loss / backward
+  // (T2-T4), sum-allreduce of w_r g_r over the DP group (T5, world > 1), Adam with 1 / sum_r w_r (T6)
   auto one_iter = [&]() -> sr_status {
     TRY(sr_sample_batch(ctx, -1, batch, p, ctx->batch_lr, ctx->batch_hr, nullptr, stream));  // device step counter
     TRY(train_grad(ctx, ctx->batch_lr, ctx->batch_hr, batch, p, loss_dev, st));
-    const float w = ctx->opt.dp_weight > 0 ? ctx->opt.dp_weight : 1.f;
-    return train_apply(ctx, 1.0f / w, nullptr, st);
+    TRY(grad_exchange(ctx, st));
+    return train_apply(ctx, (float)(1.0 / ctx->sum_w), nullptr, st);
   };
-  if (!ctx->train_graph || ctx->graph_batch != batch || ctx->graph_p != p || st == nullptr) {
-    if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; }
-    if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; }
+  // the captured graph bakes in the loss pointer and every workspace address: re-capture when any of them changed
+  const bool stale = !ctx->train_graph || ctx->graph_batch != batch || ctx->graph_p != p ||
+                     ctx->graph_loss != loss_dev || ctx->graph_gen != ctx->ws_gen;
+  if (stale || st == nullptr) {
+    if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; ctx->ws_gen++; }
+    if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; ctx->ws_gen++; }
     TRY(one_iter());  // eager iteration: grows the workspaces, configures the kernels
     --iters;
     if (st != nullptr) {  // capture one iteration (the legacy default stream cannot be captured)
@@ -1251,9 +1416,12 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
       const bool timing = ctx->timing;
       ctx->timing = false;
       cudaGraph_t g = nullptr;
+      const unsigned long long l0 = ctx->launches;
       CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
       sr_status cs = one_iter();
       cudaError_t ce = cudaStreamEndCapture(st, &g);
+      ctx->graph_kernels = ctx->launches - l0;  // captured, not run: counted per replay below
+      ctx->launches = l0;
       ctx->timing = timing;
       TRY(cs);
       CK(ce);
@@ -1261,12 +1429,14 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
       cudaGraphDestroy(g);
       ctx->graph_batch = batch;
       ctx->graph_p = p;
+      ctx->graph_loss = loss_dev;
+      ctx->graph_gen = ctx->ws_gen;
     }
   }
   for (int it = 0; it < iters; ++it) {
     if (ctx->train_graph && st != nullptr) {
       CK(cudaGraphLaunch(ctx->train_graph, st));
-      ctx->launches += 1;
+      ctx->launches += ctx->graph_kernels;
     } else {
       TRY(one_iter());
     }
@@ -1278,6 +1448,10 @@ sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
   GUARD();
   CAP_TRAIN();
   cudaStream_t st = (cudaStream_t)stream;
+  // inference reading SERVE / PREV may be in flight on other streams: the snapshot copies wait for it (a frame is
+  // never computed with a mix of old and new layer weights; the paper syncs inference at the epoch end, L1252-1253)
+  for (auto& pe : ctx->infer_evs)
+    if (pe.first != st) CK(cudaStreamWaitEvent(st, pe.second, 0));
   TRY(ensure_full_train_pack(ctx, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wf, ctx->snap[SR_SERVE].wf, ctx->pk_total * sizeof(bf16),
                      cudaMemcpyDeviceToDevice, st));
@@ -1459,6 +1633,33 @@ sr_status sr_controller_step(sr_ctx* ctx, sr_controller* c, const uint8_t* lr_de
   r.event = ev;
   r.state_after = c->state;
   *out_host = r;
+  return SR_OK;
+}
+
+sr_status sr_get_adam_state(sr_ctx* ctx, float* m_host, float* v_host, size_t n, int64_t* t_host) {
+  GUARD();
+  if (n != ctx->nparams) return fail(ctx, SR_E_INVAL, "sr_get_adam_state: size mismatch");
+  CK(cudaDeviceSynchronize());
+  if (m_host) CK(cudaMemcpy(m_host, ctx->m, n * sizeof(float), cudaMemcpyDeviceToHost));
+  if (v_host) CK(cudaMemcpy(v_host, ctx->v, n * sizeof(float), cudaMemcpyDeviceToHost));
+  if (t_host) {
+    long long t = 0;
+    CK(cudaMemcpy(&t, ctx->counters + 1, sizeof t, cudaMemcpyDeviceToHost));
+    *t_host = t;
+  }
+  return SR_OK;
+}
+
+sr_status sr_nccl_unique_id(void* id_out, size_t cap) {
+  if (!id_out || cap < sizeof(ncclUniqueId)) return SR_E_INVAL;
+  NcclApi& a = nccl();
+  if (!a.ok) {
+    fprintf(stderr, "sr_nccl_unique_id: %s\n", a.why.c_str());
+    return SR_E_NCCL;
+  }
+  ncclUniqueId id;
+  if (a.get_id(&id) != ncclSuccess) return SR_E_NCCL;
+  memcpy(id_out, &id, sizeof id);
   return SR_OK;
 }
 

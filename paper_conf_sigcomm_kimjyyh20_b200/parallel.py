@@ -1,14 +1,16 @@
-"""Host-side multi-GPU plumbing of the hot path (one process per GPU, torch.distributed over NCCL/NVLink).
+"""Host-side multi-GPU plumbing of the hot path (one process per GPU, torch.distributed for rendezvous and timing).
 
-Only sharding arithmetic and the gradient exchange live here; every FLOP runs in libsr.so.
+No arithmetic of the method lives here: sharding index ranges, the NCCL id hand-out and a max-over-ranks of a
+timing.  Every FLOP, including the data-parallel gradient exchange, runs in libsr.so.
 
 * Inference shards naturally (§6.2):
     - throughput mode: frames round-robin / contiguous per rank, no collective (`frame_shard`);
     - latency mode: one frame split into equal horizontal pieces, one per GPU (`strip_rows`, 720p -> 3 x 240
       rows, L1192-1194); the library adds an exact halo (reading R12) so stitching is bit-exact.
-* Training is data-parallel over patches (L1210-1220): the pool is partitioned by arrival sequence
-  (`pool_view`, mirrored in sr_sample_batch), each rank computes w_r * g_r, one sum-allreduce of the flat
-  fp32 gradient (NCCL; gloo on CPU for tests), then Adam with g = sum_r w_r g_r / sum_r w_r (`dp_allreduce_grad`).
+* Training is data-parallel over patches (L1210-1220): the pool is partitioned by arrival sequence (`pool_view`,
+  mirrored on the device by sr_sample_batch), each rank computes w_r * g_r, and the ctx's own NCCL communicator sums
+  them (sr_train_step / sr_train_sampled / sr_train_allreduce); Adam applies 1 / sum_r w_r.  The communicator is
+  created inside sr_create from an ncclUniqueId that rank 0 draws and `nccl_id_broadcast` hands to every rank.
 """
 from __future__ import annotations
 
@@ -30,28 +32,27 @@ def pool_view(n_avail: int, world: int, rank: int) -> tuple[int, int]:
     return n_avail * rank // world, n_avail * (rank + 1) // world
 
 
-def dp_allreduce_grad(grad, weight: float = 1.0, group=None) -> float:
-    """In-place sum-allreduce of `grad` (already scaled by this rank's weight w_r inside sr_train_grad) and of
-    the weights; returns the Adam grad_scale = 1 / sum_r w_r, so the update uses sum_r w_r g_r / sum_r w_r."""
+def nccl_id_broadcast(group=None) -> bytes:
+    """The 128-byte ncclUniqueId of the DP group: drawn by rank 0 through the library (sr_nccl_unique_id) and
+    broadcast over the process group (gloo or NCCL), so every rank passes the same bytes to SRContext(nccl_id=...)."""
+    import ctypes as C
+
     import torch
     import torch.distributed as dist
-    if not dist.is_initialized() or dist.get_world_size(group) == 1:
-        return 1.0 / weight
-    dist.all_reduce(grad, op=dist.ReduceOp.SUM, group=group)
-    w = torch.tensor([float(weight)], dtype=torch.float64, device=grad.device)
-    dist.all_reduce(w, op=dist.ReduceOp.SUM, group=group)
-    return 1.0 / float(w.item())
 
-
-def dp_allreduce_grad_dev(grad, weight_dev, group=None):
-    """Graph-capturable variant: sum-allreduce `grad` and the 1-element weight tensor `weight_dev` on the device and
-    return a device tensor holding 1 / sum_r w_r (feed it to SRContext.train_apply_dev)."""
-    import torch.distributed as dist
-    w = weight_dev.clone()
-    if dist.is_initialized() and dist.get_world_size(group) > 1:
-        dist.all_reduce(grad, op=dist.ReduceOp.SUM, group=group)
-        dist.all_reduce(w, op=dist.ReduceOp.SUM, group=group)
-    return w.reciprocal()
+    from ._lib import SRError, load
+    backend = dist.get_backend(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+    buf = torch.zeros(128, dtype=torch.uint8)
+    if dist.get_rank(group) == 0:
+        raw = C.create_string_buffer(128)
+        st = load().sr_nccl_unique_id(raw, 128)
+        if st != 0:
+            raise SRError(f"sr_nccl_unique_id failed with status {st}")
+        buf = torch.frombuffer(bytearray(raw.raw), dtype=torch.uint8).clone()
+    t = buf.to(dev)
+    dist.broadcast(t, src=0, group=group)
+    return bytes(t.cpu().numpy().tobytes())
 
 
 def max_over_ranks(value: float, device=None, group=None) -> float:

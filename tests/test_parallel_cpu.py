@@ -1,4 +1,5 @@
-"""Multi-rank host logic on CPU (gloo, world size 2): sharding arithmetic and the DP gradient exchange."""
+"""Multi-rank host logic on CPU (gloo, world size 2): sharding arithmetic, the NCCL id hand-out, max-over-ranks
+timing, and the DP exchange protocol the library runs (sum-allreduce of w_r g_r, then Adam with 1 / sum_r w_r)."""
 import os
 import socket
 import tempfile
@@ -9,7 +10,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import oracle as O
-from paper_conf_sigcomm_kimjyyh20_b200.parallel import (dp_allreduce_grad, frame_shard, max_over_ranks, pool_view,
+from paper_conf_sigcomm_kimjyyh20_b200.parallel import (frame_shard, max_over_ranks, nccl_id_broadcast, pool_view,
                                                          strip_rows)
 from synth import init_params
 
@@ -46,10 +47,16 @@ def _worker(rank, world, port, out_dir, weights):
     hr = r.integers(0, 256, size=(2, 12, 12, 3)).astype(np.uint8)
     _, g = O.train_loss_and_grad(p, lr, hr, s, B, C)
     w = weights[rank]
-    gt = torch.from_numpy(g * w)  # sr_train_grad hands back w_r * g_r
-    scale = dp_allreduce_grad(gt, weight=w)
-    agg = gt.numpy() * scale
+    # the protocol libsr runs on the device (sr_train_grad pre-scales by w_r; sr_create allreduces the weights once;
+    # sr_train_allreduce sums the gradients; k_adam applies 1 / sum_r w_r), here over gloo on the oracle's gradients
+    gt = torch.from_numpy(g * w)
+    dist.all_reduce(gt, op=dist.ReduceOp.SUM)
+    wt = torch.tensor([w], dtype=torch.float64)
+    dist.all_reduce(wt, op=dist.ReduceOp.SUM)
+    agg = gt.numpy() / float(wt.item())
     t = max_over_ranks(float(rank + 1))
+    nid = nccl_id_broadcast()
+    np.save(os.path.join(out_dir, f"id{rank}.npy"), np.frombuffer(nid, np.uint8))
     np.save(os.path.join(out_dir, f"agg{rank}.npy"), agg)
     np.save(os.path.join(out_dir, f"g{rank}.npy"), g)
     np.save(os.path.join(out_dir, f"max{rank}.npy"), np.array([t]))
@@ -62,17 +69,21 @@ def _run(weights):
         aggs = [np.load(os.path.join(d, f"agg{r}.npy")) for r in range(2)]
         gs = [np.load(os.path.join(d, f"g{r}.npy")) for r in range(2)]
         mx = [float(np.load(os.path.join(d, f"max{r}.npy"))[0]) for r in range(2)]
-    return aggs, gs, mx
+        ids = [np.load(os.path.join(d, f"id{r}.npy")) for r in range(2)]
+    return aggs, gs, mx, ids
 
 
 def test_dp_allreduce_gloo_uniform_equals_union_batch():
-    aggs, gs, mx = _run([1.0, 1.0])
+    aggs, gs, mx, ids = _run([1.0, 1.0])
     np.testing.assert_array_equal(aggs[0], aggs[1])          # every rank applies identical bits
     np.testing.assert_allclose(aggs[0], O.dp_aggregate(gs), rtol=1e-12)
     assert mx == [2.0, 2.0]
+    # rank 0's ncclUniqueId (drawn by libsr's sr_nccl_unique_id) reaches every rank byte for byte
+    assert ids[0].size == 128 and ids[0].any()
+    np.testing.assert_array_equal(ids[0], ids[1])
 
 
 def test_dp_allreduce_gloo_recency_weights():
     """Larger weight for the rank holding the newer patches (reading R11)."""
-    aggs, gs, _ = _run([1.0, 4.0])
+    aggs, gs, _, _ = _run([1.0, 4.0])
     np.testing.assert_allclose(aggs[1], O.dp_aggregate(gs, [1.0, 4.0]), rtol=1e-12)
