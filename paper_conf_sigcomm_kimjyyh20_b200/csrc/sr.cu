@@ -8,6 +8,8 @@
 #include <vector>
 #include <algorithm>
 #include <dlfcn.h>
+#include <mutex>
+#include <atomic>
 #include <nccl.h>  // types only: libnccl is dlopen'ed at sr_create when world > 1 (libsr.so loads without it)
 #include "sr_internal.h"
 #include "kernels.h"
@@ -52,6 +54,14 @@ struct Snapshot {
   float* bias = nullptr; // packed fp32 biases
 };
 
+// Activation workspace of one inference path (grown on the first call of a larger shape).  A ctx has two: frames
+// (the sr_infer family) and quality evaluation (sr_psnr_gain / sr_controller_step, issued from the training side),
+// so the two may run concurrently on different streams without sharing buffers.
+struct InferWS {
+  size_t pix = 0;
+  bf16 *x16 = nullptr, *f0 = nullptr, *fa = nullptr, *fb = nullptr, *tt = nullptr;
+};
+
 struct sr_ctx {
   int s = 2, B = 0, C = 0, Cp = 16, OUTP = 16, nconv = 0;
   sr_options opt{};
@@ -65,9 +75,8 @@ struct sr_ctx {
   bf16* wd_train = nullptr;  // dgrad-packed TRAIN weights
   bf16* wdo_train = nullptr; // dgrad weights in dy-fold layout (rolling data-grad convs)
   bool virtual_train = true; // training on the virtual wide batch with the rolling kernels
-  // inference workspace
-  size_t inf_pix = 0;
-  bf16 *x16 = nullptr, *f0 = nullptr, *fa = nullptr, *fb = nullptr, *tt = nullptr;
+  // inference workspaces: frames, quality evaluation
+  InferWS iws, qws;
   uint8_t *stage_lr = nullptr, *stage_hr = nullptr;
   cudaStream_t copy_st = nullptr, h2d_st = nullptr;  // sr_infer_host: PCIe copies overlapped with the tensor work
   std::vector<cudaEvent_t> chunk_ev;
@@ -118,7 +127,8 @@ struct sr_ctx {
   int device = 0;
   // inference calls in flight per stream (sr_publish makes its snapshot copies wait for them)
   std::vector<std::pair<cudaStream_t, cudaEvent_t>> infer_evs;
-  unsigned long long launches = 0;
+  std::mutex ev_mu;  // infer_evs is touched by the inference side (note_infer) and the training side (sr_publish)
+  std::atomic<unsigned long long> launches{0};  // kernels launched (inference and training threads)
   // optional per-kernel-class CUDA-event timing (sr_kernel_timing)
   bool timing = false;
   bool fuse_blocks = true;  // fused residual-block kernel for wide frames (sr_set_option)
@@ -342,24 +352,24 @@ static sr_status wgrad(sr_ctx* ctx, int ci, const bf16* x, const bf16* dy, int N
     if (s_ != SR_OK) return s_;  \
   } while (0)
 
-static sr_status ensure_infer_ws(sr_ctx* ctx, size_t pix) {
-  if (pix <= ctx->inf_pix) return SR_OK;
-  CK(dalloc(&ctx->x16, pix * 16));
-  CK(dalloc(&ctx->f0, pix * ctx->Cp));
-  CK(dalloc(&ctx->fa, pix * ctx->Cp));
-  CK(dalloc(&ctx->fb, pix * ctx->Cp));
-  CK(dalloc(&ctx->tt, pix * ctx->Cp));
-  ctx->inf_pix = pix;
+static sr_status ensure_infer_ws(sr_ctx* ctx, InferWS& ws, size_t pix) {
+  if (pix <= ws.pix) return SR_OK;
+  CK(dalloc(&ws.x16, pix * 16));
+  CK(dalloc(&ws.f0, pix * ctx->Cp));
+  CK(dalloc(&ws.fa, pix * ctx->Cp));
+  CK(dalloc(&ws.fb, pix * ctx->Cp));
+  CK(dalloc(&ws.tt, pix * ctx->Cp));
+  ws.pix = pix;
   return SR_OK;
 }
 
 // Inference forward (reading R1): x = v/255; f0 = head(x); f <- f + conv2(relu(conv1(f))) x B;
 // g = f0 + body(f); tail(up(g)) -> u8 with pixel shuffle + bilinear skip + clamp + RNE.
-static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
+static sr_status forward_infer(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
                                uint8_t* hr, int row0, int row1, cudaStream_t st) {
   if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const size_t pix = (size_t)n * h * w;
-  TRY(ensure_infer_ws(ctx, pix));
+  TRY(ensure_infer_ws(ctx, ws, pix));
   const int Cp = ctx->Cp;
   auto W = [&](int ci) { return sn.wf + ctx->convs[ci].pk_off; };
   auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
@@ -369,22 +379,22 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
       const double px = (double)n * h * w;
       tmark_begin(ctx, "conv_roll_16x" + std::to_string(Cp), 2.0 * 9 * 16 * Cp * px, px * (3.0 + 2.0 * Cp), st);
     }
-    cudaError_t e = launch_conv_roll_head_u8(Cp, lr, sn.wo + ctx->convs[0].pk_off, Bv(0), ctx->f0, n, h, w, st, 1);
+    cudaError_t e = launch_conv_roll_head_u8(Cp, lr, sn.wo + ctx->convs[0].pk_off, Bv(0), ws.f0, n, h, w, st, 1);
     tmark_end(ctx, st);
     ctx->launches++;
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("u8 head launch: ") + cudaGetErrorString(e));
   } else {
-    launch_pack_input(lr, pix, ctx->x16, st);
+    launch_pack_input(lr, pix, ws.x16, st);
     ctx->launches++;
     CKL();
     EpiParams ep{};
     ep.bias = Bv(0);
-    ep.out = ctx->f0;
-    TRY(conv_fwd(ctx, 16, Cp, ctx->x16, sn, 0, n, h, w, ep, st));
+    ep.out = ws.f0;
+    TRY(conv_fwd(ctx, 16, Cp, ws.x16, sn, 0, n, h, w, ep, st));
   }
-  bf16* cur = ctx->f0;
+  bf16* cur = ws.f0;
   for (int b = 0; b < ctx->B; ++b) {
-    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+    bf16* nxt = (cur == ws.fa) ? ws.fb : ws.fa;
     if (ctx->fuse_blocks && resblock_supported(Cp, w)) {  // fused block: t stays in shared memory
       if (ctx->timing) {
         const double px = (double)n * h * w;
@@ -401,13 +411,13 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
     EpiParams e1{};
     e1.bias = Bv(1 + 2 * b);
     e1.relu = 1;
-    e1.out = ctx->tt;
+    e1.out = ws.tt;
     TRY(conv_fwd(ctx, Cp, Cp, cur, sn, 1 + 2 * b, n, h, w, e1, st));
     EpiParams e2{};
     e2.bias = Bv(2 + 2 * b);
     e2.res1 = cur;
     e2.out = nxt;
-    TRY(conv_fwd(ctx, Cp, Cp, ctx->tt, sn, 2 + 2 * b, n, h, w, e2, st));
+    TRY(conv_fwd(ctx, Cp, Cp, ws.tt, sn, 2 + 2 * b, n, h, w, e2, st));
     cur = nxt;
   }
   const int cb = 1 + 2 * ctx->B, cu = cb + 1;
@@ -418,7 +428,7 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
       tmark_begin(ctx, "bodytail_" + std::to_string(Cp) + "x" + std::to_string(ctx->OUTP),
                   2.0 * 9 * Cp * (Cp + ctx->OUTP) * px, px * (4.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
     }
-    cudaError_t e = launch_bodytail(Cp, ctx->s, cur, ctx->f0, sn.wo + ctx->convs[cb].pk_off,
+    cudaError_t e = launch_bodytail(Cp, ctx->s, cur, ws.f0, sn.wo + ctx->convs[cb].pk_off,
                                     sn.wo + ctx->convs[cu].pk_off, Bv(cb), Bv(cu), lr, hr, row0, row1,
                                     ctx->opt.skip == 1, n, h, w, st);
     tmark_end(ctx, st);
@@ -426,10 +436,10 @@ static sr_status forward_infer(sr_ctx* ctx, const Snapshot& sn, const uint8_t* l
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("bodytail launch: ") + cudaGetErrorString(e));
     return SR_OK;
   }
-  bf16* gbuf = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+  bf16* gbuf = (cur == ws.fa) ? ws.fb : ws.fa;
   EpiParams eb{};
   eb.bias = Bv(cb);
-  eb.res1 = ctx->f0;
+  eb.res1 = ws.f0;
   eb.out = gbuf;
   TRY(conv_fwd(ctx, Cp, Cp, cur, sn, cb, n, h, w, eb, st));
   if (roll_supported(Cp, ctx->OUTP, w) && ctx->roll_tail) {  // rolling up conv with the tail in its epilogue
@@ -467,38 +477,38 @@ static bool use_virtual_infer(const sr_ctx* ctx, int n, int h, int w) {
          roll_supported(ctx->Cp, ctx->Cp, Wv);
 }
 
-static sr_status forward_infer_virtual(sr_ctx* ctx, const Snapshot& sn, const uint8_t* lr, int n, int p,
+static sr_status forward_infer_virtual(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, const uint8_t* lr, int n, int p,
                                        uint8_t* hr, cudaStream_t st) {
   if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const int Hv = p, Wv = n * (p + 2), sep = p + 2;
-  TRY(ensure_infer_ws(ctx, (size_t)Hv * Wv));
+  TRY(ensure_infer_ws(ctx, ws, (size_t)Hv * Wv));
   const int Cp = ctx->Cp;
   auto WO = [&](int ci) { return sn.wo + ctx->convs[ci].pk_off; };
   auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
-  launch_pack_input_virtual(lr, n, p, ctx->x16, st);
+  launch_pack_input_virtual(lr, n, p, ws.x16, st);
   ctx->launches++;
   CKL();
-  TRY(roll_ex(ctx, "infer_v", 16, Cp, ctx->x16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ctx->f0, 1, Hv, Wv,
+  TRY(roll_ex(ctx, "infer_v", 16, Cp, ws.x16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ws.f0, 1, Hv, Wv,
               st));
-  bf16* cur = ctx->f0;
+  bf16* cur = ws.f0;
   for (int b = 0; b < ctx->B; ++b) {
-    bf16* nxt = (cur == ctx->fa) ? ctx->fb : ctx->fa;
+    bf16* nxt = (cur == ws.fa) ? ws.fb : ws.fa;
     if (ctx->fuse_blocks && resblock_supported(Cp, Wv)) {
       cudaError_t e = launch_resblock(Cp, cur, WO(1 + 2 * b), WO(2 + 2 * b), Bv(1 + 2 * b), Bv(2 + 2 * b), nxt, 1, Hv,
                                       Wv, st, nullptr, nullptr, sep);
       ctx->launches++;
       if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("resblock launch: ") + cudaGetErrorString(e));
     } else {
-      TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1, sep, ctx->tt,
+      TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1, sep, ws.tt,
                   1, Hv, Wv, st));
-      TRY(roll_ex(ctx, "infer_v", Cp, Cp, ctx->tt, WO(2 + 2 * b), Bv(2 + 2 * b), cur, nullptr, nullptr, 0, sep, nxt, 1,
+      TRY(roll_ex(ctx, "infer_v", Cp, Cp, ws.tt, WO(2 + 2 * b), Bv(2 + 2 * b), cur, nullptr, nullptr, 0, sep, nxt, 1,
                   Hv, Wv, st));
     }
     cur = nxt;
   }
   const int cb = 1 + 2 * ctx->B, cu = cb + 1;
-  bf16* gbuf = (cur == ctx->fa) ? ctx->fb : ctx->fa;
-  TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(cb), Bv(cb), ctx->f0, nullptr, nullptr, 0, sep, gbuf, 1, Hv, Wv, st));
+  bf16* gbuf = (cur == ws.fa) ? ws.fb : ws.fa;
+  TRY(roll_ex(ctx, "infer_v", Cp, Cp, cur, WO(cb), Bv(cb), ws.f0, nullptr, nullptr, 0, sep, gbuf, 1, Hv, Wv, st));
   EpiParams et{};
   et.bias = Bv(cu);
   et.scale = ctx->s;
@@ -806,6 +816,7 @@ static sr_status note_infer(sr_ctx* ctx, cudaStream_t st) {
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
   CK(cudaStreamIsCapturing(st, &cs));
   if (cs != cudaStreamCaptureStatusNone) return SR_OK;  // inside a caller's graph capture: the caller orders it
+  std::lock_guard<std::mutex> lk(ctx->ev_mu);
   for (auto& pe : ctx->infer_evs)
     if (pe.first == st) { CK(cudaEventRecord(pe.second, st)); return SR_OK; }
   cudaEvent_t e;
@@ -938,8 +949,10 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
 void sr_destroy(sr_ctx* ctx) {
   if (!ctx) return;
   cudaDeviceSynchronize();
-  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->x16, ctx->f0,
-                  ctx->fa, ctx->fb, ctx->tt, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
+  for (InferWS* ws : {&ctx->iws, &ctx->qws})
+    for (bf16* q : {ws->x16, ws->f0, ws->fa, ws->fb, ws->tt})
+      if (q) cudaFree(q);
+  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
                   ctx->zero_bias, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf, ctx->cell_sse};
@@ -1021,7 +1034,7 @@ int sr_kernel_stats(sr_ctx* ctx, char* buf, size_t cap) {
 
 const char* sr_last_error(const sr_ctx* ctx) { return ctx ? ctx->err.c_str() : "null ctx"; }
 size_t sr_num_params(const sr_ctx* ctx) { return ctx ? ctx->nparams : 0; }
-uint64_t sr_launch_count(const sr_ctx* ctx) { return ctx ? ctx->launches : 0; }
+uint64_t sr_launch_count(const sr_ctx* ctx) { return ctx ? ctx->launches.load() : 0ull; }
 float* sr_grad_buffer(sr_ctx* ctx) { return ctx ? ctx->grad : nullptr; }
 
 // Every call runs on the ctx's device (restored on return), so one process may drive ctxs on several GPUs.
@@ -1094,6 +1107,23 @@ sr_status sr_get_params(sr_ctx* ctx, sr_model which, float* host_out, size_t n) 
   return SR_OK;
 }
 
+// inference of n frames (or a batch of small square images) with snapshot `which` on workspace ws
+static sr_status infer_ws(sr_ctx* ctx, InferWS& ws, sr_model which, const uint8_t* lr_dev, int n, int h, int w,
+                          uint8_t* hr_dev, cudaStream_t st) {
+  if (which == SR_BILINEAR) {
+    cudaError_t e = launch_bilinear_u8(lr_dev, n, h, w, ctx->s, hr_dev, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, cudaGetErrorString(e));
+    return SR_OK;
+  }
+  CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
+  if (use_virtual_infer(ctx, n, h, w) && ctx->virtual_train)
+    TRY(forward_infer_virtual(ctx, ws, ctx->snap[which], lr_dev, n, h, hr_dev, st));
+  else
+    TRY(forward_infer(ctx, ws, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st));
+  return note_infer(ctx, st);
+}
+
 sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, int h, int w, uint8_t* hr_dev,
                    sr_stream stream) {
   GUARD();
@@ -1107,12 +1137,7 @@ sr_status sr_infer(sr_ctx* ctx, sr_model which, const uint8_t* lr_dev, int n, in
     return SR_OK;
   }
   if (!valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_infer: bad model");
-  CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
-  if (use_virtual_infer(ctx, n, h, w) && ctx->virtual_train)
-    TRY(forward_infer_virtual(ctx, ctx->snap[which], lr_dev, n, h, hr_dev, st));
-  else
-    TRY(forward_infer(ctx, ctx->snap[which], lr_dev, n, h, w, hr_dev, 0, h, st));
-  return note_infer(ctx, st);
+  return infer_ws(ctx, ctx->iws, which, lr_dev, n, h, w, hr_dev, st);
 }
 
 sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const uint8_t* u_dev,
@@ -1237,7 +1262,7 @@ sr_status sr_infer_rows(sr_ctx* ctx, sr_model which, const uint8_t* lr_full_dev,
   const int lo = std::max(0, row0 - halo), hi = std::min(h, row1 + halo);
   const int s = ctx->s;
   CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
-  TRY(forward_infer(ctx, ctx->snap[which], lr_full_dev + (size_t)lo * w * 3, 1, hi - lo, w,
+  TRY(forward_infer(ctx, ctx->iws, ctx->snap[which], lr_full_dev + (size_t)lo * w * 3, 1, hi - lo, w,
                     hr_full_dev + (size_t)lo * s * (size_t)s * w * 3, row0 - lo, row1 - lo, st));
   return note_infer(ctx, st);
 }
@@ -1450,8 +1475,11 @@ sr_status sr_publish(sr_ctx* ctx, sr_stream stream) {
   cudaStream_t st = (cudaStream_t)stream;
   // inference reading SERVE / PREV may be in flight on other streams: the snapshot copies wait for it (a frame is
   // never computed with a mix of old and new layer weights; the paper syncs inference at the epoch end, L1252-1253)
-  for (auto& pe : ctx->infer_evs)
-    if (pe.first != st) CK(cudaStreamWaitEvent(st, pe.second, 0));
+  {
+    std::lock_guard<std::mutex> lk(ctx->ev_mu);
+    for (auto& pe : ctx->infer_evs)
+      if (pe.first != st) CK(cudaStreamWaitEvent(st, pe.second, 0));
+  }
   TRY(ensure_full_train_pack(ctx, st));
   CK(cudaMemcpyAsync(ctx->snap[SR_PREV].wf, ctx->snap[SR_SERVE].wf, ctx->pk_total * sizeof(bf16),
                      cudaMemcpyDeviceToDevice, st));
@@ -1489,7 +1517,8 @@ static sr_status mean_psnr(sr_ctx* ctx, const sr_model* models, int k, const uin
   if ((size_t)k * n > (size_t)ctx->sse_n) { CK(dalloc(&ctx->sse, (size_t)k * n)); ctx->sse_n = k * n; }
   for (int m = 0; m < k; ++m) {
     // sse of model m is launched on st right after its inference, so val_a can be reused (stream order)
-    TRY(sr_infer(ctx, models[m], lr_dev, n, p, p, ctx->val_a, (sr_stream)st));
+    if (!(valid_model(models[m]) || models[m] == SR_BILINEAR)) return fail(ctx, SR_E_INVAL, "bad model");
+    TRY(infer_ws(ctx, ctx->qws, models[m], lr_dev, n, p, p, ctx->val_a, st));  // own workspace (training side)
     launch_sse_u8(ctx->val_a, hr_dev, n, (int64_t)per, ctx->sse + (size_t)m * n, st);
     ctx->launches++;
     CKL();

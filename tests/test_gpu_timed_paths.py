@@ -69,8 +69,9 @@ def test_bench_training_graph_matches_oracle_chain():
         assert abs(loss.item() - ref_loss) / ref_loss < 1e-2, (k, loss.item(), ref_loss)
         assert rel_l2(g, ref_g) < 1e-2, (k, rel_l2(g, ref_g))
         # (b) the Adam update itself: oracle Adam from the GPU's state with the GPU's gradient, t = k
+        # (fp32 state: beta2 = 0.999 is not representable, so 1 - beta2 carries a 1.3e-5 relative error into v)
         rp, rm, rv = O.adam_step(p_prev, m_prev, v_prev, g, k)
-        assert rel_l2(m_k, rm) < 1e-5 and rel_l2(v_k, rv) < 1e-5, (k, rel_l2(m_k, rm), rel_l2(v_k, rv))
+        assert rel_l2(m_k, rm) < 1e-5 and rel_l2(v_k, rv) < 1e-4, (k, rel_l2(m_k, rm), rel_l2(v_k, rv))
         assert rel_l2(p_k - p_prev, rp - p_prev) < 1e-3, (k, rel_l2(p_k - p_prev, rp - p_prev))
         # (c) the independent fp64 oracle chain from the same start (own gradients)
         _, cg = O.train_loss_and_grad(chain_p, blr, bhr, S, B, C)
