@@ -277,3 +277,23 @@ def test_binding_rejects_bad_tensors():
         ctx.infer(good, out=torch.empty((1, 32, 30, 3), dtype=torch.uint8, device="cuda"))
     with pytest.raises(SRError):
         ctx.train_step(good, torch.zeros((1, 16, 16, 3), dtype=torch.uint8, device="cuda"))
+
+
+@pytest.mark.parametrize("n,elems,off", [(1, 3840 * 2160 * 3, 0), (64, 180 * 180 * 3, 0), (5, 1001, 3), (3, 17, 1),
+                                         (2, 70000, 7)])
+def test_sse_u8_exact(n, elems, off):
+    """k_sse_u8 (Q1's integer SSE; multi-block, 16-B vector body, unaligned heads/tails) == numpy's exact int64 sum,
+    from a whole 4K frame pair (PSNR of a 4K frame) down to ragged items at odd byte offsets."""
+    import ctypes
+    from paper_conf_sigcomm_kimjyyh20_b200 import load
+    r = np.random.default_rng(elems + n)
+    a = r.integers(0, 256, n * elems + off, dtype=np.uint8)
+    b = r.integers(0, 256, n * elems + off, dtype=np.uint8)
+    b[off: off + elems // 2] = a[off: off + elems // 2]  # an identical half (a zero partial)
+    da, db = torch.from_numpy(a).cuda(), torch.from_numpy(b).cuda()
+    out = torch.zeros(n, dtype=torch.int64, device="cuda")
+    st = load().sr_sse_u8(ctypes.c_void_p(da.data_ptr() + off), ctypes.c_void_p(db.data_ptr() + off), n, elems,
+                          ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    assert st == 0
+    d = (a[off:off + n * elems].astype(np.int64) - b[off:off + n * elems].astype(np.int64)).reshape(n, elems)
+    np.testing.assert_array_equal(out.cpu().numpy(), (d * d).sum(axis=1))
