@@ -1749,16 +1749,16 @@ sr_status sr_test_adam(float* p_dev, float* m_dev, float* v_dev, const float* g_
                        float lr, sr_stream stream) {
   if (!p_dev || !m_dev || !v_dev || !g_dev || n == 0 || steps < 1) return SR_E_INVAL;
   cudaStream_t st = (cudaStream_t)stream;
-  long long* counters = nullptr;
-  if (cudaMalloc(&counters, 2 * sizeof(long long)) != cudaSuccess) return SR_E_NOMEM;
-  cudaMemsetAsync(counters, 0, 2 * sizeof(long long), st);
+  static long long* counters = nullptr;  // test-only step counters, kept for the process
+  if (!counters) {
+    if (cudaMalloc(&counters, 2 * sizeof(long long)) != cudaSuccess) return SR_E_NOMEM;
+    if (cudaMemset(counters, 0, 2 * sizeof(long long)) != cudaSuccess) return SR_E_CUDA;
+  }
   for (int k = 0; k < steps; ++k) {
     launch_adam(p_dev, m_dev, v_dev, g_dev, n, nullptr, 1.0f, counters, lr, 0.9f, 0.999f, 1e-8f, st);
     launch_counter_add(counters + 1, 1, st);  // t (the training path advances it in the repack)
   }
-  cudaError_t e = cudaStreamSynchronize(st);
-  cudaFree(counters);
-  return e == cudaSuccess ? SR_OK : SR_E_CUDA;
+  return cudaGetLastError() == cudaSuccess ? SR_OK : SR_E_CUDA;
 }
 
 sr_status sr_test_wgrad_batch(int J, const void* const* x_devs, const void* const* dy_devs, int n, int h, int w,

@@ -82,8 +82,7 @@ def run(argv=None):
 
     torch.cuda.set_device(0)
     dev = torch.device("cuda", 0)
-    lo_p, hi_p = torch.cuda.Stream.priority_range() if hasattr(torch.cuda.Stream, "priority_range") else (0, -1)
-    hi = torch.cuda.Stream(device=dev, priority=-1)   # inference (highest priority torch exposes)
+    hi = torch.cuda.Stream(device=dev, priority=-100)  # inference: clamped to the device's highest priority
     lo = torch.cuda.Stream(device=dev, priority=0)    # training
     h2d = torch.cuda.Stream(device=dev)
     d2h = torch.cuda.Stream(device=dev)
@@ -153,6 +152,7 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
     arrivals = sorted((i / FPS + st.k / (FPS * n), st.k, i) for st in ss for i in range(per))
     done_q = queue.Queue()
     lat = []
+    parts = []  # per timed frame: (issue lag, h2d done, sr done, d2h done) in ms after arrival
     stop = threading.Event()
     t_base = [0.0]
 
@@ -161,11 +161,13 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
             item = done_q.get()
             if item is None:
                 return
-            t_arr, ev, warm = item
+            t_arr, ev, warm, evs, t_iss = item
             while not ev.query():
                 time.sleep(0.0001)
             if not warm:
                 lat.append((time.perf_counter() - t_arr) * 1e3)
+                a_rel = (t_arr - t_base[0]) * 1e3
+                parts.append(((t_iss - t_arr) * 1e3,) + tuple(base_ev.elapsed_time(e) - a_rel for e in evs))
 
     train_log = {"issued": 0, "epochs": 0, "events": [], "q_dnn": []}
     ctrls = {st.k: Controller(thresh_sat=0.05, count_sat=2, thresh_online=0.5, count_online=2) for st in ss}
@@ -207,7 +209,11 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
     comp = threading.Thread(target=completer, daemon=True)
     comp.start()
     torch.cuda.synchronize()
+    base_ev = torch.cuda.Event(enable_timing=True)
     t_base[0] = time.perf_counter() + 0.05
+    while time.perf_counter() < t_base[0]:
+        pass
+    base_ev.record(h2d)  # device-time origin = host t_base (the copy stream is idle here)
     trn = None
     if not args.no_train:
         trn = threading.Thread(target=trainer, daemon=True)
@@ -220,24 +226,25 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
             time.sleep(t_arr - now)
         slot = st.frame % RING
         st.frame += 1
+        t_iss = time.perf_counter()
         with torch.cuda.stream(h2d):
             if st.slot_done[slot] is not None:
                 h2d.wait_event(st.slot_done[slot])   # the slot's previous frame has left the device
             st.lr_dev[slot].copy_(st.host_lr[i % RING], non_blocking=True)
-            e_in = torch.cuda.Event()
+            e_in = torch.cuda.Event(enable_timing=True)
             e_in.record()
         hi.wait_event(e_in)
         with torch.cuda.stream(hi):
             st.ctx.infer(st.lr_dev[slot:slot + 1], "serve", out=st.hr_dev[slot:slot + 1])
-            e_sr = torch.cuda.Event()
+            e_sr = torch.cuda.Event(enable_timing=True)
             e_sr.record()
         d2h.wait_event(e_sr)
         with torch.cuda.stream(d2h):
             st.host_hr[slot].copy_(st.hr_dev[slot], non_blocking=True)
-            e_out = torch.cuda.Event()
+            e_out = torch.cuda.Event(enable_timing=True)
             e_out.record()
         st.slot_done[slot] = e_out
-        done_q.put((t_arr, e_out, t < args.warm_seconds))
+        done_q.put((t_arr, e_out, t < args.warm_seconds, (e_in, e_sr, e_out), t_iss))
     t_end_issue = time.perf_counter()
     stop.set()
     if trn is not None:
@@ -257,7 +264,11 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
     p99 = float(np.percentile(lat_np, 99))
     train_ok = args.no_train or train_log["issued"] >= 0.95 * need
     drain_s = t_end - t_end_issue
+    pa = np.array(parts) if parts else np.zeros((1, 4))
+    comp_p99 = {k: round(float(np.percentile(pa[:, i], 99)), 3)
+                for i, k in enumerate(("issue_lag", "h2d_done", "sr_done", "d2h_done"))}
     return {"streams": n, "frames": int(lat_np.size), "p50_ms": round(float(np.percentile(lat_np, 50)), 3),
+            "p99_components_ms_after_arrival": comp_p99,
             "p99_ms": round(p99, 3), "max_ms": round(float(lat_np.max()), 3),
             "train_iters_issued": train_log["issued"], "train_iters_needed": int(need),
             "train_patches_per_s": round(train_log["issued"] * BATCH / max(window, 1e-9), 1),
