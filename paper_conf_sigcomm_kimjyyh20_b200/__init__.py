@@ -353,6 +353,23 @@ class SRContext:
     def set_fusion(self, fuse_blocks=True):
         check(self.lib.sr_set_fusion(self.h, int(fuse_blocks)), self.h, "sr_set_fusion")
 
+    @staticmethod
+    def sm_partition(train_sms):
+        """sr_sm_partition: (infer_stream, train_stream, infer_sms, train_sms) -- torch ExternalStreams whose kernels
+        run on disjoint SM partitions (green contexts); release with SRContext.sm_partition_release()."""
+        import torch
+        lib = load()
+        si, stt = C.c_void_p(), C.c_void_p()
+        ni, nt = C.c_int(0), C.c_int(0)
+        check(lib.sr_sm_partition(int(train_sms), C.byref(si), C.byref(stt), C.byref(ni), C.byref(nt)), None,
+              "sr_sm_partition")
+        return (torch.cuda.ExternalStream(si.value), torch.cuda.ExternalStream(stt.value), int(ni.value),
+                int(nt.value))
+
+    @staticmethod
+    def sm_partition_release():
+        check(load().sr_sm_partition_release(), None, "sr_sm_partition_release")
+
     def set_sm_split(self, train_sms):
         """sr_set_sm_split: training-side calls use train_sms SMs, inference-side calls the rest (0 = all)."""
         check(self.lib.sr_set_sm_split(self.h, int(train_sms)), self.h, "sr_set_sm_split")

@@ -80,6 +80,8 @@ _SIGS = {
     "sr_kernel_timing": (_I, [_P, _I]),
     "sr_set_fusion": (_I, [_P, _I]),
     "sr_set_sm_split": (_I, [_P, _I]),
+    "sr_sm_partition": (_I, [_I, C.POINTER(_P), C.POINTER(_P), C.POINTER(_I), C.POINTER(_I)]),
+    "sr_sm_partition_release": (_I, []),
     "sr_kernel_stats": (_I, [_P, C.c_char_p, C.c_size_t]),
     "sr_test_pack_input": (_I, [_P, _I, _I, _I, _P, _P]),
     "sr_test_conv": (_I, [_P, _I, _I, _I, _I, _I, _P, _P, _P, _P, _I, _I, _P, _P]),

@@ -10,6 +10,7 @@
 #include <dlfcn.h>
 #include <mutex>
 #include <atomic>
+#include <cuda.h>  // green-context types (driver entry points resolved through the runtime)
 #include <nccl.h>  // types only: libnccl is dlopen'ed at sr_create when world > 1 (libsr.so loads without it)
 #include "sr_internal.h"
 #include "kernels.h"
@@ -119,6 +120,7 @@ struct sr_ctx {
   int graph_batch = 0, graph_p = 0;
   float* graph_loss = nullptr;
   unsigned long long graph_kernels = 0;  // our kernels in one captured iteration
+  int graph_sm = 0;                      // sm_train (grid sizes) the graph was captured with
   unsigned long long ws_gen = 0, graph_gen = 0;
   // data parallelism (T5): NCCL communicator owned by the ctx (created from sr_options.nccl_id), sum of the ranks'
   // gradient weights (allreduced once at sr_create)
@@ -1430,7 +1432,7 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
   };
   // the captured graph bakes in the loss pointer and every workspace address: re-capture when any of them changed
   const bool stale = !ctx->train_graph || ctx->graph_batch != batch || ctx->graph_p != p ||
-                     ctx->graph_loss != loss_dev || ctx->graph_gen != ctx->ws_gen;
+                     ctx->graph_loss != loss_dev || ctx->graph_gen != ctx->ws_gen || ctx->graph_sm != ctx->sm_train;
   if (stale || st == nullptr) {
     if (lb > ctx->batch_bytes_lr) { CK(dalloc(&ctx->batch_lr, lb)); ctx->batch_bytes_lr = lb; ctx->ws_gen++; }
     if (hb > ctx->batch_bytes_hr) { CK(dalloc(&ctx->batch_hr, hb)); ctx->batch_bytes_hr = hb; ctx->ws_gen++; }
@@ -1456,6 +1458,7 @@ sr_status sr_train_sampled(sr_ctx* ctx, int iters, int batch, int p, float* loss
       ctx->graph_p = p;
       ctx->graph_loss = loss_dev;
       ctx->graph_gen = ctx->ws_gen;
+      ctx->graph_sm = ctx->sm_train;
     }
   }
   for (int it = 0; it < iters; ++it) {
@@ -1662,6 +1665,98 @@ sr_status sr_controller_step(sr_ctx* ctx, sr_controller* c, const uint8_t* lr_de
   r.event = ev;
   r.state_after = c->state;
   *out_host = r;
+  return SR_OK;
+}
+
+// ---- disjoint SM partitions for concurrent inference + training (green contexts; §7: the server runs
+// inference and online training side by side)
+}  // extern "C"
+namespace {
+struct GreenApi {
+  bool ok = false;
+  CUresult (*dev_get)(CUdevice*, int) = nullptr;
+  CUresult (*get_res)(CUdevice, CUdevResource*, CUdevResourceType) = nullptr;
+  CUresult (*split)(CUdevResource*, unsigned*, const CUdevResource*, CUdevResource*, unsigned, unsigned) = nullptr;
+  CUresult (*gen_desc)(CUdevResourceDesc*, CUdevResource*, unsigned) = nullptr;
+  CUresult (*create)(CUgreenCtx*, CUdevResourceDesc, CUdevice, unsigned) = nullptr;
+  CUresult (*to_ctx)(CUcontext*, CUgreenCtx) = nullptr;
+  CUresult (*stream)(CUstream*, CUgreenCtx, unsigned, int) = nullptr;
+  CUresult (*destroy)(CUgreenCtx) = nullptr;
+};
+template <class F>
+static bool entry(const char* name, F* fn) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || !p) return false;
+  *fn = reinterpret_cast<F>(p);
+  return true;
+}
+GreenApi& green() {
+  static GreenApi g;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    g.ok = entry("cuDeviceGet", &g.dev_get) && entry("cuDeviceGetDevResource", &g.get_res) &&
+           entry("cuDevSmResourceSplitByCount", &g.split) && entry("cuDevResourceGenerateDesc", &g.gen_desc) &&
+           entry("cuGreenCtxCreate", &g.create) && entry("cuCtxFromGreenCtx", &g.to_ctx) &&
+           entry("cuGreenCtxStreamCreate", &g.stream) && entry("cuGreenCtxDestroy", &g.destroy);
+  }
+  return g;
+}
+std::vector<CUgreenCtx> g_green;  // green contexts created by sr_sm_partition (destroyed by sr_sm_partition_release)
+std::mutex g_green_mu;
+}  // namespace
+extern "C" {
+
+sr_status sr_sm_partition(int train_sms, sr_stream* infer_stream, sr_stream* train_stream, int* infer_sms,
+                          int* train_sms_out) {
+  if (!infer_stream || !train_stream || train_sms < 1) return SR_E_INVAL;
+  GreenApi& g = green();
+  if (!g.ok) return SR_E_UNSUPPORTED;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaFree(nullptr) != cudaSuccess) return SR_E_CUDA;  // primary ctx up
+  CUdevice cd;
+  CUdevResource all{}, grp[1]{}, rest{};
+  unsigned nb = 1;
+  if (g.dev_get(&cd, dev) != CUDA_SUCCESS || g.get_res(cd, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS)
+    return SR_E_CUDA;
+  if (train_sms >= (int)all.sm.smCount) return SR_E_INVAL;
+  if (g.split(grp, &nb, &all, &rest, 0, (unsigned)train_sms) != CUDA_SUCCESS || nb != 1 || rest.sm.smCount == 0)
+    return SR_E_INVAL;  // (sm_90+: partitions are multiples of 8 SMs, >= 8)
+  CUdevResourceDesc dt, di;
+  CUgreenCtx gt, gi;
+  CUcontext ct, ci;
+  CUstream st_t, st_i;
+  int lo = 0, hi = 0;
+  cudaDeviceGetStreamPriorityRange(&lo, &hi);
+  if (g.gen_desc(&dt, grp, 1) != CUDA_SUCCESS || g.gen_desc(&di, &rest, 1) != CUDA_SUCCESS) return SR_E_CUDA;
+  if (g.create(&gt, dt, cd, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) return SR_E_CUDA;
+  if (g.create(&gi, di, cd, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) { g.destroy(gt); return SR_E_CUDA; }
+  if (g.to_ctx(&ct, gt) != CUDA_SUCCESS || g.to_ctx(&ci, gi) != CUDA_SUCCESS ||
+      g.stream(&st_t, gt, CU_STREAM_NON_BLOCKING, lo) != CUDA_SUCCESS ||
+      g.stream(&st_i, gi, CU_STREAM_NON_BLOCKING, hi) != CUDA_SUCCESS) {
+    g.destroy(gt);
+    g.destroy(gi);
+    return SR_E_CUDA;
+  }
+  {
+    std::lock_guard<std::mutex> lk(g_green_mu);
+    g_green.push_back(gt);
+    g_green.push_back(gi);
+  }
+  *train_stream = reinterpret_cast<sr_stream>(st_t);
+  *infer_stream = reinterpret_cast<sr_stream>(st_i);
+  if (train_sms_out) *train_sms_out = (int)grp[0].sm.smCount;
+  if (infer_sms) *infer_sms = (int)rest.sm.smCount;
+  return SR_OK;
+}
+
+sr_status sr_sm_partition_release(void) {
+  cudaDeviceSynchronize();
+  std::lock_guard<std::mutex> lk(g_green_mu);
+  GreenApi& g = green();
+  for (CUgreenCtx c : g_green) g.destroy(c);
+  g_green.clear();
   return SR_OK;
 }
 
