@@ -423,10 +423,15 @@ extern "C" int sr_bench_roll_dbg(int cinp, int coutp, int n, int h, int w, int r
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
-  launch_conv_roll_ex(cinp, coutp, x, wt, bias, res ? r : nullptr, nullptr, nullptr, !res, 0, y, n, h, w, st);  // warm
+  // res: 0 = bias + ReLU (forward conv1), 1 = bias + residual (forward conv2), 2 = data gradient with ReLU' mask and
+  // separator columns every 50 (the training dgrad shape)
+  const bf16* r1 = res == 1 ? r : nullptr;
+  const bf16* mk = res == 2 ? r : nullptr;
+  const int relu = res == 0, sep = res == 2 ? 50 : 0;
+  const float* bb = res == 2 ? nullptr : bias;
+  launch_conv_roll_ex(cinp, coutp, x, wt, bb, r1, nullptr, mk, relu, sep, y, n, h, w, st);  // warm
   cudaEventRecord(a, st);
-  cudaError_t e = launch_conv_roll_ex(cinp, coutp, x, wt, bias, res ? r : nullptr, nullptr, nullptr, !res, 0, y, n, h,
-                                      w, st, dbg);
+  cudaError_t e = launch_conv_roll_ex(cinp, coutp, x, wt, bb, r1, nullptr, mk, relu, sep, y, n, h, w, st, dbg);
   cudaEventRecord(b, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
   cudaEventElapsedTime(ms_out, a, b);

@@ -15,7 +15,7 @@ lib.sr_bench_roll_dbg.restype = C.c_int
 lib.sr_bench_roll_dbg.argtypes = [C.c_int] * 6 + [C.c_void_p, C.c_void_p, C.c_void_p]
 st = C.c_void_p(torch.cuda.current_stream().cuda_stream)
 for shape in ((1, 48, 3200), (8, 720, 1280)):
-    for res in (0, 1):
+    for res in (0, 1, 2):
         dbg = np.zeros(16 * 256, np.int64)
         ms = C.c_float()
         lib.sr_bench_roll_dbg(48, 48, *shape, res, dbg.ctypes.data_as(C.c_void_p), C.byref(ms), st)  # warm
@@ -24,6 +24,7 @@ for shape in ((1, 48, 3200), (8, 720, 1280)):
         t0 = d[8, 0]
         print(f"shape={shape} res={res} rc={rc} event-timed {ms.value * 1e3:.1f} us; CTA-0 cycles from entry:")
         print(f"  setup+pdl done {d[10, 0] - t0}, exit {d[9, 0] - t0}")
-        names = ["in_iss", "mma_st", "acq", "in_ok", "mma_iss", "ep_got", "ep_drained", "ep_stored"]
+        names = {0: "in_iss", 1: "mma_st", 2: "acq", 3: "in_ok", 4: "mma_iss", 5: "ep_got", 6: "ep_drained",
+                 11: "ep_slot", 12: "ep_staged", 13: "ep_fenced", 7: "ep_stored"}
         for i in range(0, 12):
-            print("  %3d " % i + " ".join(f"{nm}={(d[e, i] - t0) if d[e, i] else -1:7d}" for e, nm in enumerate(names)))
+            print("  %3d " % i + " ".join(f"{nm}={(d[e, i] - t0) if d[e, i] else -1:7d}" for e, nm in names.items()))
