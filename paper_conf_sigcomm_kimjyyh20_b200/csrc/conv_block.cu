@@ -123,15 +123,26 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
-  pdl_enter();
+  // Weights and biases were written at least two kernels upstream in every chain that launches this kernel (the
+  // library's repack / publish precede at least the head conv; the kernel that wrote them completed before our
+  // predecessor passed its own griddepcontrol.wait), so they are fetched and the bias-arming tiles built before the
+  // PDL wait: on SMs the predecessor has already left, this overlaps its tail, and after the wait the producer's
+  // first activation-row TMA goes out at once.
+  if (warp == 0 && lane_id() == 0) {
+    mbar_arrive_expect_tx(&w_bar, 2 * Cfg::WBYTES);
+    bulk_load(sW1, w1, Cfg::WBYTES, &w_bar);
+    bulk_load(sW2, w2, Cfg::WBYTES, &w_bar);
+  }
   if (threadIdx.x < C) {
     reinterpret_cast<float*>(sb1v)[threadIdx.x] = b1[threadIdx.x];
     reinterpret_cast<float*>(sb2v)[threadIdx.x] = b2[threadIdx.x];
   }
-  arm_tiles_fill(sOnes, sB1, b1, C, threadIdx.x, blockDim.x);
-  arm_tiles_fill(sOnes, sB2, b2, C, threadIdx.x, blockDim.x);
+  __syncthreads();
+  arm_tiles_fill(sOnes, sB1, reinterpret_cast<const float*>(sb1v), C, threadIdx.x, blockDim.x);
+  arm_tiles_fill(sOnes, sB2, reinterpret_cast<const float*>(sb2v), C, threadIdx.x, blockDim.x);
   fence_proxy_async_smem();
   __syncthreads();
+  pdl_enter();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
   const uint32_t ring1 = tmem, ring2 = tmem + 256;
@@ -153,9 +164,6 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     // ===================== producer: weights once, then f rows y0-2 .. y1+1 of every piece =====================
     if (elect_one()) {
       tma_prefetch_desc(&tm_f);
-      mbar_arrive_expect_tx(&w_bar, 2 * Cfg::WBYTES);
-      bulk_load(sW1, w1, Cfg::WBYTES, &w_bar);
-      bulk_load(sW2, w2, Cfg::WBYTES, &w_bar);
       int s = 0;
       uint32_t ph = 0;
       SR_PIECE_BEGIN

@@ -117,11 +117,17 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
-  pdl_enter();
+  // weights + biases before the PDL wait (written >= 2 kernels upstream; see k_resblock's prologue)
+  if (warp == 0 && lane_id() == 0) {
+    mbar_arrive_expect_tx(&w_bar, Cfg::W1B + Cfg::W2B);
+    bulk_load(sW1, w1, Cfg::W1B, &w_bar);
+    bulk_load(sW2, w2, Cfg::W2B, &w_bar);
+  }
   arm_tiles_fill(sOnes, sB1, a.b1, C, threadIdx.x, blockDim.x);
   arm_tiles_fill(sOnes, sB2, a.b2, CO2, threadIdx.x, blockDim.x);
   fence_proxy_async_smem();
   __syncthreads();
+  pdl_enter();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
   const uint32_t ring1 = tmem, ring2 = tmem + Cfg::R2BASE;
@@ -144,9 +150,6 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     if (elect_one()) {
       tma_prefetch_desc(&tm_f);
       tma_prefetch_desc(&tm_lr);
-      mbar_arrive_expect_tx(&w_bar, Cfg::W1B + Cfg::W2B);
-      bulk_load(sW1, w1, Cfg::W1B, &w_bar);
-      bulk_load(sW2, w2, Cfg::W2B, &w_bar);
       int s = 0, ls = 0;
       uint32_t ph = 0, lph = 0;
       SR_PIECE_BEGIN

@@ -100,9 +100,16 @@ __device__ __forceinline__ void ld_row(const bf16* base, uint4* dst) {
 // (aux row) -> 0 in separator columns -> bf16.  M: variant bits (1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU);
 // M = 32: generic body, the variant is read from em at run time.
 template <int COUTP, int M>
-__device__ __forceinline__ void roll_stage(uint4* orow, const float* v, const uint4* aux, const uint4* r2, bool sep0,
-                                           int em) {
+__device__ __forceinline__ void roll_stage(uint4* __restrict__ orow, const float* v, const uint4* __restrict__ aux_s,
+                                           const uint4* r2, bool sep0, int em) {
   const int mm = (M & 32) ? em : M;
+  // the whole aux row (residual or mask) into registers first: the staging stores below could alias it for the
+  // compiler, which would otherwise serialise every 16-B load behind the previous chunk's store
+  uint4 aux[COUTP / 8];
+  if (mm & 5) {
+#pragma unroll
+    for (int j = 0; j < COUTP / 8; ++j) aux[j] = aux_s[j];
+  }
 #pragma unroll
   for (int j = 0; j < COUTP / 8; ++j) {
     float o[8];
@@ -169,7 +176,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   uint8_t* sOnes = sA + NAUX * ROWB;  // ring.cuh: ones x bias MMA arms a ring block
   uint8_t* sBt = sOnes + kArmOnesBytes;
   __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
-      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar, l_full[TS > 0 ? Cfg::NLR : 1],
+      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar, arm_bar, l_full[TS > 0 ? Cfg::NLR : 1],
       l_empty[TS > 0 ? Cfg::NLR : 1], u_full[U8 ? kU8Slots : 1], u_empty[U8 ? kU8Slots : 1];
   // the aux row (res1 or mask) travels by TMA; res2 (used once per backward pass) by plain loads
   const bool has_aux = a.res1 != nullptr || a.mask != nullptr;
@@ -189,6 +196,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     if (U8)
       for (int s = 0; s < kU8Slots; ++s) { mbar_init(&u_full[s], 1); mbar_init(&u_empty[s], 1); }
     mbar_init(&w_bar, 1);
+    mbar_init(&arm_bar, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
@@ -205,21 +213,33 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   // library's forward / backward chains: the kernel that packed them has completed before our predecessor passed its
   // own griddepcontrol.wait, i.e. before we were scheduled), so they are fetched before the PDL wait and the fetch
   // overlaps the predecessor's tail.  Everything the predecessor writes (activations) is read only after the wait.
-  auto load_params = [&]() {
-    if (threadIdx.x == 0) {
+  // The weights go by one bulk copy (producer thread); the bias and the ring-arming tiles are prepared by the epilogue
+  // and store warps (2..10) alone and announced to the MMA issuer through arm_bar, so the producer's first input-row
+  // TMAs are not queued behind the bias load and the tile fill.
+  if (warp == 0 && lane_id() == 0 && a.w_early) {
+    mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
+    bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
+  }
+  constexpr uint32_t kArmThreads = 9 * 32;  // warps 2..10
+  auto arm_params = [&]() {
+    const int t = (int)threadIdx.x - 64;
+    if (t < COUTP) reinterpret_cast<float*>(sbv)[t] = a.bias ? a.bias[t] : 0.f;
+    named_bar_sync(1, kArmThreads);
+    arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, t, kArmThreads);
+    fence_proxy_async_smem();
+    named_bar_sync(1, kArmThreads);
+    if (t == 0) mbar_arrive(&arm_bar);
+  };
+  if (a.w_early && warp >= 2 && warp <= 10) arm_params();
+  pdl_enter();  // predecessor complete: global inputs are valid from here on
+  if (threadIdx.x == 0) { SR_RDBG(10, 0) }  // after setup + PDL wait
+  if (!a.w_early) {
+    if (warp == 0 && lane_id() == 0) {
       mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
       bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
     }
-    if (threadIdx.x < COUTP) reinterpret_cast<float*>(sbv)[threadIdx.x] = a.bias ? a.bias[threadIdx.x] : 0.f;
-    __syncthreads();
-    arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, threadIdx.x, blockDim.x);
-    fence_proxy_async_smem();
-    __syncthreads();
-  };
-  if (a.w_early) load_params();
-  pdl_enter();  // predecessor complete: global inputs are valid from here on
-  if (threadIdx.x == 0) { SR_RDBG(10, 0) }  // after setup + PDL wait
-  if (!a.w_early) load_params();
+    if (warp >= 2 && warp <= 10) arm_params();
+  }
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
 
@@ -276,6 +296,8 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     // ===================== MMA issuer =====================
     if (elect_one()) {
       mbar_wait(&w_bar, 0);
+      mbar_wait(&arm_bar, 0);  // bias-arming tiles in place
+      tc_fence_after();
       const uint64_t bd = make_desc(smem_u32(sW), 3 * COUTP * 16, 128);
       int s = 0;
       uint32_t ph = 0;
