@@ -127,7 +127,7 @@ class ClockSampler:
 def _roofline(stats, cls, peak, peak_kind, traffic=None):
     v = stats[cls]
     achieved = v["flops"] / (v["ms"] * 1e-3) / 1e12
-    return {"bound": "tensor", "kernel": cls, "achieved": round(achieved, 1), "peak": peak, "unit": "TFLOP/s",
+    return {"bound": "tensor", "kernel": cls, "achieved": round(achieved, 1), "peak": round(peak, 1), "unit": "TFLOP/s",
             "frac": round(achieved / peak, 4), "peak_kind": peak_kind, "traffic": traffic,
             "traffic_unit": "bytes per launch (ncu dram read+write)",
             "algorithmic_bytes": round(v["bytes"] / v["launches"]), "launches": v["launches"],
@@ -153,7 +153,21 @@ def run_ours(args):
     # the DP group's NCCL communicator lives in the library (sr_options.nccl_id): rank 0 draws the id
     nccl_id = nccl_id_broadcast() if world > 1 else None
     ctx = SRContext(S, BLOCKS, CH, seed=0, world=world, rank=rank, nccl_id=nccl_id)
-    stream = torch.cuda.Stream(device=dev)  # the compute stream every call is issued on (events record on it)
+    stream = torch.cuda.Stream(device=dev)  # whole-GPU stream (setup, cfg4, cfg2)
+    # The step's inference and training run concurrently on disjoint SM partitions (sr_sm_partition, green contexts:
+    # the paper's server runs inference and online training side by side, §7): inference on `s_inf`,
+    # patch arrivals + training + publish + Algorithm 1 on `s_tr`; --partition 0 issues both on one stream instead.
+    part = None
+    if args.partition > 0:
+        try:
+            s_inf, s_tr, n_inf, n_tr = SRContext.sm_partition(args.partition)
+            ctx.set_sm_split(n_tr)
+            part = {"train_sms": n_tr, "infer_sms": n_inf}
+        except Exception as exc:  # noqa: BLE001 -- e.g. a driver without green contexts
+            print(f"[bench] SM partition unavailable ({exc}); sequential step", file=sys.stderr, flush=True)
+            part = {"error": str(exc)}
+    if part is None or "error" in part:
+        s_inf = s_tr = stream
     # ---- synthetic inputs (seeded; per-rank frame shard; every rank holds the same pool and samples its chunk)
     lr_np = synth_frames(frames, LR_H, LR_W, seed=1003 + rank)
     lr = torch.from_numpy(lr_np).to(dev)
@@ -168,16 +182,17 @@ def run_ours(args):
     state = {"q": None, "iters": 0, "epochs": 0, "arr": 0, "events": []}
     with torch.cuda.stream(stream):
         ctx.pool_push(torch.from_numpy(plr).to(dev), torch.from_numpy(phr).to(dev))
+    torch.cuda.synchronize()  # the pool is filled before the training stream samples it
     ctrl = Controller(thresh_sat=0.05, count_sat=2, thresh_online=0.5, count_online=2)
 
     def arrive():
         a = state["arr"] % (n_arr // ARRIVALS_PER_STEP)
         sl = slice(a * ARRIVALS_PER_STEP, (a + 1) * ARRIVALS_PER_STEP)
-        ctx.pool_push(arr_lr[sl], arr_hr[sl])
+        ctx.pool_push(arr_lr[sl], arr_hr[sl], stream=s_tr)
         state["arr"] += 1
 
     def epoch_eval():
-        r = ctx.controller_step(ctrl, val_lr, val_hr)
+        r = ctx.controller_step(ctrl, val_lr, val_hr, stream=s_tr)
         if r["event"]:
             state["events"].append(r["event"])
         if ctrl.state != "training":  # constant-work mode (see the docstring): keep training every epoch
@@ -186,15 +201,15 @@ def run_ours(args):
         state["epochs"] += 1
 
     def train_iters():
-        ctx.train_sampled(args.iters, BATCH, PATCH, loss)  # library-captured graph, replayed args.iters times
+        ctx.train_sampled(args.iters, BATCH, PATCH, loss, stream=s_tr)  # library-captured graph, replayed
         state["iters"] += args.iters
         if state["iters"] >= EPOCH_ITERS:  # epoch end (50 iterations, L1247-1250): publish + Algorithm 1
             state["iters"] = 0
-            ctx.publish()
+            ctx.publish(stream=s_tr)  # waits for the inference in flight on s_inf (sr_publish)
             epoch_eval()
 
     def step():
-        ctx.infer(lr, "serve", out=hr)
+        ctx.infer(lr, "serve", out=hr, stream=s_inf)
         arrive()
         train_iters()
 
@@ -203,9 +218,21 @@ def run_ours(args):
             dist.barrier()
         torch.cuda.synchronize()
 
-    with torch.cuda.stream(stream):
-        for _ in range(args.warmup):
-            step()
+    def t_start():
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(s_inf)
+        s_tr.wait_event(e)
+        return e
+
+    def t_stop(e0):
+        ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ea.record(s_inf)
+        eb.record(s_tr)
+        torch.cuda.synchronize()
+        return max(e0.elapsed_time(ea), e0.elapsed_time(eb))
+
+    for _ in range(args.warmup):
+        step()
     barrier()
     state["iters"], state["epochs"], state["events"] = 0, 0, []  # the timed region starts at an epoch boundary
     clk = ClockSampler(local)
@@ -213,14 +240,11 @@ def run_ours(args):
     l0 = ctx.launches
     ctx.kernel_timing(True)
     barrier()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with torch.cuda.stream(stream):
-        e0.record()
-        for _ in range(args.steps):
-            step()
-        e1.record()
+    e0 = t_start()
+    for _ in range(args.steps):
+        step()
+    ms = t_stop(e0)
     barrier()
-    ms = e0.elapsed_time(e1)
     epochs_timed = state["epochs"]
     launches = ctx.launches - l0
     stats = ctx.kernel_stats()
@@ -238,27 +262,26 @@ def run_ours(args):
     loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
 
     def step_e2e():
-        # a serving loop: frames in and out through the host API; patch arrivals and the training iterations are
-        # enqueued behind the inference and run while the last HR chunks drain over PCIe; the step ends when its HR
-        # frames are in host memory (sr_infer_host_wait) and its loss has been read back
-        ctx.infer_host_async(lr_host, hr_host, "serve")
+        # a serving loop: frames in and out through the host API (H2D / SR / D2H pipelined by the library on the
+        # inference stream); patch arrivals and the training iterations run beside it on the training stream; the
+        # step ends when its HR frames are in host memory (sr_infer_host_wait) and its loss has been read back
+        ctx.infer_host_async(lr_host, hr_host, "serve", stream=s_inf)
         arrive()
         train_iters()
-        loss_host.copy_(loss, non_blocking=True)
+        with torch.cuda.stream(s_tr):
+            loss_host.copy_(loss, non_blocking=True)
         ctx.infer_host_wait()
 
-    with torch.cuda.stream(stream):
-        step_e2e()
+    step_e2e()
     barrier()
     state["iters"] = 0
-    e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with torch.cuda.stream(stream):
-        e2.record()
-        for _ in range(args.steps):
-            step_e2e()
-        e3.record()
+    e2 = t_start()
+    for _ in range(args.steps):
+        step_e2e()
+    ms_e2e = max_over_ranks(t_stop(e2), device=dev)
     barrier()
-    ms_e2e = max_over_ranks(e2.elapsed_time(e3), device=dev)
+    if part is not None and "error" not in part:
+        ctx.set_sm_split(0)  # the rest runs on the whole GPU
 
     # ---- config 4: training alone at the maximum rate (sampled iterations from the captured graph)
     n_tr = 100
@@ -322,6 +345,13 @@ def run_ours(args):
         sustained = pk.get("bf16_tflops_sustained") or 1393.0
         pk_kind = "measured bf16_tflops_sustained (MEASURED_PEAKS.json)"
         dom = max(stats.items(), key=lambda kv: kv[1]["ms"])[0]
+        # with the SM partition the inference kernels run on infer_sms of the SMs: their roofline peak is that share
+        # of the measured whole-GPU peak
+        inf_share, inf_note = 1.0, ""
+        if part is not None and "error" not in part:
+            nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+            inf_share = part["infer_sms"] / nsm
+            inf_note = f" x {part['infer_sms']}/{nsm} SMs (the inference partition the kernel ran on)"
         ktot = sum(v["ms"] for v in stats.values())
         total_frames = frames * args.steps * world
         fps = total_frames / (ms * 1e-3)
@@ -343,6 +373,9 @@ def run_ours(args):
             "dtype": "bf16",
             "data": "synthetic (seeded 1/f frames + edges + strokes, pan; random-init weights)",
             "config": workload_config(frames, args.iters, world),
+            "concurrency": ({"mode": "inference and training on disjoint SM partitions (green contexts)", **part}
+                            if part is not None and "error" not in part else
+                            {"mode": "sequential on one stream", **(part or {})}),
             "train_patches_per_s": round(BATCH * args.iters * args.steps * world / (ms * 1e-3), 1),
             "quality_gain_db": round(state["q"]["q_dnn"], 4) if state["q"] else None,
             "alg1": alg1,
@@ -350,7 +383,7 @@ def run_ours(args):
             "kernel_share": {k: round(v["ms"] / ktot, 4) for k, v in sorted(stats.items(), key=lambda kv: -kv[1]["ms"])},
             "kernel_share_note": "CUDA-event time per kernel class of the eagerly launched kernels (inference, "
                                  "Algorithm-1 evaluation); the graph-replayed training kernels are in cfg4",
-            "roofline": _roofline(stats, dom, sustained, pk_kind, traffic_of(dom, frames)),
+            "roofline": _roofline(stats, dom, sustained * inf_share, pk_kind + inf_note, traffic_of(dom, frames)),
             "e2e": {"value": round(fps_e2e, 3), "unit": "frames/s",
                     "h2d_bytes_per_step": int(lr_host.numel()),
                     "d2h_bytes_per_step": int(hr_host.numel() + loss_host.numel() * 4)},
@@ -386,6 +419,8 @@ def run_ours(args):
         if not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline()
         print(json.dumps(line), flush=True)
+    if part is not None and "error" not in part:
+        SRContext.sm_partition_release()
     if world > 1:
         dist.destroy_process_group()
 
@@ -523,6 +558,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cfg2", action="store_true")
     ap.add_argument("--workload", choices=["cfg3", "live"], default="cfg3")
+    ap.add_argument("--partition", type=int, default=40,
+                    help="SMs of the training partition (green contexts); 0 = inference and training sequential")
     ap.add_argument("--ref-band", type=int, default=REF_BAND, help=argparse.SUPPRESS)
     args = ap.parse_args()
     if args.warmup < 3:

@@ -242,6 +242,16 @@ void launch_pack_weights(const float* params, const ConvDesc* convs_dev, int nco
 
 // k_adam computes the bias corrections itself from the device step counter: t = counters[1] + 1 (the counter is
 // advanced by the TRAIN repack that follows, k_pack_weights' bump) -- one launch less per training iteration.
+// HBM-bound (28 B per parameter): 16-B vector accesses for the 4-aligned body (the buffers are cudaMalloc'd), the
+// n % 4 tail by the first threads; grid = enough blocks for ~8 per SM, grid-strided.
+__device__ __forceinline__ float adam1(float& p, float& m, float& v, float g, float b1, float b2, float lr_bc1,
+                                       float inv_sqrt_bc2, float eps) {
+  m = fmaf(b1, m, (1.f - b1) * g);
+  v = fmaf(b2, v, (1.f - b2) * g * g);
+  p -= lr_bc1 * m / (sqrtf(v) * inv_sqrt_bc2 + eps);
+  return p;
+}
+
 __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
                        const float* __restrict__ grad, size_t n, const float* __restrict__ gscale_dev, float gscale,
                        const long long* __restrict__ counters, double lr, float b1, float b2, float eps) {
@@ -255,24 +265,34 @@ __global__ void k_adam(float* __restrict__ p, float* __restrict__ m, float* __re
   __syncthreads();
   const float gs = gscale * (gscale_dev ? *gscale_dev : 1.f);
   const float lr_bc1 = s_bc[0], inv_sqrt_bc2 = s_bc[1];
-  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t n4 = n / 4;
+  float4* p4 = reinterpret_cast<float4*>(p);
+  float4* m4 = reinterpret_cast<float4*>(m);
+  float4* v4 = reinterpret_cast<float4*>(v);
+  const float4* g4 = reinterpret_cast<const float4*>(grad);
   const size_t stride = (size_t)gridDim.x * blockDim.x;
-  for (; i < n; i += stride) {
-    const float g = grad[i] * gs;
-    const float mi = fmaf(b1, m[i], (1.f - b1) * g);
-    const float vi = fmaf(b2, v[i], (1.f - b2) * g * g);
-    m[i] = mi;
-    v[i] = vi;
-    p[i] -= lr_bc1 * mi / (sqrtf(vi) * inv_sqrt_bc2 + eps);
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
+    float4 pp = p4[i], mm = m4[i], vv = v4[i];
+    const float4 gg = __ldg(g4 + i);
+    adam1(pp.x, mm.x, vv.x, gg.x * gs, b1, b2, lr_bc1, inv_sqrt_bc2, eps);
+    adam1(pp.y, mm.y, vv.y, gg.y * gs, b1, b2, lr_bc1, inv_sqrt_bc2, eps);
+    adam1(pp.z, mm.z, vv.z, gg.z * gs, b1, b2, lr_bc1, inv_sqrt_bc2, eps);
+    adam1(pp.w, mm.w, vv.w, gg.w * gs, b1, b2, lr_bc1, inv_sqrt_bc2, eps);
+    p4[i] = pp;
+    m4[i] = mm;
+    v4[i] = vv;
   }
+  const size_t i = 4 * n4 + (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) adam1(p[i], m[i], v[i], grad[i] * gs, b1, b2, lr_bc1, inv_sqrt_bc2, eps);
 }
 
 void launch_adam(float* p, float* m, float* v, const float* g, size_t n, const float* gscale_dev, float gscale,
                  const long long* counters, double lr, float b1, float b2, float eps, cudaStream_t st) {
   int th = 256;
-  int blocks = (int)((n + th - 1) / th);
-  if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
-  launch_k(k_adam, dim3(blocks), dim3(th), 0, st, p, m, v, g, n, gscale_dev, gscale, counters, lr, b1, b2, eps);
+  long long blocks = (long long)((n / 4 + th - 1) / th);
+  blocks = std::max<long long>(1, std::min<long long>(blocks, 8LL * num_sms()));
+  launch_k(k_adam, dim3((unsigned)blocks), dim3(th), 0, st, p, m, v, g, n, gscale_dev, gscale, counters, lr, b1, b2,
+           eps);
 }
 
 __global__ void k_counter_add(long long* c, long long d) {
