@@ -225,11 +225,13 @@ def run_ours(args):
         return e
 
     def t_stop(e0):
-        ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ea.record(s_inf)
-        eb.record(s_tr)
+        evs = []
+        for s_ in (s_inf, s_tr, stream):
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record(s_)
+            evs.append(ev)
         torch.cuda.synchronize()
-        return max(e0.elapsed_time(ea), e0.elapsed_time(eb))
+        return max(e0.elapsed_time(ev) for ev in evs)
 
     for _ in range(args.warmup):
         step()
@@ -258,26 +260,33 @@ def run_ours(args):
 
     # ---- end-to-end: host (pinned) frames in, host frames out, through the C ABI (sr_infer_host_async)
     lr_host = torch.from_numpy(lr_np).pin_memory()
-    hr_host = torch.empty((frames, S * LR_H, S * LR_W, 3), dtype=torch.uint8).pin_memory()
+    hr_hosts = [torch.empty((frames, S * LR_H, S * LR_W, 3), dtype=torch.uint8).pin_memory() for _ in range(2)]
+    hr_host = hr_hosts[0]
     loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
+    nstep = [0]
 
     def step_e2e():
-        # a serving loop: frames in and out through the host API (H2D / SR / D2H pipelined by the library on the
-        # inference stream); patch arrivals and the training iterations run beside it on the training stream; the
-        # step ends when its HR frames are in host memory (sr_infer_host_wait) and its loss has been read back
-        ctx.infer_host_async(lr_host, hr_host, "serve", stream=s_inf)
+        # a serving loop: frames in and out through the host API (sr_infer_host_async: H2D / SR / D2H pipelined by
+        # the library, two batches in flight into two host output buffers); patch arrivals and the training
+        # iterations run beside it on the training stream and the step's loss is read back to the host
+        ctx.infer_host_async(lr_host, hr_hosts[nstep[0] & 1], "serve", stream=s_inf)
+        nstep[0] += 1
         arrive()
         train_iters()
-        with torch.cuda.stream(s_tr):
+        ev = torch.cuda.Event()
+        ev.record(s_tr)
+        stream.wait_event(ev)
+        with torch.cuda.stream(stream):
             loss_host.copy_(loss, non_blocking=True)
-        ctx.infer_host_wait()
 
     step_e2e()
+    ctx.infer_host_wait()
     barrier()
     state["iters"] = 0
     e2 = t_start()
     for _ in range(args.steps):
         step_e2e()
+    ctx.infer_host_wait()  # every step's HR frames are in host memory before the region closes
     ms_e2e = max_over_ranks(t_stop(e2), device=dev)
     barrier()
     if part is not None and "error" not in part:
@@ -419,8 +428,7 @@ def run_ours(args):
         if not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline()
         print(json.dumps(line), flush=True)
-    if part is not None and "error" not in part:
-        SRContext.sm_partition_release()
+    # (the SM partitions stay until process exit: torch may still record events on their streams at teardown)
     if world > 1:
         dist.destroy_process_group()
 

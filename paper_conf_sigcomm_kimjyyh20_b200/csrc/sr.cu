@@ -78,11 +78,15 @@ struct sr_ctx {
   bool virtual_train = true; // training on the virtual wide batch with the rolling kernels
   // inference workspaces: frames, quality evaluation
   InferWS iws, qws;
-  uint8_t *stage_lr = nullptr, *stage_hr = nullptr;
+  // sr_infer_host(_async): two staging sets used alternately, so two calls can be in flight (call k+1's H2D and
+  // compute queue behind call k's while its D2H drains); a call waits only for the call that last used its set
+  uint8_t *stage_lr[2] = {nullptr, nullptr}, *stage_hr[2] = {nullptr, nullptr};
   cudaStream_t copy_st = nullptr, h2d_st = nullptr;  // sr_infer_host: PCIe copies overlapped with the tensor work
-  std::vector<cudaEvent_t> chunk_ev;
-  bool host_pending = false;  // an sr_infer_host_async call whose D2H copies may still be in flight
-  size_t stage_lr_bytes = 0, stage_hr_bytes = 0;
+  std::vector<cudaEvent_t> chunk_ev[2];
+  cudaEvent_t host_done[2] = {nullptr, nullptr};  // last D2H of the call that used the set
+  bool host_busy[2] = {false, false};
+  unsigned long long host_calls = 0;
+  size_t stage_lr_bytes[2] = {0, 0}, stage_hr_bytes[2] = {0, 0};
   // training workspace
   size_t tr_pix = 0;
   bf16 *tx16 = nullptr, *tg = nullptr, *tdy = nullptr, *tdg = nullptr, *tdfa = nullptr, *tdfb = nullptr,
@@ -954,7 +958,13 @@ void sr_destroy(sr_ctx* ctx) {
   for (InferWS* ws : {&ctx->iws, &ctx->qws})
     for (bf16* q : {ws->x16, ws->f0, ws->fa, ws->fb, ws->tt})
       if (q) cudaFree(q);
-  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->stage_lr, ctx->stage_hr, ctx->tx16, ctx->tg, ctx->tdy,
+  for (int k = 0; k < 2; ++k) {
+    if (ctx->stage_lr[k]) cudaFree(ctx->stage_lr[k]);
+    if (ctx->stage_hr[k]) cudaFree(ctx->stage_hr[k]);
+    for (auto e : ctx->chunk_ev[k]) if (e) cudaEventDestroy(e);
+    if (ctx->host_done[k]) cudaEventDestroy(ctx->host_done[k]);
+  }
+  void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
                   ctx->zero_bias, ctx->pool_lr,
                   ctx->pool_hr, ctx->batch_lr, ctx->batch_hr, ctx->val_a, ctx->sse, ctx->yuv_lr, ctx->yuv_hr, ctx->crop_buf, ctx->cell_sse};
@@ -969,7 +979,6 @@ void sr_destroy(sr_ctx* ctx) {
   for (auto& pe : ctx->infer_evs) cudaEventDestroy(pe.second);
   if (ctx->comm) nccl().destroy(ctx->comm);
   if (ctx->train_graph) cudaGraphExecDestroy(ctx->train_graph);
-  for (auto e : ctx->chunk_ev) if (e) cudaEventDestroy(e);
   if (ctx->copy_st) cudaStreamDestroy(ctx->copy_st);
   if (ctx->h2d_st) cudaStreamDestroy(ctx->h2d_st);
   for (auto& r : ctx->trec) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
@@ -1168,18 +1177,23 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
                                  uint8_t* hr_host, sr_stream stream, bool sync) {
   CAP_INFER();
   if (!lr_host || !hr_host || n < 1 || h < 1 || w < 1) return fail(ctx, SR_E_INVAL, "sr_infer_host: bad args");
-  if (ctx->host_pending) {  // the staging buffers and chunk events are reused: finish the previous async call
-    CK(cudaStreamSynchronize(ctx->copy_st));
-    ctx->host_pending = false;
+  const int set = (int)(ctx->host_calls & 1);
+  if (ctx->host_busy[set]) {  // the call two back used this staging set: its D2H copies must have drained
+    CK(cudaEventSynchronize(ctx->host_done[set]));
+    ctx->host_busy[set] = false;
   }
   cudaStream_t st = (cudaStream_t)stream;
   const size_t fl = (size_t)h * w * 3, fh = fl * ctx->s * ctx->s;
   const size_t lb = (size_t)n * fl, hb = (size_t)n * fh;
-  if (lb > ctx->stage_lr_bytes) { CK(dalloc(&ctx->stage_lr, lb)); ctx->stage_lr_bytes = lb; }
-  if (hb > ctx->stage_hr_bytes) { CK(dalloc(&ctx->stage_hr, hb)); ctx->stage_hr_bytes = hb; }
+  if (lb > ctx->stage_lr_bytes[set]) { CK(dalloc(&ctx->stage_lr[set], lb)); ctx->stage_lr_bytes[set] = lb; }
+  if (hb > ctx->stage_hr_bytes[set]) { CK(dalloc(&ctx->stage_hr[set], hb)); ctx->stage_hr_bytes[set] = hb; }
+  uint8_t* const stage_lr = ctx->stage_lr[set];
+  uint8_t* const stage_hr = ctx->stage_hr[set];
   if (!ctx->copy_st) {
     CK(cudaStreamCreateWithFlags(&ctx->copy_st, cudaStreamNonBlocking));
     CK(cudaStreamCreateWithFlags(&ctx->h2d_st, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&ctx->host_done[0], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ctx->host_done[1], cudaEventDisableTiming));
   }
   // Chunked pipeline: all H2D copies go first on their own stream (per-chunk events), chunk k is super-resolved
   // on `stream` as soon as its frames landed, and its D2H runs on a third stream while chunk k+1 computes.
@@ -1201,32 +1215,34 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
     }
   }
   const int nch = (int)c0s.size() - 1;
-  while ((int)ctx->chunk_ev.size() < 2 * nch + 1) {
+  while ((int)ctx->chunk_ev[set].size() < 2 * nch + 1) {
     cudaEvent_t e;
     CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    ctx->chunk_ev.push_back(e);
+    ctx->chunk_ev[set].push_back(e);
   }
-  cudaEvent_t* ev = ctx->chunk_ev.data();  // [0] start, [1 + c] chunk c landed, [1 + nch + c] chunk c done
+  cudaEvent_t* ev = ctx->chunk_ev[set].data();  // [0] start, [1 + c] chunk c landed, [1 + nch + c] chunk c done
   CK(cudaEventRecord(ev[0], st));
   CK(cudaStreamWaitEvent(ctx->h2d_st, ev[0], 0));  // copies follow earlier work on `stream`
   CK(cudaStreamWaitEvent(ctx->copy_st, ev[0], 0));
   for (int c = 0; c < nch; ++c) {
     const int f0 = c0s[c], fn = c0s[c + 1] - c0s[c];
-    CK(cudaMemcpyAsync(ctx->stage_lr + f0 * fl, lr_host + f0 * fl, fn * fl, cudaMemcpyHostToDevice, ctx->h2d_st));
+    CK(cudaMemcpyAsync(stage_lr + f0 * fl, lr_host + f0 * fl, fn * fl, cudaMemcpyHostToDevice, ctx->h2d_st));
     CK(cudaEventRecord(ev[1 + c], ctx->h2d_st));
   }
   for (int c = 0; c < nch; ++c) {
     const int f0 = c0s[c], fn = c0s[c + 1] - c0s[c];
     CK(cudaStreamWaitEvent(st, ev[1 + c], 0));
-    TRY(sr_infer(ctx, which, ctx->stage_lr + f0 * fl, fn, h, w, ctx->stage_hr + f0 * fh, stream));
+    TRY(sr_infer(ctx, which, stage_lr + f0 * fl, fn, h, w, stage_hr + f0 * fh, stream));
     CK(cudaEventRecord(ev[1 + nch + c], st));
     CK(cudaStreamWaitEvent(ctx->copy_st, ev[1 + nch + c], 0));
-    CK(cudaMemcpyAsync(hr_host + f0 * fh, ctx->stage_hr + f0 * fh, fn * fh, cudaMemcpyDeviceToHost, ctx->copy_st));
+    CK(cudaMemcpyAsync(hr_host + f0 * fh, stage_hr + f0 * fh, fn * fh, cudaMemcpyDeviceToHost, ctx->copy_st));
   }
+  CK(cudaEventRecord(ctx->host_done[set], ctx->copy_st));
+  ctx->host_calls++;
   if (sync) {
-    CK(cudaStreamSynchronize(ctx->copy_st));
+    CK(cudaEventSynchronize(ctx->host_done[set]));
   } else {
-    ctx->host_pending = true;
+    ctx->host_busy[set] = true;
   }
   return SR_OK;
 }
@@ -1245,10 +1261,11 @@ sr_status sr_infer_host_async(sr_ctx* ctx, sr_model which, const uint8_t* lr_hos
 
 sr_status sr_infer_host_wait(sr_ctx* ctx) {
   GUARD();
-  if (ctx->host_pending) {
-    CK(cudaStreamSynchronize(ctx->copy_st));
-    ctx->host_pending = false;
-  }
+  for (int k = 0; k < 2; ++k)
+    if (ctx->host_busy[k]) {
+      CK(cudaEventSynchronize(ctx->host_done[k]));
+      ctx->host_busy[k] = false;
+    }
   return SR_OK;
 }
 
