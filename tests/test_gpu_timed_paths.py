@@ -297,3 +297,20 @@ def test_sse_u8_exact(n, elems, off):
     assert st == 0
     d = (a[off:off + n * elems].astype(np.int64) - b[off:off + n * elems].astype(np.int64)).reshape(n, elems)
     np.testing.assert_array_equal(out.cpu().numpy(), (d * d).sum(axis=1))
+
+
+def test_infer_host_async_two_in_flight():
+    """sr_infer_host_async with two staging sets: consecutive calls overlap (up to two in flight, a third waits for
+    the first); every batch lands intact in its own host buffer, bit-identical to sr_infer on device buffers."""
+    s, b, c = 3, 2, 16
+    ctx = _ctx(s, b, c, seed=33)
+    lrs = [synth_frames(5, 96, 160, seed=40 + k) for k in range(4)]
+    ref = [ctx.infer(torch.from_numpy(x).cuda(), "serve").cpu() for x in lrs]
+    lr_h = [torch.from_numpy(x).pin_memory() for x in lrs]
+    outs = [torch.zeros((5, 288, 480, 3), dtype=torch.uint8).pin_memory() for _ in range(4)]
+    st = torch.cuda.Stream()
+    for k in range(4):
+        ctx.infer_host_async(lr_h[k], outs[k], "serve", stream=st)
+    ctx.infer_host_wait()
+    for k in range(4):
+        assert torch.equal(outs[k], ref[k]), k
