@@ -1198,9 +1198,10 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
   // Chunked pipeline: all H2D copies go first on their own stream (per-chunk events), chunk k is super-resolved
   // on `stream` as soon as its frames landed, and its D2H runs on a third stream while chunk k+1 computes.
   // PCIe (55 GB/s measured) then hides behind the tensor work; only the last chunk's D2H is exposed.
-  // Chunk sizes: ~96 MB of HR output per chunk, except a one-frame first chunk (compute starts after one frame's
-  // H2D) and a one-frame last chunk (only one frame's D2H is left exposed after the last kernel).
-  const int F = std::max(1, std::min(n, (int)std::max<size_t>(1, (size_t)(96u << 20) / std::max<size_t>(fh, 1))));
+  // Chunk sizes: ~240 MB of HR output per chunk (fewer, larger inference launches; with two calls in flight the
+  // other call's work hides the longer exposed copies), except a one-frame first chunk (compute starts after one
+  // frame's H2D) and a one-frame last chunk (only one frame's D2H is left exposed after the last kernel).
+  const int F = std::max(1, std::min(n, (int)std::max<size_t>(1, (size_t)(240u << 20) / std::max<size_t>(fh, 1))));
   std::vector<int> c0s;  // first frame of each chunk (+ n at the end)
   {
     int f = 0;
