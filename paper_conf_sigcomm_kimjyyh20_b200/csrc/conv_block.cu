@@ -424,9 +424,7 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       if (warp == 6 && lane_id() == 0) { SR_DBG(14, q + 1) }
       if (emit) {
         if (lane_ok && !(exp & 2)) {
-          // chunk-planar staging row [chunk][126 px][16 B]: conflict-free 16-B stores (a pixel-major row would make
-          // each one 2-way conflicted on the shared-memory port the MMAs are bound by)
-          uint8_t* orow = sO + os * OUTB + m * 16;
+          uint4* orow = reinterpret_cast<uint4*>(sO + os * OUTB + m * C * 2);
 #pragma unroll
           for (int j = 0; j < C / 8; ++j) {
             const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&res[j]);
@@ -455,13 +453,13 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
             u.y = pack_bf16x2(a[2], a[3]);
             u.z = pack_bf16x2(a[4], a[5]);
             u.w = pack_bf16x2(a[6], a[7]);
-            *reinterpret_cast<uint4*>(orow + j * (kBlkTW * 16)) = u;
+            orow[j] = u;
           }
         }
         fence_proxy_async_smem();
         named_bar_sync(2, 128);
         if (leader && !(exp & 2)) {
-          tma_store_5d(&tm_out, sO + os * OUTB, 0, x0, r, 0, n);
+          tma_store_4d(&tm_out, sO + os * OUTB, 0, x0, r, n);
           bulk_commit();
           bulk_wait_read<kBlkNO - 2>();
           SR_DBG(6, q + 1)
@@ -512,8 +510,7 @@ cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf1
                             bf16* tsave, int sep, int exp, const bf16* mask, const bf16* res2) {
   CUtensorMap tf, to;
   if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  if (make_act_tmap(&to, out, N, H, W, cp, kBlkTW, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, cp, kBlkTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   const long long rows = (long long)N * ((W + kBlkTW - 1) / kBlkTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;

@@ -99,13 +99,8 @@ __device__ __forceinline__ void ld_row(const bf16* base, uint4* dst) {
 // One output row of one lane into the staging row: v (bias included) + res1 (aux row) + res2 -> ReLU -> x 1[mask > 0]
 // (aux row) -> 0 in separator columns -> bf16.  M: variant bits (1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU);
 // M = 32: generic body, the variant is read from em at run time.
-// Staging and aux rows are chunk-planar, [channel chunk of 8][128 pixels][16 B] (kRollPlaneO bytes per chunk): a
-// lane's 16-B accesses to one chunk are consecutive across the warp, so they are bank-conflict free (a pixel-major
-// row, 2 x COUTP bytes per pixel, makes every 16-B access 2-way conflicted on the shared-memory port that also feeds
-// the MMAs).
-static constexpr uint32_t kRollPlaneO = kRollTW * 16;
 template <int COUTP, int M>
-__device__ __forceinline__ void roll_stage(uint8_t* __restrict__ orow, const float* v, const uint8_t* __restrict__ aux_s,
+__device__ __forceinline__ void roll_stage(uint4* __restrict__ orow, const float* v, const uint4* __restrict__ aux_s,
                                            const uint4* r2, bool sep0, int em) {
   const int mm = (M & 32) ? em : M;
   // the whole aux row (residual or mask) into registers first: the staging stores below could alias it for the
@@ -113,7 +108,7 @@ __device__ __forceinline__ void roll_stage(uint8_t* __restrict__ orow, const flo
   uint4 aux[COUTP / 8];
   if (mm & 5) {
 #pragma unroll
-    for (int j = 0; j < COUTP / 8; ++j) aux[j] = *reinterpret_cast<const uint4*>(aux_s + j * kRollPlaneO);
+    for (int j = 0; j < COUTP / 8; ++j) aux[j] = aux_s[j];
   }
 #pragma unroll
   for (int j = 0; j < COUTP / 8; ++j) {
@@ -154,7 +149,7 @@ __device__ __forceinline__ void roll_stage(uint8_t* __restrict__ orow, const flo
     u.y = pack_bf16x2(o[2], o[3]);
     u.z = pack_bf16x2(o[4], o[5]);
     u.w = pack_bf16x2(o[6], o[7]);
-    *reinterpret_cast<uint4*>(orow + j * kRollPlaneO) = u;
+    orow[j] = u;
   }
 }
 
@@ -290,7 +285,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         if (has_aux && i >= 1 && i - 1 < y1 - y0) {  // aux row of output row y0+i-1 (needed after input row y0+i)
           mbar_wait(&x_empty[xs], xph ^ 1);
           mbar_arrive_expect_tx(&x_full[xs], kRollTW * COUTP * 2);
-          tma_load_5d(sA + xs * ROWB, &tm_aux, &x_full[xs], 0, x0, y0 + i - 1, 0, n);  // chunk-planar
+          tma_load_4d(sA + xs * ROWB, &tm_aux, &x_full[xs], 0, x0, y0 + i - 1, n);
           if (++xs == NAUX) { xs = 0; xph ^= 1; }
         }
       }
@@ -403,7 +398,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
           if (TS > 0)  // the S HR rows of LR row r
             tma_store_4d(&tm_out, sO + b * ROWB, 0, x0 * TS * 3 / 16, TS * r, n);
           else
-            tma_store_5d(&tm_out, sO + b * ROWB, 0, x0, r, 0, n);  // chunk-planar staging row
+            tma_store_4d(&tm_out, sO + b * ROWB, 0, x0, r, n);
           bulk_commit();
           bulk_wait_read<1>();        // the previous store has read its staging row
           if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
@@ -515,12 +510,12 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         }
         continue;
       }
-      const uint8_t* aux = sA + (int)(xi % NAUX) * ROWB + m * 16;
+      const uint4* aux = reinterpret_cast<const uint4*>(sA + (int)(xi % NAUX) * ROWB + m * COUTP * 2);
       if (has_aux) mbar_wait(&x_full[xi % NAUX], (uint32_t)(xi / NAUX) & 1u);
       mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);  // the store warp has read this staging row
       if (warp == 2 && lane_id() == 0) { SR_RDBG(11, q + 1) }
       if (lane_ok) {
-        uint8_t* orow = stage + os * ROWB + m * 16;
+        uint4* orow = reinterpret_cast<uint4*>(stage + os * ROWB + m * COUTP * 2);
         // the epilogue variant is uniform across the launch: dispatch once per row to straight-line code
         // (a generic body predicates every variant's instructions -- ~600 per row -- and the per-row chain of
         // the epilogue group is what bounds the launch)
@@ -591,8 +586,7 @@ cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* w
   if (!roll_head_u8_supported(coutp, W, lr)) return cudaErrorNotSupported;
   CUtensorMap ti, to;
   if (make_u8_rows_tmap(&ti, lr, N, H, 3LL * W, 26, 1) != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  if (make_act_tmap(&to, out, N, H, W, coutp, kRollTW, 1, coutp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, nullptr, nullptr, 0, 0, 0, 0, w_early};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
   int grid = num_sms();
@@ -624,13 +618,10 @@ cudaError_t launch_conv_roll_ex(int cinp, int coutp, const void* in, const bf16*
   CUtensorMap ti, to;
   if (make_act_tmap(&ti, in, N, H, W, cinp, kRollTW + 2, 1, cinp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
     return cudaErrorInvalidValue;
-  // output and aux rows as chunk-planar boxes ([chunk][128 px][8 ch]; see roll_stage)
-  if (make_act_tmap(&to, out, N, H, W, coutp, kRollTW, 1, coutp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   CUtensorMap tx;
   const void* auxp = res1 ? (const void*)res1 : (mask ? (const void*)mask : (const void*)out);
-  if (make_act_tmap(&tx, auxp, N, H, W, coutp, kRollTW, 1, coutp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
-    return cudaErrorInvalidValue;
+  if (make_row_tmap(&tx, auxp, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (res1 && mask) return cudaErrorNotSupported;  // one TMA aux stream per launch
   RollArgs a{bias, res1, res2, mask, relu, sep, N, H, W, dbg, nullptr, nullptr, 0, 0, 0, 0, w_early};
   const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
