@@ -23,6 +23,14 @@ sys.path.insert(0, ROOT)
 
 
 def main():
+    import argparse
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--only", default="", help="comma list of: adam_small,adam64m,gather,sse4k,sseval,infer")
+    args = ap.parse_args()
+    only = set(x for x in args.only.split(",") if x)
+
+    def want(k):
+        return not only or k in only
     import numpy as np
     import torch
     from paper_conf_sigcomm_kimjyyh20_b200 import SRContext, load
@@ -47,7 +55,7 @@ def main():
         return e0.elapsed_time(e1) / reps
 
     # ---- Adam
-    for n in (366363, 64 << 20):
+    for n in [n for n, k in ((366363, "adam_small"), (64 << 20, "adam64m")) if want(k)]:
         p = torch.randn(n, device="cuda") * 0.05
         m = torch.zeros(n, device="cuda")
         v = torch.zeros(n, device="cuda")
@@ -64,23 +72,34 @@ def main():
     ctx.pool_push(torch.from_numpy(plr).cuda(), torch.from_numpy(phr).cuda())
     blr = torch.empty((64, 48, 48, 3), dtype=torch.uint8, device="cuda")
     bhr = torch.empty((64, 144, 144, 3), dtype=torch.uint8, device="cuda")
-    ms = timeit(lambda: ctx.sample_batch(-1, 64, 48, out=(blr, bhr, None)))
-    rows.append(("k_sample_gather", "64 x (48^2 + 144^2) x 3 B", 2 * 64 * (48 * 48 + 144 * 144) * 3, ms))
+    if want("gather"):
+        ms = timeit(lambda: ctx.sample_batch(-1, 64, 48, out=(blr, bhr, None)))
+        rows.append(("k_sample_gather", "64 x (48^2 + 144^2) x 3 B", 2 * 64 * (48 * 48 + 144 * 144) * 3, ms))
     # ---- SSE: one 4K frame pair; the bench's 64 validation patches (180x180 HR)
     a = torch.from_numpy(synth_frames(1, 2160, 3840, seed=1)).cuda()
     b = torch.from_numpy(synth_frames(1, 2160, 3840, seed=2)).cuda()
     out = torch.zeros(64, dtype=torch.int64, device="cuda")
     el = 2160 * 3840 * 3
-    ms = timeit(lambda: lib.sr_sse_u8(ctypes.c_void_p(a.data_ptr()), ctypes.c_void_p(b.data_ptr()), 1, el,
-                                      ctypes.c_void_p(out.data_ptr()), sp))
-    rows.append(("k_sse_u8", "one 4K frame pair", 2 * el, ms))
+    if want("sse4k"):
+        ms = timeit(lambda: lib.sr_sse_u8(ctypes.c_void_p(a.data_ptr()), ctypes.c_void_p(b.data_ptr()), 1, el,
+                                          ctypes.c_void_p(out.data_ptr()), sp))
+        rows.append(("k_sse_u8", "one 4K frame pair", 2 * el, ms))
     va = torch.from_numpy(phr[:64].copy()).cuda()
     vb = torch.from_numpy(phr[64:128].copy()).cuda()
     el = 180 * 180 * 3
-    ms = timeit(lambda: lib.sr_sse_u8(ctypes.c_void_p(va.data_ptr()), ctypes.c_void_p(vb.data_ptr()), 64, el,
-                                      ctypes.c_void_p(out.data_ptr()), sp))
-    rows.append(("k_sse_u8", "64 validation patches 180x180", 2 * 64 * el, ms))
+    if want("sseval"):
+        ms = timeit(lambda: lib.sr_sse_u8(ctypes.c_void_p(va.data_ptr()), ctypes.c_void_p(vb.data_ptr()), 64, el,
+                                          ctypes.c_void_p(out.data_ptr()), sp))
+        rows.append(("k_sse_u8", "64 validation patches 180x180", 2 * 64 * el, ms))
     # ---- head conv from u8 (inference of 30 720p frames, timed per kernel class by the library)
+    if not want("infer"):
+        out_rows = []
+        for name, shape, by, ms in rows:
+            gbs = by / (ms * 1e-3) / 1e9
+            out_rows.append({"kernel": name, "shape": shape, "algorithmic_bytes": int(by), "ms": round(ms, 5),
+                             "GB/s": round(gbs, 1), "frac_of_hbm": round(gbs / peak, 4)})
+        print(json.dumps({"hbm_peak_gbs": peak, "rows": out_rows}, indent=1))
+        return
     lr = torch.from_numpy(synth_frames(30, 720, 1280, seed=1003)).cuda()
     hr = torch.empty((30, 2160, 3840, 3), dtype=torch.uint8, device="cuda")
     for _ in range(3):
