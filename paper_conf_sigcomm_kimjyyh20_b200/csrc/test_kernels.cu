@@ -568,3 +568,9 @@ extern "C" int sr_bench_bodytail_dbg(int cp, int s, int n, int h, int w, long lo
   cudaFree(x); cudaFree(f0); cudaFree(lr); cudaFree(hr); cudaFree(w1); cudaFree(w2); cudaFree(bias); cudaFree(dbg);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
+
+// Benchmarking only: cap the persistent grids of subsequent launches (0 = all SMs), as sr_set_sm_split does per call.
+extern "C" int sr_test_grid_cap(int cap) {
+  sr::set_grid_cap(cap);
+  return 0;
+}

@@ -14,7 +14,16 @@ lib = load()
 lib.sr_bench_roll_dbg.restype = C.c_int
 lib.sr_bench_roll_dbg.argtypes = [C.c_int] * 6 + [C.c_void_p, C.c_void_p, C.c_void_p]
 st = C.c_void_p(torch.cuda.current_stream().cuda_stream)
-for shape in ((1, 48, 3200), (8, 720, 1280)):
+# GRID=n: n CTAs (the bench's training partition has 40 SMs); PART=n: run on an n-SM green-context partition
+grid = int(os.environ.get("GRID", "0"))
+if grid:
+    lib.sr_test_grid_cap(grid)
+if os.environ.get("PART"):
+    from paper_conf_sigcomm_kimjyyh20_b200 import SRContext  # noqa: E402
+    _, pst, _, _ = SRContext.sm_partition(int(os.environ["PART"]))
+    st = C.c_void_p(pst.cuda_stream)
+shapes = ((1, 48, 3200),) if os.environ.get("TRAIN_ONLY") else ((1, 48, 3200), (8, 720, 1280))
+for shape in shapes:
     for res in (0, 1, 2):
         dbg = np.zeros(16 * 256, np.int64)
         ms = C.c_float()
