@@ -14,9 +14,10 @@
 // Each CTA takes a contiguous range of (column strip, row) work (equal rows per CTA); input rows are read once
 // per strip piece (+2 halo rows per piece).  Strips are 128 output pixels (= MMA M).
 //
-// Warp roles (352 threads): warp 0 TMA producer, warp 1 TMEM alloc + MMA issuer, warps 2..9 epilogue in two groups
-// of 4 that take alternate output rows (all channels) and hand finished rows to warp 10, which issues the TMA
-// stores.  The per-row epilogue chain (drain, re-arm, residual, stage) is latency-bound: two rows in flight and no
+// Warp roles (384 threads): warp 0 TMA producer of the input rows, warp 1 TMEM alloc + MMA issuer, warps 2..9
+// epilogue in two groups of 4 that take alternate output rows (all channels) and hand finished rows to warp 10,
+// which issues the TMA stores; warp 11 issues the aux-row (residual / mask) and tail LR-row TMAs on its own, so
+// waiting for an aux slot the epilogue has not released yet never holds back the input rows the MMAs need.  The per-row epilogue chain (drain, re-arm, residual, stage) is latency-bound: two rows in flight and no
 // barrier or store wait on it.
 #include <cuda.h>
 #include "ptx.cuh"
@@ -29,7 +30,7 @@
 
 namespace sr {
 
-static constexpr int kRollThreads = 352;  // + warp 10: TMA-store warp
+static constexpr int kRollThreads = 384;  // warp 10: TMA-store warp, warp 11: aux / LR-row TMA producer
 static constexpr int kRollNO = 3;    // output staging rows per epilogue group
 static constexpr int kRollTW = 128;  // output pixels per strip (= MMA M)
 
@@ -154,7 +155,7 @@ __device__ __forceinline__ void roll_stage(uint4* __restrict__ orow, const float
 }
 
 // U8 (head conv only, CINP = 16): the input is the u8 RGB frame itself.  The producer TMA-loads u8 rows (16-B
-// chunk map, W % 16 == 0) into a small ring in the aux area and warp 11 expands each row into the bf16 A slot
+// chunk map, W % 16 == 0) into a small ring in the aux area and warps 12, 13 expand each row into the bf16 A slot
 // (x = v/255 in channels 0..2, exactly k_pack_input's arithmetic; channel chunk 1 is a zero plane written once),
 // so k_pack_input's 32 B/px write and the head's 32 B/px read become a 3 B/px read.
 static constexpr int kU8Slots = 8;
@@ -253,18 +254,18 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     pos += y1 - y0;                                                                   \
     const int n = col / tiles_x, x0 = (col - n * tiles_x) * kRollTW;                  \
     const int n_in = y1 - y0 + 2;                                                     \
-    (void)n; (void)x0;
+    (void)n; (void)x0; (void)n_in;
 #define SR_PIECE_END }
 
   if (warp == 0) {
     // ===================== TMA producer: weights, then input rows y0-1 .. y1 of each piece =====================
     if (elect_one()) {
       tma_prefetch_desc(&tm_in);
-      int s = 0, xs = 0, ls = 0, us = 0;
-      uint32_t ph = 0, xph = 0, lph = 0, uph = 0;
+      int s = 0, us = 0;
+      uint32_t ph = 0, uph = 0;
       SR_PIECE_BEGIN
       for (int i = 0; i < n_in; ++i) {
-        if constexpr (U8) {  // u8 row y0-1+i, pixels x0-1 .. x0+128 (+ chunk alignment), for warp 11 to expand
+        if constexpr (U8) {  // u8 row y0-1+i, pixels x0-1 .. x0+128 (+ chunk alignment), for warps 12, 13 to expand
           mbar_wait(&u_empty[us], uph ^ 1);
           mbar_arrive_expect_tx(&u_full[us], 16 * 26);
           tma_load_4d(sA + us * kU8Slot, &tm_in, &u_full[us], 0, (3 * x0 - 3) >> 4, y0 - 1 + i, n);
@@ -276,16 +277,28 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
           if (++s == kRollIn) { s = 0; ph ^= 1; }
         }
         SR_RDBG(0, i)
-        if (TS > 0 && a.tail_tma && i >= 1 && i - 1 < y1 - y0) {  // LR rows r-2..r+2 of output row r = y0+i-1
+      }
+      SR_PIECE_END
+    }
+    __syncwarp();
+  } else if (warp == 11) {
+    // ===================== aux producer: residual / mask rows and the tail's LR neighbourhood rows =============
+    if ((has_aux || (TS > 0 && a.tail_tma)) && elect_one()) {
+      tma_prefetch_desc(&tm_aux);
+      int xs = 0, ls = 0;
+      uint32_t xph = 0, lph = 0;
+      SR_PIECE_BEGIN
+      for (int r = y0; r < y1; ++r) {  // output rows of the piece, in emission order
+        if (TS > 0 && a.tail_tma) {  // LR rows r-2..r+2 of output row r
           mbar_wait(&l_empty[ls], lph ^ 1);
           mbar_arrive_expect_tx(&l_full[ls], 16 * kTailLrChunks * 5);
-          tma_load_4d(sA + ls * kTailLrSlot, &tm_aux, &l_full[ls], 0, 3 * x0 / 16 - 1, y0 + i - 3, n);
+          tma_load_4d(sA + ls * kTailLrSlot, &tm_aux, &l_full[ls], 0, 3 * x0 / 16 - 1, r - 2, n);
           if (++ls == Cfg::NLR) { ls = 0; lph ^= 1; }
         }
-        if (has_aux && i >= 1 && i - 1 < y1 - y0) {  // aux row of output row y0+i-1 (needed after input row y0+i)
+        if (has_aux) {  // aux row of output row r
           mbar_wait(&x_empty[xs], xph ^ 1);
           mbar_arrive_expect_tx(&x_full[xs], kRollTW * COUTP * 2);
-          tma_load_4d(sA + xs * ROWB, &tm_aux, &x_full[xs], 0, x0, y0 + i - 1, n);
+          tma_load_4d(sA + xs * ROWB, &tm_aux, &x_full[xs], 0, x0, r, n);
           if (++xs == NAUX) { xs = 0; xph ^= 1; }
         }
       }
@@ -330,15 +343,15 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       SR_PIECE_END
     }
     __syncwarp();
-  } else if (U8 && warp >= 11) {
-    // ===================== u8 -> bf16 A-operand expansion (head conv): warps 11, 12 take alternate rows ==========
+  } else if (U8 && warp >= 12) {
+    // ===================== u8 -> bf16 A-operand expansion (head conv): warps 12, 13 take alternate rows ==========
     int s = 0, us = 0;
     uint32_t ph = 0, uph = 0;
     long long rowc = 0;  // rows seen so far (both warps count every row; each converts its parity)
     SR_PIECE_BEGIN
     const int lbase = 16 * ((3 * x0 - 3) >> 4);
     for (int i = 0; i < n_in; ++i, ++rowc) {
-      if ((int)(rowc & 1) != warp - 11) {
+      if ((int)(rowc & 1) != warp - 12) {
         if (++us == kU8Slots) { us = 0; uph ^= 1; }
         if (++s == kRollIn) { s = 0; ph ^= 1; }
         continue;
