@@ -27,7 +27,6 @@
 #include "kernels.h"
 #include "launch.cuh"
 #include "tail.cuh"
-#include "rot.cuh"
 
 namespace sr {
 
@@ -105,12 +104,13 @@ template <int COUTP, int M>
 __device__ __forceinline__ void roll_stage(uint4* __restrict__ orow, const float* v, const uint4* __restrict__ aux_s,
                                            const uint4* r2, bool sep0, int em) {
   const int mm = (M & 32) ? em : M;
-  // the whole aux row (residual or mask) into registers first (lane-rotated chunk order: conflict-free, rot.cuh);
-  // the staging stores below could alias it for the compiler, which would otherwise serialise every 16-B load
-  // behind the previous chunk's store
+  // the whole aux row (residual or mask) into registers first: the staging stores below could alias it for the
+  // compiler, which would otherwise serialise every 16-B load behind the previous chunk's store
   uint4 aux[COUTP / 8];
-  if (mm & 5) ld_pix_rot<COUTP / 8>(reinterpret_cast<const uint8_t*>(aux_s), aux);
-  uint4 ov[COUTP / 8];
+  if (mm & 5) {
+#pragma unroll
+    for (int j = 0; j < COUTP / 8; ++j) aux[j] = aux_s[j];
+  }
 #pragma unroll
   for (int j = 0; j < COUTP / 8; ++j) {
     float o[8];
@@ -150,9 +150,8 @@ __device__ __forceinline__ void roll_stage(uint4* __restrict__ orow, const float
     u.y = pack_bf16x2(o[2], o[3]);
     u.z = pack_bf16x2(o[4], o[5]);
     u.w = pack_bf16x2(o[6], o[7]);
-    ov[j] = u;
+    orow[j] = u;
   }
-  st_pix_rot<COUTP / 8>(reinterpret_cast<uint8_t*>(orow), ov);
 }
 
 // U8 (head conv only, CINP = 16): the input is the u8 RGB frame itself.  The producer TMA-loads u8 rows (16-B
