@@ -366,15 +366,17 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     SR_PIECE_BEGIN
     const bool lane_ok = m < kBlkTW && x0 + m < W;
     const bool sep0 = sep > 0 && (((x0 + m) % max(sep, 1)) == 0 || ((x0 + m) % max(sep, 1)) == sep - 1);
-    // the residual row is loaded one row ahead (res_nx), so its L2 latency overlaps a whole row-step
-    uint4 res_nx[C / 8];
+    // the residual row is loaded ahead (res_nx: one row; at C <= 32, where a row-step is only ~660 cycles, two rows
+    // through res_nx2), so its L2/HBM latency overlaps whole row-steps
+    constexpr int kAhead = (C <= 32 && !BWD) ? 2 : 1;  // (BWD keeps res2 one row ahead alongside)
+    uint4 res_nx[C / 8], res_nx2[kAhead > 1 ? C / 8 : 1];
     uint4 r2_nx[BWD ? C / 8 : 1];
     auto ld_res = [&](int q) {
       if (q >= 1 && q <= n_t - 2 && lane_ok && !(exp & 1)) {
         const size_t pix = (((size_t)n * H + y0 - 1 + q) * W) + x0 + m;
         const uint4* rp = reinterpret_cast<const uint4*>(fres + pix * C);
 #pragma unroll
-        for (int j = 0; j < C / 8; ++j) res_nx[j] = __ldg(rp + j);
+        for (int j = 0; j < C / 8; ++j) (kAhead > 1 ? res_nx2 : res_nx)[j] = __ldg(rp + j);
         if (BWD && res2) {
           const uint4* rp2 = reinterpret_cast<const uint4*>(res2 + pix * C);
 #pragma unroll
@@ -383,6 +385,11 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       }
     };
     ld_res(-1);
+    if constexpr (kAhead > 1) {
+#pragma unroll
+      for (int j = 0; j < C / 8; ++j) res_nx[j] = res_nx2[j];
+      ld_res(0);
+    }
     for (int q = -1; q <= n_t; ++q) {         // out rows of conv2 = output rows y0-1+q
       const long long g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
@@ -390,11 +397,15 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       uint4 res[C / 8], rs2[BWD ? C / 8 : 1];
 #pragma unroll
       for (int j = 0; j < C / 8; ++j) res[j] = res_nx[j];
+      if constexpr (kAhead > 1) {
+#pragma unroll
+        for (int j = 0; j < C / 8; ++j) res_nx[j] = res_nx2[j];
+      }
       if (BWD && res2) {
 #pragma unroll
         for (int j = 0; j < C / 8; ++j) rs2[j] = r2_nx[j];
       }
-      ld_res(q + 1);
+      ld_res(q + kAhead);
       const int b = ring_idx<RB>(g);
       mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
       tc_fence_after();
