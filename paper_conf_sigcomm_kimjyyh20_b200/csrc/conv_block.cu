@@ -194,9 +194,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       for (int st = 0; st < n_f; ++st) {
         SR_DBG(7, st)
         const long long g = G1 + st;
-        for (; acq1 < g + 3; ++acq1) mbar_wait_probe(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
+        for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
         SR_DBG(8, st)
-        mbar_wait_probe(&f_full[fs], fph);
+        mbar_wait(&f_full[fs], fph);
         SR_DBG(9, st)
         tc_fence_after();
         if (st == 0) {  // the piece's first two rows receive no earlier contribution
@@ -231,9 +231,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       for (int k = 0; k < n_t; ++k) {
         SR_DBG(10, k + 3)
         const long long g = G2 + k;
-        for (; acq2 < g + 3; ++acq2) mbar_wait_probe(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
+        for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
         SR_DBG(11, k + 3)
-        mbar_wait_probe(&t_full[ts], tph);
+        mbar_wait(&t_full[ts], tph);
         SR_DBG(12, k + 3)
         tc_fence_after();
         if (k == 0) {

@@ -319,9 +319,9 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       for (int i = 0; i < n_in; ++i) {
         const long long g = G + i;  // out row completed by this step (dy = 2 target)
         SR_RDBG(1, i)
-        for (; acq < g + 3; ++acq) mbar_wait_probe(&r_free[ring_idx<RB>(acq)], (uint32_t)(acq / RB) & 1u);
+        for (; acq < g + 3; ++acq) mbar_wait(&r_free[ring_idx<RB>(acq)], (uint32_t)(acq / RB) & 1u);
         SR_RDBG(2, i)
-        mbar_wait_probe(&in_full[s], ph);
+        mbar_wait(&in_full[s], ph);
         SR_RDBG(3, i)
         tc_fence_after();
         if (i == 0) {  // the piece's first two rows receive no earlier contribution

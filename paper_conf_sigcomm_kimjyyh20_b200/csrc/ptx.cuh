@@ -52,19 +52,6 @@ __device__ __forceinline__ bool mbar_try_wait(uint32_t addr, uint32_t phase) {
       : "memory");
   return ok != 0;
 }
-// Non-suspending probe of a phase parity (mbarrier.test_wait): for the MMA issuers, whose barriers have usually
-// completed long before they are checked.
-__device__ __forceinline__ bool mbar_test_wait(uint32_t addr, uint32_t phase) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred P;\n\t"
-      "mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
-      "selp.b32 %0, 1, 0, P;\n\t}"
-      : "=r"(ok)
-      : "r"(addr), "r"(phase)
-      : "memory");
-  return ok != 0;
-}
 // Blocking wait on a phase parity.  A pipeline bug would otherwise hang the GPU: after ~2^35 cycles
 // (~17 s) the wait traps so the launch fails with an error instead.
 __device__ __forceinline__ long long globaltimer() {
@@ -73,12 +60,6 @@ __device__ __forceinline__ long long globaltimer() {
   return t;
 }
 
-// Issuer-side wait: a cheap non-suspending probe first (the common case: already complete), then mbar_wait.
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase);
-__device__ __forceinline__ void mbar_wait_probe(uint64_t* bar, uint32_t phase) {
-  if (mbar_test_wait(smem_u32(bar), phase)) return;
-  mbar_wait(bar, phase);
-}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
   const uint32_t addr = smem_u32(bar);
   if (mbar_try_wait(addr, phase)) return;
