@@ -93,8 +93,11 @@ def run(argv=None):
             st = Stream(len(streams), torch, SRContext, synth_frames, synth_patch_pool, dev)
             with torch.cuda.stream(hi):   # warm the inference path (workspace, kernels)
                 st.ctx.infer(st.lr_dev[:1], "serve", out=st.hr_dev[:1])
-            with torch.cuda.stream(lo):   # warm + capture the training iteration
-                st.ctx.train_sampled(2, BATCH, PATCH, st.loss)
+            with torch.cuda.stream(lo):   # warm + capture the training iteration; warm the epoch-end path (its
+                st.ctx.train_sampled(2, BATCH, PATCH, st.loss)  # workspaces are allocated here, not in the window)
+                st.ctx.publish()
+                st.ctx.controller_step(Controller(thresh_sat=0.05, count_sat=2, thresh_online=0.5, count_online=2),
+                                       st.val_lr, st.val_hr)
             torch.cuda.synchronize()
             streams.append(st)
         return streams[:n]
@@ -162,8 +165,7 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
             if item is None:
                 return
             t_arr, ev, warm, evs, t_iss = item
-            while not ev.query():
-                time.sleep(0.0001)
+            ev.synchronize()  # (releases the GIL while it waits)
             if not warm:
                 lat.append((time.perf_counter() - t_arr) * 1e3)
                 a_rel = (t_arr - t_base[0]) * 1e3
@@ -184,7 +186,11 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
                 time.sleep(min(0.01, due - now))
                 continue
             warm = tick * 0.5 < args.warm_seconds
-            for st in ss:
+            for si_, st in enumerate(ss):
+                # spread the streams' slices over the tick, so the host work is not one burst
+                t_due = due + 0.5 * si_ / len(ss)
+                while time.perf_counter() < t_due and not stop.is_set():
+                    time.sleep(min(0.002, max(0.0, t_due - time.perf_counter())))
                 with torch.cuda.stream(lo):
                     a = st.arrivals % 20
                     if tick % 2 == 0:
