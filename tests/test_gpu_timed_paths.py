@@ -314,3 +314,27 @@ def test_infer_host_async_two_in_flight():
     ctx.infer_host_wait()
     for k in range(4):
         assert torch.equal(outs[k], ref[k]), k
+
+
+def test_nccl_allreduce_on_partition_stream():
+    """bench.py at N > 1 runs the DP iteration (with the library's in-graph ncclAllReduce) on the training partition's
+    green-context stream: a one-rank communicator there gives the same parameters as no communicator."""
+    import ctypes
+    from paper_conf_sigcomm_kimjyyh20_b200 import SRContext, load
+    buf = ctypes.create_string_buffer(128)
+    assert load().sr_nccl_unique_id(buf, 128) == 0
+    a = _ctx(3, 2, 32, seed=3, nccl_id=buf.raw)
+    b = _ctx(3, 2, 32, seed=3)
+    plr, phr, _ = synth_patch_pool(64, 3, 180, seed=5, frame_hw=(1080, 1800))
+    for c in (a, b):
+        c.pool_push(torch.from_numpy(plr).cuda(), torch.from_numpy(phr).cuda())
+    torch.cuda.synchronize()
+    si, stt, ni, nt = SRContext.sm_partition(40)
+    assert nt == 40 and ni > 0
+    for c in (a, b):
+        c.set_sm_split(nt)
+        c.train_sampled(4, 16, 48, stream=stt)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(a.get_params("train"), b.get_params("train"))
+    for c in (a, b):
+        c.set_sm_split(0)
