@@ -34,6 +34,7 @@
 #include "sr_internal.h"
 #include "ring.cuh"
 #include "launch.cuh"
+#include "rot.cuh"
 
 namespace sr {
 
@@ -435,7 +436,8 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       if (warp == 6 && lane_id() == 0) { SR_DBG(14, q + 1) }
       if (emit) {
         if (lane_ok && !(exp & 2)) {
-          uint4* orow = reinterpret_cast<uint4*>(sO + os * OUTB + m * C * 2);
+          uint8_t* orow = sO + os * OUTB + m * C * 2;
+          uint4 ov[C / 8];
 #pragma unroll
           for (int j = 0; j < C / 8; ++j) {
             const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&res[j]);
@@ -464,8 +466,11 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
             u.y = pack_bf16x2(a[2], a[3]);
             u.z = pack_bf16x2(a[4], a[5]);
             u.w = pack_bf16x2(a[6], a[7]);
-            orow[j] = u;
+            ov[j] = u;
           }
+          // lane-rotated chunk order: conflict-free 16-B stores into the pixel-major staging row (rot.cuh; at
+          // C = 32 the 64-B pixel stride makes a plain chunk loop 4-way conflicted)
+          st_pix_rot<C / 8>(orow, ov);
         }
         fence_proxy_async_smem();
         named_bar_sync(2, 128);
