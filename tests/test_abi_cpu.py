@@ -52,3 +52,18 @@ def test_product_path_has_no_oracle_or_cpu_fallback():
         pass
     finally:
         _lib._lib = None
+
+
+def test_nccl_unique_id_and_missing_library():
+    """sr_nccl_unique_id draws a 128-byte id through the dlopen'ed libnccl (no GPU needed), returns SR_E_INVAL for a
+    short buffer, and SR_E_NCCL when libnccl cannot be loaded (SR_NCCL_LIB pointing nowhere, fresh process)."""
+    import subprocess
+    import sys
+    code = ("import ctypes, sys; sys.path.insert(0, %r); from paper_conf_sigcomm_kimjyyh20_b200 import load; "
+            "lib = load(); b = ctypes.create_string_buffer(128); s = ctypes.create_string_buffer(16); "
+            "print(lib.sr_nccl_unique_id(b, 128), lib.sr_nccl_unique_id(s, 16), int(any(b.raw)))" % ROOT)
+    ok = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=120)
+    assert ok.stdout.split() == ["0", "-1", "1"], ok.stdout + ok.stderr
+    env = dict(os.environ, SR_NCCL_LIB="/nonexistent/libnccl.so.2")
+    bad = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=120, env=env)
+    assert bad.stdout.split()[0] == "-4", bad.stdout + bad.stderr
