@@ -88,6 +88,7 @@ _SIGS = {
     "sr_test_wgrad": (_I, [_P, _P, _I, _I, _I, _I, _I, _P, _P, _P]),
     "sr_test_wgrad_batch": (_I, [_I, _P, _P, _I, _I, _I, _P, _P, _P, _P]),
     "sr_test_adam": (_I, [_P, _P, _P, _P, C.c_size_t, _I, C.c_float, _P]),
+    "sr_test_mma2": (_I, [_P, _P, _P, _I, _I, _P]),
     "sr_test_mma": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _P, _P]),
     "sr_test_tma": (_I, [_P, _I, _I, _I, _I, _I, _I, _I, _I, _I, _I, _P, _P]),
 }

@@ -574,3 +574,90 @@ extern "C" int sr_test_grid_cap(int cap) {
   sr::set_grid_cap(cap);
   return 0;
 }
+
+// ---- CTA-pair prototype (pair.cuh): D[256 x N] = A[256 x K] B[N x K]^T with one cta_group::2 MMA chain.
+// CTA r of the pair holds A rows [128 r, 128 r + 128) (K-major, SWIZZLE_NONE) and B rows [N/2 r, N/2 r + N/2);
+// A arrives by a 2-D TMA box per CTA counted on the LEADER's barrier (cta_group::2 TMA), B by thread copies
+// (fence + remote arrive); the leader issues the MMAs and multicasts the commit; each CTA drains its 128 lanes.
+#include "pair.cuh"
+namespace sr {
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1)
+k_test_mma2(const __grid_constant__ CUtensorMap tma, const __nv_bfloat16* __restrict__ B, float* __restrict__ D,
+            int N, int K) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ __align__(8) uint64_t a_full, b_ready, done;
+  __shared__ uint32_t tmem_base;
+  const uint32_t rank = cluster_rank();
+  uint8_t* sA = smem;                    // [K/8 chunks][128 rows][16 B] via the 2-D box (8 elems x 128 rows) per chunk
+  uint8_t* sB = smem + 128 * K * 2;      // [K/8][N/2 rows][16 B]
+  const int NH = N / 2;
+  if (threadIdx.x == 0) {
+    mbar_init(&a_full, 2);   // one expect_tx arrival per CTA (leader's copy used)
+    mbar_init(&b_ready, 2);  // one arrival per CTA
+    mbar_init(&done, 1);
+    fence_barrier_init();
+  }
+  if (warp_id() == 0) tmem_alloc2<256>(&tmem_base);
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base;
+  // B half by threads
+  for (int i = threadIdx.x; i < NH * K; i += blockDim.x) {
+    const int n = i / K, k = i % K;
+    *reinterpret_cast<__nv_bfloat16*>(sB + (k / 8) * (NH * 16) + n * 16 + (k % 8) * 2) = B[(rank * NH + n) * K + k];
+  }
+  fence_proxy_async_smem();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t la = cluster_addr(&a_full, 0);
+    mbar_arrive_expect_tx_cluster(la, 128u * K * 2u);
+    for (int c = 0; c < K / 8; ++c) tma_load_2d_pair(sA + c * 2048, &tma, la, c * 8, (int)rank * 128);
+    mbar_arrive_cluster(cluster_addr(&b_ready, 0));
+  }
+  if (rank == 0 && threadIdx.x == 0) {
+    mbar_wait_cluster(&a_full, 0);
+    mbar_wait_cluster(&b_ready, 0);
+    tc_fence_after();
+    const uint32_t idesc = make_idesc(256, N, 0, 0);
+    const uint64_t ad = make_desc(smem_u32(sA), 2048, 128), bd = make_desc(smem_u32(sB), NH * 16, 128);
+    for (int k = 0; k < K / 16; ++k)
+      mma2_bf16_ss(tmem, desc_add(ad, k * 2 * 2048), desc_add(bd, k * 2 * NH * 16), idesc, k > 0);
+    mma2_commit_mc(&done, 0x3);
+  }
+  mbar_wait(&done, 0);
+  tc_fence_after();
+  const int q = warp_id(), lane = lane_id();
+  for (int c = 0; c < N; c += 8) {
+    float v[8];
+    tmem_ld8(tmem + ((uint32_t)(q * 32) << 16) + c, v);
+    tmem_ld_wait();
+    for (int e = 0; e < 8; ++e) D[(size_t)(rank * 128 + q * 32 + lane) * N + c + e] = v[e];
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  if (warp_id() == 0) tmem_dealloc2<256>(tmem);
+}
+}  // namespace sr
+
+// A [256][K] bf16 row-major, B [N][K] bf16 row-major -> D [256][N] fp32 (device pointers).  N % 16 == 0, N <= 256,
+// K % 16 == 0, K <= 64.
+extern "C" int sr_test_mma2(const void* A, const void* B, float* D, int N, int K, void* stream) {
+  using namespace sr;
+  auto fn = get_encode_fn();
+  if (!fn || N % 16 || N > 256 || K % 16 || K > 64) return SR_E_INVAL;
+  CUtensorMap tm;
+  cuuint64_t dims[2] = {(cuuint64_t)K, 256};
+  cuuint64_t strides[1] = {(cuuint64_t)K * 2};
+  cuuint32_t box[2] = {8, 128};
+  cuuint32_t es[2] = {1, 1};
+  if (fn(&tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(A), dims, strides, box, es,
+         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return SR_E_CUDA;
+  const size_t smem = 128 * K * 2 + (N / 2) * K * 2 + 1024;
+  cudaFuncSetAttribute(k_test_mma2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_test_mma2<<<2, 128, smem, (cudaStream_t)stream>>>(tm, (const __nv_bfloat16*)B, D, N, K);
+  cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
+  return e == cudaSuccess ? SR_OK : SR_E_CUDA;
+}

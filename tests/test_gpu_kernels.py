@@ -229,3 +229,20 @@ def test_sse_exact(lib):
     torch.cuda.synchronize()
     exp = ((a.astype(np.int64) - b.astype(np.int64)) ** 2).sum(axis=1)
     np.testing.assert_array_equal(out.cpu().numpy(), exp)
+
+
+@pytest.mark.parametrize("n,k", [(144, 48), (96, 64), (48, 16), (32, 32)])
+def test_cta_pair_mma_m256(n, k):
+    """tcgen05 cta_group::2 (pair.cuh): one M = 256 MMA chain over a 2-CTA cluster -- A rows split by CTA, B's N split
+    by CTA, A loaded by cta_group::2 TMA counted on the leader's barrier, multicast commit -- equals A @ B^T."""
+    from paper_conf_sigcomm_kimjyyh20_b200 import load
+    import ctypes
+    r = np.random.default_rng(n * 7 + k)
+    A = torch.from_numpy(r.standard_normal((256, k)).astype(np.float32)).to(torch.bfloat16).cuda()
+    B = torch.from_numpy(r.standard_normal((n, k)).astype(np.float32)).to(torch.bfloat16).cuda()
+    D = torch.zeros((256, n), dtype=torch.float32, device="cuda")
+    st = load().sr_test_mma2(ctypes.c_void_p(A.data_ptr()), ctypes.c_void_p(B.data_ptr()),
+                             ctypes.c_void_p(D.data_ptr()), n, k, ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    assert st == 0
+    ref = A.float() @ B.float().T
+    torch.testing.assert_close(D, ref, rtol=1e-5, atol=1e-4)
