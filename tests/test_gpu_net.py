@@ -661,3 +661,19 @@ def test_tiled_layouts_follow_fold_only_training_steps():
     g1 = ctx.grad_buffer().clone()
     fresh.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo2)
     assert torch.equal(g1, fresh.grad_buffer()) and lo1.item() == lo2.item()
+
+
+@pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (37, 272), 2), ((2, 3, 32), (29, 400), 3), ((3, 2, 48), (90, 700), 1),
+                                      ((2, 2, 32), (17, 1280), 1), ((3, 1, 48), (8, 126), 3)])
+def test_pair_resblock_equals_single_cta(cfg, hw, n):
+    """Residual blocks on CTA pairs (tcgen05 cta_group::2, M = 256 over two SMs, B split by N; default for wide
+    frames) == the single-CTA kernel (set_fusion bit 7), bit for bit: the same MMA sequence per output element.
+    Odd and even total strip counts (a dummy strip in the last pair), ragged last strips, several frames."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=81)
+    lr = torch.from_numpy(synth_frames(n, hw[0], hw[1], seed=82)).cuda()
+    a = ctx.infer(lr, "serve").clone()
+    ctx.set_fusion(1 | 128)
+    b = ctx.infer(lr, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
