@@ -50,11 +50,11 @@ struct B2Cfg {
   static constexpr uint32_t OFF_B1 = OFF_A2 + SLABS * R_A2 * 16;
   static constexpr uint32_t OFF_B2 = OFF_B1 + SLABS * R_B1 * 16;
   static constexpr uint32_t WBYTES = OFF_B2 + SLABS * R_B2 * 16;
-  static constexpr uint32_t WB_AL = (WBYTES + 1023u) & ~1023u;
+  static constexpr uint32_t WB_AL = (WBYTES + 127u) & ~127u;
   static constexpr uint32_t PLANE = 130 * 16;
   static constexpr uint32_t ROWB = ((CCH * PLANE) + 127u) & ~127u;
   static constexpr uint32_t OUTB = ((kB2TW * C * 2) + 1023u) & ~1023u;
-  static constexpr uint32_t ARMB = ((kArmOnesBytes + 2 * (C / 2) * 32) + 1023u) & ~1023u;  // ones + 2 half bias tiles
+  static constexpr uint32_t ARMB = ((kArmOnesBytes + 2 * (C / 2) * 32) + 127u) & ~127u;  // ones + 2 half bias tiles
   static constexpr size_t SMEM = 1024 + 2 * (size_t)WB_AL + (size_t)NF * ROWB + (size_t)NT * ROWB +
                                  (size_t)NO * OUTB + ARMB;
 };
@@ -461,9 +461,10 @@ static cudaError_t launch_block2_t(const CUtensorMap& tf, const CUtensorMap& to,
 }
 
 bool resblock2_supported(int cp, int W) {
+  constexpr size_t kStatic = 1024;  // barriers, TMEM address, bias staging (static shared memory)
   if (W < 96) return false;
-  if (cp == 32) return B2Cfg<32>::SMEM <= 227 * 1024;
-  if (cp == 48) return B2Cfg<48>::SMEM <= 227 * 1024;
+  if (cp == 32) return B2Cfg<32>::SMEM + kStatic <= 227 * 1024;
+  if (cp == 48) return B2Cfg<48>::SMEM + kStatic <= 227 * 1024;
   return false;
 }
 
