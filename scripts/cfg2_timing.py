@@ -9,6 +9,8 @@ from paper_conf_sigcomm_kimjyyh20_b200 import SRContext  # noqa: E402
 from synth import synth_frames  # noqa: E402
 
 ctx = SRContext(2, 8, 32, seed=0)
+if os.environ.get("SR_FUSION"):  # A/B of kernel variants (sr_set_fusion bits)
+    ctx.set_fusion(int(os.environ["SR_FUSION"]))
 lr = torch.from_numpy(synth_frames(30, 540, 960, seed=1002)).cuda()
 hr = torch.empty((30, 1080, 1920, 3), dtype=torch.uint8, device="cuda")
 for _ in range(3):
