@@ -215,7 +215,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       for (int i = 0; i < n_f; ++i) {
         mbar_wait(&f_empty[s], ph ^ 1);
         const uint32_t lf = cluster_addr(&f_full[s], 0);
-        mbar_arrive_expect_tx_cluster(lf, CCH * PLANE);
+        mbar_arrive_expect_tx_remote(lf, CCH * PLANE);
         tma_load_5d_pair(sF + s * ROWB, &tm_f, lf, 0, x0 - 2, y0 - 2 + i, 0, n);
         if (++s == NF) { s = 0; ph ^= 1; }
       }
@@ -230,9 +230,9 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
     // ===================== conv1 MMA issuer (leader): step st consumes f row st of both CTAs ====================
     if (elect_one()) {
       mbar_wait(&w_bar, 0);  // this CTA's weight regions have landed (the arming tiles before the cluster sync)
-      mbar_arrive_cluster(cluster_addr(&setup_bar, 0));
+      mbar_arrive_remote(cluster_addr(&setup_bar, 0));  // (the arming tiles were ordered by the cluster barrier)
       if (lead) {
-        mbar_wait_cluster(&setup_bar, 0);
+        mbar_wait(&setup_bar, 0);
         tc_fence_after();
         int fs = 0;
         uint32_t fph = 0;
@@ -240,8 +240,8 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
         SR_PIECE_BEGIN
         for (int st = 0; st < n_f; ++st) {
           const long long g = G1 + st;
-          for (; acq1 < g + 3; ++acq1) mbar_wait_cluster(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
-          mbar_wait_cluster(&f_full[fs], fph);
+          for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
+          mbar_wait(&f_full[fs], fph);
           tc_fence_after();
           if (st == 0) {
             ring_arm2<C, RB>(ring1, g, smem_u32(sOnes), smem_u32(sB1));
@@ -265,7 +265,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
   } else if (warp == 10) {
     // ===================== conv2 MMA issuer (leader): step k consumes t row k of both CTAs =====================
     if (lead && elect_one()) {
-      mbar_wait_cluster(&setup_bar, 0);
+      mbar_wait(&setup_bar, 0);
       tc_fence_after();
       int ts = 0;
       uint32_t tph = 0;
@@ -273,7 +273,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       SR_PIECE_BEGIN
       for (int k = 0; k < n_t; ++k) {
         const long long g = G2 + k;
-        for (; acq2 < g + 3; ++acq2) mbar_wait_cluster(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
+        for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
         mbar_wait_cluster(&t_full[ts], tph);
         tc_fence_after();
         if (k == 0) {
@@ -300,7 +300,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
     const int m = quarter * 32 + lane_id();
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
     for (int b = 0; b < RB; ++b)
-      if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&r1_free[b], 0));
+      if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r1_free[b], 0));
     int ts = 0;
     uint32_t tph = 0;
     long long G = 0;
@@ -322,7 +322,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
-      if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&r1_free[b], 0));
+      if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r1_free[b], 0));
       if (emit) {
         uint8_t* dst = sT + ts * ROWB + m * 16;
 #pragma unroll
@@ -356,7 +356,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
     const bool leader = (warp == 6 && lane_id() == 0);
     for (int b = 0; b < RB; ++b)
-      if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&r2_free[b], 0));
+      if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
     int os = 0;
     long long G = 0;
     SR_PIECE_BEGIN
@@ -398,7 +398,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
-      if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&r2_free[b], 0));
+      if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
       if (emit) {
         if (lane_ok) {
           uint8_t* orow = sO + os * OUTB + m * C * 2;

@@ -30,6 +30,15 @@ __device__ __forceinline__ void mbar_arrive_expect_tx_cluster(uint32_t caddr, ui
   asm volatile("mbarrier.arrive.expect_tx.release.cluster.shared::cluster.b64 _, [%0], %1;" ::"r"(caddr), "r"(bytes)
                : "memory");
 }
+// the same with the default (.release.cta) semantics: for signals that order no generic-proxy data across the pair
+// (TMEM blocks freed after tcgen05.ld + fence, TMA byte counts) -- a cluster-scope release would first wait for
+// every outstanding memory operation of the thread (e.g. the epilogue's residual prefetch)
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t caddr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(caddr) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx_remote(uint32_t caddr, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cluster.b64 _, [%0], %1;" ::"r"(caddr), "r"(bytes) : "memory");
+}
 // wait on a local mbarrier whose arrivals may come from the peer CTA (acquire at cluster scope)
 __device__ __forceinline__ bool mbar_try_wait_cluster(uint32_t addr, uint32_t phase) {
   uint32_t ok;
