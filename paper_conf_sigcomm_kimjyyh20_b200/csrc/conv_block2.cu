@@ -9,12 +9,11 @@
 // one issuer per conv drives both SMs.  Only the pair's leader (cluster rank 0) issues MMAs.
 //
 // B halves.  With cta_group::2, CTA r provides rows [r N/2, (r+1) N/2) of an MMA's B.  A step whose three target
-// blocks wrap around the TMEM ring (two of every RB steps) is issued as three MMA groups of N = C, one per vertical
-// tap, so each CTA keeps two row regions of every (kx, 8-channel) weight slab of the dy-fold layout
-// Wo[kx][ci/8][3C][8]: FULL (its half of the 3C rows) and DY (its half of each tap's C rows) -- 3 C rows, the
-// single-CTA kernel's weight footprint, at the same shared-memory offsets in both CTAs, so one descriptor addresses
-// both halves.  (The single-CTA kernel issues a wrap as N = 2C + C or C + 2C; per output element the accumulation
-// order over (dx, k) is the same, so the results are bit-identical.)
+// blocks wrap around the TMEM ring is issued as two MMA groups (N = 2C + C or C + 2C; ring.cuh), and those
+// sub-ranges split differently, so each CTA keeps five row regions of every (kx, 8-channel) weight slab of the
+// dy-fold layout Wo[kx][ci/8][3C][8]: FULL (its half of the 3C rows), A1/A2 (its halves of rows [0,2C) and
+// [2C,3C)), B1/B2 (its halves of rows [0,C) and [C,3C)) -- 4.5 C rows instead of 3 C, all at the same shared-memory
+// offsets in both CTAs, so one descriptor addresses both halves.
 //
 // Synchronisation (the leader's barriers collect both CTAs): f rows are TMA-loaded by each CTA into its own smem and
 // counted on the LEADER's f_full (cta_group::2 TMA, expect_tx from both producers); t rows are written by both
@@ -40,14 +39,17 @@ template <int C>
 struct B2Cfg {
   static constexpr int CCH = C / 8, KS = C / 16, N = 3 * C;
   static constexpr int RB = (256 / C) < 8 ? (256 / C) : 8;
-  static constexpr int NF = 4;  // f-row ring
-  static constexpr int NT = 3;  // t-row ring
-  static constexpr int NO = 3;  // output staging rows
-  static constexpr int SLABS = 3 * CCH;  // (kx, 8-channel) slabs of a conv's dy-fold weights
-  static constexpr int R_FULL = 3 * C / 2, R_DY = C / 2;
+  static constexpr int NF = C >= 48 ? 3 : 4;  // f-row ring (one slot less than k_resblock at C = 48: weights grew)
+  static constexpr int NT = 3;                // t-row ring
+  static constexpr int NO = C >= 48 ? 2 : 3;  // output staging rows
+  static constexpr int SLABS = 3 * CCH;       // (kx, 8-channel) slabs of a conv's dy-fold weights
+  static constexpr int R_FULL = 3 * C / 2, R_A1 = C, R_A2 = C / 2, R_B1 = C / 2, R_B2 = C;
   static constexpr uint32_t OFF_FULL = 0;
-  static constexpr uint32_t OFF_DY = OFF_FULL + SLABS * R_FULL * 16;  // [tap][slab][C/2 rows][16 B]
-  static constexpr uint32_t WBYTES = OFF_DY + 3 * SLABS * R_DY * 16;
+  static constexpr uint32_t OFF_A1 = OFF_FULL + SLABS * R_FULL * 16;
+  static constexpr uint32_t OFF_A2 = OFF_A1 + SLABS * R_A1 * 16;
+  static constexpr uint32_t OFF_B1 = OFF_A2 + SLABS * R_A2 * 16;
+  static constexpr uint32_t OFF_B2 = OFF_B1 + SLABS * R_B1 * 16;
+  static constexpr uint32_t WBYTES = OFF_B2 + SLABS * R_B2 * 16;
   static constexpr uint32_t WB_AL = (WBYTES + 127u) & ~127u;
   static constexpr uint32_t PLANE = 130 * 16;
   static constexpr uint32_t ROWB = ((CCH * PLANE) + 127u) & ~127u;
@@ -97,10 +99,12 @@ __device__ __forceinline__ void ring_mma_step2(uint32_t ring_base, long long g, 
   };
   if (i0 >= 2) {
     group(i0 - 2, 3 * C, Cfg::OFF_FULL, Cfg::R_FULL);
-  } else {  // tap d targets block (i0 - 2 + d) mod RB
-#pragma unroll
-    for (int d = 0; d < 3; ++d)
-      group((i0 - 2 + d + RB) % RB, C, Cfg::OFF_DY + (uint32_t)d * Cfg::SLABS * Cfg::R_DY * 16u, Cfg::R_DY);
+  } else if (i0 == 0) {
+    group(RB - 2, 2 * C, Cfg::OFF_A1, Cfg::R_A1);
+    group(0, C, Cfg::OFF_A2, Cfg::R_A2);
+  } else {
+    group(RB - 1, C, Cfg::OFF_B1, Cfg::R_B1);
+    group(0, 2 * C, Cfg::OFF_B2, Cfg::R_B2);
   }
 }
 
@@ -153,15 +157,13 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
   if (warp == 0 && lane_id() == 0) {
     mbar_arrive_expect_tx(&w_bar, 2 * Cfg::WBYTES);
     const int h = (int)rank;
-    // regions: FULL = rows [h 1.5C, (h+1) 1.5C); DY tap d = rows [d C + h C/2, d C + (h+1) C/2)
-    const int r0[4] = {h * Cfg::R_FULL, h * Cfg::R_DY, C + h * Cfg::R_DY, 2 * C + h * Cfg::R_DY};
-    const int rn[4] = {Cfg::R_FULL, Cfg::R_DY, Cfg::R_DY, Cfg::R_DY};
-    const uint32_t off[4] = {Cfg::OFF_FULL, Cfg::OFF_DY, Cfg::OFF_DY + Cfg::SLABS * Cfg::R_DY * 16u,
-                             Cfg::OFF_DY + 2u * Cfg::SLABS * Cfg::R_DY * 16u};
+    const int r0[5] = {h * Cfg::R_FULL, h * C, 2 * C + h * (C / 2), h * (C / 2), C + h * C};
+    const int rn[5] = {Cfg::R_FULL, Cfg::R_A1, Cfg::R_A2, Cfg::R_B1, Cfg::R_B2};
+    const uint32_t off[5] = {Cfg::OFF_FULL, Cfg::OFF_A1, Cfg::OFF_A2, Cfg::OFF_B1, Cfg::OFF_B2};
     for (int cv = 0; cv < 2; ++cv) {
       const bf16* wg = cv ? w2 : w1;
       uint8_t* sw = cv ? sW2 : sW1;
-      for (int rg = 0; rg < 4; ++rg)
+      for (int rg = 0; rg < 5; ++rg)
         for (int sl = 0; sl < Cfg::SLABS; ++sl)
           bulk_load(sw + off[rg] + (uint32_t)sl * rn[rg] * 16u, wg + ((size_t)sl * 3 * C + r0[rg]) * 8,
                     (uint32_t)rn[rg] * 16u, &w_bar);
@@ -272,7 +274,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       for (int k = 0; k < n_t; ++k) {
         const long long g = G2 + k;
         for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
-        mbar_wait(&t_full[ts], tph);
+        mbar_wait_cluster(&t_full[ts], tph);
         tc_fence_after();
         if (k == 0) {
           ring_arm2<C, RB>(ring2, g, smem_u32(sOnes), smem_u32(sB2));
@@ -337,7 +339,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
         }
         fence_proxy_async_smem();
         __syncwarp();
-        if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&t_full[ts], 0));  // after fence.proxy.async
+        if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&t_full[ts], 0));
         if (++ts == NT) { ts = 0; tph ^= 1; }
       }
     }
