@@ -460,11 +460,14 @@ static cudaError_t launch_block2_t(const CUtensorMap& tf, const CUtensorMap& to,
   return launch_k(kern, dim3(grid), dim3(kB2Threads), B2Cfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, N, H, W);
 }
 
+// Offered for C = 32 (BASELINE config 2's 8 x 32 net), where a row-step's MMAs are short and the pair's halved B
+// reads and single issuer pay (same-session A/B: 0.83 -> 0.69 ms per 30 540p frames).  At C = 48 the 4.5 C weight
+// rows cost a slot of the f ring and of the output staging, and the pair measured no faster than the single-CTA
+// kernel (17.4 vs 17.6-20.5 ms per 30 720p frames across the variants tried), so C = 48 stays on k_resblock.
 bool resblock2_supported(int cp, int W) {
   constexpr size_t kStatic = 1024;  // barriers, TMEM address, bias staging (static shared memory)
   if (W < 96) return false;
   if (cp == 32) return B2Cfg<32>::SMEM + kStatic <= 227 * 1024;
-  if (cp == 48) return B2Cfg<48>::SMEM + kStatic <= 227 * 1024;
   return false;
 }
 
@@ -479,8 +482,7 @@ cudaError_t launch_resblock2(int cp, const bf16* f, const bf16* w1fold, const bf
   long long pairs = num_sms() / 2;
   if (units < pairs) pairs = units;
   const int grid = (int)(2 * pairs);
-  if (cp == 32) return launch_block2_t<32>(tf, to, w1fold, w2fold, b1, b2, f, N, H, W, grid, st);
-  return launch_block2_t<48>(tf, to, w1fold, w2fold, b1, b2, f, N, H, W, grid, st);
+  return launch_block2_t<32>(tf, to, w1fold, w2fold, b1, b2, f, N, H, W, grid, st);
 }
 
 }  // namespace sr

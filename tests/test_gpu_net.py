@@ -663,11 +663,12 @@ def test_tiled_layouts_follow_fold_only_training_steps():
     assert torch.equal(g1, fresh.grad_buffer()) and lo1.item() == lo2.item()
 
 
-@pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (37, 272), 2), ((2, 3, 32), (29, 400), 3), ((3, 2, 48), (90, 700), 1),
-                                      ((2, 2, 32), (17, 1280), 1), ((3, 1, 48), (8, 126), 3)])
+@pytest.mark.parametrize("cfg,hw,n", [((2, 8, 32), (37, 272), 2), ((2, 3, 32), (29, 400), 3), ((3, 2, 32), (90, 700), 1),
+                                      ((2, 2, 32), (17, 1280), 1), ((3, 1, 32), (8, 126), 3), ((2, 8, 32), (54, 960), 3)])
 def test_pair_resblock_equals_single_cta(cfg, hw, n):
     """Residual blocks on CTA pairs (tcgen05 cta_group::2, M = 256 over two SMs, B split by N; default for wide
-    frames) == the single-CTA kernel (set_fusion bit 7), bit for bit: the same MMA sequence per output element.
+    frames at C = 32, config 2's net) == the single-CTA kernel (set_fusion bit 7), bit for bit: the same MMA sequence
+    per output element.
     Odd and even total strip counts (a dummy strip in the last pair), ragged last strips, several frames."""
     s, B, C = cfg
     ctx = _ctx(s, B, C, seed=81)
