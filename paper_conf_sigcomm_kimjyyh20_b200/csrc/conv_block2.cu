@@ -17,7 +17,8 @@
 //
 // Synchronisation (the leader's barriers collect both CTAs): f rows are TMA-loaded by each CTA into its own smem and
 // counted on the LEADER's f_full (cta_group::2 TMA, expect_tx from both producers); t rows are written by both
-// CTAs' conv1 epilogues and announced on the leader's t_full (fence.proxy.async + release.cluster arrive); ring
+// CTAs' conv1 epilogues (each SM's tensor core reads its own CTA's rows) and announced on the leader's t_full
+// (fence.proxy.async, then a remote arrive: a cluster-scope release there cost 30% in an A/B); ring
 // blocks are freed on the leader's r1_free / r2_free by both CTAs' epilogues; the leader's commits multicast
 // r*_ready, f_empty and t_empty to both CTAs.  Weights and bias-arming tiles of both CTAs are announced on the
 // leader's setup_bar.  Results are bit-identical to k_resblock: the same MMA sequence per output element.
@@ -274,7 +275,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       for (int k = 0; k < n_t; ++k) {
         const long long g = G2 + k;
         for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
-        mbar_wait_cluster(&t_full[ts], tph);
+        mbar_wait(&t_full[ts], tph);
         tc_fence_after();
         if (k == 0) {
           ring_arm2<C, RB>(ring2, g, smem_u32(sOnes), smem_u32(sB2));
@@ -339,7 +340,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
         }
         fence_proxy_async_smem();
         __syncwarp();
-        if (lane_id() == 0) mbar_arrive_cluster(cluster_addr(&t_full[ts], 0));
+        if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&t_full[ts], 0));  // after fence.proxy.async
         if (++ts == NT) { ts = 0; tph ^= 1; }
       }
     }
