@@ -216,6 +216,8 @@ def run_ours(args):
     def barrier():
         if world > 1:
             dist.barrier()
+        for s_ in (s_inf, s_tr):  # the partitions' streams (green contexts) explicitly
+            s_.synchronize()
         torch.cuda.synchronize()
 
     def t_start():
@@ -230,6 +232,8 @@ def run_ours(args):
             ev = torch.cuda.Event(enable_timing=True)
             ev.record(s_)
             evs.append(ev)
+        for ev in evs:
+            ev.synchronize()
         torch.cuda.synchronize()
         return max(e0.elapsed_time(ev) for ev in evs)
 

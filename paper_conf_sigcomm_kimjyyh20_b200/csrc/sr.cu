@@ -17,6 +17,20 @@
 
 using namespace sr;
 
+// Streams of the green-context SM partitions (sr_sm_partition).  The synchronous calls below wait for them too:
+// a device-wide synchronize of the primary context is not documented to cover work on green-context streams.
+static std::vector<cudaStream_t> g_part_streams;
+static std::mutex g_part_mu;
+static cudaError_t sync_all() {
+  cudaError_t e = cudaDeviceSynchronize();
+  std::lock_guard<std::mutex> lk(g_part_mu);
+  for (cudaStream_t s : g_part_streams) {
+    const cudaError_t e2 = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) e = e2;
+  }
+  return e;
+}
+
 // ---------------------------------------------------------------------------------- NCCL (T5)
 // The data-parallel gradient exchange is one sum-allreduce of the flat fp32 gradient over NVLink/NVSwitch.  libnccl
 // is resolved at run time (SR_NCCL_LIB, else the soname "libnccl.so.2": the copy torch already loaded if any, else the
@@ -959,7 +973,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
 
 void sr_destroy(sr_ctx* ctx) {
   if (!ctx) return;
-  cudaDeviceSynchronize();
+  sync_all();
   for (InferWS* ws : {&ctx->iws, &ctx->qws})
     for (bf16* q : {ws->x16, ws->f0, ws->fa, ws->fb, ws->tt})
       if (q) cudaFree(q);
@@ -1022,7 +1036,7 @@ sr_status sr_kernel_timing(sr_ctx* ctx, int enable) {
 
 int sr_kernel_stats(sr_ctx* ctx, char* buf, size_t cap) {
   if (!ctx || !buf || cap == 0) return SR_E_INVAL;
-  if (cudaDeviceSynchronize() != cudaSuccess) return SR_E_CUDA;
+  if (sync_all() != cudaSuccess) return SR_E_CUDA;
   struct Acc { long long n = 0; double ms = 0, flops = 0, bytes = 0; };
   std::vector<std::pair<std::string, Acc>> acc;
   for (size_t i = 0; i < ctx->tnext; ++i) {
@@ -1096,14 +1110,14 @@ sr_status sr_set_params(sr_ctx* ctx, const float* host_in, size_t n) {
     CK(cudaMemcpy(ctx->snap[k].bias, ctx->snap[SR_TRAIN].bias, ctx->b_total * sizeof(float),
                   cudaMemcpyDeviceToDevice));
   }
-  CK(cudaDeviceSynchronize());
+  CK(sync_all());
   return SR_OK;
 }
 
 sr_status sr_get_params(sr_ctx* ctx, sr_model which, float* host_out, size_t n) {
   GUARD();
   if (!host_out || n != ctx->nparams || !valid_model(which)) return fail(ctx, SR_E_INVAL, "sr_get_params: bad args");
-  CK(cudaDeviceSynchronize());
+  CK(sync_all());
   if (which == SR_TRAIN) {
     CK(cudaMemcpy(host_out, ctx->params, n * sizeof(float), cudaMemcpyDeviceToHost));
     return SR_OK;
@@ -1390,7 +1404,7 @@ size_t sr_pool_size(const sr_ctx* ctx) {
 sr_status sr_pool_stats(sr_ctx* ctx, int64_t* arrivals, int64_t* clamped) {
   GUARD();
   long long h[2] = {0, 0};
-  CK(cudaDeviceSynchronize());
+  CK(sync_all());
   CK(cudaMemcpy(h, ctx->counters + 3, sizeof h, cudaMemcpyDeviceToHost));
   if (arrivals) *arrivals = h[0];
   if (clamped) *clamped = h[1];
@@ -1768,6 +1782,11 @@ sr_status sr_sm_partition(int train_sms, sr_stream* infer_stream, sr_stream* tra
     g_green.push_back(gt);
     g_green.push_back(gi);
   }
+  {
+    std::lock_guard<std::mutex> lk(g_part_mu);
+    g_part_streams.push_back(reinterpret_cast<cudaStream_t>(st_t));
+    g_part_streams.push_back(reinterpret_cast<cudaStream_t>(st_i));
+  }
   *train_stream = reinterpret_cast<sr_stream>(st_t);
   *infer_stream = reinterpret_cast<sr_stream>(st_i);
   if (train_sms_out) *train_sms_out = (int)grp[0].sm.smCount;
@@ -1776,7 +1795,11 @@ sr_status sr_sm_partition(int train_sms, sr_stream* infer_stream, sr_stream* tra
 }
 
 sr_status sr_sm_partition_release(void) {
-  cudaDeviceSynchronize();
+  sync_all();
+  {
+    std::lock_guard<std::mutex> lk(g_part_mu);
+    g_part_streams.clear();
+  }
   std::lock_guard<std::mutex> lk(g_green_mu);
   GreenApi& g = green();
   for (CUgreenCtx c : g_green) g.destroy(c);
@@ -1787,7 +1810,7 @@ sr_status sr_sm_partition_release(void) {
 sr_status sr_get_adam_state(sr_ctx* ctx, float* m_host, float* v_host, size_t n, int64_t* t_host) {
   GUARD();
   if (n != ctx->nparams) return fail(ctx, SR_E_INVAL, "sr_get_adam_state: size mismatch");
-  CK(cudaDeviceSynchronize());
+  CK(sync_all());
   if (m_host) CK(cudaMemcpy(m_host, ctx->m, n * sizeof(float), cudaMemcpyDeviceToHost));
   if (v_host) CK(cudaMemcpy(v_host, ctx->v, n * sizeof(float), cudaMemcpyDeviceToHost));
   if (t_host) {

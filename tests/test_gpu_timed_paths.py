@@ -334,7 +334,10 @@ def test_nccl_allreduce_on_partition_stream():
     for c in (a, b):
         c.set_sm_split(nt)
         c.train_sampled(4, 16, 48, stream=stt)
+    stt.synchronize()  # the partition's own stream (green context)
     torch.cuda.synchronize()
+    ta, tb = a.adam_state()[2], b.adam_state()[2]
+    assert ta == tb == 4, (ta, tb)
     np.testing.assert_array_equal(a.get_params("train"), b.get_params("train"))
     for c in (a, b):
         c.set_sm_split(0)
