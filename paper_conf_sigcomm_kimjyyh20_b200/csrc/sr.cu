@@ -98,6 +98,8 @@ struct sr_ctx {
   cudaStream_t copy_st = nullptr, h2d_st = nullptr;  // sr_infer_host: PCIe copies overlapped with the tensor work
   std::vector<cudaEvent_t> chunk_ev[2];
   cudaEvent_t host_done[2] = {nullptr, nullptr};  // last D2H of the call that used the set
+  cudaEvent_t set_read[2] = {nullptr, nullptr};   // last inference chunk of the call that used the set (its LR read)
+  bool set_used[2] = {false, false};
   bool host_busy[2] = {false, false};
   unsigned long long host_calls = 0;
   size_t stage_lr_bytes[2] = {0, 0}, stage_hr_bytes[2] = {0, 0};
@@ -982,6 +984,7 @@ void sr_destroy(sr_ctx* ctx) {
     if (ctx->stage_hr[k]) cudaFree(ctx->stage_hr[k]);
     for (auto e : ctx->chunk_ev[k]) if (e) cudaEventDestroy(e);
     if (ctx->host_done[k]) cudaEventDestroy(ctx->host_done[k]);
+    if (ctx->set_read[k]) cudaEventDestroy(ctx->set_read[k]);
   }
   void* ptrs[] = {ctx->convs_dev, ctx->params, ctx->m, ctx->v, ctx->grad, ctx->wd_train, ctx->wdo_train, ctx->tx16, ctx->tg, ctx->tdy,
                   ctx->tdg, ctx->tdfa, ctx->tdfb, ctx->tdt, ctx->ws_w, ctx->wg_sync, ctx->loss_sum, ctx->counters,
@@ -1214,6 +1217,8 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
     CK(cudaStreamCreateWithFlags(&ctx->h2d_st, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&ctx->host_done[0], cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ctx->host_done[1], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ctx->set_read[0], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ctx->set_read[1], cudaEventDisableTiming));
   }
   // Chunked pipeline: all H2D copies go first on their own stream (per-chunk events), chunk k is super-resolved
   // on `stream` as soon as its frames landed, and its D2H runs on a third stream while chunk k+1 computes.
@@ -1223,7 +1228,11 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
   // frame's H2D) and a one-frame last chunk (only one frame's D2H is left exposed after the last kernel).
   const int F = std::max(1, std::min(n, (int)std::max<size_t>(1, (size_t)(240u << 20) / std::max<size_t>(fh, 1))));
   std::vector<int> c0s;  // first frame of each chunk (+ n at the end)
-  {
+  if (!sync && n >= 2) {
+    // two calls in flight: this call's H2D overlaps the previous call's compute and its D2H the next call's, so
+    // the batch goes as two chunks (fewer, larger inference launches)
+    c0s = {0, (n + 1) / 2, n};
+  } else {
     int f = 0;
     c0s.push_back(0);
     if (n >= 3 && F > 1) { f = 1; c0s.push_back(f); }
@@ -1236,15 +1245,16 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
     }
   }
   const int nch = (int)c0s.size() - 1;
+  (void)F;
   while ((int)ctx->chunk_ev[set].size() < 2 * nch + 1) {
     cudaEvent_t e;
     CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     ctx->chunk_ev[set].push_back(e);
   }
   cudaEvent_t* ev = ctx->chunk_ev[set].data();  // [0] start, [1 + c] chunk c landed, [1 + nch + c] chunk c done
-  CK(cudaEventRecord(ev[0], st));
-  CK(cudaStreamWaitEvent(ctx->h2d_st, ev[0], 0));  // copies follow earlier work on `stream`
-  CK(cudaStreamWaitEvent(ctx->copy_st, ev[0], 0));
+  // the H2D into this staging set waits only for the inference that last read it (two calls back), not for all
+  // earlier work on `stream`: it overlaps the previous call's compute
+  if (ctx->set_used[set]) CK(cudaStreamWaitEvent(ctx->h2d_st, ctx->set_read[set], 0));
   for (int c = 0; c < nch; ++c) {
     const int f0 = c0s[c], fn = c0s[c + 1] - c0s[c];
     CK(cudaMemcpyAsync(stage_lr + f0 * fl, lr_host + f0 * fl, fn * fl, cudaMemcpyHostToDevice, ctx->h2d_st));
@@ -1255,6 +1265,10 @@ static sr_status infer_host_impl(sr_ctx* ctx, sr_model which, const uint8_t* lr_
     CK(cudaStreamWaitEvent(st, ev[1 + c], 0));
     TRY(sr_infer(ctx, which, stage_lr + f0 * fl, fn, h, w, stage_hr + f0 * fh, stream));
     CK(cudaEventRecord(ev[1 + nch + c], st));
+    if (c == nch - 1) {
+      CK(cudaEventRecord(ctx->set_read[set], st));
+      ctx->set_used[set] = true;
+    }
     CK(cudaStreamWaitEvent(ctx->copy_st, ev[1 + nch + c], 0));
     CK(cudaMemcpyAsync(hr_host + f0 * fh, stage_hr + f0 * fh, fn * fh, cudaMemcpyDeviceToHost, ctx->copy_st));
   }
