@@ -341,3 +341,32 @@ def test_nccl_allreduce_on_partition_stream():
     np.testing.assert_array_equal(a.get_params("train"), b.get_params("train"))
     for c in (a, b):
         c.set_sm_split(0)
+
+
+def test_dp_error_paths():
+    """world > 1 without a communicator: sr_train_step / sr_train_sampled / sr_train_allreduce refuse (SR_E_STATE) and
+    leave TRAIN untouched, while the caller-exchange split (sr_train_grad + sr_train_apply) works; sr_dp_weight_sum is
+    0 there (unknown); sr_sm_partition rejects impossible splits."""
+    from paper_conf_sigcomm_kimjyyh20_b200 import SRContext, SRError
+    ctx = _ctx(2, 1, 16, seed=4, world=2, rank=1)
+    assert ctx.dp_weight_sum == 0.0
+    lrp, hrp, _ = synth_patch_pool(8, 2, 48, seed=9, frame_hw=(192, 384))
+    lr, hr = torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda()
+    p0 = ctx.get_params("train")
+    with pytest.raises(SRError):
+        ctx.train_step(lr, hr)
+    ctx2 = _ctx(2, 1, 16, seed=4, world=2, rank=1)
+    with pytest.raises(SRError):
+        ctx2.train_allreduce()
+    ctx3 = _ctx(2, 1, 16, seed=4, world=2, rank=1)
+    ctx3.pool_push(lr, hr)
+    with pytest.raises(SRError):
+        ctx3.train_sampled(1, 4, 16)
+    np.testing.assert_array_equal(_ctx(2, 1, 16, seed=4, world=2, rank=1).get_params("train"), p0)
+    ok = _ctx(2, 1, 16, seed=4, world=2, rank=1)
+    ok.train_grad(lr, hr)
+    ok.train_apply(1.0)  # the caller's own exchange (here: none) and 1 / sum w
+    assert not np.array_equal(ok.get_params("train"), p0)
+    for bad in (0, 148, 1000):
+        with pytest.raises(SRError):
+            SRContext.sm_partition(bad)
