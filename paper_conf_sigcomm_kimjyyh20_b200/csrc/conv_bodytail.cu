@@ -74,7 +74,11 @@ struct BtArgs {
 #define SR_BDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
 
-template <int C, int CO2, int S>
+// BIC: bicubic skip (else bilinear).  A template parameter, so each kernel carries only its own tail code
+// (k_bodytail<48,32,3> -3.4% with the bicubic code compiled out, scripts/bt_time.py A/B).  The kernel is very
+// sensitive to code shape: compiling the (null-checked) clock64 stamps out made it 10% slower, a runtime
+// experiment mask 13% slower -- measure every change to it.
+template <int C, int CO2, int S, bool BIC>
 __global__ void __launch_bounds__(kBtThreads, 1)
 k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_lr,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const BtArgs a) {
@@ -356,7 +360,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       if (lane_ok) {
         uint8_t o[S * S * 3];
         tail_u8_px<S>(smem_u32(sL + ls * kBtLrSlot) - (uint32_t)lbase + 0u, 16 * kBtLrChunks, 0, r, xc, H, W, v,
-                      a.bicubic, o);
+                      BIC ? 1 : 0, o);
 #pragma unroll
         for (int i = 0; i < S; ++i) {
           const uint32_t sh = (uint32_t)(reinterpret_cast<uintptr_t>(hrow0 + (size_t)i * sW * 3) & 15);
@@ -395,13 +399,13 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-template <int C, int CO2, int S>
+template <int C, int CO2, int S, bool BIC>
 static cudaError_t launch_bt_t(const CUtensorMap& tf, const CUtensorMap& tl, const bf16* w1, const bf16* w2,
                                const BtArgs& a, int grid, cudaStream_t st) {
   if constexpr (!BtCfg<C, CO2, S>::FITS) {
     return cudaErrorNotSupported;
   } else {
-    auto kern = k_bodytail<C, CO2, S>;
+    auto kern = k_bodytail<C, CO2, S, BIC>;
     static bool configured = false;
     if (!configured) {
       cudaError_t e =
@@ -441,7 +445,9 @@ cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const 
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
 #define SR_BT_CASE(C, S) \
-  if (cp == C && s == S) return launch_bt_t<C, (S == 2 ? 16 : (S == 3 ? 32 : 48)), S>(tf, tl, w1fold, w2fold, a, grid, st);
+  if (cp == C && s == S)                                                                                   \
+    return bicubic ? launch_bt_t<C, (S == 2 ? 16 : (S == 3 ? 32 : 48)), S, true>(tf, tl, w1fold, w2fold, a, grid, st) \
+                   : launch_bt_t<C, (S == 2 ? 16 : (S == 3 ? 32 : 48)), S, false>(tf, tl, w1fold, w2fold, a, grid, st);
   SR_BT_CASE(16, 2) SR_BT_CASE(16, 3) SR_BT_CASE(16, 4)
   SR_BT_CASE(32, 2) SR_BT_CASE(32, 3) SR_BT_CASE(32, 4)
   SR_BT_CASE(48, 2) SR_BT_CASE(48, 3) SR_BT_CASE(48, 4)

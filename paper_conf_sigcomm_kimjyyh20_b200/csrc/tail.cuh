@@ -283,15 +283,33 @@ __device__ __forceinline__ void tail_u8_px(uint32_t L, int lpitch, int lbase, in
     }
     return;
   }
+  // the 9 bytes of pixels X-1 .. X+1 of an LR row come from 3 aligned words (one wavefront each, instead of 9
+  // byte loads), then edge replication replaces the pixel outside the frame (the slot holds the strip's pixels
+  // with a margin, so the words are inside it)
   float nb[3][3][3];
+  const uint32_t b0 = 3u * (uint32_t)X - 3u;  // byte of pixel X-1 (wraps at X = 0; that pixel is replaced)
+  const bool lclamp = X == 0, rclamp = X + 1 >= W;
 #pragma unroll
   for (int a = 0; a < 3; ++a) {
-    const uint32_t lrow = L + (min(max(Y + a - 1, 0), H - 1) - Y + 2) * lpitch - lbase;
+    const uint32_t ad = L + (min(max(Y + a - 1, 0), H - 1) - Y + 2) * lpitch - lbase + b0;
+    const uint32_t wa = ad & ~3u, sft = 8u * (ad & 3u);
+    uint32_t w0, w1, w2;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w0) : "r"(wa));
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w1) : "r"(wa + 4));
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w2) : "r"(wa + 8));
+    const uint32_t q0 = __funnelshift_r(w0, w1, sft), q1 = __funnelshift_r(w1, w2, sft), q2 = w2 >> sft;
+    float px[9];
 #pragma unroll
-    for (int b = 0; b < 3; ++b) {
-      const uint32_t p = lrow + 3 * min(max(X + b - 1, 0), W - 1);
+    for (int k = 0; k < 4; ++k) {
+      px[k] = (float)((q0 >> (8 * k)) & 0xffu);
+      px[4 + k] = (float)((q1 >> (8 * k)) & 0xffu);
+    }
+    px[8] = (float)(q2 & 0xffu);
 #pragma unroll
-      for (int c = 0; c < 3; ++c) nb[a][b][c] = lds_u8f(p + c);
+    for (int c = 0; c < 3; ++c) {
+      nb[a][1][c] = px[3 + c];
+      nb[a][0][c] = lclamp ? px[3 + c] : px[c];
+      nb[a][2][c] = rclamp ? px[3 + c] : px[6 + c];
     }
   }
   float hx[3][S][3];

@@ -560,11 +560,13 @@ extern "C" int sr_bench_bodytail_dbg(int cp, int s, int n, int h, int w, long lo
   cudaEventCreate(&b);
   launch_bodytail(cp, s, x, f0, w1, w2, bias, bias, lr, hr, 0, h, 0, n, h, w, st);  // warm
   cudaEventRecord(a, st);
-  cudaError_t e = launch_bodytail(cp, s, x, f0, w1, w2, bias, bias, lr, hr, 0, h, 0, n, h, w, st, dbg);
+  // dbg_host == nullptr: the production (stamp-free) kernel variant is timed
+  cudaError_t e = launch_bodytail(cp, s, x, f0, w1, w2, bias, bias, lr, hr, 0, h, 0, n, h, w, st,
+                                  dbg_host ? dbg : nullptr);
   cudaEventRecord(b, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
   cudaEventElapsedTime(ms_out, a, b);
-  cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
+  if (dbg_host) cudaMemcpy(dbg_host, dbg, 16 * 256 * 8, cudaMemcpyDeviceToHost);
   cudaFree(x); cudaFree(f0); cudaFree(lr); cudaFree(hr); cudaFree(w1); cudaFree(w2); cudaFree(bias); cudaFree(dbg);
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
