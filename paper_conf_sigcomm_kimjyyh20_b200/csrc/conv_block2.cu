@@ -76,7 +76,7 @@ __device__ __forceinline__ void arm_half_fill(uint8_t* btile, const float* bias,
 }
 
 template <int C, int RB>
-__device__ __forceinline__ void ring_arm2(uint32_t ring_base, long long g, uint32_t ones_saddr, uint32_t btile_saddr) {
+__device__ __forceinline__ void ring_arm2(uint32_t ring_base, unsigned g, uint32_t ones_saddr, uint32_t btile_saddr) {
   constexpr uint32_t id = make_idesc(256, C, 0, 0);
   mma2_bf16_ss(ring_base + ring_idx<RB>(g) * C, make_desc(ones_saddr, 2048, 128),
                make_desc(btile_saddr, (C / 2) * 16, 128), id, 0u);
@@ -84,7 +84,7 @@ __device__ __forceinline__ void ring_arm2(uint32_t ring_base, long long g, uint3
 
 // one input-row step of a dy-fold conv on the pair (see ring_mma_step in ring.cuh for the single-CTA form)
 template <int C, int RB>
-__device__ __forceinline__ void ring_mma_step2(uint32_t ring_base, long long g, uint64_t ad, uint32_t sw,
+__device__ __forceinline__ void ring_mma_step2(uint32_t ring_base, unsigned g, uint64_t ad, uint32_t sw,
                                                uint32_t kstride) {
   using Cfg = B2Cfg<C>;
   constexpr int CCH = Cfg::CCH, KS = Cfg::KS;
@@ -237,10 +237,10 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
         tc_fence_after();
         int fs = 0;
         uint32_t fph = 0;
-        long long G1 = 0, acq1 = 0;
+        unsigned G1 = 0, acq1 = 0;
         SR_PIECE_BEGIN
         for (int st = 0; st < n_f; ++st) {
-          const long long g = G1 + st;
+          const unsigned g = G1 + st;
           for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB>(acq1)], (uint32_t)(acq1 / RB) & 1u);
           mbar_wait(&f_full[fs], fph);
           tc_fence_after();
@@ -270,10 +270,10 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       tc_fence_after();
       int ts = 0;
       uint32_t tph = 0;
-      long long G2 = 0, acq2 = 0;
+      unsigned G2 = 0, acq2 = 0;
       SR_PIECE_BEGIN
       for (int k = 0; k < n_t; ++k) {
-        const long long g = G2 + k;
+        const unsigned g = G2 + k;
         for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB>(acq2)], (uint32_t)(acq2 / RB) & 1u);
         mbar_wait(&t_full[ts], tph);
         tc_fence_after();
@@ -304,12 +304,12 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r1_free[b], 0));
     int ts = 0;
     uint32_t tph = 0;
-    long long G = 0;
+    unsigned G = 0;
     SR_PIECE_BEGIN
     const int tcol = x0 - 1 + m;
     const bool col_ok = tcol >= 0 && tcol < W;
     for (int q = -1; q <= n_f; ++q) {  // out rows of conv1 = t rows y0-2+q
-      const long long g = G + q + 1;
+      const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_f - 2;
       const int trow = y0 - 2 + q;
       const bool ok = col_ok && trow >= 0 && trow < H;
@@ -359,7 +359,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
     for (int b = 0; b < RB; ++b)
       if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
     int os = 0;
-    long long G = 0;
+    unsigned G = 0;
     SR_PIECE_BEGIN
     const bool lane_ok = m < kB2TW && x0 + m < W;
     constexpr int kAhead = C <= 32 ? 2 : 1;
@@ -379,7 +379,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       ld_res(0);
     }
     for (int q = -1; q <= n_t; ++q) {  // out rows of conv2 = output rows y0-1+q
-      const long long g = G + q + 1;
+      const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
       const int r = y0 - 1 + q;
       uint4 res[C / 8];

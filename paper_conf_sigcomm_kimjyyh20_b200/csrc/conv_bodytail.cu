@@ -180,10 +180,10 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       const uint64_t bd1 = make_desc(smem_u32(sW1), 3 * C * 16, 128);
       int fs = 0;
       uint32_t fph = 0;
-      long long G1 = 0, acq1 = 0;
+      unsigned G1 = 0, acq1 = 0;
       SR_PIECE_BEGIN
       for (int st = 0; st < n_f; ++st) {
-        const long long g = G1 + st;
+        const unsigned g = G1 + st;
         SR_BDBG(7, st)
         for (; acq1 < g + 3; ++acq1) mbar_wait(&r1_free[ring_idx<RB1>(acq1)], (uint32_t)(acq1 / RB1) & 1u);
         SR_BDBG(8, st)
@@ -216,10 +216,10 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       const uint64_t bd2 = make_desc(smem_u32(sW2), 3 * CO2 * 16, 128);
       int ts = 0;
       uint32_t tph = 0;
-      long long G2 = 0, acq2 = 0;
+      unsigned G2 = 0, acq2 = 0;
       SR_PIECE_BEGIN
       for (int k = 0; k < n_t; ++k) {
-        const long long g = G2 + k;
+        const unsigned g = G2 + k;
         SR_BDBG(10, k + 3)
         for (; acq2 < g + 3; ++acq2) mbar_wait(&r2_free[ring_idx<RB2>(acq2)], (uint32_t)(acq2 / RB2) & 1u);
         SR_BDBG(11, k + 3)
@@ -254,7 +254,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       if (lane_id() == 0) mbar_arrive(&r1_free[b]);
     int ts = 0;
     uint32_t tph = 0;
-    long long G = 0;
+    unsigned G = 0;
     SR_PIECE_BEGIN
     const int tcol = x0 - 1 + m;
     const bool col_ok = tcol >= 0 && tcol < W;
@@ -269,7 +269,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
     };
     ld_res(-1);
     for (int q = -1; q <= n_f; ++q) {  // out rows of conv1 = g rows y0-2+q
-      const long long g = G + q + 1;
+      const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_f - 2;
       const int trow = y0 - 2 + q;
       const bool ok = col_ok && trow >= 0 && trow < H;
@@ -327,16 +327,16 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         if (lane_id() == 0) mbar_arrive(&r2_free[b]);
     const int sH = S * H, sW = S * W;
     int os = 0;
-    long long G = 0, emitted = 0;  // emitted: output rows of both groups so far (LR ring order)
+    unsigned G = 0, emitted = 0;  // emitted: output rows of both groups so far (LR ring order)
     SR_PIECE_BEGIN
     const int xc = x0 + m;
     const bool lane_ok = m < kBtTW && xc < W;
     const int lbase = 16 * ((3 * x0 - 6) >> 4);  // LR byte of the slot's first chunk
     const int nbytes = min(kBtTW, W - x0) * 3 * S;  // HR bytes of this strip per row
     for (int q = -1; q <= n_t; ++q) {  // out rows of conv2 = output rows y0-1+q
-      const long long g = G + q + 1;
+      const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
-      const long long xi = emitted;  // LR ring index of this row (if emitted)
+      const unsigned xi = emitted;  // LR ring index of this row (if emitted)
       emitted += emit;
       if ((int)(g & 1) != grp) continue;
       const int ls = (int)(xi % NLR);

@@ -314,10 +314,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       const uint64_t bd = make_desc(smem_u32(sW), 3 * COUTP * 16, 128);
       int s = 0;
       uint32_t ph = 0;
-      long long G = 0, acq = 0;
+      unsigned G = 0, acq = 0;
       SR_PIECE_BEGIN
       for (int i = 0; i < n_in; ++i) {
-        const long long g = G + i;  // out row completed by this step (dy = 2 target)
+        const unsigned g = G + i;  // out row completed by this step (dy = 2 target)
         SR_RDBG(1, i)
         for (; acq < g + 3; ++acq) mbar_wait(&r_free[ring_idx<RB>(acq)], (uint32_t)(acq / RB) & 1u);
         SR_RDBG(2, i)
@@ -399,10 +399,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       int os[2] = {0, 0};
       uint32_t oph[2] = {0, 0};
       int pend_b = -1;  // staging slot (global index) of the previously issued store
-      long long G = 0;
+      unsigned G = 0;
       SR_PIECE_BEGIN
       for (int q = 1; q <= n_in - 2; ++q) {
-        const long long g = G + q + 1;
+        const unsigned g = G + q + 1;
         const int grp = (int)(g & 1);
         const int b = grp * kRollNO + os[grp];
         mbar_wait(&o_full[b], oph[grp]);
@@ -441,7 +441,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       if (lane_id() == 0) mbar_arrive(&r_free[b]);
     int os = 0;
     float tr_lsum = 0.f;  // training tail: this thread's loss partial
-    long long G = 0, emitted = 0;  // emitted: output rows of both groups so far (aux ring order)
+    unsigned G = 0, emitted = 0;  // emitted: output rows of both groups so far (aux ring order)
     SR_PIECE_BEGIN
     const int xc = x0 + m;
     const bool lane_ok = xc < W;
@@ -449,9 +449,9 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     // epilogue variant bits: 1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU
     const int emode = (a.res1 ? 1 : 0) | (a.res2 ? 2 : 0) | (a.mask ? 4 : 0) | (a.sep > 0 ? 8 : 0) | (a.relu ? 16 : 0);
     for (int q = -1; q <= n_in; ++q) {
-      const long long g = G + q + 1;
+      const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_in - 2;
-      const long long xi = emitted;  // aux ring index of this row (if emitted)
+      const unsigned xi = emitted;  // aux ring index of this row (if emitted)
       emitted += emit;
       if ((int)(g & 1) != grp) continue;
       const int r = y0 - 1 + q;

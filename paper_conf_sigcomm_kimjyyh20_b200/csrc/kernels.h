@@ -52,6 +52,7 @@ cudaError_t launch_conv_roll_tail(int cinp, int coutp, int s, const void* in, co
                                   int w_early = 0);
 // fused body conv (+ f0) + up conv + tail (g kept in shared memory); needs W % 16 == 0 and a 16-B aligned LR frame
 bool bodytail_supported(int cp, int s, int W, const void* lr, const void* hr);
+void set_block_gen(int g);  // benchmarking only
 cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const bf16* w1fold, const bf16* w2fold,
                             const float* b1, const float* b2, const uint8_t* lr, uint8_t* hr, int hr_row0,
                             int hr_row1, int bicubic, int N, int H, int W, cudaStream_t st,

@@ -247,7 +247,7 @@ __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.
 // C columns; one input-row step writes blocks of rows g+2 (dy0), g+1 (dy1), g (dy2), contiguous unless the ring
 // wraps inside the three (idx(g) < 2), in which case the step is issued as two MMA groups.
 template <int RB>
-__host__ __device__ constexpr int ring_idx(long long g) {
+__host__ __device__ constexpr int ring_idx(unsigned g) {
   return (int)((RB - (g % RB)) % RB);
 }
 }  // namespace sr

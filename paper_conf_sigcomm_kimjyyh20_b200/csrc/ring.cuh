@@ -14,7 +14,7 @@ namespace sr {
 // A operand = one input row: APX bytes per pixel row of a K-atom (16 for SWIZZLE_NONE 8-channel chunks, 32 for
 // SWIZZLE_32B 16-channel blocks); kstride = bytes from one K step (16 channels) to the next.
 template <int CINP, int COUTP, int RB, int APX = 16>
-__device__ __forceinline__ void ring_mma_step(uint32_t ring_base, long long g, uint64_t ad, uint64_t bd,
+__device__ __forceinline__ void ring_mma_step(uint32_t ring_base, unsigned g, uint64_t ad, uint64_t bd,
                                               uint32_t kstride) {
   constexpr int CCH = CINP / 8, KS = CINP / 16, N = 3 * COUTP;
   const int i0 = ring_idx<RB>(g);
@@ -97,7 +97,7 @@ __device__ __forceinline__ void arm_tiles_fill(uint8_t* ones, uint8_t* btile, co
 }
 
 template <int COUTP, int RB>
-__device__ __forceinline__ void ring_arm(uint32_t ring_base, long long g, uint32_t ones_saddr, uint32_t btile_saddr) {
+__device__ __forceinline__ void ring_arm(uint32_t ring_base, unsigned g, uint32_t ones_saddr, uint32_t btile_saddr) {
   constexpr uint32_t id = make_idesc(128, COUTP, 0, 0);
   mma_bf16_ss(ring_base + ring_idx<RB>(g) * COUTP, make_desc(ones_saddr, 2048, 128),
               make_desc(btile_saddr, COUTP * 16, 128), id, 0u);

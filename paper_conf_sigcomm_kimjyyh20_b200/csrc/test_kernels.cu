@@ -571,6 +571,12 @@ extern "C" int sr_bench_bodytail_dbg(int cp, int s, int n, int h, int w, long lo
   return (e == cudaSuccess && e2 == cudaSuccess) ? SR_OK : SR_E_CUDA;
 }
 
+// Benchmarking only: run the residual block's more general instantiation (conv_block.cu GEN) with null extras.
+extern "C" int sr_test_block_gen(int g) {
+  sr::set_block_gen(g);
+  return 0;
+}
+
 // Benchmarking only: cap the persistent grids of subsequent launches (0 = all SMs), as sr_set_sm_split does per call.
 extern "C" int sr_test_grid_cap(int cap) {
   sr::set_grid_cap(cap);
