@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libsr.so")
-SOURCES = ["conv.cu", "conv_roll.cu", "conv_block.cu", "conv_block2.cu", "conv_bodytail.cu", "conv_wgrad.cu", "kernels.cu", "sr.cu", "test_kernels.cu"]
+SOURCES = ["conv.cu", "conv_roll.cu", "conv_block.cu", "conv_block2.cu", "conv_block_split.cu", "conv_bodytail.cu", "conv_wgrad.cu", "kernels.cu", "sr.cu", "test_kernels.cu"]
 OBJDIR = os.path.join(ROOT, "build", "obj")
 
 

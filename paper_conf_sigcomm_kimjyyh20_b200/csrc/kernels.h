@@ -69,6 +69,10 @@ cudaError_t launch_conv_roll_tail_train(int cinp, int coutp, int s, const void* 
 bool resblock_supported(int cp, int W);
 // the residual block on CTA pairs (conv_block2.cu, tcgen05 cta_group::2; inference only, bit-identical output)
 bool resblock2_supported(int cp, int W);
+bool resblock_split_supported(int cp, int W);
+cudaError_t launch_resblock_split(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
+                                  const float* b2, bf16* out, int N, int H, int W, cudaStream_t st,
+                                  long long* dbg = nullptr);
 cudaError_t launch_resblock2(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,
                              const float* b2, bf16* out, int N, int H, int W, cudaStream_t st);
 cudaError_t launch_resblock(int cp, const bf16* f, const bf16* w1fold, const bf16* w2fold, const float* b1,

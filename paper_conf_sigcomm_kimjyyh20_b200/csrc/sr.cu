@@ -160,6 +160,7 @@ struct sr_ctx {
   bool fuse_bodytail = true;  // body conv + up conv + tail as one kernel, g in smem (sr_set_fusion bit 5 clears)
   bool fuse_head = true;      // head conv reads the u8 frame directly (sr_set_fusion bit 6 clears)
   bool pair_blocks = true;    // residual blocks of wide frames on CTA pairs, cta_group::2 (sr_set_fusion bit 7 clears)
+  bool split_blocks = false;  // inference residual blocks on CTA pairs split by conv (sr_set_fusion bit 8 sets)
   int sm_train = 0;           // sr_set_sm_split: SMs given to the training kernels (0 = all SMs to every call)
   bool train_fold_only = false;  // TRAIN's tiled layouts (wf, wd) may be stale: rebuild before reading them
   int sm_total = 0;
@@ -424,7 +425,11 @@ static sr_status forward_infer(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, con
         tmark_begin(ctx, "resblock_" + std::to_string(Cp), 2 * 2.0 * 9 * Cp * Cp * px, px * 2.0 * 2 * Cp, st);
       }
       cudaError_t e =
-          ctx->pair_blocks && resblock2_supported(Cp, w)
+          ctx->split_blocks && resblock_split_supported(Cp, w)
+              ? launch_resblock_split(Cp, cur, sn.wo + ctx->convs[1 + 2 * b].pk_off,
+                                      sn.wo + ctx->convs[2 + 2 * b].pk_off, Bv(1 + 2 * b), Bv(2 + 2 * b), nxt, n, h, w,
+                                      st)
+          : ctx->pair_blocks && resblock2_supported(Cp, w)
               ? launch_resblock2(Cp, cur, sn.wo + ctx->convs[1 + 2 * b].pk_off, sn.wo + ctx->convs[2 + 2 * b].pk_off,
                                  Bv(1 + 2 * b), Bv(2 + 2 * b), nxt, n, h, w, st)
               : launch_resblock(Cp, cur, sn.wo + ctx->convs[1 + 2 * b].pk_off, sn.wo + ctx->convs[2 + 2 * b].pk_off,
@@ -1017,6 +1022,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->fuse_bodytail = (fuse_blocks & 32) == 0; // bit 5 set: body conv and up conv + tail as two kernels
   ctx->fuse_head = (fuse_blocks & 64) == 0;     // bit 6 set: k_pack_input + head conv on the bf16 copy
   ctx->pair_blocks = (fuse_blocks & 128) == 0;  // bit 7 set: single-CTA residual blocks instead of CTA pairs
+  ctx->split_blocks = (fuse_blocks & 256) != 0; // bit 8 set: inference blocks on conv-split CTA pairs
   return SR_OK;
 }
 

@@ -388,10 +388,16 @@ extern "C" int sr_bench_resblock(int c, int n, int h, int w, int iters, float* m
   cudaEventCreate(&b);
   const char* ex = std::getenv("SR_BLOCK_EXP");  // benchmarking experiments (see k_resblock)
   const int exp = ex ? std::atoi(ex) : 0;
-  cudaError_t e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, dbg_host ? dbg : nullptr, nullptr, 0, exp);
+  const char* sp = std::getenv("SR_BLOCK_SPLIT");  // 1: the conv-split CTA-pair kernel; 2: the cta_group::2 pair
+  const int split = sp ? std::atoi(sp) : 0;
+  auto launch = [&](long long* d) {
+    return split == 1 ? launch_resblock_split(c, x, w1, w2, bias, bias, y, n, h, w, st, d)
+         : split == 2 ? launch_resblock2(c, x, w1, w2, bias, bias, y, n, h, w, st)
+                      : launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, d, nullptr, 0, exp);
+  };
+  cudaError_t e = launch(dbg_host ? dbg : nullptr);
   cudaEventRecord(a, st);
-  for (int i = 0; i < iters && e == cudaSuccess; ++i)
-    e = launch_resblock(c, x, w1, w2, bias, bias, y, n, h, w, st, nullptr, nullptr, 0, exp);
+  for (int i = 0; i < iters && e == cudaSuccess; ++i) e = launch(nullptr);
   cudaEventRecord(b, st);
   cudaError_t e2 = cudaStreamSynchronize(st);
   float ms = 0.f;

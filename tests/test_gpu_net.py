@@ -678,3 +678,21 @@ def test_pair_resblock_equals_single_cta(cfg, hw, n):
     b = ctx.infer(lr, "serve")
     torch.cuda.synchronize()
     assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (37, 272), 2), ((3, 2, 48), (90, 700), 1), ((2, 2, 48), (8, 126), 3),
+                                      ((2, 8, 32), (54, 960), 3), ((2, 3, 16), (29, 400), 2), ((3, 2, 48), (720, 1280), 1)])
+def test_split_resblock_equals_single_cta(cfg, hw, n):
+    """Residual blocks on CTA pairs split by conv (conv_block_split.cu: conv1 on one SM, conv2 on the other, t rows
+    through distributed shared memory; set_fusion bit 8) == the single-CTA kernel (bit 7), bit for bit: the same MMA
+    sequence per output element in both rings.  Ragged last strips, pieces shorter than a ring, several frames,
+    and a full 720p frame (many pieces per pair)."""
+    s, B, C = cfg
+    ctx = _ctx(s, B, C, seed=91)
+    lr = torch.from_numpy(synth_frames(n, hw[0], hw[1], seed=92)).cuda()
+    ctx.set_fusion(1 | 128)
+    a = ctx.infer(lr, "serve").clone()
+    ctx.set_fusion(1 | 128 | 256)
+    b = ctx.infer(lr, "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
