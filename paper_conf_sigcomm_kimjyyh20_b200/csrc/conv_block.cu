@@ -87,6 +87,9 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   // 11 conv2 blocks acquired, 12 t row ready, 13 epi1 freed a block (by row), 14 epi2 freed a block (by row)
   using Cfg = BlkCfg<C>;
   constexpr int CCH = Cfg::CCH, RB = Cfg::RB;
+  // the bias-arming MMAs take their ones operand from 8 spare TMEM columns after ring 1 when there are any
+  // (C = 48: columns 240..247; C = 16: 128..135), saving a 4 KB shared-memory read per arm
+  constexpr bool kOnesTmem = RB * C + 8 <= 256;
   constexpr uint32_t PLANE = Cfg::PLANE, ROWB = Cfg::ROWB, OUTB = Cfg::OUTB;
 
   extern __shared__ uint8_t smem_raw[];
@@ -124,6 +127,14 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
   tc_fence_before();
   __syncthreads();
+  if constexpr (kOnesTmem) {
+    if (warp >= 2 && warp < 6) {  // warps 2..5 cover the four TMEM lane quarters
+      tc_fence_after();
+      ones_tmem_fill(tmem_base_sh + ((uint32_t)((warp & 3) * 32) << 16) + RB * C);
+      tmem_st_wait();
+      tc_fence_before();
+    }
+  }
   // Weights and biases were written at least two kernels upstream in every chain that launches this kernel (the
   // library's repack / publish precede at least the head conv; the kernel that wrote them completed before our
   // predecessor passed its own griddepcontrol.wait), so they are fetched and the bias-arming tiles built before the
@@ -146,7 +157,15 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   pdl_enter();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
-  const uint32_t ring1 = tmem, ring2 = tmem + 256;
+  const uint32_t ring1 = tmem, ring2 = tmem + 256, ones_t = tmem + RB * C;
+  auto arm1 = [&](unsigned gg) {
+    if constexpr (kOnesTmem) ring_arm_ts<C, RB>(ring1, gg, ones_t, smem_u32(sB1));
+    else ring_arm<C, RB>(ring1, gg, smem_u32(sOnes), smem_u32(sB1));
+  };
+  auto arm2 = [&](unsigned gg) {
+    if constexpr (kOnesTmem) ring_arm_ts<C, RB>(ring2, gg, ones_t, smem_u32(sB2));
+    else ring_arm<C, RB>(ring2, gg, smem_u32(sOnes), smem_u32(sB2));
+  };
 
   const int tiles_x = (W + kBlkTW - 1) / kBlkTW;
   const long long total = (long long)N * tiles_x * H;
@@ -201,10 +220,10 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_DBG(9, st)
         tc_fence_after();
         if (st == 0) {  // the piece's first two rows receive no earlier contribution
-          ring_arm<C, RB>(ring1, g, smem_u32(sOnes), smem_u32(sB1));
-          ring_arm<C, RB>(ring1, g + 1, smem_u32(sOnes), smem_u32(sB1));
+          arm1(g);
+          arm1(g + 1);
         }
-        ring_arm<C, RB>(ring1, g + 2, smem_u32(sOnes), smem_u32(sB1));  // its first contribution comes now
+        arm1(g + 2);  // its first contribution comes now
         if (!(exp & 32))
           ring_mma_step<C, C, RB>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, 2 * PLANE);
         mma_commit(&r1_ready[ring_idx<RB>(g)]);  // out row g (dy=2 target) is complete
@@ -238,10 +257,10 @@ k_resblock(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_DBG(12, k + 3)
         tc_fence_after();
         if (k == 0) {
-          ring_arm<C, RB>(ring2, g, smem_u32(sOnes), smem_u32(sB2));
-          ring_arm<C, RB>(ring2, g + 1, smem_u32(sOnes), smem_u32(sB2));
+          arm2(g);
+          arm2(g + 1);
         }
-        ring_arm<C, RB>(ring2, g + 2, smem_u32(sOnes), smem_u32(sB2));
+        arm2(g + 2);
         if (!(exp & 16))
           ring_mma_step<C, C, RB>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, 2 * PLANE);
         mma_commit(&r2_ready[ring_idx<RB>(g)]);

@@ -130,11 +130,29 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   arm_tiles_fill(sOnes, sB1, a.b1, C, threadIdx.x, blockDim.x);
   arm_tiles_fill(sOnes, sB2, a.b2, CO2, threadIdx.x, blockDim.x);
   fence_proxy_async_smem();
+  // the arming MMAs take their ones operand from 8 spare TMEM columns after ring 1 when there are any (ring.cuh)
+  constexpr bool kOnesTmem = RB1 * C + 8 <= Cfg::R2BASE;
+  if constexpr (kOnesTmem) {
+    if (warp >= 2 && warp < 6) {
+      tc_fence_after();
+      ones_tmem_fill(tmem_base_sh + ((uint32_t)((warp & 3) * 32) << 16) + RB1 * C);
+      tmem_st_wait();
+      tc_fence_before();
+    }
+  }
   __syncthreads();
   pdl_enter();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
-  const uint32_t ring1 = tmem, ring2 = tmem + Cfg::R2BASE;
+  const uint32_t ring1 = tmem, ring2 = tmem + Cfg::R2BASE, ones_t = tmem + RB1 * C;
+  auto arm1 = [&](unsigned gg) {
+    if constexpr (kOnesTmem) ring_arm_ts<C, RB1>(ring1, gg, ones_t, smem_u32(sB1));
+    else ring_arm<C, RB1>(ring1, gg, smem_u32(sOnes), smem_u32(sB1));
+  };
+  auto arm2 = [&](unsigned gg) {
+    if constexpr (kOnesTmem) ring_arm_ts<CO2, RB2>(ring2, gg, ones_t, smem_u32(sB2));
+    else ring_arm<CO2, RB2>(ring2, gg, smem_u32(sOnes), smem_u32(sB2));
+  };
 
   const int tiles_x = (W + kBtTW - 1) / kBtTW;
   const long long total = (long long)N * tiles_x * H;
@@ -191,10 +209,10 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_BDBG(9, st)
         tc_fence_after();
         if (st == 0) {
-          ring_arm<C, RB1>(ring1, g, smem_u32(sOnes), smem_u32(sB1));
-          ring_arm<C, RB1>(ring1, g + 1, smem_u32(sOnes), smem_u32(sB1));
+          arm1(g);
+          arm1(g + 1);
         }
-        ring_arm<C, RB1>(ring1, g + 2, smem_u32(sOnes), smem_u32(sB1));
+        arm1(g + 2);
         ring_mma_step<C, C, RB1>(ring1, g, make_desc(smem_u32(sF + fs * ROWB), PLANE, 128), bd1, 2 * PLANE);
         mma_commit(&r1_ready[ring_idx<RB1>(g)]);
         mma_commit(&f_empty[fs]);
@@ -227,10 +245,10 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         SR_BDBG(12, k + 3)
         tc_fence_after();
         if (k == 0) {
-          ring_arm<CO2, RB2>(ring2, g, smem_u32(sOnes), smem_u32(sB2));
-          ring_arm<CO2, RB2>(ring2, g + 1, smem_u32(sOnes), smem_u32(sB2));
+          arm2(g);
+          arm2(g + 1);
         }
-        ring_arm<CO2, RB2>(ring2, g + 2, smem_u32(sOnes), smem_u32(sB2));
+        arm2(g + 2);
         ring_mma_step<C, CO2, RB2>(ring2, g, make_desc(smem_u32(sT + ts * ROWB), PLANE, 128), bd2, 2 * PLANE);
         mma_commit(&r2_ready[ring_idx<RB2>(g)]);
         mma_commit(&t_empty[ts]);

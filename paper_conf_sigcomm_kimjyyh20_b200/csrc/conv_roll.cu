@@ -222,12 +222,22 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     bulk_load(sW, wfold, Cfg::WBYTES, &w_bar);
   }
   constexpr uint32_t kArmThreads = 9 * 32;  // warps 2..10
+  // the arming MMAs take their ones operand from 8 spare TMEM columns after the ring when there are any (ring.cuh)
+  constexpr bool kOnesTmem = RB * COUTP + 8 <= 512;
   auto arm_params = [&]() {
     const int t = (int)threadIdx.x - 64;
     if (t < COUTP) reinterpret_cast<float*>(sbv)[t] = a.bias ? a.bias[t] : 0.f;
     named_bar_sync(1, kArmThreads);
     arm_tiles_fill(sOnes, sBt, reinterpret_cast<const float*>(sbv), COUTP, t, kArmThreads);
     fence_proxy_async_smem();
+    if constexpr (kOnesTmem) {
+      if (warp >= 2 && warp <= 5) {  // the four TMEM lane quarters
+        tc_fence_after();
+        ones_tmem_fill(tmem_base_sh + ((uint32_t)((warp & 3) * 32) << 16) + RB * COUTP);
+        tmem_st_wait();
+        tc_fence_before();
+      }
+    }
     named_bar_sync(1, kArmThreads);
     if (t == 0) mbar_arrive(&arm_bar);
   };
@@ -312,6 +322,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       mbar_wait(&arm_bar, 0);  // bias-arming tiles in place
       tc_fence_after();
       const uint64_t bd = make_desc(smem_u32(sW), 3 * COUTP * 16, 128);
+      auto arm = [&](unsigned gg) {
+        if constexpr (kOnesTmem) ring_arm_ts<COUTP, RB>(tmem, gg, tmem + RB * COUTP, smem_u32(sBt));
+        else ring_arm<COUTP, RB>(tmem, gg, smem_u32(sOnes), smem_u32(sBt));
+      };
       int s = 0;
       uint32_t ph = 0;
       unsigned G = 0, acq = 0;
@@ -325,10 +339,10 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
         SR_RDBG(3, i)
         tc_fence_after();
         if (i == 0) {  // the piece's first two rows receive no earlier contribution
-          ring_arm<COUTP, RB>(tmem, g, smem_u32(sOnes), smem_u32(sBt));
-          ring_arm<COUTP, RB>(tmem, g + 1, smem_u32(sOnes), smem_u32(sBt));
+          arm(g);
+          arm(g + 1);
         }
-        ring_arm<COUTP, RB>(tmem, g + 2, smem_u32(sOnes), smem_u32(sBt));  // its first contribution comes now
+        arm(g + 2);  // its first contribution comes now
         ring_mma_step<CINP, COUTP, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, 2 * PLANE);
         mma_commit(&r_ready[ring_idx<RB>(g)]);
         mma_commit(&in_empty[s]);

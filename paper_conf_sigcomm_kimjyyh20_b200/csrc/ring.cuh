@@ -103,4 +103,23 @@ __device__ __forceinline__ void ring_arm(uint32_t ring_base, unsigned g, uint32_
               make_desc(btile_saddr, COUTP * 16, 128), id, 0u);
 }
 
+// The same with the ones operand held in TMEM (8 columns: A[m][k] = 1 for k < 3, bf16 pairs per 32-bit column),
+// written once by ones_tmem_fill: the arming MMA then reads only the bias tile from shared memory (the 4 KB ones
+// tile per arm otherwise goes through the shared-memory port the conv MMAs saturate).
+template <int COUTP, int RB>
+__device__ __forceinline__ void ring_arm_ts(uint32_t ring_base, unsigned g, uint32_t ones_tmem, uint32_t btile_saddr) {
+  constexpr uint32_t id = make_idesc(128, COUTP, 0, 0);
+  mma_bf16_ts(ring_base + ring_idx<RB>(g) * COUTP, ones_tmem, make_desc(btile_saddr, COUTP * 16, 128), id, 0u);
+}
+// one warp writes its 32 lanes of the TMEM ones operand (caller: tcgen05.wait::st + fence before the MMA issuer)
+__device__ __forceinline__ void ones_tmem_fill(uint32_t taddr_lane) {
+  const __nv_bfloat162 one_one = __floats2bfloat162_rn(1.f, 1.f), one_zero = __floats2bfloat162_rn(1.f, 0.f);
+  float v[8];
+  v[0] = __uint_as_float(*reinterpret_cast<const uint32_t*>(&one_one));
+  v[1] = __uint_as_float(*reinterpret_cast<const uint32_t*>(&one_zero));
+#pragma unroll
+  for (int i = 2; i < 8; ++i) v[i] = 0.f;
+  tmem_st8(taddr_lane, v);
+}
+
 }  // namespace sr
