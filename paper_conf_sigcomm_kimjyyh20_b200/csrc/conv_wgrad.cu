@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(kWrThreads, 1) k_wgrad_multi(const __grid_cons
   } else if (warp == 1) {
     // ===================== MMA issuer
     if (elect_one()) {
-      long long xq0 = 0, xw = 0, dq = 0;  // global X input index of the piece's first row, X inputs waited, dY rows
+      unsigned xq0 = 0, xw = 0, dq = 0;  // global X input index of the piece's first row, X inputs waited, dY rows
       bool first = true;
       uint32_t seg = 0;
       SR_WPIECE_BEGIN
@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(kWrThreads, 1) k_wgrad_multi(const __grid_cons
     float acc8[8];
 #pragma unroll
     for (int e = 0; e < 8; ++e) acc8[e] = 0.f;
-    long long dq = 0;
+    unsigned dq = 0;
     uint32_t seg = 0;
     SR_WPIECE_BEGIN
     const int coutp = jb.coutp, cinp = jb.cinp;
