@@ -27,6 +27,8 @@
 #include "kernels.h"
 #include "launch.cuh"
 #include "tail.cuh"
+#include <algorithm>
+#include <vector>
 
 namespace sr {
 
@@ -721,6 +723,534 @@ cudaError_t launch_conv_roll(int cinp, int coutp, const void* in, const bf16* wf
                              const bf16* res, int relu, bf16* out, int N, int H, int W, cudaStream_t st, int w_early) {
   return launch_conv_roll_ex(cinp, coutp, in, wfold, bias, res, nullptr, nullptr, relu, 0, out, N, H, W, st, nullptr,
                              w_early);
+}
+
+
+// ====================================================================================================================
+// k_conv_chain: a whole chain of C -> C rolling convs (the residual blocks + body conv of a training forward pass, or
+// the data-gradient chain of its backward pass) in ONE persistent cooperative launch.  Opt-in (sr_set_fusion bit 9,
+// SR_CHAIN=1): measured, it does not beat one PDL-overlapped k_conv_roll launch per conv.
+//
+// Why it was built: at the training shape (64 patches of 48 x 48 side by side = 1 x 48 x 3200) a conv is 6.4 GFLOP,
+// ~8 rows per CTA on 148 SMs, so each k_conv_roll launch is ~3-4 us of ramp (barriers, TMEM, weights, the first
+// input rows' TMA latency) + ~10 row-steps + ~2 us of drain (profiles/r02_roll_timeline.txt).  Here every CTA keeps
+// the same work for all layers of the chain and walks them in order: the TMEM ring, barriers and counters keep
+// running across layer boundaries, the next layer's weights are fetched as soon as the MMAs of the previous one have
+// completed, and a layer's input row is loaded as soon as the CTAs that produce it (same strip and the two
+// neighbouring strips, for the 1-pixel halo columns) have published it -- no grid-wide barrier, no relaunch.
+// Work split (chain_pieces): with >= 1 CTA per column strip, two phases -- each CTA owns one band of the top half and
+// one band of the bottom half of the rows and walks layer l as [top band, bottom band], so the store -> publish ->
+// load latency of a layer boundary is covered by the other phase's work.
+//
+// Cross-CTA protocol (all CTAs co-resident: cooperative launch): sync[0] = launch generation, sync[1] = exit count,
+// sync[2 + col * H + row] = flag of output row (col, row).  Once the bulk group of a piece has completed
+// (cp.async.bulk.wait_group 0) the store thread hands the piece to the publisher warp through shared memory, which
+// issues the proxy + gpu-scope fences and stores gen * 64 + layer + 1 into the piece's row flags.  A producer
+// polls the flags of the rows it is about to load (input rows: layer - 1, three columns; res1 aux rows: the layer
+// that wrote them) with one lane per flag, fences (acquire) and orders its TMA loads after them with
+// fence.proxy.async.  Flags only grow, so no reset is needed between launches; the last CTA to exit advances the
+// generation.  Math per layer: exactly k_conv_roll's (same MMAs in the same order, same ring, same epilogue
+// variants): the outputs are bit-identical to one k_conv_roll launch per layer (tests/test_gpu_timed_paths.py).
+static constexpr int kChainMax = 20;
+struct ChainLayer {
+  CUtensorMap tin, tout, taux;
+  const bf16* w;
+  const float* bias;
+  const bf16* res2;
+  int emode;    // roll_stage variant bits: 1 res1, 2 res2, 4 mask, 8 separators, 16 ReLU
+  int aux_dep;  // >= 0: the aux (res1) rows were written by layer aux_dep of this launch; -1: by an earlier kernel
+};
+static constexpr int kChainMaxCta = 192;
+struct ChainPiece {
+  short col, y0, y1, pad;
+};
+struct ChainParams {
+  ChainLayer L[kChainMax];
+  int nl, N, H, W, sep;
+  int nph;      // 0: each CTA takes a contiguous (strip, row) range (<= 4 pieces); 1, 2: pieces from pc[cta][0..nph)
+  ChainPiece pc[kChainMaxCta][2];
+  unsigned* sync;
+  int dbg_cta;
+  unsigned long long* dbg;  // benchmarking only: per (CTA, layer) globaltimer stamps [8] (sr_test_chain_dbg)
+};
+#define SR_RDBG2(l, i, k) \
+  if (p.dbg && blockIdx.x == (unsigned)p.dbg_cta && (i) < 64) \
+    p.dbg[(size_t)gridDim.x * kChainMax * 8 + ((size_t)(l) * 64 + (i)) * 4 + (k)] = (unsigned long long)globaltimer();
+#define SR_CDBG(l, k) \
+  if (p.dbg) p.dbg[((size_t)blockIdx.x * kChainMax + (l)) * 8 + (k)] = (unsigned long long)globaltimer();
+
+// bias of one layer into its arming tile (B[n][k]: hi, mid, lo bf16 terms at k = 0, 1, 2; ring.cuh)
+__device__ __forceinline__ void chain_bias_tile(uint8_t* btile, const float* bias, int coutp, int tid, int nthreads) {
+  for (int i = tid; i < coutp * 16; i += nthreads) {
+    const int n = i / 16, k = i % 16;
+    const float b = bias ? __ldg(bias + n) : 0.f;
+    const __nv_bfloat16 hi = __float2bfloat16(b);
+    const __nv_bfloat16 mid = __float2bfloat16(b - __bfloat162float(hi));
+    const __nv_bfloat16 lo = __float2bfloat16(b - __bfloat162float(hi) - __bfloat162float(mid));
+    const __nv_bfloat16 v = k == 0 ? hi : k == 1 ? mid : k == 2 ? lo : __float2bfloat16(0.f);
+    *reinterpret_cast<__nv_bfloat16*>(btile + (n % 8) * 16 + (n / 8) * 128 + (k / 8) * (coutp * 16) + (k % 8) * 2) = v;
+  }
+}
+
+static constexpr int kChainThreads = kRollThreads;
+template <int C>
+__global__ void __launch_bounds__(kChainThreads, 1) k_conv_chain(const __grid_constant__ ChainParams p) {
+  using Cfg = RollCfg<C, C>;
+  constexpr int RB = Cfg::RB, kRollIn = Cfg::NIN, NAUX = Cfg::NAUX;
+  constexpr uint32_t PLANE = Cfg::PLANE, IN_STRIDE = Cfg::IN_STRIDE, ROWB = Cfg::ROWB;
+  static_assert(RB * C + 8 <= 512, "chain: the ones operand lives in TMEM");
+  static_assert(2 * C * 32 <= (int)kArmOnesBytes, "chain: two bias tiles in the (unused) ones-tile area");
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* sW = smem;
+  uint8_t* sIn = sW + Cfg::WB_AL;
+  uint8_t* sO = sIn + kRollIn * IN_STRIDE;
+  uint8_t* sA = sO + 2 * kRollNO * ROWB;
+  uint8_t* sBt = sA + NAUX * ROWB;  // two bias-arming tiles (layer parity)
+  __shared__ __align__(8) uint64_t in_full[kRollIn], in_empty[kRollIn], r_ready[RB], r_free[RB], x_full[NAUX],
+      x_empty[NAUX], o_full[2 * kRollNO], o_free[2 * kRollNO], w_bar, w_free, arm_bar[2];
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ unsigned gen_sh;
+  // pieces whose stores have completed, handed from the store thread to the publisher (piece index, layer): entries
+  // [0, pub_w) written; the publisher trails by at most one layer, far less than the ring
+  constexpr int kPubRing = 128;
+  __shared__ uint8_t pub_pc[kPubRing], pub_l[kPubRing];
+  __shared__ volatile uint32_t pub_w;
+
+  const int N = p.N, H = p.H, W = p.W, nl = p.nl;
+  const int warp = warp_id();
+  if (warp == 0 && lane_id() == 0) {
+    for (int s = 0; s < kRollIn; ++s) { mbar_init(&in_full[s], 1); mbar_init(&in_empty[s], 1); }
+    for (int s = 0; s < RB; ++s) { mbar_init(&r_ready[s], 1); mbar_init(&r_free[s], 4); }
+    for (int s = 0; s < NAUX; ++s) { mbar_init(&x_full[s], 1); mbar_init(&x_empty[s], 4); }
+    for (int s = 0; s < 2 * kRollNO; ++s) { mbar_init(&o_full[s], 4); mbar_init(&o_free[s], 1); }
+    mbar_init(&w_bar, 1);
+    mbar_init(&w_free, 1);
+    mbar_init(&arm_bar[0], 1);
+    mbar_init(&arm_bar[1], 1);
+    fence_barrier_init();
+    pub_w = 0;
+  }
+  if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
+  tc_fence_before();
+  __syncthreads();
+  if (warp >= 2 && warp <= 5) {  // the TMEM ones operand of the arming MMAs (four lane quarters)
+    tc_fence_after();
+    ones_tmem_fill(tmem_base_sh + ((uint32_t)((warp & 3) * 32) << 16) + RB * C);
+    tmem_st_wait();
+    tc_fence_before();
+  }
+  pdl_enter();  // the chain's input, the external aux rows and the packed weights are complete from here on
+  if (threadIdx.x == 0) gen_sh = *reinterpret_cast<volatile unsigned*>(p.sync);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const unsigned base = gen_sh * 64u;  // flag value of layer l: base + l + 1
+  unsigned* const flags = p.sync + 2;
+
+  const int tiles_x = (W + kRollTW - 1) / kRollTW;
+  const long long total = (long long)N * tiles_x * H;
+  // this CTA's pieces (column strip, rows [y0, y1)), the same for every layer
+  int pcol[4], py0[4], py1[4], npc = 0;
+  if (p.nph > 0) {
+    for (int k = 0; k < p.nph; ++k) {
+      const ChainPiece& q = p.pc[blockIdx.x][k];
+      pcol[npc] = q.col; py0[npc] = q.y0; py1[npc] = q.y1; ++npc;
+    }
+  } else {
+    const long long beg = total * blockIdx.x / gridDim.x, end = total * (blockIdx.x + 1) / gridDim.x;
+    for (long long pos = beg; pos < end && npc < 4;) {
+      const int col = (int)(pos / H), y0 = (int)(pos - (long long)col * H);
+      const int y1 = (int)min((long long)H, y0 + (end - pos));
+      pos += y1 - y0;
+      pcol[npc] = col; py0[npc] = y0; py1[npc] = y1; ++npc;
+    }
+  }
+  uint32_t rows_mine = 0;
+  for (int k = 0; k < npc; ++k) rows_mine += py1[k] - py0[k];
+  (void)rows_mine;
+#define SR_PIECE_BEGIN                                                                \
+  for (int pi = 0; pi < npc; ++pi) {                                                  \
+    const int col = pcol[pi], y0 = py0[pi], y1 = py1[pi];                             \
+    const int n = col / tiles_x, x0 = (col - n * tiles_x) * kRollTW;                  \
+    const int n_in = y1 - y0 + 2;                                                     \
+    (void)n; (void)x0; (void)n_in;
+#define SR_PIECE_END }
+
+  if (warp == 0) {
+    // ===================== producer: layer weights, then each input row once its three producers published it ====
+    // The warp polls the flags of the next up-to-8 input rows x 3 columns (the 1-pixel halo of the neighbouring
+    // strips) in one round (one lane per flag); lane 0 issues the weight and row TMAs.
+    const bool lead = lane_id() == 0;
+    int s = 0, xs = 0;
+    uint32_t ph = 0, xph = 0;
+    for (int l = 0; l < nl; ++l) {
+      const ChainLayer& Ly = p.L[l];
+      if (lead) {
+        tma_prefetch_desc(&Ly.tin);
+        if (l > 0) mbar_wait(&w_free, (uint32_t)(l - 1) & 1u);  // the previous layer's MMAs have completed
+        mbar_arrive_expect_tx(&w_bar, Cfg::WBYTES);
+        bulk_load(sW, Ly.w, Cfg::WBYTES, &w_bar);
+        SR_CDBG(l, 5)
+      }
+      const bool has_aux = (Ly.emode & 5) != 0;
+      if (lead && has_aux) tma_prefetch_desc(&Ly.taux);
+      bool first_piece = true;
+      SR_PIECE_BEGIN
+      const int sx = col - n * tiles_x;
+      const bool has_l = sx > 0, has_r = sx + 1 < tiles_x;
+      int ready = l > 0 ? 0 : n_in;  // input rows [0, ready) of the piece confirmed published
+      if (has_aux && Ly.aux_dep >= 0) {  // res1 rows: own rows (same strip and rows) of an earlier layer
+        for (int r = y0 + lane_id(); r < y1; r += 32)
+          flag_spin(flags + (size_t)col * H + r, base + (unsigned)Ly.aux_dep + 1u);
+        fence_acq_rel_gpu();
+        __syncwarp();
+        if (lead) fence_proxy_async_global();
+      }
+      for (int i = 0; i < n_in; ++i) {
+        const int y = y0 - 1 + i;
+        if (i >= ready) {  // input row y = output row y of layer l - 1 in strips sx - 1 .. sx + 1
+          const int k = lane_id(), ii = i + k / 3, dc = k % 3 - 1;
+          const int yy = y0 - 1 + ii;
+          const bool mine = k < 24 && ii < n_in && yy >= 0 && yy < H && (dc == 0 || (dc < 0 ? has_l : has_r));
+          const unsigned* f = flags + (size_t)(col + dc) * H + yy;
+          const unsigned tgt = base + (unsigned)l;
+          const long long t0 = clock64();
+          for (;;) {
+            const bool ok = !mine || (int)(ld_relaxed_gpu(f) - tgt) >= 0;
+            const unsigned bad = __ballot_sync(0xffffffffu, !ok);
+            const int nrd = bad ? (__ffs(bad) - 1) / 3 : 8;  // leading rows with all three flags set
+            if (nrd > 0) { ready = i + nrd; break; }
+            __nanosleep(20);
+            if (clock64() - t0 > (1ll << 34)) __trap();
+          }
+          fence_acq_rel_gpu();
+          __syncwarp();
+          if (lead) fence_proxy_async_global();
+        }
+        if (lead) {
+          if (first_piece && i == 0) { SR_CDBG(l, 0) }
+          SR_RDBG2(l, i, 0)
+          mbar_wait(&in_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&in_full[s], Cfg::IN_BOX);
+          tma_load_5d(sIn + s * IN_STRIDE, &Ly.tin, &in_full[s], 0, x0 - 1, y, 0, n);
+          if (has_aux && i >= 1 && i <= n_in - 2) {  // the aux row of output emission i (needed after input i + 1)
+            const int r = y0 - 1 + i;
+            mbar_wait(&x_empty[xs], xph ^ 1);
+            mbar_arrive_expect_tx(&x_full[xs], kRollTW * C * 2);
+            tma_load_4d(sA + xs * ROWB, &Ly.taux, &x_full[xs], 0, x0, r, n);
+          }
+        }
+        if (has_aux && i >= 1 && i <= n_in - 2 && ++xs == NAUX) { xs = 0; xph ^= 1; }
+        if (++s == kRollIn) { s = 0; ph ^= 1; }
+      }
+      first_piece = false;
+      __syncwarp();
+      SR_PIECE_END
+    }
+  } else if (warp == 11) {
+    // ===================== publisher: flags of the pieces the store thread reports written ======================
+    // (a gpu-scope fence costs ~1.5k cycles; issued here it never holds back the store thread's staging slots)
+    const uint32_t total = (uint32_t)(nl * npc);  // pieces handed over: every piece of every layer
+    uint32_t r = 0;
+    const long long t0 = clock64();
+    while (r < total) {
+      const uint32_t w = pub_w;
+      if (w == r) {
+        __nanosleep(32);
+        if (clock64() - t0 > (1ll << 36)) __trap();
+        continue;
+      }
+      __syncwarp();
+      __threadfence_block();
+      if (lane_id() == 0) {
+        fence_proxy_async_global();
+        fence_acq_rel_gpu();
+      }
+      __syncwarp();
+      for (; r < w; ++r) {
+        const int pi = pub_pc[r % kPubRing], l = pub_l[r % kPubRing];
+        const int col = pcol[pi], y0 = py0[pi], y1 = py1[pi];
+        for (int y = y0 + lane_id(); y < y1; y += 32) st_relaxed_gpu(flags + (size_t)col * H + y, base + (unsigned)l + 1u);
+        if (pi == npc - 1) { SR_CDBG(l, 4) }
+      }
+      __syncwarp();
+    }
+  } else if (warp == 1) {
+    // ===================== MMA issuer =====================
+    if (elect_one()) {
+      const uint64_t bd = make_desc(smem_u32(sW), 3 * C * 16, 128);
+      const uint32_t ones = tmem + RB * C;
+      int s = 0;
+      uint32_t ph = 0;
+      unsigned G = 0, acq = 0;
+      for (int l = 0; l < nl; ++l) {
+        mbar_wait(&w_bar, (uint32_t)l & 1u);
+        mbar_wait(&arm_bar[l & 1], (uint32_t)(l >> 1) & 1u);
+        tc_fence_after();
+        const uint32_t bt = smem_u32(sBt + (l & 1) * C * 32);
+        const unsigned Gl = G;
+        SR_PIECE_BEGIN
+        for (int i = 0; i < n_in; ++i) {
+          const unsigned g = G + i;
+          for (; acq < g + 3; ++acq) mbar_wait(&r_free[ring_idx<RB>(acq)], (uint32_t)(acq / RB) & 1u);
+          mbar_wait(&in_full[s], ph);
+          tc_fence_after();
+          if (i == 0) {
+            ring_arm_ts<C, RB>(tmem, g, ones, bt);
+            ring_arm_ts<C, RB>(tmem, g + 1, ones, bt);
+          }
+          ring_arm_ts<C, RB>(tmem, g + 2, ones, bt);
+          ring_mma_step<C, C, RB>(tmem, g, make_desc(smem_u32(sIn + s * IN_STRIDE), PLANE, 128), bd, 2 * PLANE);
+          if (G == Gl && i == 0) { SR_CDBG(l, 1) }
+          if (G == Gl) { SR_RDBG2(l, i, 1) }
+          mma_commit(&r_ready[ring_idx<RB>(g)]);
+          mma_commit(&in_empty[s]);
+          if (i == n_in - 1) {
+            mma_commit(&r_ready[ring_idx<RB>(g + 1)]);
+            mma_commit(&r_ready[ring_idx<RB>(g + 2)]);
+          }
+          if (++s == kRollIn) { s = 0; ph ^= 1; }
+        }
+        G += n_in + 2;
+        SR_PIECE_END
+        mma_commit(&w_free);  // fires when every MMA of this layer (and the arms) has completed
+        SR_CDBG(l, 2)
+      }
+    }
+    __syncwarp();
+  } else if (warp == 10) {
+    // ===================== store warp: TMA-store finished rows; publish each piece's rows once written ==========
+    const bool lead = lane_id() == 0;
+    int os[2] = {0, 0};
+    uint32_t oph[2] = {0, 0};
+    unsigned G = 0;
+    for (int l = 0; l < nl; ++l) {
+      const ChainLayer& Ly = p.L[l];
+      if (lead) tma_prefetch_desc(&Ly.tout);
+      SR_PIECE_BEGIN
+      if (lead) {
+        // The rows of a piece are published together once its last store has completed, by the publisher warp (a
+        // gpu-scope fence issued here, behind outstanding bulk stores, costs ~1.5k cycles and holds back the staging
+        // slots the epilogue waits for).
+        int pend_b = -1;
+        for (int q = 1; q <= n_in - 2; ++q) {
+          const unsigned g = G + q + 1;
+          const int grp = (int)(g & 1);
+          const int b = grp * kRollNO + os[grp];
+          mbar_wait(&o_full[b], oph[grp]);
+          SR_RDBG2(l, q, 3)
+          tma_store_4d(&Ly.tout, sO + b * ROWB, 0, x0, y0 - 1 + q, n);
+          bulk_commit();
+          bulk_wait_read<1>();  // the previous store has read its staging row
+          if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
+          pend_b = b;
+          if (++os[grp] == kRollNO) { os[grp] = 0; oph[grp] ^= 1; }
+        }
+        SR_CDBG(l, 3)
+        bulk_wait<0>();
+        if (pend_b >= 0) mbar_arrive(&o_free[pend_b]);
+        const uint32_t w = pub_w;  // hand the piece to the publisher warp
+        pub_pc[w % kPubRing] = (uint8_t)pi;
+        pub_l[w % kPubRing] = (uint8_t)l;
+        __threadfence_block();
+        pub_w = w + 1;
+      }
+      __syncwarp();
+      G += n_in + 2;
+      SR_PIECE_END
+    }
+  } else {
+    // ===================== epilogue: 2 groups x 4 warps (alternate rows); also build the next layers' bias tiles =
+    const int quarter = warp & 3;
+    const int grp = (warp - 2) >> 2;
+    const int m = quarter * 32 + lane_id();
+    const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+    const int et = (int)threadIdx.x - 64;  // 0 .. 255 over the eight epilogue warps
+    uint8_t* stage = sO + grp * kRollNO * ROWB;
+    auto arm_layer = [&](int l) {  // bias tile of layer l into slot l & 1 (its previous user, layer l - 2, is drained)
+      chain_bias_tile(sBt + (l & 1) * C * 32, p.L[l].bias, C, et, 256);
+      fence_proxy_async_smem();
+      named_bar_sync(1, 256);
+      if (et == 0) mbar_arrive(&arm_bar[l & 1]);
+    };
+    arm_layer(0);
+    if (nl > 1) arm_layer(1);
+    uint32_t ophase = 0;
+    for (int b = grp; b < RB; b += 2)
+      if (lane_id() == 0) mbar_arrive(&r_free[b]);
+    int os = 0;
+    unsigned G = 0, xi = 0;  // xi: aux rows consumed so far (layers with an aux row only)
+    for (int l = 0; l < nl; ++l) {
+      const ChainLayer& Ly = p.L[l];
+      if (l >= 1 && l + 1 < nl) arm_layer(l + 1);
+      const int emode = Ly.emode;
+      const bool has_aux = (emode & 5) != 0;
+      const bf16* res2 = Ly.res2;
+      const unsigned Gl = G;
+      SR_PIECE_BEGIN
+      const int xc = x0 + m;
+      const bool lane_ok = xc < W;
+      const bool sep0 = p.sep > 0 && ((xc % p.sep) == 0 || (xc % p.sep) == p.sep - 1);
+      for (int q = -1; q <= n_in; ++q) {
+        const unsigned g = G + q + 1;
+        const bool emit = q >= 1 && q <= n_in - 2;
+        const unsigned xr = xi;
+        if (emit && has_aux) ++xi;
+        if ((int)(g & 1) != grp) continue;
+        const int r = y0 - 1 + q;
+        const size_t pix = (((size_t)n * H + r) * W) + xc;
+        uint4 r2[C / 8];
+        if (emit && lane_ok && (emode & 2)) ld_row<C>(res2 + pix * C, r2);
+        const int b = ring_idx<RB>(g);
+        mbar_wait(&r_ready[b], (uint32_t)(g / RB) & 1u);
+        tc_fence_after();
+        float v[C];
+        ring_load<C>(tmem + lane_off + b * C, v);
+        tc_fence_before();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&r_free[b]);
+        if (!emit) continue;
+        if (warp == 2 + 4 * grp && lane_id() == 0 && G == Gl) { SR_RDBG2(l, q, 2) }
+        const uint4* aux = reinterpret_cast<const uint4*>(sA + (int)(xr % NAUX) * ROWB + m * C * 2);
+        if (has_aux) mbar_wait(&x_full[xr % NAUX], (uint32_t)(xr / NAUX) & 1u);
+        mbar_wait(&o_free[grp * kRollNO + os], ophase ^ 1);
+        if (lane_ok) {
+          uint4* orow = reinterpret_cast<uint4*>(stage + os * ROWB + m * C * 2);
+          switch (emode) {
+            case 8: roll_stage<C, 8>(orow, v, aux, r2, sep0, emode); break;
+            case 1 | 8: roll_stage<C, 1 | 8>(orow, v, aux, r2, sep0, emode); break;
+            case 1 | 2 | 8: roll_stage<C, 1 | 2 | 8>(orow, v, aux, r2, sep0, emode); break;
+            case 4 | 8: roll_stage<C, 4 | 8>(orow, v, aux, r2, sep0, emode); break;
+            case 16 | 8: roll_stage<C, 16 | 8>(orow, v, aux, r2, sep0, emode); break;
+            default: roll_stage<C, 32>(orow, v, aux, r2, sep0, emode); break;
+          }
+        }
+        if (has_aux) {
+          __syncwarp();
+          if (lane_id() == 0) mbar_arrive(&x_empty[xr % NAUX]);
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&o_full[grp * kRollNO + os]);
+        if (++os == kRollNO) { os = 0; ophase ^= 1; }
+      }
+      G += n_in + 2;
+      SR_PIECE_END
+    }
+  }
+#undef SR_PIECE_BEGIN
+#undef SR_PIECE_END
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tmem);
+  if (threadIdx.x == 0) {  // the last CTA out advances the generation for the next launch
+    __threadfence();
+    const unsigned prev = atomicAdd(p.sync + 1, 1u);
+    if (prev == gridDim.x - 1) {
+      p.sync[1] = 0;
+      __threadfence();
+      atomicAdd(p.sync, 1u);
+    }
+  }
+}
+
+static unsigned long long* g_chain_dbg = nullptr;
+void set_chain_dbg(void* p) { g_chain_dbg = reinterpret_cast<unsigned long long*>(p); }
+
+bool chain_supported(int cp, int W, int nl) {
+  if (nl < 1 || nl > kChainMax || W < 96) return false;
+  return (cp == 32 && RollCfg<32, 32>::FITS) || (cp == 48 && RollCfg<48, 48>::FITS);
+}
+
+size_t chain_sync_words(int N, int H, int W) {
+  return 2 + (size_t)N * ((W + kRollTW - 1) / kRollTW) * H;
+}
+
+// Work split of a chain launch (the same for every layer).  With at least one CTA per column strip: two phases --
+// every CTA takes one band of the top half of the rows and one band of the bottom half (bands of neighbouring
+// strips cover the same rows), and walks layer l as [top band, bottom band]: the rows a top band needs for layer
+// l + 1 were all published during the previous top-band phase, a whole bottom-band phase before (and the bottom
+// half's row a boundary band needs comes last in its pass), so the layer boundary's store -> publish -> load latency
+// is hidden by the other phase's work instead of idling the tensor pipe.  Bands are paired tall with short.
+// Otherwise: contiguous (strip, row) ranges (<= 4 pieces per CTA).
+static bool chain_pieces(ChainParams& prm, int N, int H, int W, int grid) {
+  const int S = N * ((W + kRollTW - 1) / kRollTW);
+  if (grid >= S && grid <= kChainMaxCta && H >= 8 && grid <= S * (H / 2) &&
+      std::getenv("SR_CHAIN_CONTIG") == nullptr) {
+    const int hs[3] = {0, H / 2, H};
+    std::vector<ChainPiece> ph[2];
+    for (int h = 0; h < 2; ++h) {
+      const int q = grid / S, rm = grid % S, rows = hs[h + 1] - hs[h];
+      for (int sc = 0; sc < S; ++sc) {
+        const int k = q + ((h == 0 ? sc : S - 1 - sc) < rm ? 1 : 0);  // extra bands on different strips per phase
+        for (int j = 0; j < k; ++j)
+          ph[h].push_back(ChainPiece{(short)sc, (short)(hs[h] + rows * j / k), (short)(hs[h] + rows * (j + 1) / k), 0});
+      }
+    }
+    auto ht = [](const ChainPiece& a) { return a.y1 - a.y0; };
+    std::stable_sort(ph[0].begin(), ph[0].end(), [&](const ChainPiece& a, const ChainPiece& b) { return ht(a) > ht(b); });
+    std::stable_sort(ph[1].begin(), ph[1].end(), [&](const ChainPiece& a, const ChainPiece& b) { return ht(a) < ht(b); });
+    for (int c = 0; c < grid; ++c) { prm.pc[c][0] = ph[0][c]; prm.pc[c][1] = ph[1][c]; }
+    prm.nph = 2;
+    return true;
+  }
+  const long long total = (long long)S * H;
+  const long long maxlen = (total + grid - 1) / grid;
+  if ((maxlen + H - 1) / H + 1 > 4) return false;
+  prm.nph = 0;
+  return true;
+}
+
+template <int C>
+static cudaError_t launch_chain_t(const ChainParams& prm, int grid, cudaStream_t st) {
+  auto kern = k_conv_chain<C>;
+  constexpr size_t smem = RollCfg<C, C>::SMEM;
+  static bool configured = false;
+  if (!configured) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    configured = true;
+  }
+  return launch_coop(kern, dim3(grid), dim3(kChainThreads), smem, st, prm);
+}
+
+cudaError_t launch_conv_chain(int cp, const ChainLayerDesc* layers, int nl, int sep, int N, int H, int W,
+                              unsigned* sync, cudaStream_t st) {
+  if (!chain_supported(cp, W, nl) || !sync) return cudaErrorNotSupported;
+  ChainParams prm{};  // ~9 KB of kernel parameters (tensor maps by value: a captured graph keeps its own copy)
+  for (int l = 0; l < nl; ++l) {
+    const ChainLayerDesc& d = layers[l];
+    ChainLayer& L = prm.L[l];
+    if (make_act_tmap(&L.tin, d.in, N, H, W, cp, kRollTW + 2, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS)
+      return cudaErrorInvalidValue;
+    if (make_row_tmap(&L.tout, d.out, N, H, W, cp, kRollTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+    if (d.res1 && d.mask) return cudaErrorNotSupported;
+    const void* auxp = d.res1 ? (const void*)d.res1 : (d.mask ? (const void*)d.mask : (const void*)d.out);
+    if (make_row_tmap(&L.taux, auxp, N, H, W, cp, kRollTW, cp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+    L.w = d.w;
+    L.bias = d.bias;
+    L.res2 = d.res2;
+    L.emode = (d.res1 ? 1 : 0) | (d.res2 ? 2 : 0) | (d.mask ? 4 : 0) | (sep > 0 ? 8 : 0) | (d.relu ? 16 : 0);
+    L.aux_dep = d.res1 ? d.aux_dep : -1;
+    if (L.aux_dep >= l) return cudaErrorInvalidValue;
+  }
+  prm.nl = nl;
+  prm.N = N;
+  prm.H = H;
+  prm.W = W;
+  prm.sep = sep;
+  prm.sync = sync;
+  prm.dbg = g_chain_dbg;
+  if (const char* e = std::getenv("SR_CHAIN_DBG_CTA")) prm.dbg_cta = std::atoi(e);
+  const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  if (!chain_pieces(prm, N, H, W, grid)) return cudaErrorNotSupported;
+  if (cp == 32) return launch_chain_t<32>(prm, grid, st);
+  return launch_chain_t<48>(prm, grid, st);
 }
 
 }  // namespace sr

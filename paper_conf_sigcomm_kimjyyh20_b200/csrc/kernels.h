@@ -66,6 +66,25 @@ cudaError_t launch_conv_roll_tail_train(int cinp, int coutp, int s, const void* 
                                         const float* bias, const uint8_t* lr, const uint8_t* hr_ref, bf16* dy,
                                         double* loss_sum, int vsep, int vp, int l1, int bicubic, int N, int H, int W,
                                         cudaStream_t st, int w_early);
+// a chain of C -> C rolling convs in one persistent cooperative launch (k_conv_chain, conv_roll.cu); each layer is
+// k_conv_roll's conv with the same epilogue variants; aux_dep: index of the earlier layer of the chain whose output
+// res1 is (-1: written by an earlier kernel); sync: chain_sync_words() zero-initialised words owned by the caller
+struct ChainLayerDesc {
+  const void* in;
+  bf16* out;
+  const bf16* w;
+  const float* bias;
+  const bf16* res1;
+  const bf16* res2;
+  const bf16* mask;
+  int relu;
+  int aux_dep;
+};
+bool chain_supported(int cp, int W, int nl);
+void set_chain_dbg(void* p);  // benchmarking only: globaltimer stamps of k_conv_chain
+size_t chain_sync_words(int N, int H, int W);
+cudaError_t launch_conv_chain(int cp, const ChainLayerDesc* layers, int nl, int sep, int N, int H, int W,
+                              unsigned* sync, cudaStream_t st);
 bool resblock_supported(int cp, int W);
 // the residual block on CTA pairs (conv_block2.cu, tcgen05 cta_group::2; inference only, bit-identical output)
 bool resblock2_supported(int cp, int W);

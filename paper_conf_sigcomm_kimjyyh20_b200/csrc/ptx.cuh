@@ -262,4 +262,28 @@ __device__ __forceinline__ void pdl_enter() {
   pdl_wait();
   pdl_trigger();
 }
+
+// ---- cross-CTA row flags (k_conv_chain): the rows a CTA wrote with TMA stores are published, once their bulk group
+// has completed, by one proxy fence + one gpu-scope fence and then plain relaxed flag stores (one per row, from the
+// lanes of the store warp); a consumer warp polls the flags it needs with relaxed loads in parallel (one per lane),
+// then fences (acquire) and orders its own TMA loads after them with a proxy fence
+__device__ __forceinline__ unsigned ld_relaxed_gpu(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_gpu(unsigned* p, unsigned v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+// until *p >= target (wrap-safe); traps after ~2^34 cycles so a dependency bug fails the launch instead of hanging
+__device__ __forceinline__ void flag_spin(const unsigned* p, unsigned target) {
+  if ((int)(ld_relaxed_gpu(p) - target) >= 0) return;
+  const long long t0 = clock64();
+  while ((int)(ld_relaxed_gpu(p) - target) < 0) {
+    __nanosleep(20);
+    if (clock64() - t0 > (1ll << 34)) __trap();
+  }
+}
 }  // namespace sr

@@ -161,6 +161,9 @@ struct sr_ctx {
   bool fuse_head = true;      // head conv reads the u8 frame directly (sr_set_fusion bit 6 clears)
   bool pair_blocks = true;    // residual blocks of wide frames on CTA pairs, cta_group::2 (sr_set_fusion bit 7 clears)
   bool split_blocks = false;  // inference residual blocks on CTA pairs split by conv (sr_set_fusion bit 8 sets)
+  bool chain = false;         // training: block convs + body conv (forward) and the data-gradient chain as one
+                              // persistent launch each (k_conv_chain; sr_set_fusion bit 9 or SR_CHAIN=1 sets)
+  unsigned* chain_sync[2] = {nullptr, nullptr};  // k_conv_chain generation + row flags (forward, backward)
   int sm_train = 0;           // sr_set_sm_split: SMs given to the training kernels (0 = all SMs to every call)
   bool train_fold_only = false;  // TRAIN's tiled layouts (wf, wd) may be stale: rebuild before reading them
   int sm_total = 0;
@@ -172,6 +175,10 @@ struct sr_ctx {
 };
 
 // ------------------------------------------------------------------------------------------ helpers
+static bool env_chain() {  // SR_CHAIN=1: training conv chains as persistent k_conv_chain launches (A/B switch)
+  const char* e = std::getenv("SR_CHAIN");
+  return e && e[0] == '1';
+}
 static sr_status fail(sr_ctx* c, sr_status st, const std::string& msg) {
   if (c) {
     c->err = msg;
@@ -300,6 +307,21 @@ static sr_status roll_ex(sr_ctx* ctx, const char* cls, int cinp, int coutp, cons
   tmark_end(ctx, st);
   ctx->launches++;
   if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("roll launch: ") + cudaGetErrorString(e));
+  return SR_OK;
+}
+
+// a chain of C -> C training convs as one persistent launch (k_conv_chain), timed as one class
+static sr_status chain_launch(sr_ctx* ctx, const char* cls, const std::vector<ChainLayerDesc>& L, int sep, int H,
+                              int W, unsigned* sync, cudaStream_t st) {
+  const int Cp = ctx->Cp;
+  if (ctx->timing) {
+    const double px = (double)H * W * L.size();
+    tmark_begin(ctx, std::string(cls) + "_" + std::to_string(Cp), 2.0 * 9 * Cp * Cp * px, px * 2.0 * 2 * Cp, st);
+  }
+  cudaError_t e = launch_conv_chain(Cp, L.data(), (int)L.size(), sep, 1, H, W, sync, st);
+  tmark_end(ctx, st);
+  ctx->launches++;
+  if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("chain launch: ") + cudaGetErrorString(e));
   return SR_OK;
 }
 
@@ -568,6 +590,11 @@ static sr_status ensure_train_ws(sr_ctx* ctx, size_t pix) {
   CK(dalloc(&ctx->tdt, pix * Cp));
   for (auto& p : ctx->tdf) CK(dalloc(&p, pix * Cp));
   for (auto& p : ctx->tdtb) CK(dalloc(&p, pix * Cp));
+  for (auto& p : ctx->chain_sync) {  // >= chain_sync_words(1, H, W) for any H x W = pix with W >= 96
+    const size_t words = 66 + pix / 48;
+    CK(dalloc(&p, words));
+    CK(cudaMemset(p, 0, words * sizeof(unsigned)));
+  }
   ctx->tr_pix = pix;
   return SR_OK;
 }
@@ -592,7 +619,20 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
   // ---- forward (saving f_0..f_B, t_1..t_B, g)
   TRY(roll_ex(ctx, "train_fwd", 16, Cp, ctx->tx16, WO(0), Bv(0), nullptr, nullptr, nullptr, 0, sep, ctx->tf[0], 1,
               Hv, Wv, st));
-  for (int b = 0; b < B; ++b) {
+  const int cb = 1 + 2 * B, cu = cb + 1;
+  const bool use_chain = ctx->chain && chain_supported(Cp, Wv, 2 * B + 1) &&
+                         chain_sync_words(1, Hv, Wv) <= 66 + pix / 48;
+  if (use_chain) {  // the B blocks (conv1 ReLU -> t_b, conv2 + f_b -> f_b+1) and the body conv (+ f_0) in one launch
+    std::vector<ChainLayerDesc> L;
+    for (int b = 0; b < B; ++b) {
+      L.push_back({ctx->tf[b], ctx->tts[b], WO(1 + 2 * b), Bv(1 + 2 * b), nullptr, nullptr, nullptr, 1, -1});
+      L.push_back({ctx->tts[b], ctx->tf[b + 1], WO(2 + 2 * b), Bv(2 + 2 * b), ctx->tf[b], nullptr, nullptr, 0,
+                   b == 0 ? -1 : 2 * b - 1});
+    }
+    L.push_back({ctx->tf[B], ctx->tg, WO(cb), Bv(cb), ctx->tf[0], nullptr, nullptr, 0, -1});
+    TRY(chain_launch(ctx, "train_fwd_chain", L, sep, Hv, Wv, ctx->chain_sync[0], st));
+  }
+  for (int b = 0; b < B && !use_chain; ++b) {
     if (ctx->fuse_blocks && resblock_supported(Cp, Wv)) {  // fused block, t also saved for the backward pass
       if (ctx->timing) {
         const double px = (double)Hv * Wv;
@@ -610,9 +650,9 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
     TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tts[b], WO(2 + 2 * b), Bv(2 + 2 * b), ctx->tf[b], nullptr, nullptr, 0,
                 sep, ctx->tf[b + 1], 1, Hv, Wv, st));
   }
-  const int cb = 1 + 2 * B, cu = cb + 1;
-  TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tf[B], WO(cb), Bv(cb), ctx->tf[0], nullptr, nullptr, 0, sep, ctx->tg, 1,
-              Hv, Wv, st));
+  if (!use_chain)
+    TRY(roll_ex(ctx, "train_fwd", Cp, Cp, ctx->tf[B], WO(cb), Bv(cb), ctx->tf[0], nullptr, nullptr, 0, sep, ctx->tg, 1,
+                Hv, Wv, st));
   {
     EpiParams e{};
     e.bias = Bv(cu);
@@ -650,9 +690,22 @@ static sr_status train_grad_virtual(sr_ctx* ctx, const uint8_t* lr, const uint8_
   // ---- backward: the data-gradient chain (every df_b, dt_b kept), then all weight gradients in one batched launch
   TRY(roll_ex(ctx, "train_dgrad", OUTP, Cp, ctx->tdy, WDO(cu), nullptr, nullptr, nullptr, nullptr, 0, sep, ctx->tdg, 1,
               Hv, Wv, st));
-  TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdg, WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr,
-              0, sep, ctx->tdf[B], 1, Hv, Wv, st));
-  for (int b = B - 1; b >= 0; --b) {
+  if (use_chain) {  // body dgrad, then per block (last first): dt_b = dgrad_conv2(df_b+1) x 1[t_b > 0] and
+                    // df_b = dgrad_conv1(dt_b) + df_b+1 (+ dg at b = 0), in one launch
+    std::vector<ChainLayerDesc> L;
+    L.push_back({ctx->tdg, ctx->tdf[B], WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr, 0, -1});
+    for (int b = B - 1; b >= 0; --b) {
+      const int l2 = (int)L.size();
+      L.push_back({ctx->tdf[b + 1], ctx->tdtb[b], WDO(2 + 2 * b), nullptr, nullptr, nullptr, ctx->tts[b], 0, -1});
+      L.push_back({ctx->tdtb[b], ctx->tdf[b], WDO(1 + 2 * b), nullptr, ctx->tdf[b + 1], b == 0 ? ctx->tdg : nullptr,
+                   nullptr, 0, l2 - 1});
+    }
+    TRY(chain_launch(ctx, "train_dgrad_chain", L, sep, Hv, Wv, ctx->chain_sync[1], st));
+  } else {
+    TRY(roll_ex(ctx, "train_dgrad", Cp, Cp, ctx->tdg, WDO(cb), nullptr, B == 0 ? ctx->tdg : nullptr, nullptr, nullptr,
+                0, sep, ctx->tdf[B], 1, Hv, Wv, st));
+  }
+  for (int b = B - 1; b >= 0 && !use_chain; --b) {
     if (ctx->fuse_blocks && ctx->fuse_bwd && resblock_supported(Cp, Wv)) {
       // the block's data gradient in one fused kernel (k_resblock in mask mode): dt = dgrad_conv2(df) * 1[t > 0]
       // stays in shared memory (and is saved for the wgrad), df' = df + dgrad_conv1(dt) (+ dg into f0 at b = 0)
@@ -866,6 +919,7 @@ sr_status sr_create(int scale, int blocks, int channels, const sr_options* opt, 
   *out = nullptr;
   if ((scale < 2 || scale > 4) || blocks < 0 || channels < 1 || channels > 64) return SR_E_INVAL;
   sr_ctx* ctx = new sr_ctx();
+  ctx->chain = env_chain();
   ctx->s = scale;
   ctx->B = blocks;
   ctx->C = channels;
@@ -1002,6 +1056,7 @@ void sr_destroy(sr_ctx* ctx) {
   for (auto p : ctx->tts) if (p) cudaFree(p);
   for (auto p : ctx->tdf) if (p) cudaFree(p);
   for (auto p : ctx->tdtb) if (p) cudaFree(p);
+  for (auto p : ctx->chain_sync) if (p) cudaFree(p);
   if (ctx->publish_ev) cudaEventDestroy(ctx->publish_ev);
   for (auto& pe : ctx->infer_evs) cudaEventDestroy(pe.second);
   if (ctx->comm) nccl().destroy(ctx->comm);
@@ -1023,6 +1078,7 @@ sr_status sr_set_fusion(sr_ctx* ctx, int fuse_blocks) {
   ctx->fuse_head = (fuse_blocks & 64) == 0;     // bit 6 set: k_pack_input + head conv on the bf16 copy
   ctx->pair_blocks = (fuse_blocks & 128) == 0;  // bit 7 set: single-CTA residual blocks instead of CTA pairs
   ctx->split_blocks = (fuse_blocks & 256) != 0; // bit 8 set: inference blocks on conv-split CTA pairs
+  ctx->chain = (fuse_blocks & 512) != 0 || env_chain();  // bit 9 set: training conv chains as k_conv_chain
   return SR_OK;
 }
 

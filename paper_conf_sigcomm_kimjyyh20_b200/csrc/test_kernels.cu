@@ -675,3 +675,10 @@ extern "C" int sr_test_mma2(const void* A, const void* B, float* D, int N, int K
   cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
   return e == cudaSuccess ? SR_OK : SR_E_CUDA;
 }
+
+namespace sr { void set_chain_dbg(void* p); }
+// benchmarking only: k_conv_chain writes per (CTA, layer) globaltimer stamps into dev (u64 [grid][20][8]); nullptr off
+extern "C" int sr_test_chain_dbg(void* dev) {
+  sr::set_chain_dbg(dev);
+  return 0;
+}

@@ -153,6 +153,38 @@ def test_train_sampled_recaptures_on_new_loss_pointer():
     assert l1.item() > 0 and l2.item() > 0 and l1.item() != l2.item()
 
 
+@pytest.mark.parametrize("cfg,n,p", [((3, 8, 48), 64, 48), ((2, 8, 32), 30, 48), ((3, 2, 48), 5, 40),
+                                     ((2, 3, 32), 3, 60)])
+def test_chain_equals_per_layer_launches(cfg, n, p):
+    """The persistent chain launches (k_conv_chain: the forward blocks + body conv, and the data-gradient chain, each
+    one cooperative launch with cross-CTA row flags; opt-in, set_fusion bit 9) against one k_conv_roll launch per
+    conv (set_fusion 0, the blocks unfused): the same MMAs in the same order and the same epilogues -> loss and
+    gradient bit-identical, over several consecutive calls (the flag generation advances per launch), and within the
+    north-star bars of the oracle.  Shapes: the bench's (64 x 48x48: 25 column strips, two-phase bands), the C = 32
+    net, and ragged widths (a partial last strip; fewer CTAs than strips: contiguous pieces)."""
+    s, Bn, Cn = cfg
+    lrp, hrp, _ = synth_patch_pool(n, s, s * p, seed=51, frame_hw=(s * p * 3, s * p * 4))
+    lr, hr = torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda()
+    out = []
+    for mode in (512, 0):
+        ctx = _ctx(s, Bn, Cn, seed=52)
+        ctx.set_fusion(mode)
+        p0 = ctx.get_params("train")
+        runs = []
+        for _ in range(3):
+            loss = torch.zeros(1, device="cuda")
+            ctx.train_grad(lr, hr, loss)
+            runs.append((loss.item(), ctx.grad_buffer().clone()))
+        out.append(runs)
+    for (la, ga), (lb, gb) in zip(out[0], out[1]):
+        assert la == lb
+        assert torch.equal(ga, gb)
+    if n <= 8:
+        ref_loss, ref_g = O.train_loss_and_grad(p0, lrp, hrp, s, Bn, Cn)
+        assert abs(out[0][0][0] - ref_loss) / ref_loss < 1e-2
+        assert rel_l2(out[0][0][1].cpu().numpy(), ref_g) < 1e-2
+
+
 def test_whole_720p_frame_elementwise():
     """One whole 720p frame through the x3 8x48 net (the bench's net and frame size) against the oracle, every
     output element: |du8| <= 2 and PSNR within 0.05 dB of the oracle's against the HR original."""
