@@ -412,7 +412,7 @@ def run_ours(args):
                 "frac_of_sustained": round(TRAIN_FLOP / (tr_ms * 1e-3) / 1e12 / sustained, 4),
                 "allreduce_us": round(allreduce_us, 2) if allreduce_us is not None else None,
                 "allreduce_bytes": ctx.num_params * 4,
-                "roofline": _roofline(tstats, tdom, sustained, pk_kind),
+                "roofline": _roofline(tstats, tdom, sustained, pk_kind, traffic_of(tdom, 1, PATCH, BATCH * (PATCH + 2))),
                 "kernel_share": {k: round(v["ms"] / tktot, 4)
                                  for k, v in sorted(tstats.items(), key=lambda kv: -kv[1]["ms"])},
                 "kernel_share_note": "eager event-timed launches of the same kernels (sample, forward, backward; "
@@ -427,7 +427,7 @@ def run_ours(args):
                 "workload": f"BASELINE config 2: {frames} x 540p -> 1080p x2, 8 blocks x 32 ch, inference only",
                 "frames_per_s": round(c2fps, 2), "ms_per_batch": round(c2["c2_ms"] / args.steps, 3),
                 "tflops": round(c2fps * C2_H * C2_W * C2_FLOP_PER_LR_PX / 1e12, 1),
-                "roofline": _roofline(cst, cdom, sustained, pk_kind),
+                "roofline": _roofline(cst, cdom, sustained, pk_kind, traffic_of(cdom, frames, C2_H, C2_W)),
                 "kernel_share": {k: round(v["ms"] / sum(x["ms"] for x in cst.values()), 4)
                                  for k, v in sorted(cst.items(), key=lambda kv: -kv[1]["ms"])},
             }
@@ -530,17 +530,21 @@ def run_reference(args):
     }), flush=True)
 
 
-def traffic_of(kernel_class, frames):
-    """DRAM bytes per launch of the dominant kernel from the committed ncu capture (profiles/r01_traffic.json),
-    when it was taken on the same launch shape; else None."""
-    try:
-        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
-            t = json.load(f).get(kernel_class)
-    except (OSError, ValueError):
-        return None
-    if not t or t.get("frames") != frames or (t.get("h"), t.get("w")) != (LR_H, LR_W):
-        return None
-    return int(t["dram_read"] + t["dram_write"])
+def traffic_of(kernel_class, frames, h=None, w=None):
+    """DRAM bytes per launch of a dominant kernel from the committed ncu captures (profiles/r01_traffic.json: the
+    headline's inference kernels; profiles/r02_traffic.json: the cfg4 / cfg2 side lines), when taken on the same
+    launch shape; else None."""
+    h = LR_H if h is None else h
+    w = LR_W if w is None else w
+    for name in ("r02_traffic.json", "r01_traffic.json"):
+        try:
+            with open(os.path.join(ROOT, "profiles", name)) as f:
+                t = json.load(f).get(kernel_class)
+        except (OSError, ValueError):
+            continue
+        if t and t.get("frames") == frames and (t.get("h"), t.get("w")) == (h, w):
+            return int(t["dram_read"] + t["dram_write"])
+    return None
 
 
 def _free_port():
