@@ -185,6 +185,27 @@ def test_chain_equals_per_layer_launches(cfg, n, p):
         assert rel_l2(out[0][0][1].cpu().numpy(), ref_g) < 1e-2
 
 
+@pytest.mark.parametrize("train_sms", [40, 24])
+def test_chain_on_partition_grids(train_sms):
+    """k_conv_chain at the bench's training shape (64 x 48x48 -> 25 column strips) with the grid of a training
+    partition (sr_set_sm_split): 40 CTAs = two-phase bands of unequal height (15 strips x 2 bands, 10 x 1), 24 CTAs =
+    fewer CTAs than strips -> contiguous pieces spanning strips; bit-identical to the per-layer launches."""
+    s, Bn, Cn = 3, 8, 48
+    lrp, hrp, _ = synth_patch_pool(64, s, s * 48, seed=61, frame_hw=(s * 48 * 3, s * 48 * 4))
+    lr, hr = torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda()
+    out = []
+    for mode in (512, 0):
+        ctx = _ctx(s, Bn, Cn, seed=62)
+        ctx.set_fusion(mode)
+        ctx.set_sm_split(train_sms)
+        loss = torch.zeros(1, device="cuda")
+        ctx.train_grad(lr, hr, loss)
+        out.append((loss.item(), ctx.grad_buffer().clone()))
+        ctx.set_sm_split(0)
+    assert out[0][0] == out[1][0]
+    assert torch.equal(out[0][1], out[1][1])
+
+
 def test_whole_720p_frame_elementwise():
     """One whole 720p frame through the x3 8x48 net (the bench's net and frame size) against the oracle, every
     output element: |du8| <= 2 and PSNR within 0.05 dB of the oracle's against the HR original."""
