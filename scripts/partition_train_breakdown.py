@@ -6,8 +6,10 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sigcomm_kimjyyh20_b200 import SRContext
 from synth import synth_patch_pool
 
+fusion = int(os.environ.get("SR_FUSION", "1"))
 for n in [int(x) for x in sys.argv[1:]] or [40, 32]:
     ctx = SRContext(3, 8, 48, seed=0)
+    ctx.set_fusion(fusion)
     s_inf, s_tr, n_inf, n_tr = SRContext.sm_partition(n)
     ctx.set_sm_split(n_tr)
     dev = torch.device("cuda")
@@ -36,7 +38,7 @@ for n in [int(x) for x in sys.argv[1:]] or [40, 32]:
     s_tr.synchronize()
     st = ctx.kernel_stats()
     tot = sum(v["ms"] for v in st.values())
-    print(f"train_sms={n_tr}: graph {ms:.3f} ms/iter; eager per iter {tot / 5:.3f} ms: " +
+    print(f"fusion={fusion} train_sms={n_tr}: graph {ms:.3f} ms/iter; eager per iter {tot / 5:.3f} ms: " +
           ", ".join(f"{k} {v['ms'] / 5 * 1e3:.0f}us" for k, v in sorted(st.items(), key=lambda kv: -kv[1]["ms"])))
     ctx.set_sm_split(0)
     del ctx
