@@ -35,6 +35,7 @@ def build(force=False, verbose=True):
     os.makedirs(OBJDIR, exist_ok=True)
     flags = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-Xcompiler", "-fPIC",
              "-Xptxas", "-v" if os.environ.get("SR_PTXAS_V") else "-O3", "-I", os.path.join(ROOT, "include")]
+    flags += os.environ.get("SR_NVCC_DEFS", "").split()  # A/B builds only, e.g. "-DSR_BLOCK_DIRECT_OUT=1"
     nvcc = nvcc_path()
 
     def compile_one(src):
