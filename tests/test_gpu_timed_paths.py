@@ -11,6 +11,9 @@
 * Whole-frame inference: one 720p frame x3 8x48 element-wise (|du8| <= 2, PSNR within 0.05 dB) and frame 29 of the
   bench's 30-frame batch bit-identical to the frame inferred alone (offsets > 2^31 bytes in the activations).
 * The paper's own 120-px HR training patch (LR 60 at x2, 40 at x3).
+* The other BASELINE configs at their own sizes: config 2 (x2 8x32, a whole 540p frame element-wise + frame 29 of a
+  30-frame batch), config 5 (x2 8x48 1080p: a band of the whole-frame output against the oracle on the band + halo),
+  config 4's second net (x2 8x32, 64 x 48x48: gradient and Adam step).
 """
 import numpy as np
 import pytest
@@ -229,6 +232,58 @@ def test_frame_29_of_bench_batch_equals_frame_alone():
     torch.cuda.synchronize()
     assert torch.equal(batch[29], alone[0])
     assert torch.equal(batch[0], first[0])
+
+
+def test_cfg2_whole_540p_frame_elementwise_and_batch_tail():
+    """BASELINE config 2's net and frame (x2, 8 blocks x 32 ch, 540p -> 1080p; residual blocks on CTA pairs): one
+    whole frame element-wise against the oracle (|du8| <= 2, PSNR within 0.05 dB against the HR original), and
+    frame 29 of the bench's 30-frame batch bit-identical to that frame inferred alone."""
+    s, b, c = 2, 8, 32
+    ctx = _ctx(s, b, c, seed=0)
+    lr, hr = synth_frames(1, 540, 960, seed=1002, scale=s)
+    got = ctx.infer(torch.from_numpy(lr).cuda(), "serve").cpu().numpy()
+    ref = O.infer_u8(ctx.get_params("serve"), lr, s, b, c)
+    d = np.abs(got.astype(np.int64) - ref.astype(np.int64))
+    assert d.max() <= 2, d.max()
+    assert abs(psnr(got, hr) - psnr(ref, hr)) < 0.05
+    lr30 = torch.from_numpy(synth_frames(30, 540, 960, seed=1002)).cuda()
+    batch = ctx.infer(lr30, "serve")
+    alone = ctx.infer(lr30[29:30].contiguous(), "serve")
+    torch.cuda.synchronize()
+    assert torch.equal(batch[29], alone[0])
+
+
+def test_cfg5_1080p_x2_band_elementwise():
+    """BASELINE config 5's net and frame (x2, 8 x 48, 1080p -> 2160p): the HR rows of a 64-row LR band in the middle
+    of a whole-frame inference against the oracle run on that band plus its receptive-field halo (2B + 4 = 20 LR
+    rows each side; R12), element-wise (|du8| <= 2) -- the full 1080p frame is beyond the oracle's seconds budget."""
+    s, b, c = 2, 8, 48
+    ctx = _ctx(s, b, c, seed=0)
+    lr, _ = synth_frames(1, 1080, 1920, seed=1005, scale=s)
+    got = ctx.infer(torch.from_numpy(lr).cuda(), "serve").cpu().numpy()
+    r0, r1, R = 500, 564, 2 * b + 4
+    band = np.ascontiguousarray(lr[:, r0 - R:r1 + R])
+    ref = O.infer_u8(ctx.get_params("serve"), band, s, b, c)[:, s * R:s * (R + r1 - r0)]
+    d = np.abs(got[:, s * r0:s * r1].astype(np.int64) - ref.astype(np.int64))
+    assert d.max() <= 2, d.max()
+
+
+def test_cfg4_secondary_net_gradient_batch64():
+    """BASELINE config 4's second net (x2, 8 x 32) at the bench's batch (64 patches of 48 x 48, virtual wide batch of
+    64 x 50 columns): loss within 1e-2 and gradient rel L2 <= 1e-2 against the oracle, one Adam step rel L2 <= 1e-3."""
+    s, b, c = 2, 8, 32
+    ctx = _ctx(s, b, c, seed=7)
+    lrp, hrp, _ = synth_patch_pool(64, s, s * 48, seed=1008, frame_hw=(960, 1600))
+    p0 = ctx.get_params("train")
+    lo = torch.zeros(1, device="cuda")
+    ctx.train_grad(torch.from_numpy(lrp).cuda(), torch.from_numpy(hrp).cuda(), lo)
+    g = ctx.grad_buffer().cpu().numpy().copy()
+    ref_loss, ref_g = O.train_loss_and_grad(p0, lrp, hrp, s, b, c)
+    assert abs(lo.item() - ref_loss) / ref_loss < 1e-2
+    assert rel_l2(g, ref_g) < 1e-2, rel_l2(g, ref_g)
+    ctx.train_apply(1.0)
+    rp, _, _ = O.adam_step(p0, np.zeros_like(p0), np.zeros_like(p0), ref_g, 1)
+    assert rel_l2(ctx.get_params("train"), rp) < 1e-3
 
 
 @pytest.mark.parametrize("s,p", [(2, 60), (3, 40)])
