@@ -27,6 +27,7 @@
 #include "kernels.h"
 #include "launch.cuh"
 #include "tail.cuh"
+#include "color.cuh"
 #include <algorithm>
 #include <vector>
 
@@ -88,6 +89,12 @@ struct RollArgs {
   bf16* dy;
   double* loss_sum;
   int vsep, vp, l1;
+  // YUV head (U8 && YUV): the input is an I420 frame -- tm_in maps the Y plane's rows, U / V ([N][H/2][W/2]) are read
+  // directly; the expansion warps convert with the library's BT.601 integer conversion (color.cuh) and also write
+  // the frame's RGB u8 copy (rgb_out [N][H][W][3], each strip's own pixels and rows) for the tail's skip
+  const uint8_t* yuv_u;
+  const uint8_t* yuv_v;
+  uint8_t* rgb_out;
 };
 #define SR_RDBG(ev, idx) \
   if (DBG && a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -164,7 +171,8 @@ static constexpr int kU8Slots = 8;
 static constexpr uint32_t kU8Slot = 512;  // 26 chunks = 416 B per u8 row
 // DBG: the instantiation with the CTA-0 clock64 stamps (benchmarking tools only; the production instantiations
 // carry no stamp code -- each predicated stamp sits on a latency-bound epilogue chain)
-template <int CINP, int COUTP, int TS, bool U8 = false, bool DBG = false>
+static constexpr int kYuvChunks = 10;  // Y bytes [16 cb, 16 cb + 160) cover pixels x0-1 .. x0+128
+template <int CINP, int COUTP, int TS, bool U8 = false, bool DBG = false, bool YUV = false>
 __global__ void __launch_bounds__(kRollThreads + (U8 ? 64 : 0), 1)
 k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_out,
             const __grid_constant__ CUtensorMap tm_aux, const bf16* __restrict__ wfold, const RollArgs a) {
@@ -281,8 +289,13 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       for (int i = 0; i < n_in; ++i) {
         if constexpr (U8) {  // u8 row y0-1+i, pixels x0-1 .. x0+128 (+ chunk alignment), for warps 12, 13 to expand
           mbar_wait(&u_empty[us], uph ^ 1);
-          mbar_arrive_expect_tx(&u_full[us], 16 * 26);
-          tma_load_4d(sA + us * kU8Slot, &tm_in, &u_full[us], 0, (3 * x0 - 3) >> 4, y0 - 1 + i, n);
+          if constexpr (YUV) {  // Y row y0-1+i, pixels x0-1 .. x0+128
+            mbar_arrive_expect_tx(&u_full[us], 16 * kYuvChunks);
+            tma_load_4d(sA + us * kU8Slot, &tm_in, &u_full[us], 0, (x0 - 1) >> 4, y0 - 1 + i, n);
+          } else {
+            mbar_arrive_expect_tx(&u_full[us], 16 * 26);
+            tma_load_4d(sA + us * kU8Slot, &tm_in, &u_full[us], 0, (3 * x0 - 3) >> 4, y0 - 1 + i, n);
+          }
           if (++us == kU8Slots) { us = 0; uph ^= 1; }
         } else {
           mbar_wait(&in_empty[s], ph ^ 1);
@@ -367,7 +380,7 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
     uint32_t ph = 0, uph = 0;
     long long rowc = 0;  // rows seen so far (both warps count every row; each converts its parity)
     SR_PIECE_BEGIN
-    const int lbase = 16 * ((3 * x0 - 3) >> 4);
+    const int lbase = YUV ? 16 * ((x0 - 1) >> 4) : 16 * ((3 * x0 - 3) >> 4);
     for (int i = 0; i < n_in; ++i, ++rowc) {
       if ((int)(rowc & 1) != warp - 12) {
         if (++us == kU8Slots) { us = 0; uph ^= 1; }
@@ -376,17 +389,43 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
       }
       mbar_wait(&u_full[us], uph);
       mbar_wait(&in_empty[s], ph ^ 1);
-      const uint32_t src = smem_u32(sA + us * kU8Slot) + (uint32_t)(3 * (x0 - 1) - lbase);
       uint8_t* dst = sIn + s * IN_STRIDE;
       constexpr int kIt = (kRollTW + 2 + 31) / 32;
       float px[kIt][3];
+      if constexpr (YUV) {  // I420 -> RGB (color.cuh) per pixel; zero outside the frame (the conv's zero padding)
+        const uint32_t src = smem_u32(sA + us * kU8Slot) + (uint32_t)(x0 - 1 - lbase);
+        const int y = y0 - 1 + i;
+        const bool row_ok = y >= 0 && y < H, own_row = i >= 1 && i <= n_in - 2;
+        const size_t crow = ((size_t)n * (H / 2) + (y >> 1)) * (size_t)(W / 2);
 #pragma unroll
-      for (int k = 0; k < kIt; ++k) {  // all loads first, so their latencies overlap
-        const int p = lane_id() + 32 * k;
-        const uint32_t q = src + 3 * min(p, kRollTW + 1);
-        px[k][0] = lds_u8f(q);
-        px[k][1] = lds_u8f(q + 1);
-        px[k][2] = lds_u8f(q + 2);
+        for (int k = 0; k < kIt; ++k) {
+          const int p = lane_id() + 32 * k, x = x0 - 1 + p;
+          const bool ok = row_ok && p < kRollTW + 2 && x >= 0 && x < W;
+          uint8_t rgb[3] = {0, 0, 0};
+          if (ok) {
+            const int Y = (int)lds_u8f(src + p);
+            yuv_to_rgb(Y, __ldg(a.yuv_u + crow + (x >> 1)), __ldg(a.yuv_v + crow + (x >> 1)), rgb);
+            if (own_row && p >= 1 && p <= kRollTW) {
+              uint8_t* o = a.rgb_out + (((size_t)n * H + y) * W + x) * 3;
+              o[0] = rgb[0];
+              o[1] = rgb[1];
+              o[2] = rgb[2];
+            }
+          }
+          px[k][0] = (float)rgb[0];
+          px[k][1] = (float)rgb[1];
+          px[k][2] = (float)rgb[2];
+        }
+      } else {
+        const uint32_t src = smem_u32(sA + us * kU8Slot) + (uint32_t)(3 * (x0 - 1) - lbase);
+#pragma unroll
+        for (int k = 0; k < kIt; ++k) {  // all loads first, so their latencies overlap
+          const int p = lane_id() + 32 * k;
+          const uint32_t q = src + 3 * min(p, kRollTW + 1);
+          px[k][0] = lds_u8f(q);
+          px[k][1] = lds_u8f(q + 1);
+          px[k][2] = lds_u8f(q + 2);
+        }
       }
 #pragma unroll
       for (int k = 0; k < kIt; ++k) {
@@ -589,13 +628,13 @@ k_conv_roll(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ C
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-template <int CINP, int COUTP, int TS = 0, bool U8 = false, bool DBG = false>
+template <int CINP, int COUTP, int TS = 0, bool U8 = false, bool DBG = false, bool YUV = false>
 static cudaError_t launch_roll_t(const CUtensorMap& ti, const CUtensorMap& to, const CUtensorMap& tx,
                                  const bf16* wfold, const RollArgs& a, int grid, cudaStream_t st) {
   if constexpr (!RollCfg<CINP, COUTP>::FITS) {
     return cudaErrorNotSupported;
   } else {
-    auto kern = k_conv_roll<CINP, COUTP, TS, U8, DBG>;
+    auto kern = k_conv_roll<CINP, COUTP, TS, U8, DBG, YUV>;
     constexpr size_t smem = RollCfg<CINP, COUTP>::SMEM;
     static bool configured = false;
     if (!configured) {
@@ -625,6 +664,30 @@ cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* w
   if (coutp == 16) return launch_roll_t<16, 16, 0, true>(ti, to, to, wfold, a, grid, st);
   if (coutp == 32) return launch_roll_t<16, 32, 0, true>(ti, to, to, wfold, a, grid, st);
   return launch_roll_t<16, 48, 0, true>(ti, to, to, wfold, a, grid, st);
+}
+
+bool roll_head_yuv_supported(int coutp, int W, const void* y, const void* u, const void* v) {
+  auto al16 = [](const void* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; };
+  return W >= 96 && W % 32 == 0 && al16(y) && al16(u) && al16(v) && (coutp == 16 || coutp == 32 || coutp == 48);
+}
+
+cudaError_t launch_conv_roll_head_yuv(int coutp, const uint8_t* y, const uint8_t* u, const uint8_t* v,
+                                      uint8_t* rgb_out, const bf16* wfold, const float* bias, bf16* out, int N, int H,
+                                      int W, cudaStream_t st, int w_early) {
+  if (!roll_head_yuv_supported(coutp, W, y, u, v) || (H & 1)) return cudaErrorNotSupported;
+  CUtensorMap ti, to;
+  if (make_u8_rows_tmap(&ti, y, N, H, W, kYuvChunks, 1) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (make_row_tmap(&to, out, N, H, W, coutp, kRollTW, coutp) != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  RollArgs a{bias, nullptr, nullptr, nullptr, 0, 0, N, H, W, nullptr, nullptr, nullptr, 0, 0, 0, 0, w_early};
+  a.yuv_u = u;
+  a.yuv_v = v;
+  a.rgb_out = rgb_out;
+  const long long rows = (long long)N * ((W + kRollTW - 1) / kRollTW) * H;
+  int grid = num_sms();
+  if (rows < grid) grid = (int)rows;
+  if (coutp == 16) return launch_roll_t<16, 16, 0, true, false, true>(ti, to, to, wfold, a, grid, st);
+  if (coutp == 32) return launch_roll_t<16, 32, 0, true, false, true>(ti, to, to, wfold, a, grid, st);
+  return launch_roll_t<16, 48, 0, true, false, true>(ti, to, to, wfold, a, grid, st);
 }
 
 static bool ch_ok(int c) { return c == 16 || c == 32 || c == 48 || c == 64; }

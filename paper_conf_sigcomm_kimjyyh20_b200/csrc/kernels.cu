@@ -2,6 +2,7 @@
 // recency-weighted sampler + patch gather, integer SSE (PSNR), bilinear-only baseline.
 #include <algorithm>
 #include "ptx.cuh"
+#include "color.cuh"
 #include "sr_internal.h"
 #include "kernels.h"
 #include "launch.cuh"
@@ -30,15 +31,7 @@ void launch_pack_input(const uint8_t* lr, size_t npix, bf16* x, cudaStream_t st)
 }
 
 // ------------------------------------------------------------------ I420 <-> RGB (BT.601 studio swing, reading R21)
-// Integer conversion: C = Y - 16, D = U - 128, E = V - 128; R = (298 C + 409 E + 128) >> 8, G = (298 C - 100 D -
-// 208 E + 128) >> 8, B = (298 C + 516 D + 128) >> 8, clamped; chroma (y/2, x/2) is shared by its 2x2 block.
-__device__ __forceinline__ uint8_t clip8(int v) { return (uint8_t)min(max(v, 0), 255); }
-__device__ __forceinline__ void yuv_to_rgb(int Y, int U, int V, uint8_t* o) {
-  const int c = Y - 16, d = U - 128, e = V - 128;
-  o[0] = clip8((298 * c + 409 * e + 128) >> 8);
-  o[1] = clip8((298 * c - 100 * d - 208 * e + 128) >> 8);
-  o[2] = clip8((298 * c + 516 * d + 128) >> 8);
-}
+// yuv_to_rgb / clip8: color.cuh (shared with the fused I420 head conv)
 
 // one thread per pixel: planes y [n][h][w], u/v [n][h/2][w/2] -> rgb [n][h][w][3]
 __global__ void k_i420_to_rgb(const uint8_t* __restrict__ y, const uint8_t* __restrict__ u,

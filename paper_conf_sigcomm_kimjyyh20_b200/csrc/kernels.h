@@ -61,6 +61,12 @@ cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const 
 bool roll_head_u8_supported(int coutp, int W, const void* lr);
 cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* wfold, const float* bias, bf16* out,
                                      int N, int H, int W, cudaStream_t st, int w_early);
+// head conv straight from an I420 frame (Y rows by TMA, U / V read directly, BT.601 integer conversion fused into the
+// u8 expansion; also writes the frame's RGB copy rgb_out for the tail); needs W % 32 == 0, even H, 16-B aligned planes
+bool roll_head_yuv_supported(int coutp, int W, const void* y, const void* u, const void* v);
+cudaError_t launch_conv_roll_head_yuv(int coutp, const uint8_t* y, const uint8_t* u, const uint8_t* v,
+                                      uint8_t* rgb_out, const bf16* wfold, const float* bias, bf16* out, int N, int H,
+                                      int W, cudaStream_t st, int w_early);
 // rolling up conv + training tail (loss partial into *loss_sum, dy rows; vsep > 0: virtual patch batch)
 cudaError_t launch_conv_roll_tail_train(int cinp, int coutp, int s, const void* in, const bf16* wfold,
                                         const float* bias, const uint8_t* lr, const uint8_t* hr_ref, bf16* dy,

@@ -411,15 +411,31 @@ static sr_status ensure_infer_ws(sr_ctx* ctx, InferWS& ws, size_t pix) {
 
 // Inference forward (reading R1): x = v/255; f0 = head(x); f <- f + conv2(relu(conv1(f))) x B;
 // g = f0 + body(f); tail(up(g)) -> u8 with pixel shuffle + bilinear skip + clamp + RNE.
+struct YuvIn {  // an I420 LR frame batch: planes y [n][h][w], u / v [n][h/2][w/2]
+  const uint8_t *y, *u, *v;
+};
+
+// yuv (optional): the LR frames arrive as I420; the head conv converts them itself (the I420 -> RGB conversion fused
+// into its u8 expansion) and writes the RGB copy into `lr` (a ctx buffer) for the tail's skip.
 static sr_status forward_infer(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
-                               uint8_t* hr, int row0, int row1, cudaStream_t st) {
+                               uint8_t* hr, int row0, int row1, cudaStream_t st, const YuvIn* yuv = nullptr) {
   if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const size_t pix = (size_t)n * h * w;
   TRY(ensure_infer_ws(ctx, ws, pix));
   const int Cp = ctx->Cp;
   auto W = [&](int ci) { return sn.wf + ctx->convs[ci].pk_off; };
   auto Bv = [&](int ci) { return sn.bias + ctx->convs[ci].b_off; };
-  if (ctx->fuse_head && roll_supported(16, Cp, w) && roll_head_u8_supported(Cp, w, lr)) {
+  if (yuv) {
+    if (ctx->timing) {
+      const double px = (double)n * h * w;
+      tmark_begin(ctx, "conv_roll_yuv_16x" + std::to_string(Cp), 2.0 * 9 * 16 * Cp * px, px * (1.5 + 3.0 + 2.0 * Cp), st);
+    }
+    cudaError_t e = launch_conv_roll_head_yuv(Cp, yuv->y, yuv->u, yuv->v, const_cast<uint8_t*>(lr),
+                                              sn.wo + ctx->convs[0].pk_off, Bv(0), ws.f0, n, h, w, st, 1);
+    tmark_end(ctx, st);
+    ctx->launches++;
+    if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("I420 head launch: ") + cudaGetErrorString(e));
+  } else if (ctx->fuse_head && roll_supported(16, Cp, w) && roll_head_u8_supported(Cp, w, lr)) {
     // head conv straight from the u8 frame (x = v/255 expanded in shared memory; no k_pack_input pass)
     if (ctx->timing) {
       const double px = (double)n * h * w;
@@ -1248,10 +1264,22 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
   const size_t lb = (size_t)n * h * w * 3, hb = lb * s * s;
   if (lb > ctx->yuv_lr_bytes) { CK(dalloc(&ctx->yuv_lr, lb)); ctx->yuv_lr_bytes = lb; }
   if (hb > ctx->yuv_hr_bytes) { CK(dalloc(&ctx->yuv_hr, hb)); ctx->yuv_hr_bytes = hb; }
-  launch_i420_to_rgb(y_dev, u_dev, v_dev, n, h, w, ctx->yuv_lr, st);
-  ctx->launches++;
-  CKL();
-  TRY(sr_infer(ctx, which, ctx->yuv_lr, n, h, w, ctx->yuv_hr, stream));
+  // wide frames: the I420 -> RGB conversion runs inside the head conv (which also leaves the RGB copy for the tail);
+  // otherwise (narrow / small-image batches, the bilinear model, set_fusion bit 6) a separate conversion pass
+  const bool fused = ctx->fuse_head && valid_model(which) && which != SR_BILINEAR &&
+                     !(use_virtual_infer(ctx, n, h, w) && ctx->virtual_train) && roll_supported(16, ctx->Cp, w) &&
+                     roll_head_yuv_supported(ctx->Cp, w, y_dev, u_dev, v_dev);
+  if (fused) {
+    const YuvIn yuv{y_dev, u_dev, v_dev};
+    CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
+    TRY(forward_infer(ctx, ctx->iws, ctx->snap[which], ctx->yuv_lr, n, h, w, ctx->yuv_hr, 0, h, st, &yuv));
+    TRY(note_infer(ctx, st));
+  } else {
+    launch_i420_to_rgb(y_dev, u_dev, v_dev, n, h, w, ctx->yuv_lr, st);
+    ctx->launches++;
+    CKL();
+    TRY(sr_infer(ctx, which, ctx->yuv_lr, n, h, w, ctx->yuv_hr, stream));
+  }
   launch_rgb_to_i420(ctx->yuv_hr, n, s * h, s * w, hy_dev, hu_dev, hv_dev, st);
   ctx->launches++;
   CKL();
