@@ -15,4 +15,14 @@ __device__ __forceinline__ void yuv_to_rgb(int Y, int U, int V, uint8_t* o) {
   o[2] = clip8((298 * c + 516 * d + 128) >> 8);
 }
 
+// RGB -> I420: Y per pixel; U / V from a 2x2 block's rounded mean colour (sums of the four R, G, B)
+__device__ __forceinline__ uint8_t rgb_to_y(int R, int G, int B) {
+  return (uint8_t)(((66 * R + 129 * G + 25 * B + 128) >> 8) + 16);
+}
+__device__ __forceinline__ void rgb_sums_to_uv(int sr, int sg, int sb, uint8_t& u, uint8_t& v) {
+  const int R = (sr + 2) >> 2, G = (sg + 2) >> 2, B = (sb + 2) >> 2;
+  u = (uint8_t)(((-38 * R - 74 * G + 112 * B + 128) >> 8) + 128);
+  v = (uint8_t)(((112 * R - 94 * G - 18 * B + 128) >> 8) + 128);
+}
+
 }  // namespace sr

@@ -28,6 +28,7 @@
 #include "ring.cuh"
 #include "launch.cuh"
 #include "tail.cuh"
+#include "color.cuh"
 
 namespace sr {
 
@@ -70,6 +71,11 @@ struct BtArgs {
   int hr_row0, hr_row1;  // LR rows whose HR rows are written (strip mode)
   int bicubic;
   long long* dbg;  // benchmarking only: CTA-0 clock64 stamps [event][row]
+  // I420 output (k_bodytail<..., YO = true>, S = 2 or 4: a lane's S x S HR block holds whole 2x2 chroma blocks):
+  // planes hy [N][sH][sW], hu / hv [N][sH/2][sW/2] instead of the RGB frame hr
+  uint8_t* hy;
+  uint8_t* hu;
+  uint8_t* hv;
 };
 #define SR_BDBG(ev, idx) \
   if (a.dbg && blockIdx.x == 0 && (idx) >= 0 && (idx) < 256) a.dbg[(ev) * 256 + (idx)] = clock64();
@@ -78,7 +84,7 @@ struct BtArgs {
 // (k_bodytail<48,32,3> -3.4% with the bicubic code compiled out, scripts/bt_time.py A/B).  The kernel is very
 // sensitive to code shape: compiling the (null-checked) clock64 stamps out made it 10% slower, a runtime
 // experiment mask 13% slower -- measure every change to it.
-template <int C, int CO2, int S, bool BIC>
+template <int C, int CO2, int S, bool BIC, bool YO = false>
 __global__ void __launch_bounds__(kBtThreads, 1)
 k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_lr,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const BtArgs a) {
@@ -374,6 +380,76 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       mbar_wait(&l_full[ls], lph);
       if (tid == 0) { SR_BDBG(14, q + 1) }
       uint8_t* stg = sO + (grp * kBtNO + os) * OUTB;
+      if constexpr (YO) {  // I420 out: Y rows (S), U and V rows (S/2 each) staged like the RGB rows, then copied out
+        static_assert(S % 2 == 0, "I420 output: whole 2x2 chroma blocks per lane");
+        constexpr uint32_t HRPY = ((kBtTW * S + 15u) & ~15u) + 16u, HRPC = ((kBtTW * S / 2 + 15u) & ~15u) + 16u;
+        static_assert(S * HRPY + S * HRPC <= OUTB, "I420 staging fits the RGB staging slot");
+        uint8_t* const stgY = stg;
+        uint8_t* const stgU = stg + S * HRPY;
+        uint8_t* const stgV = stgU + (S / 2) * HRPC;
+        const size_t sWc = (size_t)sW / 2, sHc = (size_t)sH / 2;
+        uint8_t* const yrow0 = a.hy + ((size_t)n * sH + (size_t)S * r) * sW + (size_t)S * x0;
+        uint8_t* const urow0 = a.hu + ((size_t)n * sHc + (size_t)(S / 2) * r) * sWc + (size_t)(S / 2) * x0;
+        uint8_t* const vrow0 = a.hv + ((size_t)n * sHc + (size_t)(S / 2) * r) * sWc + (size_t)(S / 2) * x0;
+        if (lane_ok) {
+          uint8_t o[S * S * 3];
+          tail_u8_px<S>(smem_u32(sL + ls * kBtLrSlot) - (uint32_t)lbase + 0u, 16 * kBtLrChunks, 0, r, xc, H, W, v,
+                        BIC ? 1 : 0, o);
+#pragma unroll
+          for (int i = 0; i < S; ++i) {
+            const uint32_t sh = (uint32_t)(reinterpret_cast<uintptr_t>(yrow0 + (size_t)i * sW) & 15);
+            const uint32_t dst = smem_u32(stgY + i * HRPY) + sh + S * m;
+#pragma unroll
+            for (int j = 0; j < S; ++j)
+              sts_u8(dst + j, rgb_to_y(o[i * 3 * S + 3 * j], o[i * 3 * S + 3 * j + 1], o[i * 3 * S + 3 * j + 2]));
+          }
+#pragma unroll
+          for (int bi = 0; bi < S / 2; ++bi) {
+            const uint32_t shu = (uint32_t)(reinterpret_cast<uintptr_t>(urow0 + (size_t)bi * sWc) & 15);
+            const uint32_t shv = (uint32_t)(reinterpret_cast<uintptr_t>(vrow0 + (size_t)bi * sWc) & 15);
+#pragma unroll
+            for (int bj = 0; bj < S / 2; ++bj) {
+              int sr = 0, sg = 0, sb = 0;
+#pragma unroll
+              for (int dy = 0; dy < 2; ++dy)
+#pragma unroll
+                for (int dx = 0; dx < 2; ++dx) {
+                  const int k = (2 * bi + dy) * 3 * S + 3 * (2 * bj + dx);
+                  sr += o[k]; sg += o[k + 1]; sb += o[k + 2];
+                }
+              uint8_t uu, vv;
+              rgb_sums_to_uv(sr, sg, sb, uu, vv);
+              sts_u8(smem_u32(stgU + bi * HRPC) + shu + (S / 2) * m + bj, uu);
+              sts_u8(smem_u32(stgV + bi * HRPC) + shv + (S / 2) * m + bj, vv);
+            }
+          }
+        }
+        named_bar_sync(2 + grp, 128);  // staging complete (and the LR slot read by every lane of the group)
+        if (tid == 0) mbar_arrive(&l_empty[ls]);
+        if (r >= a.hr_row0 && r < a.hr_row1) {
+          const int npx = min(kBtTW, W - x0);
+          auto copy_row = [&](uint8_t* d, const uint8_t* srow, int nb) {  // 16-B stores, ragged ends bytewise
+            const int sh = (int)(reinterpret_cast<uintptr_t>(d) & 15);
+            const uint8_t* src = srow + sh;
+            const int pre = min((16 - sh) & 15, nb);
+            const int nch = (nb - pre) >> 4;
+            const int post = nb - pre - 16 * nch;
+            for (int k = tid; k < nch; k += 128)
+              *reinterpret_cast<uint4*>(d + pre + 16 * k) = *reinterpret_cast<const uint4*>(src + pre + 16 * k);
+            if (tid < pre) d[tid] = src[tid];
+            else if (tid >= 32 && tid < 32 + post) d[pre + 16 * nch + tid - 32] = src[pre + 16 * nch + tid - 32];
+          };
+#pragma unroll
+          for (int i = 0; i < S; ++i) copy_row(yrow0 + (size_t)i * sW, stgY + i * HRPY, npx * S);
+#pragma unroll
+          for (int bi = 0; bi < S / 2; ++bi) {
+            copy_row(urow0 + (size_t)bi * sWc, stgU + bi * HRPC, npx * S / 2);
+            copy_row(vrow0 + (size_t)bi * sWc, stgV + bi * HRPC, npx * S / 2);
+          }
+        }
+        os = os == kBtNO - 1 ? 0 : os + 1;
+        continue;
+      }
       uint8_t* hrow0 = a.hr + (((size_t)n * sH + (size_t)S * r) * sW + (size_t)S * x0) * 3;
       if (lane_ok) {
         uint8_t o[S * S * 3];
@@ -417,13 +493,13 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-template <int C, int CO2, int S, bool BIC>
+template <int C, int CO2, int S, bool BIC, bool YO = false>
 static cudaError_t launch_bt_t(const CUtensorMap& tf, const CUtensorMap& tl, const bf16* w1, const bf16* w2,
                                const BtArgs& a, int grid, cudaStream_t st) {
-  if constexpr (!BtCfg<C, CO2, S>::FITS) {
+  if constexpr (!BtCfg<C, CO2, S>::FITS || (YO && S % 2 != 0)) {
     return cudaErrorNotSupported;
   } else {
-    auto kern = k_bodytail<C, CO2, S, BIC>;
+    auto kern = k_bodytail<C, CO2, S, BIC, YO>;
     static bool configured = false;
     if (!configured) {
       cudaError_t e =
@@ -454,14 +530,25 @@ bool bodytail_supported(int cp, int s, int W, const void* lr, const void* hr) {
 
 cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const bf16* w1fold, const bf16* w2fold,
                             const float* b1, const float* b2, const uint8_t* lr, uint8_t* hr, int hr_row0,
-                            int hr_row1, int bicubic, int N, int H, int W, cudaStream_t st, long long* dbg) {
+                            int hr_row1, int bicubic, int N, int H, int W, cudaStream_t st, long long* dbg,
+                            uint8_t* hy, uint8_t* hu, uint8_t* hv) {
   CUtensorMap tf, tl;
   if (make_act_tmap(&tf, f, N, H, W, cp, 130, 1, cp / 8, CHUNK_ROW_PIX) != CUDA_SUCCESS) return cudaErrorInvalidValue;
   if (make_u8_rows_tmap(&tl, lr, N, H, 3LL * W, kBtLrChunks, 5) != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  BtArgs a{b1, b2, f0, lr, hr, N, H, W, hr_row0, hr_row1, bicubic, dbg};
+  BtArgs a{b1, b2, f0, lr, hr, N, H, W, hr_row0, hr_row1, bicubic, dbg, hy, hu, hv};
   const long long rows = (long long)N * ((W + kBtTW - 1) / kBtTW) * H;
   int grid = num_sms();
   if (rows < grid) grid = (int)rows;
+  if (hy) {  // I420 output (s = 2, 4)
+    if (!hu || !hv || s == 3) return cudaErrorNotSupported;
+#define SR_BT_YO(C, S) \
+    if (cp == C && s == S)                                                                                      \
+      return bicubic ? launch_bt_t<C, (S == 2 ? 16 : 48), S, true, true>(tf, tl, w1fold, w2fold, a, grid, st)   \
+                     : launch_bt_t<C, (S == 2 ? 16 : 48), S, false, true>(tf, tl, w1fold, w2fold, a, grid, st);
+    SR_BT_YO(16, 2) SR_BT_YO(16, 4) SR_BT_YO(32, 2) SR_BT_YO(32, 4) SR_BT_YO(48, 2) SR_BT_YO(48, 4)
+#undef SR_BT_YO
+    return cudaErrorNotSupported;
+  }
 #define SR_BT_CASE(C, S) \
   if (cp == C && s == S)                                                                                   \
     return bicubic ? launch_bt_t<C, (S == 2 ? 16 : (S == 3 ? 32 : 48)), S, true>(tf, tl, w1fold, w2fold, a, grid, st) \

@@ -63,12 +63,10 @@ __global__ void k_rgb_to_i420(const uint8_t* __restrict__ rgb, int n, int h, int
     for (int dx = 0; dx < 2; ++dx) {
       const size_t p = ((size_t)f * h + 2 * by + dy) * w + 2 * bx + dx;
       const int R = rgb[p * 3], G = rgb[p * 3 + 1], B = rgb[p * 3 + 2];
-      y[p] = (uint8_t)(((66 * R + 129 * G + 25 * B + 128) >> 8) + 16);
+      y[p] = rgb_to_y(R, G, B);
       sr += R; sg += G; sb += B;
     }
-  const int R = (sr + 2) >> 2, G = (sg + 2) >> 2, B = (sb + 2) >> 2;
-  u[i] = (uint8_t)(((-38 * R - 74 * G + 112 * B + 128) >> 8) + 128);
-  v[i] = (uint8_t)(((112 * R - 94 * G - 18 * B + 128) >> 8) + 128);
+  rgb_sums_to_uv(sr, sg, sb, u[i], v[i]);
 }
 
 // LR counterparts of arriving HR patches (§5.2): pp x pp RGB crops of decoded frame 0 at LR top-left

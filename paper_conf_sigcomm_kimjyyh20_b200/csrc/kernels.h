@@ -56,7 +56,8 @@ void set_block_gen(int g);  // benchmarking only
 cudaError_t launch_bodytail(int cp, int s, const bf16* f, const bf16* f0, const bf16* w1fold, const bf16* w2fold,
                             const float* b1, const float* b2, const uint8_t* lr, uint8_t* hr, int hr_row0,
                             int hr_row1, int bicubic, int N, int H, int W, cudaStream_t st,
-                            long long* dbg = nullptr);
+                            long long* dbg = nullptr, uint8_t* hy = nullptr, uint8_t* hu = nullptr,
+                            uint8_t* hv = nullptr);
 // head conv straight from the u8 frame (k_pack_input fused in); needs W % 16 == 0 and a 16-B aligned frame
 bool roll_head_u8_supported(int coutp, int W, const void* lr);
 cudaError_t launch_conv_roll_head_u8(int coutp, const uint8_t* lr, const bf16* wfold, const float* bias, bf16* out,

@@ -414,11 +414,18 @@ static sr_status ensure_infer_ws(sr_ctx* ctx, InferWS& ws, size_t pix) {
 struct YuvIn {  // an I420 LR frame batch: planes y [n][h][w], u / v [n][h/2][w/2]
   const uint8_t *y, *u, *v;
 };
+struct YuvOut {  // the I420 HR output planes: y [n][sh][sw], u / v [n][sh/2][sw/2]
+  uint8_t *y, *u, *v;
+};
 
 // yuv (optional): the LR frames arrive as I420; the head conv converts them itself (the I420 -> RGB conversion fused
 // into its u8 expansion) and writes the RGB copy into `lr` (a ctx buffer) for the tail's skip.
+// yo (optional, s = 2 or 4): the fused body + tail kernel writes the HR frames as I420 planes instead of RGB into hr
+// (a lane's s x s HR block holds whole 2x2 chroma blocks); *yo_done says whether it did (else hr holds RGB).
 static sr_status forward_infer(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, const uint8_t* lr, int n, int h, int w,
-                               uint8_t* hr, int row0, int row1, cudaStream_t st, const YuvIn* yuv = nullptr) {
+                               uint8_t* hr, int row0, int row1, cudaStream_t st, const YuvIn* yuv = nullptr,
+                               const YuvOut* yo = nullptr, bool* yo_done = nullptr) {
+  if (yo_done) *yo_done = false;
   if (&sn == &ctx->snap[SR_TRAIN]) TRY(ensure_full_train_pack(ctx, st));
   const size_t pix = (size_t)n * h * w;
   TRY(ensure_infer_ws(ctx, ws, pix));
@@ -498,12 +505,15 @@ static sr_status forward_infer(sr_ctx* ctx, InferWS& ws, const Snapshot& sn, con
       tmark_begin(ctx, "bodytail_" + std::to_string(Cp) + "x" + std::to_string(ctx->OUTP),
                   2.0 * 9 * Cp * (Cp + ctx->OUTP) * px, px * (4.0 * Cp + 3.0 * (1 + ctx->s * ctx->s)), st);
     }
+    const bool i420 = yo && ctx->s % 2 == 0;
     cudaError_t e = launch_bodytail(Cp, ctx->s, cur, ws.f0, sn.wo + ctx->convs[cb].pk_off,
                                     sn.wo + ctx->convs[cu].pk_off, Bv(cb), Bv(cu), lr, hr, row0, row1,
-                                    ctx->opt.skip == 1, n, h, w, st);
+                                    ctx->opt.skip == 1, n, h, w, st, nullptr, i420 ? yo->y : nullptr,
+                                    i420 ? yo->u : nullptr, i420 ? yo->v : nullptr);
     tmark_end(ctx, st);
     ctx->launches++;
     if (e != cudaSuccess) return fail(ctx, SR_E_CUDA, std::string("bodytail launch: ") + cudaGetErrorString(e));
+    if (yo_done) *yo_done = i420;
     return SR_OK;
   }
   bf16* gbuf = (cur == ws.fa) ? ws.fb : ws.fa;
@@ -1264,15 +1274,24 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
   const size_t lb = (size_t)n * h * w * 3, hb = lb * s * s;
   if (lb > ctx->yuv_lr_bytes) { CK(dalloc(&ctx->yuv_lr, lb)); ctx->yuv_lr_bytes = lb; }
   if (hb > ctx->yuv_hr_bytes) { CK(dalloc(&ctx->yuv_hr, hb)); ctx->yuv_hr_bytes = hb; }
-  // wide frames: the I420 -> RGB conversion runs inside the head conv (which also leaves the RGB copy for the tail);
-  // otherwise (narrow / small-image batches, the bilinear model, set_fusion bit 6) a separate conversion pass
-  const bool fused = ctx->fuse_head && valid_model(which) && which != SR_BILINEAR &&
-                     !(use_virtual_infer(ctx, n, h, w) && ctx->virtual_train) && roll_supported(16, ctx->Cp, w) &&
-                     roll_head_yuv_supported(ctx->Cp, w, y_dev, u_dev, v_dev);
-  if (fused) {
-    const YuvIn yuv{y_dev, u_dev, v_dev};
+  // Frames on the rolling / fused path (a DNN model, not a small-image batch): the I420 -> RGB conversion runs inside
+  // the head conv when it can (W % 32 == 0; it also leaves the RGB copy for the tail) and, at s = 2 / 4, the fused
+  // body + tail kernel writes the I420 planes itself; whatever is not fused runs as a separate conversion pass.
+  const bool direct = valid_model(which) && which != SR_BILINEAR && !(use_virtual_infer(ctx, n, h, w) && ctx->virtual_train);
+  bool yo_done = false;
+  if (direct) {
+    const bool fused_in = ctx->fuse_head && roll_supported(16, ctx->Cp, w) &&
+                          roll_head_yuv_supported(ctx->Cp, w, y_dev, u_dev, v_dev);
+    if (!fused_in) {
+      launch_i420_to_rgb(y_dev, u_dev, v_dev, n, h, w, ctx->yuv_lr, st);
+      ctx->launches++;
+      CKL();
+    }
+    const YuvIn yin{y_dev, u_dev, v_dev};
+    const YuvOut yout{hy_dev, hu_dev, hv_dev};
     CK(cudaStreamWaitEvent(st, ctx->publish_ev, 0));
-    TRY(forward_infer(ctx, ctx->iws, ctx->snap[which], ctx->yuv_lr, n, h, w, ctx->yuv_hr, 0, h, st, &yuv));
+    TRY(forward_infer(ctx, ctx->iws, ctx->snap[which], ctx->yuv_lr, n, h, w, ctx->yuv_hr, 0, h, st,
+                      fused_in ? &yin : nullptr, &yout, &yo_done));
     TRY(note_infer(ctx, st));
   } else {
     launch_i420_to_rgb(y_dev, u_dev, v_dev, n, h, w, ctx->yuv_lr, st);
@@ -1280,9 +1299,11 @@ sr_status sr_infer_i420(sr_ctx* ctx, sr_model which, const uint8_t* y_dev, const
     CKL();
     TRY(sr_infer(ctx, which, ctx->yuv_lr, n, h, w, ctx->yuv_hr, stream));
   }
-  launch_rgb_to_i420(ctx->yuv_hr, n, s * h, s * w, hy_dev, hu_dev, hv_dev, st);
-  ctx->launches++;
-  CKL();
+  if (!yo_done) {
+    launch_rgb_to_i420(ctx->yuv_hr, n, s * h, s * w, hy_dev, hu_dev, hv_dev, st);
+    ctx->launches++;
+    CKL();
+  }
   return SR_OK;
 }
 

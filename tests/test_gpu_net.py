@@ -380,12 +380,13 @@ def test_i420_dnn_path(cfg, hw):
 
 
 @pytest.mark.parametrize("cfg,hw,n", [((3, 8, 48), (90, 160), 2), ((2, 2, 32), (38, 224), 3), ((4, 2, 16), (20, 96), 1),
-                                      ((2, 8, 48), (66, 320), 1)])
-def test_i420_fused_head_equals_separate_pass(cfg, hw, n):
-    """Wide frames (W % 32 == 0): the I420 -> RGB conversion fused into the head conv's u8 expansion (Y rows by TMA,
-    U / V read directly, the RGB copy for the tail written by the head) against the separate conversion pass
-    (set_fusion bit 6: conversion pass, then k_pack_input + head): bit-identical planes, two launches fewer; ragged
-    strips (224 = 128 + 96) included."""
+                                      ((2, 8, 48), (66, 320), 1), ((4, 1, 48), (18, 352), 2)])
+def test_i420_fused_boundary_equals_separate_passes(cfg, hw, n):
+    """The I420 boundary fused into the path (wide frames): I420 -> RGB inside the head conv's u8 expansion (W % 32
+    == 0), and at x2 / x4 RGB -> I420 inside the fused body + tail kernel's staged store (a lane's s x s HR block holds
+    whole 2x2 chroma blocks; x3 keeps the conversion pass) -- against the separate conversion passes around the RGB
+    path (set_fusion bits 6 and 5: conversion, k_pack_input + head, ..., body conv + rolling tail, conversion):
+    bit-identical planes with fewer launches; ragged strips (224 = 128 + 96, 352 = 2 x 126 + 100) included."""
     s, B, C = cfg
     ctx = _ctx(s, B, C, seed=9)
     y, u, v = _i420_frames(n, hw[0], hw[1], seed=43)
@@ -393,13 +394,13 @@ def test_i420_fused_head_equals_separate_pass(cfg, hw, n):
     l0 = ctx.launches
     a = [t.clone() for t in ctx.infer_i420(*planes)]
     l1 = ctx.launches
-    ctx.set_fusion(1 | 64)
+    ctx.set_fusion(1 | 64 | 32)
     b = ctx.infer_i420(*planes)
     l2 = ctx.launches
     torch.cuda.synchronize()
     for ga, gb in zip(a, b):
         assert torch.equal(ga, gb)
-    assert (l1 - l0) + 2 == (l2 - l1)  # separate: k_i420_to_rgb + k_pack_input + head; fused: the head alone
+    assert (l1 - l0) + 2 <= (l2 - l1)
 
 
 def test_pool_push_i420_crops_the_decoded_frame():
