@@ -46,14 +46,25 @@ RING = 3
 class Stream:
     """One ingest stream: its own SR context (per-stream DNN), frame rings and patch pool."""
 
-    def __init__(self, k, torch, SRContext, synth_frames, synth_patch_pool, dev):
+    def __init__(self, k, torch, SRContext, synth_frames, synth_patch_pool, dev, i420=False):
         self.k = k
+        self.i420 = i420
         self.ctx = SRContext(S5, B5, C5, seed=k)
         lr = synth_frames(RING, H5, W5, seed=5000 + k)
-        self.host_lr = torch.from_numpy(lr).pin_memory()
-        self.lr_dev = torch.empty((RING, H5, W5, 3), dtype=torch.uint8, device=dev)
-        self.hr_dev = torch.empty((RING, S5 * H5, S5 * W5, 3), dtype=torch.uint8, device=dev)
-        self.host_hr = torch.empty((RING, S5 * H5, S5 * W5, 3), dtype=torch.uint8).pin_memory()
+        if i420:
+            # what WebRTC hands the server: planar I420 (Y [h,w], U/V [h/2,w/2]); synthetic planes taken from the
+            # synthetic frame's channels (input synthesis only, not the library's colour conversion)
+            planes = (lr[..., 0], lr[:, ::2, ::2, 1], lr[:, ::2, ::2, 2])
+            self.host_lr = [torch.from_numpy(p.copy()).pin_memory() for p in planes]
+            self.lr_dev = [torch.empty(p.shape, dtype=torch.uint8, device=dev) for p in planes]
+            hr_shapes = ((RING, S5 * H5, S5 * W5), (RING, S5 * H5 // 2, S5 * W5 // 2), (RING, S5 * H5 // 2, S5 * W5 // 2))
+            self.hr_dev = [torch.empty(sh, dtype=torch.uint8, device=dev) for sh in hr_shapes]
+            self.host_hr = [torch.empty(sh, dtype=torch.uint8).pin_memory() for sh in hr_shapes]
+        else:
+            self.host_lr = [torch.from_numpy(lr).pin_memory()]
+            self.lr_dev = [torch.empty((RING, H5, W5, 3), dtype=torch.uint8, device=dev)]
+            self.hr_dev = [torch.empty((RING, S5 * H5, S5 * W5, 3), dtype=torch.uint8, device=dev)]
+            self.host_hr = [torch.empty((RING, S5 * H5, S5 * W5, 3), dtype=torch.uint8).pin_memory()]
         plr, phr, _ = synth_patch_pool(256, S5, S5 * POOL_LR, seed=6000 + k, frame_hw=(1080, 1920))
         alr, ahr, _ = synth_patch_pool(60, S5, S5 * POOL_LR, seed=7000 + k, frame_hw=(1080, 1920))
         self.ctx.pool_push(torch.from_numpy(plr).to(dev), torch.from_numpy(phr).to(dev))
@@ -66,6 +77,23 @@ class Stream:
         self.iters = 0
         self.arrivals = 0
 
+    # one frame: host -> device (slot), super-resolution (sr_infer, or sr_infer_i420 with the fused I420 boundary),
+    # device -> host
+    def h2d(self, slot, i):
+        for d, h in zip(self.lr_dev, self.host_lr):
+            d[slot].copy_(h[i % RING], non_blocking=True)
+
+    def sr(self, slot):
+        if self.i420:
+            self.ctx.infer_i420(*(d[slot:slot + 1] for d in self.lr_dev), "serve",
+                                out=tuple(d[slot:slot + 1] for d in self.hr_dev))
+        else:
+            self.ctx.infer(self.lr_dev[0][slot:slot + 1], "serve", out=self.hr_dev[0][slot:slot + 1])
+
+    def d2h(self, slot):
+        for h, d in zip(self.host_hr, self.hr_dev):
+            h[slot].copy_(d[slot], non_blocking=True)
+
 
 def run(argv=None):
     ap = argparse.ArgumentParser()
@@ -73,6 +101,7 @@ def run(argv=None):
     ap.add_argument("--seconds", type=float, default=6.0, help="paced video seconds per S (>= 5: one epoch end)")
     ap.add_argument("--warm-seconds", type=float, default=1.0)
     ap.add_argument("--no-train", action="store_true")
+    ap.add_argument("--i420", action="store_true", help="frames in and out as planar I420 (sr_infer_i420)")
     args, _ = ap.parse_known_args(argv)
 
     import numpy as np
@@ -90,9 +119,9 @@ def run(argv=None):
 
     def get_streams(n):
         while len(streams) < n:
-            st = Stream(len(streams), torch, SRContext, synth_frames, synth_patch_pool, dev)
+            st = Stream(len(streams), torch, SRContext, synth_frames, synth_patch_pool, dev, i420=args.i420)
             with torch.cuda.stream(hi):   # warm the inference path (workspace, kernels)
-                st.ctx.infer(st.lr_dev[:1], "serve", out=st.hr_dev[:1])
+                st.sr(0)
             with torch.cuda.stream(lo):   # warm + capture the training iteration; warm the epoch-end path (its
                 st.ctx.train_sampled(2, BATCH, PATCH, st.loss)  # workspaces are allocated here, not in the window)
                 st.ctx.publish()
@@ -108,9 +137,9 @@ def run(argv=None):
     for i in range(40):
         t0 = time.perf_counter()
         with torch.cuda.stream(hi):
-            s0.lr_dev[0].copy_(s0.host_lr[i % RING], non_blocking=True)
-            s0.ctx.infer(s0.lr_dev[:1], "serve", out=s0.hr_dev[:1])
-            s0.host_hr[0].copy_(s0.hr_dev[0], non_blocking=True)
+            s0.h2d(0, i)
+            s0.sr(0)
+            s0.d2h(0)
         hi.synchronize()
         if i >= 10:
             delays.append((time.perf_counter() - t0) * 1e3)
@@ -139,7 +168,10 @@ def run(argv=None):
                                "(x2, 8x48), H2D + sr_infer (high-priority stream) + D2H per frame; per-stream "
                                "training 10 it/s (batch 64, 48x48) + 3 patch arrivals/s + publish and Algorithm-1 "
                                "evaluation every 50 iterations (low-priority stream)",
-                   "seconds_per_point": args.seconds, "train": not args.no_train},
+                   "seconds_per_point": args.seconds, "train": not args.no_train,
+                   "frames": ("planar I420 in and out (sr_infer_i420: I420 -> RGB inside the head conv, RGB -> I420 "
+                              "inside the body + tail store; 3.1 MB in / 12.4 MB out per frame)") if args.i420
+                   else "RGB u8 in and out (6.2 MB in / 24.9 MB out per frame)"},
         "single_frame_delay": single,
         "sweep": sweep,
         "tflops_per_stream": round(FPS * H5 * W5 * FLOP_PER_LR_PX / 1e12, 2),
@@ -236,17 +268,17 @@ def paced_run(ss, n, args, torch, np, hi, lo, h2d, d2h, Controller):
         with torch.cuda.stream(h2d):
             if st.slot_done[slot] is not None:
                 h2d.wait_event(st.slot_done[slot])   # the slot's previous frame has left the device
-            st.lr_dev[slot].copy_(st.host_lr[i % RING], non_blocking=True)
+            st.h2d(slot, i)
             e_in = torch.cuda.Event(enable_timing=True)
             e_in.record()
         hi.wait_event(e_in)
         with torch.cuda.stream(hi):
-            st.ctx.infer(st.lr_dev[slot:slot + 1], "serve", out=st.hr_dev[slot:slot + 1])
+            st.sr(slot)
             e_sr = torch.cuda.Event(enable_timing=True)
             e_sr.record()
         d2h.wait_event(e_sr)
         with torch.cuda.stream(d2h):
-            st.host_hr[slot].copy_(st.hr_dev[slot], non_blocking=True)
+            st.d2h(slot)
             e_out = torch.cuda.Event(enable_timing=True)
             e_out.record()
         st.slot_done[slot] = e_out
