@@ -833,7 +833,7 @@ struct ChainParams {
   int nph;      // 0: each CTA takes a contiguous (strip, row) range (<= 4 pieces); 1, 2: pieces from pc[cta][0..nph)
   ChainPiece pc[kChainMaxCta][2];
   unsigned* sync;
-  int dbg_cta;
+  int dbg_cta;              // benchmarking only: the CTA whose per-row stamps are kept (SR_CHAIN_DBG_CTA)
   unsigned long long* dbg;  // benchmarking only: per (CTA, layer) globaltimer stamps [8] (sr_test_chain_dbg)
 };
 #define SR_RDBG2(l, i, k) \
@@ -931,9 +931,6 @@ __global__ void __launch_bounds__(kChainThreads, 1) k_conv_chain(const __grid_co
       pcol[npc] = col; py0[npc] = y0; py1[npc] = y1; ++npc;
     }
   }
-  uint32_t rows_mine = 0;
-  for (int k = 0; k < npc; ++k) rows_mine += py1[k] - py0[k];
-  (void)rows_mine;
 #define SR_PIECE_BEGIN                                                                \
   for (int pi = 0; pi < npc; ++pi) {                                                  \
     const int col = pcol[pi], y0 = py0[pi], y1 = py1[pi];                             \
