@@ -33,11 +33,15 @@
 
 namespace sr {
 
-static constexpr int kB2Threads = 352;  // warps: 0 producer, 1 conv1 issuer, 2..5 conv1 epi, 6..9 conv2 epi, 10 conv2 issuer
+// warps: 0 producer, 1 conv1 issuer, 2..5 conv1 epi, 6..9 conv2 epi (group 0), 10 conv2 issuer, at C <= 32 also
+// 11..14 conv2 epi (group 1): the conv2 epilogue groups take alternate output rows
+static constexpr int kB2Threads = 352;
 static constexpr int kB2TW = 126;
 
 template <int C>
 struct B2Cfg {
+  static constexpr int EPI2 = C <= 32 ? 2 : 1;  // conv2 epilogue groups (rows alternate between them)
+  static constexpr int THREADS = kB2Threads + (EPI2 - 1) * 128;
   static constexpr int CCH = C / 8, KS = C / 16, N = 3 * C;
   static constexpr int RB = (256 / C) < 8 ? (256 / C) : 8;
   static constexpr int NF = C >= 48 ? 3 : 4;  // f-row ring (one slot less than k_resblock at C = 48: weights grew)
@@ -57,7 +61,7 @@ struct B2Cfg {
   static constexpr uint32_t OUTB = ((kB2TW * C * 2) + 1023u) & ~1023u;
   static constexpr uint32_t ARMB = ((kArmOnesBytes + 2 * (C / 2) * 32) + 127u) & ~127u;  // ones + 2 half bias tiles
   static constexpr size_t SMEM = 1024 + 2 * (size_t)WB_AL + (size_t)NF * ROWB + (size_t)NT * ROWB +
-                                 (size_t)NO * OUTB + ARMB;
+                                 (size_t)EPI2 * NO * OUTB + ARMB;
 };
 
 // Bias-arming B tile of this CTA's half of the N = C columns: rows n < C/2 hold bias[half + n] split into three bf16
@@ -110,7 +114,7 @@ __device__ __forceinline__ void ring_mma_step2(uint32_t ring_base, unsigned g, u
 }
 
 template <int C>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kB2Threads, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(B2Cfg<C>::THREADS, 1)
 k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_out,
             const bf16* __restrict__ w1, const bf16* __restrict__ w2, const float* __restrict__ b1,
             const float* __restrict__ b2, const bf16* __restrict__ fres, const int N, const int H, const int W) {
@@ -125,7 +129,7 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
   uint8_t* sF = sW2 + Cfg::WB_AL;
   uint8_t* sT = sF + NF * ROWB;
   uint8_t* sO = sT + NT * ROWB;
-  uint8_t* sOnes = sO + NO * OUTB;
+  uint8_t* sOnes = sO + Cfg::EPI2 * NO * OUTB;
   uint8_t* sB1 = sOnes + kArmOnesBytes;
   uint8_t* sB2 = sB1 + (C / 2) * 32;
   __shared__ __align__(8) uint64_t f_full[NF], f_empty[NF], t_full[NT], t_empty[NT], r1_ready[RB], r1_free[RB],
@@ -350,46 +354,50 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       mbar_wait(&t_empty[ts], tph ^ 1);
       if (++ts == NT) { ts = 0; tph ^= 1; }
     }
-  } else if (warp < 10) {
+  } else if (warp < 10 || warp >= 11) {
     // ===================== conv2 epilogue (both CTAs): drain rows -> + residual f -> smem -> TMA store ==========
+    // (EPI2 groups: group grp takes the output rows with g % EPI2 == grp, its own staging slots and named barrier)
+    constexpr int EPI2 = Cfg::EPI2;
+    const int grp = warp >= 11 ? 1 : 0;
     const int quarter = warp & 3;
     const int m = quarter * 32 + lane_id();
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
-    const bool leader = (warp == 6 && lane_id() == 0);
-    for (int b = 0; b < RB; ++b)
-      if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
+    const bool leader = (warp == (grp ? 11 : 6) && lane_id() == 0);
+    if (grp == 0)
+      for (int b = 0; b < RB; ++b)
+        if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
     int os = 0;
     unsigned G = 0;
     SR_PIECE_BEGIN
     const bool lane_ok = m < kB2TW && x0 + m < W;
-    constexpr int kAhead = C <= 32 ? 2 : 1;
-    uint4 res_nx[C / 8], res_nx2[kAhead > 1 ? C / 8 : 1];
+    // the residual row of this group's next kept output row is loaded while the current one is processed
+    uint4 res_nx[C / 8];
     auto ld_res = [&](int q) {
       if (q >= 1 && q <= n_t - 2 && lane_ok) {
         const size_t pix = (((size_t)n * H + y0 - 1 + q) * W) + x0 + m;
         const uint4* rp = reinterpret_cast<const uint4*>(fres + pix * C);
 #pragma unroll
-        for (int j = 0; j < C / 8; ++j) (kAhead > 1 ? res_nx2 : res_nx)[j] = __ldg(rp + j);
+        for (int j = 0; j < C / 8; ++j) res_nx[j] = __ldg(rp + j);
       }
     };
-    ld_res(-1);
-    if constexpr (kAhead > 1) {
-#pragma unroll
-      for (int j = 0; j < C / 8; ++j) res_nx[j] = res_nx2[j];
-      ld_res(0);
+    auto own = [&](int q) { return (int)((G + q + 1) % EPI2) == grp; };
+    int qn = -1;  // this group's next row index
+    while (qn <= n_t && !own(qn)) ++qn;
+    {
+      int qf = qn;  // first kept row of the group
+      while (qf <= n_t && !(own(qf) && qf >= 1 && qf <= n_t - 2)) ++qf;
+      ld_res(qf);
     }
-    for (int q = -1; q <= n_t; ++q) {  // out rows of conv2 = output rows y0-1+q
+    for (int q = qn; q <= n_t; q += EPI2) {  // out rows of conv2 = output rows y0-1+q
       const unsigned g = G + q + 1;
       const bool emit = q >= 1 && q <= n_t - 2;
       const int r = y0 - 1 + q;
       uint4 res[C / 8];
+      if (emit) {
 #pragma unroll
-      for (int j = 0; j < C / 8; ++j) res[j] = res_nx[j];
-      if constexpr (kAhead > 1) {
-#pragma unroll
-        for (int j = 0; j < C / 8; ++j) res_nx[j] = res_nx2[j];
+        for (int j = 0; j < C / 8; ++j) res[j] = res_nx[j];
+        ld_res(q + EPI2);
       }
-      ld_res(q + kAhead);
       const int b = ring_idx<RB>(g);
       mbar_wait(&r2_ready[b], (uint32_t)(g / RB) & 1u);
       tc_fence_after();
@@ -401,8 +409,9 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
       __syncwarp();
       if (lane_id() == 0) mbar_arrive_remote(cluster_addr(&r2_free[b], 0));
       if (emit) {
+        uint8_t* const slot = sO + (grp * NO + os) * OUTB;
         if (lane_ok) {
-          uint8_t* orow = sO + os * OUTB + m * C * 2;
+          uint8_t* orow = slot + m * C * 2;
           uint4 ov[C / 8];
 #pragma unroll
           for (int j = 0; j < C / 8; ++j) {
@@ -424,9 +433,9 @@ k_resblock2(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CU
           st_pix_rot<C / 8>(orow, ov);
         }
         fence_proxy_async_smem();
-        named_bar_sync(2, 128);
+        named_bar_sync(2 + grp, 128);
         if (leader && !dummy) {
-          tma_store_4d(&tm_out, sO + os * OUTB, 0, x0, r, n);
+          tma_store_4d(&tm_out, slot, 0, x0, r, n);
           bulk_commit();
           bulk_wait_read<NO - 2>();
         } else if (leader) {
@@ -458,7 +467,7 @@ static cudaError_t launch_block2_t(const CUtensorMap& tf, const CUtensorMap& to,
     if (e != cudaSuccess) return e;
     configured = true;
   }
-  return launch_k(kern, dim3(grid), dim3(kB2Threads), B2Cfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, N, H, W);
+  return launch_k(kern, dim3(grid), dim3(B2Cfg<C>::THREADS), B2Cfg<C>::SMEM, st, tf, to, w1, w2, b1, b2, f, N, H, W);
 }
 
 // Offered for C = 32 (BASELINE config 2's 8 x 32 net), where a row-step's MMAs are short and the pair's halved B
