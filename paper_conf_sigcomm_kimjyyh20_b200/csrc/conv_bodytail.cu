@@ -33,6 +33,12 @@
 namespace sr {
 
 static constexpr int kBtThreads = 480;  // 15 warps: two tail epilogue groups
+// C <= 32: a second body-conv epilogue group (warps 15..18) on alternate g rows
+template <int C>
+struct BtThreads {
+  static constexpr int EPI1 = C <= 32 ? 2 : 1;
+  static constexpr int N = kBtThreads + (EPI1 - 1) * 128;
+};
 static constexpr int kBtTW = 126;  // output pixels per strip
 static constexpr int kBtNF = 4;    // f-row ring
 static constexpr int kBtNT = 4;    // g-row ring
@@ -85,7 +91,7 @@ struct BtArgs {
 // sensitive to code shape: compiling the (null-checked) clock64 stamps out made it 10% slower, a runtime
 // experiment mask 13% slower -- measure every change to it.
 template <int C, int CO2, int S, bool BIC, bool YO = false>
-__global__ void __launch_bounds__(kBtThreads, 1)
+__global__ void __launch_bounds__(BtThreads<C>::N, 1)
 k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUtensorMap tm_lr,
            const bf16* __restrict__ w1, const bf16* __restrict__ w2, const BtArgs a) {
   using Cfg = BtCfg<C, CO2, S>;
@@ -269,6 +275,87 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
       SR_PIECE_END
     }
     __syncwarp();
+  } else if (BtThreads<C>::EPI1 == 2 && (warp < 6 || warp >= 15)) {
+    // ============ conv1 epilogue, two groups (C <= 32): alternate g rows; g slots follow the emitted-row order ======
+    constexpr int EPI1 = BtThreads<C>::EPI1;
+    const int grp = warp >= 15 ? 1 : 0;
+    const int quarter = warp & 3;
+    const int m = quarter * 32 + lane_id();
+    const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+    if (grp == 0)
+      for (int b = 0; b < RB1; ++b)
+        if (lane_id() == 0) mbar_arrive(&r1_free[b]);
+    unsigned G = 0, E = 0;  // E: g rows emitted by both groups in earlier pieces
+    SR_PIECE_BEGIN
+    const int tcol = x0 - 1 + m;
+    const bool col_ok = tcol >= 0 && tcol < W;
+    uint4 res_nx[CCH];  // f0 row of this group's next kept row
+    auto ld_res = [&](int q) {
+      const int trow = y0 - 2 + q;
+      if (q >= 1 && q <= n_f - 2 && col_ok && trow >= 0 && trow < H) {
+        const uint4* rp = reinterpret_cast<const uint4*>(a.f0 + ((((size_t)n * H + trow) * W) + tcol) * C);
+#pragma unroll
+        for (int j = 0; j < CCH; ++j) res_nx[j] = __ldg(rp + j);
+      }
+    };
+    auto own = [&](int q) { return (int)((G + q + 1) % EPI1) == grp; };
+    int q0 = -1;
+    while (q0 <= n_f && !own(q0)) ++q0;
+    {
+      int qf = q0;
+      while (qf <= n_f && !(own(qf) && qf >= 1 && qf <= n_f - 2)) ++qf;
+      ld_res(qf);
+    }
+    for (int q = q0; q <= n_f; q += EPI1) {  // out rows of conv1 = g rows y0-2+q
+      const unsigned g = G + q + 1;
+      const bool emit = q >= 1 && q <= n_f - 2;
+      const int trow = y0 - 2 + q;
+      const bool ok = col_ok && trow >= 0 && trow < H;
+      uint4 res[CCH];
+      if (emit) {
+#pragma unroll
+        for (int j = 0; j < CCH; ++j) res[j] = res_nx[j];
+        ld_res(q + EPI1);
+      }
+      const unsigned ti = E + (unsigned)(q - 1);
+      const int ts = (int)(ti % kBtNT);
+      const uint32_t tph = (ti / kBtNT) & 1u;
+      if (emit) mbar_wait(&t_empty[ts], tph ^ 1);
+      const int b = ring_idx<RB1>(g);
+      mbar_wait(&r1_ready[b], (uint32_t)(g / RB1) & 1u);
+      tc_fence_after();
+      float v[C];
+      ring_load<C>(ring1 + lane_off + b * C, v);
+      tc_fence_before();
+      __syncwarp();
+      if (lane_id() == 0) mbar_arrive(&r1_free[b]);
+      if (emit) {
+        uint8_t* dst = sT + ts * ROWB + m * 16;
+#pragma unroll
+        for (int j = 0; j < CCH; ++j) {
+          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&res[j]);
+          float o[8];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 f2 = __bfloat1622float2(h2[e]);
+            o[2 * e] = ok ? v[8 * j + 2 * e] + f2.x : 0.f;
+            o[2 * e + 1] = ok ? v[8 * j + 2 * e + 1] + f2.y : 0.f;
+          }
+          uint4 u;
+          u.x = pack_bf16x2(o[0], o[1]);
+          u.y = pack_bf16x2(o[2], o[3]);
+          u.z = pack_bf16x2(o[4], o[5]);
+          u.w = pack_bf16x2(o[6], o[7]);
+          *reinterpret_cast<uint4*>(dst + j * PLANE) = u;
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane_id() == 0) mbar_arrive(&t_full[ts]);
+      }
+    }
+    G += n_f + 2;
+    E += n_f - 2;
+    SR_PIECE_END
   } else if (warp < 6) {
     // ============ conv1 epilogue: drain finished rows -> + b (armed) + f0 -> g smem ring (0 outside the frame) ======
     const int quarter = warp & 3;
@@ -507,7 +594,7 @@ static cudaError_t launch_bt_t(const CUtensorMap& tf, const CUtensorMap& tl, con
       if (e != cudaSuccess) return e;
       configured = true;
     }
-    return launch_k(kern, dim3(grid), dim3(kBtThreads), BtCfg<C, CO2, S>::SMEM, st, tf, tl, w1, w2, a);
+    return launch_k(kern, dim3(grid), dim3(BtThreads<C>::N), BtCfg<C, CO2, S>::SMEM, st, tf, tl, w1, w2, a);
   }
 }
 
