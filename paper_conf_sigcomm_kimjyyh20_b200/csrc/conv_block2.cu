@@ -44,8 +44,9 @@ struct B2Cfg {
   static constexpr int THREADS = kB2Threads + (EPI2 - 1) * 128;
   static constexpr int CCH = C / 8, KS = C / 16, N = 3 * C;
   static constexpr int RB = (256 / C) < 8 ? (256 / C) : 8;
-  static constexpr int NF = C >= 48 ? 3 : 4;  // f-row ring (one slot less than k_resblock at C = 48: weights grew)
-  static constexpr int NT = 3;                // t-row ring
+  static constexpr int NF = C >= 48 ? 3 : 5;  // f-row ring (C = 48: one slot less than k_resblock, weights grew;
+                                              // C = 32: 5 measured 5% faster than 4, 6-7 no better)
+  static constexpr int NT = C >= 48 ? 3 : 5;  // t-row ring (the cross-CTA t hand-off needs depth at C = 32)
   static constexpr int NO = C >= 48 ? 2 : 3;  // output staging rows
   static constexpr int SLABS = 3 * CCH;       // (kx, 8-channel) slabs of a conv's dy-fold weights
   static constexpr int R_FULL = 3 * C / 2, R_A1 = C, R_A2 = C / 2, R_B1 = C / 2, R_B2 = C;
