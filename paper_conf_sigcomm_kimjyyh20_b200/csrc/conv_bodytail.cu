@@ -40,8 +40,8 @@ struct BtThreads {
   static constexpr int N = kBtThreads + (EPI1 - 1) * 128;
 };
 static constexpr int kBtTW = 126;  // output pixels per strip
-static constexpr int kBtNF = 4;    // f-row ring
-static constexpr int kBtNT = 4;    // g-row ring
+static constexpr int kBtNF = 4;    // f-row ring (C = 48)
+static constexpr int kBtNT = 4;    // g-row ring (C = 48)
 static constexpr int kBtNO = 3;    // HR staging slots per tail group
 static constexpr int kBtLrChunks = 26;  // LR bytes [16 cb, 16 cb + 416) cover pixels x0-2 .. x0+129
 static constexpr uint32_t kBtLrSlot = (16 * kBtLrChunks * 5 + 127) & ~127u;
@@ -59,8 +59,15 @@ struct BtCfg {
   static constexpr uint32_t HRP = ((kBtTW * S * 3 + 15u) & ~15u) + 16u;  // staging row pitch (+16: alignment shift)
   static constexpr uint32_t OUTB = ((S * HRP) + 127u) & ~127u;
   static constexpr uint32_t ARMB = ((kArmOnesBytes + C * 32 + CO2 * 32) + 1023u) & ~1023u;
-  static constexpr size_t BASE = 1024 + W1_AL + W2_AL + (size_t)kBtNF * ROWB + (size_t)kBtNT * ROWB +
-                                 (size_t)2 * kBtNO * OUTB + ARMB;
+  // f- and g-row ring depths: 4 at C = 48 (shared memory is full); at C <= 32 as deep as fits with >= 8 LR slots,
+  // up to 8 (config 2's body + tail: 0.91 -> 0.77 ms per 30 540p frames from 4 to 8, profiles/r02_ab_bodytail.log)
+  static constexpr size_t base_at(int d) {
+    return 1024 + W1_AL + W2_AL + (size_t)2 * d * ROWB + (size_t)2 * kBtNO * OUTB + ARMB;
+  }
+  static constexpr int fit_lr(int d) { return (int)(((long long)227 * 1024 - 2048 - (long long)base_at(d)) / kBtLrSlot); }
+  static constexpr int DEPTH = C >= 48 ? kBtNF : (fit_lr(8) >= 8 ? 8 : (fit_lr(6) >= 8 ? 6 : kBtNF));
+  static constexpr int NF = DEPTH, NT = DEPTH;
+  static constexpr size_t BASE = base_at(DEPTH);
   static constexpr int NLR_FIT = (int)((227 * 1024 - 2048 - BASE) / kBtLrSlot);  // 2 KB: static smem (barriers)
   static constexpr int NLR = NLR_FIT > 12 ? 12 : NLR_FIT;
   static constexpr bool FITS = NLR >= 4;
@@ -103,27 +110,28 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
   uint8_t* sW1 = smem;
   uint8_t* sW2 = sW1 + Cfg::W1_AL;
   uint8_t* sF = sW2 + Cfg::W2_AL;
-  uint8_t* sT = sF + kBtNF * ROWB;
-  uint8_t* sO = sT + kBtNT * ROWB;
+  constexpr int kNF = Cfg::NF, kNT = Cfg::NT;
+  uint8_t* sT = sF + kNF * ROWB;
+  uint8_t* sO = sT + kNT * ROWB;
   uint8_t* sOnes = sO + 2 * kBtNO * OUTB;
   uint8_t* sB1 = sOnes + kArmOnesBytes;
   uint8_t* sB2 = sB1 + C * 32;
   uint8_t* sL = sOnes + Cfg::ARMB;
-  __shared__ __align__(8) uint64_t f_full[kBtNF], f_empty[kBtNF], t_full[kBtNT], t_empty[kBtNT], r1_ready[RB1],
+  __shared__ __align__(8) uint64_t f_full[kNF], f_empty[kNF], t_full[kNT], t_empty[kNT], r1_ready[RB1],
       r1_free[RB1], r2_ready[RB2], r2_free[RB2], l_full[NLR], l_empty[NLR], w_bar;
   __shared__ uint32_t tmem_base_sh;
 
   const int N = a.N, H = a.H, W = a.W;
   const int warp = warp_id();
   // spare g positions 128, 129 of every plane of every g slot are read by the two invalid conv2 lanes: zero them
-  for (int i = threadIdx.x; i < kBtNT * CCH * 2; i += blockDim.x) {
+  for (int i = threadIdx.x; i < kNT * CCH * 2; i += blockDim.x) {
     const int slot = i / (CCH * 2), rem = i % (CCH * 2);
     *reinterpret_cast<uint4*>(sT + slot * ROWB + (rem / 2) * PLANE + (128 + rem % 2) * 16) = make_uint4(0, 0, 0, 0);
   }
   fence_proxy_async_smem();
   if (warp == 0 && lane_id() == 0) {
-    for (int s = 0; s < kBtNF; ++s) { mbar_init(&f_full[s], 1); mbar_init(&f_empty[s], 1); }
-    for (int s = 0; s < kBtNT; ++s) { mbar_init(&t_full[s], 4); mbar_init(&t_empty[s], 1); }
+    for (int s = 0; s < kNF; ++s) { mbar_init(&f_full[s], 1); mbar_init(&f_empty[s], 1); }
+    for (int s = 0; s < kNT; ++s) { mbar_init(&t_full[s], 4); mbar_init(&t_empty[s], 1); }
     for (int s = 0; s < RB1; ++s) { mbar_init(&r1_ready[s], 1); mbar_init(&r1_free[s], 4); }
     for (int s = 0; s < RB2; ++s) { mbar_init(&r2_ready[s], 1); mbar_init(&r2_free[s], 4); }
     for (int s = 0; s < NLR; ++s) { mbar_init(&l_full[s], 1); mbar_init(&l_empty[s], 1); }
@@ -192,7 +200,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         mbar_arrive_expect_tx(&f_full[s], CCH * PLANE);
         tma_load_5d(sF + s * ROWB, &tm_f, &f_full[s], 0, x0 - 2, y0 - 2 + i, 0, n);
         SR_BDBG(0, i)
-        if (++s == kBtNF) { s = 0; ph ^= 1; }
+        if (++s == kNF) { s = 0; ph ^= 1; }
         if (i >= 4) {  // f row y0-2+i is the last one output row r = y0+i-4 needs: its LR rows r-2 .. r+2 now
           mbar_wait(&l_empty[ls], lph ^ 1);
           mbar_arrive_expect_tx(&l_full[ls], 16 * kBtLrChunks * 5);
@@ -233,7 +241,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           mma_commit(&r1_ready[ring_idx<RB1>(g + 1)]);
           mma_commit(&r1_ready[ring_idx<RB1>(g + 2)]);
         }
-        if (++fs == kBtNF) { fs = 0; fph ^= 1; }
+        if (++fs == kNF) { fs = 0; fph ^= 1; }
       }
       G1 += n_f + 2;
       SR_PIECE_END
@@ -269,7 +277,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
           mma_commit(&r2_ready[ring_idx<RB2>(g + 1)]);
           mma_commit(&r2_ready[ring_idx<RB2>(g + 2)]);
         }
-        if (++ts == kBtNT) { ts = 0; tph ^= 1; }
+        if (++ts == kNT) { ts = 0; tph ^= 1; }
       }
       G2 += n_t + 2;
       SR_PIECE_END
@@ -318,8 +326,8 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         ld_res(q + EPI1);
       }
       const unsigned ti = E + (unsigned)(q - 1);
-      const int ts = (int)(ti % kBtNT);
-      const uint32_t tph = (ti / kBtNT) & 1u;
+      const int ts = (int)(ti % kNT);
+      const uint32_t tph = (ti / kNT) & 1u;
       if (emit) mbar_wait(&t_empty[ts], tph ^ 1);
       const int b = ring_idx<RB1>(g);
       mbar_wait(&r1_ready[b], (uint32_t)(g / RB1) & 1u);
@@ -421,7 +429,7 @@ k_bodytail(const __grid_constant__ CUtensorMap tm_f, const __grid_constant__ CUt
         __syncwarp();
         if (lane_id() == 0) mbar_arrive(&t_full[ts]);
         if (warp == 2 && lane_id() == 0) { SR_BDBG(4, q + 1) }
-        if (++ts == kBtNT) { ts = 0; tph ^= 1; }
+        if (++ts == kNT) { ts = 0; tph ^= 1; }
       }
     }
     G += n_f + 2;
