@@ -579,7 +579,9 @@ def main():
     ap.add_argument("--partition", type=int, default=40,
                     help="SMs of the training partition (green contexts); 0 = inference and training sequential")
     ap.add_argument("--ref-band", type=int, default=REF_BAND, help=argparse.SUPPRESS)
-    args = ap.parse_args()
+    args, extra = ap.parse_known_args()
+    if extra and args.workload != "live":  # the live harness takes its own options (--streams, --seconds, --i420, ...)
+        ap.error(f"unrecognized arguments: {' '.join(extra)}")
     if args.warmup < 3:
         raise SystemExit("bench: --warmup must be >= 3")
     if "WORLD_SIZE" not in os.environ and args.gpus > 1:
